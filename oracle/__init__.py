@@ -1,0 +1,201 @@
+"""ctypes wrapper of the CPU oracle (TEST INFRASTRUCTURE ONLY).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+``--impl reference`` legs may import this package.  The product path
+(paper_conf_ipps_heislersdms24_b200) never imports it, and it never takes an
+input from the CUDA path.  See bte_oracle.h for the method and citations.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "bte_oracle.c")
+_HDR = os.path.join(_HERE, "bte_oracle.h")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+OK, EINVAL, ENOCONV = 0, 1, 5
+
+
+def build(force=False):
+    """Compile liboracle.so with gcc (plain -O2, no fast-math, OpenMP)."""
+    stale = (not os.path.exists(_LIB) or
+             os.path.getmtime(_LIB) < max(os.path.getmtime(_SRC), os.path.getmtime(_HDR)))
+    if force or stale:
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fno-fast-math", "-shared", "-fPIC",
+                               _SRC, "-o", _LIB, "-lm"])
+    return _LIB
+
+
+class _Problem(C.Structure):
+    _fields_ = [
+        ("dim", C.c_int32), ("n_cells", C.c_int64),
+        ("face_offsets", C.c_void_p), ("face_nbr", C.c_void_p), ("face_area", C.c_void_p),
+        ("face_normal", C.c_void_p), ("cell_volume", C.c_void_p),
+        ("n_bands", C.c_int32), ("omega", C.c_void_p), ("vg", C.c_void_p), ("tau", C.c_void_p),
+        ("C", C.c_void_p),
+        ("n_dirs", C.c_int32), ("s", C.c_void_p), ("w", C.c_void_p),
+        ("n_bfaces", C.c_int64), ("bkind", C.c_void_p), ("t_wall", C.c_void_p),
+        ("temp_rule", C.c_int32), ("newton_rtol", C.c_double), ("newton_maxit", C.c_int32),
+    ]
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(build())
+        P = C.POINTER(_Problem)
+        vp, i32, i64, dbl = C.c_void_p, C.c_int32, C.c_int64, C.c_double
+        _lib.oracle_I0.argtypes = [dbl, dbl, dbl]
+        _lib.oracle_I0.restype = dbl
+        _lib.oracle_weight.argtypes = [P, i32]
+        _lib.oracle_weight.restype = dbl
+        _lib.oracle_reflection_map.argtypes = [P, vp]
+        _lib.oracle_update_intensity.argtypes = [P, vp, vp, vp, vp, dbl, i32, i32]
+        _lib.oracle_update_intensity.restype = None
+        _lib.oracle_energy.argtypes = [P, vp, i32, i32, vp]
+        _lib.oracle_energy.restype = None
+        _lib.oracle_newton.argtypes = [P, vp, vp, vp]
+        _lib.oracle_equilibrium.argtypes = [P, vp, i32, i32, vp]
+        _lib.oracle_equilibrium.restype = None
+        _lib.oracle_run.argtypes = [P, dbl, i64, vp, vp]
+        _lib.oracle_step_cells_equilibrium.argtypes = [P, vp, vp, vp, i64, dbl, vp, vp]
+    return _lib
+
+
+def _ptr(a):
+    return a.ctypes.data_as(C.c_void_p)
+
+
+class Problem:
+    """A mesh + band table + direction set + BCs as the oracle sees them."""
+
+    def __init__(self, mesh, bands, dirs, bcs, temp_rule=0, rtol=1e-12, maxit=50):
+        f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
+        i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
+        i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
+        self.keep = dict(
+            face_offsets=i64(mesh["face_offsets"]), face_nbr=i64(mesh["face_nbr"]),
+            face_area=f64(mesh["face_area"]), face_normal=f64(mesh["face_normal"]),
+            cell_volume=f64(mesh["cell_volume"]),
+            omega=f64(bands["omega"]), vg=f64(bands["vg"]), tau=f64(bands["tau"]), C=f64(bands["C"]),
+            s=f64(dirs["s"]), w=f64(dirs["w"]),
+            bkind=i32(bcs["kind"]), t_wall=f64(bcs["t_wall"]),
+        )
+        k = self.keep
+        self.nc, self.nb, self.nd = int(mesh["n_cells"]), int(bands["n_bands"]), int(dirs["n_dirs"])
+        self.nbf = int(bcs["n_bfaces"])
+        self.s = _Problem(
+            dim=int(mesh["dim"]), n_cells=self.nc,
+            face_offsets=_ptr(k["face_offsets"]).value, face_nbr=_ptr(k["face_nbr"]).value,
+            face_area=_ptr(k["face_area"]).value, face_normal=_ptr(k["face_normal"]).value,
+            cell_volume=_ptr(k["cell_volume"]).value,
+            n_bands=self.nb, omega=_ptr(k["omega"]).value, vg=_ptr(k["vg"]).value,
+            tau=_ptr(k["tau"]).value, C=_ptr(k["C"]).value,
+            n_dirs=self.nd, s=_ptr(k["s"]).value, w=_ptr(k["w"]).value,
+            n_bfaces=self.nbf, bkind=_ptr(k["bkind"]).value, t_wall=_ptr(k["t_wall"]).value,
+            temp_rule=int(temp_rule), newton_rtol=float(rtol), newton_maxit=int(maxit),
+        )
+        self._r = None
+
+    @property
+    def ref(self):
+        return C.byref(self.s)
+
+    # -- pieces of the method -------------------------------------------------
+    def I0(self, b, T):
+        return lib().oracle_I0(float(self.keep["C"][b]), float(self.keep["omega"][b]), float(T))
+
+    def weight(self, b):
+        return lib().oracle_weight(self.ref, int(b))
+
+    def weights(self):
+        return np.array([self.weight(b) for b in range(self.nb)])
+
+    def reflection_map(self):
+        if self._r is None:
+            r = np.empty((max(self.nbf, 1), self.nd), dtype=np.int32)
+            rc = lib().oracle_reflection_map(self.ref, _ptr(r))
+            if rc != OK:
+                raise ValueError("specular reflection not closed on the direction set")
+            self._r = r
+        return self._r
+
+    def equilibrium(self, T, b_lo=0, b_hi=None):
+        b_hi = self.nb if b_hi is None else b_hi
+        T = np.ascontiguousarray(np.broadcast_to(np.asarray(T, np.float64), (self.nc,)))
+        I = np.empty((b_hi - b_lo, self.nd, self.nc))
+        lib().oracle_equilibrium(self.ref, _ptr(T), int(b_lo), int(b_hi), _ptr(I))
+        return I
+
+    def update_intensity(self, T, I, dt, b_lo=0, b_hi=None):
+        b_hi = self.nb if b_hi is None else b_hi
+        T = np.ascontiguousarray(T, np.float64)
+        I = np.ascontiguousarray(I, np.float64)
+        out = np.zeros_like(I)
+        lib().oracle_update_intensity(self.ref, _ptr(self.reflection_map()), _ptr(T), _ptr(I),
+                                      _ptr(out), float(dt), int(b_lo), int(b_hi))
+        return out
+
+    def energy(self, I, b_lo=0, b_hi=None):
+        b_hi = self.nb if b_hi is None else b_hi
+        I = np.ascontiguousarray(I, np.float64)
+        E = np.empty(self.nc)
+        lib().oracle_energy(self.ref, _ptr(I), int(b_lo), int(b_hi), _ptr(E))
+        return E
+
+    def newton(self, E, T_guess):
+        E = np.ascontiguousarray(E, np.float64)
+        T = np.array(np.broadcast_to(np.asarray(T_guess, np.float64), (self.nc,)))
+        iters = np.zeros(self.nc, dtype=np.int32)
+        rc = lib().oracle_newton(self.ref, _ptr(E), _ptr(T), _ptr(iters))
+        if rc != OK:
+            raise RuntimeError(f"oracle newton failed rc={rc}")
+        return T, iters
+
+    def run(self, I, T, dt, nsteps):
+        """nsteps explicit steps from (I, T); returns new copies."""
+        I = np.array(I, dtype=np.float64, order="C")
+        T = np.array(T, dtype=np.float64, order="C")
+        assert I.shape == (self.nb, self.nd, self.nc)
+        self.reflection_map()  # raise early on an unclosed map
+        rc = lib().oracle_run(self.ref, float(dt), int(nsteps), _ptr(I), _ptr(T))
+        if rc != OK:
+            raise RuntimeError(f"oracle run failed rc={rc}")
+        return I, T
+
+    def step_cells_equilibrium(self, T0, cells, dt):
+        T0 = np.ascontiguousarray(T0, np.float64)
+        cells = np.ascontiguousarray(cells, np.int64)
+        out = np.empty((cells.size, self.nb, self.nd))
+        T1 = np.empty(cells.size)
+        rc = lib().oracle_step_cells_equilibrium(self.ref, _ptr(self.reflection_map()), _ptr(T0),
+                                                 _ptr(cells), int(cells.size), float(dt),
+                                                 _ptr(out), _ptr(T1))
+        if rc != OK:
+            raise RuntimeError(f"oracle sampled step failed rc={rc}")
+        return out, T1
+
+    # -- initial state ----------------------------------------------------------
+    def initial_state(self, t_init, ic_eps=0.0, seed=None, mult_fn=None):
+        """IC of the synthetic configs: I = I0_b(t_init) * multiplier, then
+        T = temperature of that field (Newton from t_init)."""
+        T = np.full(self.nc, float(t_init))
+        I = self.equilibrium(T)
+        if ic_eps:
+            from paper_conf_ipps_heislersdms24_b200.inputs import ic_multiplier, SEED
+            for b in range(self.nb):
+                I[b] *= ic_multiplier(self.nd, self.nc, b, ic_eps, SEED if seed is None else seed)
+            T, _ = self.newton(self.energy(I), T)
+        return I, T
+
+
+def problem_from_config(cfg, **kw):
+    return Problem(cfg.mesh, cfg.bands, cfg.dirs, cfg.bcs, temp_rule=cfg.temp_rule, **kw)
