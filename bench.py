@@ -1,0 +1,345 @@
+#!/usr/bin/env python
+"""Benchmark: cell.dir.band updates/s of the explicit phonon-BTE step on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4] [--impl ours|reference]
+
+N > 1 is launched by torch.distributed.run (one rank per GPU); band-rows are
+sharded across ranks with one NCCL all-reduce of the per-cell energy per step
+(strong scaling: the problem is fixed, each rank owns ~nb/N rows).
+
+A step is one pass of the whole hot path (upwind flux + relaxation + boundary
+faces + energy reduction + all-reduce + Newton temperature solve) over the
+workload.  Default workload: BASELINE.json configs[3], 3-D 64 x 64 x 32 hex
+mesh, 40 spectral bands (55 band-rows), 400 directions, Fig.-1 walls, seeded
++-10 % IC; FP64.  Each state copy is 23 GB, far larger than the 126 MB L2, so
+no L2 flush is needed between steps.
+
+Prints ONE JSON line on rank 0 (see DESIGN.md 6 for every key).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "cell*dir*band updates/s"
+WORKLOADS = {
+    "C3": "2-D 120x120 quad mesh (525 um), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
+    "C4": "3-D 64x64x32 hex mesh (8.2 um cells), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
+    "C5": "3-D 96x96x96 hex mesh (8.2 um cells), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
+}
+BYTES_PER_UPDATE = 16  # algorithmic: read I^n once, write I^{n+1} once
+
+
+def _peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            pk = json.load(f)
+        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def _traffic_from_profiles(config):
+    """Per-launch DRAM bytes of the interior flux kernel from the committed
+    `ncu --set full` summary, if one exists for this workload."""
+    path = os.path.join(ROOT, "profiles", "ncu_flux_summary.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        if d.get("config") == config:
+            return d.get("dram_bytes_per_launch")
+    except Exception:
+        pass
+    return None
+
+
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks and throttle reasons during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        rows = []
+        try:
+            for line in open(self.path):
+                f = [x.strip() for x in line.split(",")]
+                if len(f) >= 9:
+                    rows.append(f)
+        except Exception:
+            pass
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        smax = max(float(r[2]) for r in rows if r[2].replace(".", "").isdigit())
+        loaded = [x for x in sm if x > 0.5 * smax] or sm
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def _dist():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def cpu_baseline(cfg, budget_s=15.0, max_rows=16):
+    """The oracle as it stands, on this host's cores, on a bounded sample of the
+    workload: the full mesh and direction set, the first k band-rows, 1 step."""
+    import numpy as np
+    import oracle
+    from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+
+    cores = os.cpu_count() or 1
+    os.environ.setdefault("OMP_NUM_THREADS", str(cores))
+
+    def run(k, steps):
+        bands = gen.select_bands(cfg.bands, np.arange(k))
+        p = oracle.Problem(cfg.mesh, bands, cfg.dirs, cfg.bcs, temp_rule=cfg.temp_rule)
+        T = np.full(cfg.mesh["n_cells"], cfg.t_init)
+        I = p.equilibrium(T)
+        p.reflection_map()
+        t0 = time.perf_counter()
+        p.run(I, T, cfg.dt, steps)
+        return time.perf_counter() - t0
+
+    t1 = run(1, 1)
+    k = int(max(1, min(max_rows, cfg.bands["n_bands"], budget_s / max(t1, 1e-3))))
+    steps = 1
+    t = run(k, steps)
+    upd = cfg.mesh["n_cells"] * cfg.dirs["n_dirs"] * k * steps
+    return {"value": upd / t, "unit": METRIC.replace("updates/s", "updates/s"), "cores": cores,
+            "kind": "oracle",
+            "sample": f"{cfg.name}: full mesh ({cfg.mesh['n_cells']} cells) x {cfg.dirs['n_dirs']} dirs x first {k} "
+                      f"of {cfg.bands['n_bands']} band-rows, {steps} step(s), {t:.2f} s, OMP_NUM_THREADS={os.environ['OMP_NUM_THREADS']}"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle on the same workload/metric (rank 0 only)."""
+    rank, world, _ = _dist()
+    if rank != 0:
+        return
+    from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+    cfg = gen.make_config(args.config)
+    vals = []
+    cb = None
+    for i in range(args.warmup + args.steps):
+        r = cpu_baseline(cfg, budget_s=5.0)
+        if i >= args.warmup:
+            vals.append(r["value"])
+            cb = r
+    v = statistics.median(vals)
+    cb = dict(cb, value=v)
+    line = {"metric": METRIC, "value": v, "unit": "updates/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "higher_is_better": True, "impl": "reference", "dtype": "f64",
+            "data": "synthetic", "scaling": "strong",
+            "config": {"workload": WORKLOADS[args.config], "name": args.config},
+            "vs_baseline": None, "cpu_baseline": cb,
+            "e2e": {"value": v, "unit": "updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+
+    rank, world, local = _dist()
+    assert world == args.gpus or (world == 1 and args.gpus == 1), "launch N>1 with torch.distributed.run"
+    torch.cuda.set_device(local)
+    pg = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        pg = dist
+    from paper_conf_ipps_heislersdms24_b200 import bte
+    from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+
+    cfg = gen.make_config(args.config)
+    nccl_id = None
+    if world > 1:
+        from paper_conf_ipps_heislersdms24_b200.dist import share_nccl_id
+        nccl_id = share_nccl_id(pg, rank)
+    stream = torch.cuda.current_stream()
+    s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream,
+                               profile=True, band_group=args.band_group, block_threads=args.block_threads,
+                               max_spare_slabs=args.max_spare)
+    bte.apply_ic(s, cfg)
+    nb_loc = s.b_hi - s.b_lo
+    nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
+    dt = cfg.dt
+
+    def barrier():
+        if pg is not None:
+            pg.barrier()
+
+    # ---- warm-up
+    s.step(dt, args.warmup)
+    torch.cuda.synchronize()
+    s.reset_stats()
+
+    # ---- timed region: K steps, device-resident state
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        s.step(dt, args.steps)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    ms = e0.elapsed_time(e1)
+    st = s.stats()
+    clocks = clk.summary()
+    if pg is not None:
+        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        pg.all_reduce(t, op=pg.ReduceOp.MAX)
+        ms = float(t.item())
+    total_updates = nc * nd * nb * args.steps  # whole job, all ranks
+    value = total_updates / (ms / 1e3)
+
+    # ---- roofline of the dominant kernel (interior flux), from the library's
+    # CUDA events on the launching stream over the timed region
+    n_int = st["n_interior_cells"]
+    launches_int = args.steps * (-(-nb_loc // max(1, st["spare_slabs"])))
+    t_int = st["ms_flux_interior"] / max(1, launches_int) / 1e3
+    alg_bytes = BYTES_PER_UPDATE * n_int * nd * nb_loc / (-(-nb_loc // max(1, st["spare_slabs"])))
+    peak, peak_src = _peaks()
+    achieved = alg_bytes / t_int / 1e9 if t_int > 0 else None
+    traffic = _traffic_from_profiles(args.config)
+    roof = {"bound": "hbm", "kernel": "bte::flux_kernel (interior cells)", "achieved": achieved, "peak": peak,
+            "unit": "GB/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+            "peak_source": peak_src,
+            "alg_bytes_per_launch": alg_bytes,
+            "kernel_ms_per_launch": t_int * 1e3,
+            "share_of_step": st["ms_flux_interior"] / ms if ms > 0 else None,
+            "step_alg_GBs": BYTES_PER_UPDATE * nc * nd * nb_loc * args.steps / (ms / 1e3) / 1e9}
+    phases = {k: st[k] / args.steps for k in ("ms_flux_interior", "ms_flux_boundary", "ms_allreduce", "ms_newton")}
+
+    # ---- end-to-end through the public API with host buffers: upload the state
+    # (pinned host -> device) once, then every step bte_step + read T back.
+    e2e = None
+    if not args.no_e2e:
+        e2e = _e2e(s, pg, world, nb_loc, nb, nd, nc, dt, total_updates, args)
+
+    cb = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cb = cpu_baseline(cfg)
+    _emit(locals())
+
+
+def _e2e(s, pg, world, nb_loc, nb, nd, nc, dt, total_updates, args):
+    import torch
+    def barrier():
+        if pg is not None:
+            pg.barrier()
+    pin_I = torch.empty((nb_loc, nd, nc), dtype=torch.float64).pin_memory()
+    pin_T = torch.empty((nc,), dtype=torch.float64).pin_memory()
+    s.intensity(out=pin_I.numpy())
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    s.set_intensity(pin_I)
+    for _ in range(args.steps):
+        s.step(dt, 1)
+        s.temperature(out=pin_T.numpy())
+    torch.cuda.synchronize()
+    e2e_s = time.perf_counter() - t0
+    if pg is not None:
+        t = torch.tensor([e2e_s], device="cuda", dtype=torch.float64)
+        pg.all_reduce(t, op=pg.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    e2e = {"value": total_updates / e2e_s, "unit": "updates/s",
+           "h2d_bytes_per_step": int(nb * nd * nc * 8 / args.steps),
+           "d2h_bytes_per_step": int(nc * 8 * world),
+           "how": "timed: bte_set_intensity(state from pinned host) once + K x (bte_step(dt,1) + "
+                  "bte_get_temperature(pinned host)); wall clock, max over ranks"}
+    return e2e
+
+
+def _emit(v):
+    rank, world, args, s, pg = v["rank"], v["world"], v["args"], v["s"], v["pg"]
+    value, ms, nc, nd, nb, dt, roof, cb, e2e, clocks, st, phases = (
+        v[k] for k in ("value", "ms", "nc", "nd", "nb", "dt", "roof", "cb", "e2e", "clocks", "st", "phases"))
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "updates/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WORKLOADS[args.config], "name": args.config, "n_cells": nc, "n_dirs": nd,
+                       "n_band_rows": nb, "dt": dt, "parallelism": f"band-shard x{world}",
+                       "l2": "state 23 GB/copy >> 126 MB L2 (no flush needed)" if args.config != "C3"
+                             else "state 2.5 GB/copy >> L2"},
+            "roofline": roof, "cpu_baseline": cb, "e2e": e2e, "clocks": clocks,
+            "gpu_launches": st["kernel_launches"], "phases_ms_per_step": phases,
+            "newton_iter_max": st["newton_iter_max"], "band_group": st["band_group"],
+            "block_threads": st["block_threads"], "dir_chunks": st["dir_chunks"],
+            "spare_slabs": st["spare_slabs"],
+        }
+        print(json.dumps(line), flush=True)
+    s.close()
+    if pg is not None:
+        pg.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C4", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--band-group", type=int, default=0)
+    ap.add_argument("--block-threads", type=int, default=0)
+    ap.add_argument("--max-spare", type=int, default=0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

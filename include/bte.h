@@ -1,0 +1,227 @@
+/*
+ * bte.h -- C ABI of the B200-native explicit step of the non-gray phonon
+ * Boltzmann transport equation (E. Heisler, S. Mazumder, S. Saurav,
+ * A. Deshmukh, H. Sundar, "Automating GPU Scalability for Complex Scientific
+ * Models: Phonon Boltzmann Transport Equation", IPDPS 2024).
+ *
+ * Citations "Lnnn" are lines of the paper text (/root/reference/PAPER.md,
+ * not shipped); "SURVEY 8(c) #k" are the readings listed in DESIGN.md.
+ *
+ * What one step computes (all FP64), for every band-row b, direction d, cell c:
+ *
+ *   I'[b][d][c] = I + dt ( (I0_b(T_c) - I) / tau_b
+ *                          - (v_b / V_c) sum_f A_f (s_d . n_f) I_hat_f )      (Eq. 3, 5)
+ *   I_hat_f = I[b][d][c]                if s_d . n_f > 0   (first-order upwind,
+ *           = I[b][d][nbr(f)]           interior face       L264-267, L644-647)
+ *           = I0_b(T_wall(f))           isothermal wall     (Eq. 6)
+ *           = I[b][r_f(d)][c]           symmetric wall, s_r = s_d - 2 (s_d.n_f) n_f
+ *   E_c = sum_b c_b sum_d w_d I'[b][d][c]                                     (L412-418)
+ *   T_c' solves W sum_b c_b I0_b(T) = E_c  (Newton from T_c, W = sum_d w_d)   (L407-418, L555-561)
+ *   I0_b(T) = C_b / expm1(hbar omega_b / (kB T))
+ *   c_b = 1/(v_b tau_b) (temp_rule 0, default) or 1/v_b (temp_rule 1)
+ *
+ * Storage is band-major I[b][d][c] (L777-840: band-parallel loop order) with
+ * the cell index fastest.  Band-rows are sharded across ranks (L760-775): rank g
+ * of P owns rows [floor(g nb/P), floor((g+1) nb/P)); bands couple only through
+ * the per-cell energy, which is summed across ranks with one NCCL all-reduce of
+ * n_cells doubles per step.
+ *
+ * Conventions for every call:
+ *   - All pointers passed IN are borrowed for the duration of the call only and
+ *     are HOST pointers unless stated otherwise; inputs are deep-copied.
+ *   - Output buffers are caller-allocated HOST memory; getters synchronise the
+ *     library's stream before returning.
+ *   - Cell order at the ABI is always the caller's order (the library reorders
+ *     internally and undoes it in the getters).
+ *   - Errors are returned as bte_status; nothing aborts or throws across the
+ *     ABI.  bte_last_error() gives the message of the last failure.
+ *   - One context per host thread at a time.
+ */
+#ifndef BTE_H
+#define BTE_H
+
+#include <stdint.h>
+
+#if defined(BTE_BUILD) && defined(__GNUC__)
+#define BTE_API __attribute__((visibility("default")))
+#else
+#define BTE_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bte_ctx bte_ctx; /* opaque; owned by the caller until bte_destroy */
+
+typedef enum {
+    BTE_OK = 0,
+    BTE_EINVAL = 1,  /* invalid argument / input data (message says which) */
+    BTE_ENOMEM = 2,  /* device or host allocation failed */
+    BTE_ECUDA = 3,   /* CUDA runtime error */
+    BTE_ENCCL = 4,   /* NCCL missing or failed */
+    BTE_ENOCONV = 5, /* per-cell temperature solve did not converge (E <= 0 or NaN) */
+    BTE_ESTATE = 6   /* call not valid in the current state */
+} bte_status;
+
+/* Face-based finite-volume mesh (Eq. 3: polygonal/polyhedral cells with m
+ * faces of area A_i, L286-292).  2-D meshes are 3-D with unit depth: face areas
+ * are edge lengths, volumes are cell areas and every normal has n_z = 0
+ * (SURVEY 8(c) #18).  Each cell lists its own faces; an interior face therefore
+ * appears once in each of its two cells with opposite normals.
+ * Limits: at most 8 faces per cell, n_cells < 2^31. */
+typedef struct {
+    int32_t dim;                 /* 2 or 3 */
+    int64_t n_cells;
+    const int64_t *face_offsets; /* [n_cells+1], CSR offsets into the face arrays */
+    const int64_t *face_nbr;     /* [n_faces]: >= 0 neighbour cell id;
+                                    < 0: boundary face id = -1 - face_nbr */
+    const double *face_area;     /* [n_faces], > 0 */
+    const double *face_normal;   /* [n_faces][3], unit, outward from the owning cell */
+    const double *cell_volume;   /* [n_cells], > 0 */
+} bte_mesh;
+
+/* Band-rows: one row per (spectral band, polarization) present (L507-514). */
+typedef struct {
+    int32_t n_bands;
+    const double *omega;         /* [n_bands] centre angular frequency, rad/s, > 0 */
+    const double *d_omega;       /* [n_bands] width, rad/s (metadata; may be NULL) */
+    const double *vg;            /* [n_bands] group velocity |v_g|_b, m/s, > 0 */
+    const double *tau;           /* [n_bands] relaxation time, s, in (0, +inf] */
+    const int32_t *polarization; /* [n_bands] 0 = LA, 1 = TA (metadata; may be NULL) */
+    const double *i0_prefactor;  /* [n_bands] C_b > 0; required */
+} bte_bands;
+
+/* Discrete directions (L514-518, L654-664): unit vectors and solid-angle weights. */
+typedef struct {
+    int32_t n_dirs;
+    const double *s; /* [n_dirs][3], unit */
+    const double *w; /* [n_dirs], > 0 */
+} bte_dirs;
+
+/* Boundary conditions per boundary face id (Eq. 6). */
+#define BTE_BC_ISOTHERMAL 0
+#define BTE_BC_SYMMETRY 1
+typedef struct {
+    int64_t n_bfaces;
+    const int32_t *kind;  /* [n_bfaces] BTE_BC_ISOTHERMAL or BTE_BC_SYMMETRY */
+    const double *t_wall; /* [n_bfaces] wall temperature (K, > 0) of isothermal faces */
+} bte_bcs;
+
+/* bte_options.flags */
+#define BTE_FLAG_PROFILE 1u /* record CUDA events around every phase (see bte_stats) */
+
+typedef struct {
+    double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */
+    int32_t temp_rule;        /* 0: c_b = 1/(v_b tau_b) (default); 1: c_b = 1/v_b */
+    double newton_rtol;       /* stop when |dT| <= rtol T (default 1e-12) */
+    int32_t newton_max_iter;  /* default 50; bisection fallback after that */
+    int32_t rank, world;      /* band sharding; world == 1: single GPU, no NCCL */
+    int32_t device;           /* CUDA device ordinal */
+    const void *nccl_unique_id; /* world > 1: 128-byte ncclUniqueId from bte_nccl_unique_id()
+                                   on rank 0, broadcast by the caller.  NULL with world > 1:
+                                   no communicator; the caller reduces the energy itself
+                                   through the split-step calls (bte_step returns ESTATE) */
+    void *stream;             /* cudaStream_t to launch on (NULL: library-owned stream) */
+    uint32_t flags;           /* BTE_FLAG_* */
+    int32_t max_spare_slabs;  /* band slabs of workspace: <= 0 auto (double buffer when it
+                                 fits, else slab rotation), k > 0 forces at most k */
+    int32_t block_threads;    /* 0 auto; else 64..1024, multiple of 32 */
+    int32_t band_group;       /* 0 auto; else 1..8 band-rows per thread */
+} bte_options;
+
+/* Per-context counters since creation / the last bte_reset_stats. Phase
+ * times need BTE_FLAG_PROFILE and are sums of CUDA-event intervals on the
+ * library stream. */
+typedef struct {
+    int64_t steps;
+    int64_t kernel_launches;   /* kernels launched by bte_step */
+    int64_t updates;           /* (cell, dir, band) unknowns advanced on this rank */
+    double ms_flux_interior;   /* interior-cell flux + relaxation + energy partial */
+    double ms_flux_boundary;   /* boundary-cell kernel */
+    double ms_allreduce;       /* slot reduce + NCCL all-reduce (world > 1) */
+    double ms_newton;          /* temperature solve + I0 refresh */
+    double ms_total;           /* first to last event of the profiled steps */
+    int32_t newton_iter_max;   /* max Newton iterations of any cell */
+    int32_t spare_slabs;       /* workspace band slabs in use */
+    int32_t n_interior_cells;
+    int32_t band_group;
+    int32_t block_threads;
+    int32_t dir_chunks;        /* direction chunks per launch (grid.y factor) */
+} bte_stats;
+
+/* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,
+ * rank 0 / world 1 / device 0, everything else 0/NULL). */
+BTE_API bte_status bte_options_default(bte_options *o);
+
+/* Validate and deep-copy the problem, build the device layout (interior cells
+ * first, padded per-cell face slots, reflection maps, isothermal ghost tables)
+ * and initialise I = I0_b(t_init), T = t_init.  Collective when world > 1.
+ * EINVAL on: dim not 2/3; non-positive V, A, w, C, omega, v or tau; non-unit
+ * normals or directions; n_z != 0 in 2-D; a face id out of range; > 8 faces in
+ * a cell; a symmetric wall whose reflected direction is not in the set (1e-10);
+ * all temperature weights zero; more than 128 band-rows on one rank. */
+BTE_API bte_status bte_create(const bte_mesh *mesh, const bte_bands *bands, const bte_dirs *dirs,
+                      const bte_bcs *bcs, const bte_options *opts, bte_ctx **out);
+
+/* n explicit steps of size dt (Eq. 2-3).  Collective when world > 1; returns
+ * after the steps completed.  EINVAL if dt <= 0 or dt exceeds the positivity
+ * bound 1 / max_{c,b,d} (1/tau_b + v_b sum_f (A_f/V_c) max(s_d.n_f, 0))
+ * (see bte_dt_bound).  ENOCONV if a cell's temperature solve failed. */
+BTE_API bte_status bte_step(bte_ctx *ctx, double dt, int64_t n);
+
+/* Largest admissible dt (the positivity bound above, over all bands). */
+BTE_API bte_status bte_dt_bound(const bte_ctx *ctx, double *dt_max);
+
+/* T[n_cells] (host, caller order).  T is replicated on every rank. */
+BTE_API bte_status bte_get_temperature(const bte_ctx *ctx, double *T);
+
+/* I[b_hi-b_lo][n_dirs][n_cells] (host, caller order) for global band-rows
+ * [b_lo, b_hi), which must lie inside this rank's bte_band_range. */
+BTE_API bte_status bte_get_intensity(const bte_ctx *ctx, int32_t b_lo, int32_t b_hi, double *I);
+
+/* Overwrite rows [b_lo, b_hi) of I (same layout as bte_get_intensity).  T is
+ * NOT changed; call bte_solve_temperature after the last row is set. */
+BTE_API bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const double *I);
+
+/* T <- temperature of the current I (energy reduction, all-reduce, Newton from
+ * the current T), and I0 refreshed.  Collective when world > 1. */
+BTE_API bte_status bte_solve_temperature(bte_ctx *ctx);
+
+/* Set T (host, caller order) and I = I0_b(T_c) for every local row (local
+ * thermal equilibrium).  Not collective. */
+BTE_API bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T);
+
+/* This rank's band-rows [b_lo, b_hi). */
+BTE_API bte_status bte_band_range(const bte_ctx *ctx, int32_t *b_lo, int32_t *b_hi);
+
+/* Split step, for callers that reduce the energy themselves (e.g. tests of
+ * band sharding on one device): begin = flux/relaxation of the local rows and
+ * the local energy partial; get/set energy move E[n_cells] (host, caller
+ * order); finish = temperature solve from the set energy, I0 refresh and state
+ * advance.  bte_step(ctx, dt, 1) == begin; (reduce E); finish. */
+BTE_API bte_status bte_step_begin(bte_ctx *ctx, double dt);
+BTE_API bte_status bte_get_energy(const bte_ctx *ctx, double *E);
+BTE_API bte_status bte_set_energy(bte_ctx *ctx, const double *E);
+BTE_API bte_status bte_step_finish(bte_ctx *ctx);
+
+/* Counters (see bte_stats). */
+BTE_API bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st);
+BTE_API bte_status bte_reset_stats(bte_ctx *ctx);
+
+/* 128-byte NCCL unique id (call on rank 0 only, then broadcast). ENCCL if the
+ * NCCL library cannot be loaded (BTE_NCCL_LIB overrides the search). */
+BTE_API bte_status bte_nccl_unique_id(void *id128);
+
+/* Message of the last failure on ctx (ctx may be NULL: last bte_create /
+ * global failure of this thread).  Never NULL. */
+BTE_API const char *bte_last_error(const bte_ctx *ctx);
+BTE_API const char *bte_status_string(bte_status s);
+
+/* Release device memory, streams and the NCCL communicator.  NULL is a no-op. */
+BTE_API void bte_destroy(bte_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BTE_H */

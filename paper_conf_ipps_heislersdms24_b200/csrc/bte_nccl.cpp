@@ -1,0 +1,96 @@
+// bte_nccl.cpp -- dlopen wrapper over the NCCL C API (see bte_nccl.h).
+#include "bte_nccl.h"
+
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+
+namespace bte {
+namespace nccl {
+namespace {
+
+struct Api {
+    void *h = nullptr;
+    ncclResult_t (*getUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*commInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*allReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+    const char *(*getErrorString)(ncclResult_t) = nullptr;
+    std::string why;
+};
+
+Api *api() {
+    static Api a;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char *cands[] = {getenv("BTE_NCCL_LIB"), "libnccl.so.2", "libnccl.so",
+                               "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
+        for (const char *p : cands) {
+            if (!p || !*p) continue;
+            a.h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
+            if (a.h) break;
+        }
+        if (!a.h) {
+            a.why = "cannot dlopen libnccl.so.2 (set BTE_NCCL_LIB)";
+            return;
+        }
+        a.getUniqueId = (decltype(a.getUniqueId))dlsym(a.h, "ncclGetUniqueId");
+        a.commInitRank = (decltype(a.commInitRank))dlsym(a.h, "ncclCommInitRank");
+        a.allReduce = (decltype(a.allReduce))dlsym(a.h, "ncclAllReduce");
+        a.commDestroy = (decltype(a.commDestroy))dlsym(a.h, "ncclCommDestroy");
+        a.getErrorString = (decltype(a.getErrorString))dlsym(a.h, "ncclGetErrorString");
+        if (!a.getUniqueId || !a.commInitRank || !a.allReduce || !a.commDestroy || !a.getErrorString) {
+            a.why = "libnccl is missing a required symbol";
+            a.h = nullptr;
+        }
+    });
+    return a.h ? &a : nullptr;
+}
+
+const char *why() { return "NCCL unavailable: cannot load libnccl.so.2 with the required symbols (set BTE_NCCL_LIB)"; }
+
+}  // namespace
+
+bool unique_id(void *id128, std::string *err) {
+    Api *a = api();
+    if (!a) return *err = why(), false;
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId must be 128 bytes");
+    ncclUniqueId id;
+    ncclResult_t r = a->getUniqueId(&id);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    std::memcpy(id128, &id, sizeof id);
+    return true;
+}
+
+bool init(Comm *c, const void *id128, int rank, int world, std::string *err) {
+    Api *a = api();
+    if (!a) return *err = why(), false;
+    ncclUniqueId id;
+    std::memcpy(&id, id128, sizeof id);
+    ncclComm_t comm = nullptr;
+    ncclResult_t r = a->commInitRank(&comm, world, id, rank);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    c->comm = comm;
+    return true;
+}
+
+bool allreduce_sum_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    ncclResult_t r = a->allReduce(buf, buf, (size_t)n, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    return true;
+}
+
+void destroy(Comm &c) {
+    Api *a = api();
+    if (a && c.comm) a->commDestroy((ncclComm_t)c.comm);
+    c.comm = nullptr;
+}
+
+}  // namespace nccl
+}  // namespace bte

@@ -1,0 +1,281 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Element by element on the same seeded inputs: relative 1e-10 on I and 1e-9 on
+T (north star), at sizes that span several thread blocks with ragged tails, in
+every launch configuration the library can pick (band groups, block sizes,
+direction chunking, slab rotation), plus sampled outputs at the full bench
+size.
+"""
+import dataclasses
+
+import numpy as np
+import pytest
+
+from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+from tests._parity import RTOL_I, RTOL_T, assert_parity, gpu_run, oracle_run, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def bte():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    from paper_conf_ipps_heislersdms24_b200 import bte as mod
+    return mod
+
+
+def _cfg(name, steps=None, **kw):
+    cfg = gen.make_config(name)
+    if steps is not None:
+        cfg = dataclasses.replace(cfg, nsteps=steps)
+    return dataclasses.replace(cfg, **kw) if kw else cfg
+
+
+# ------------------------------------------------------------------ configs
+def test_c1_full_50_steps(bte, oracle_mod):
+    cfg = _cfg("C1")
+    Io, To = oracle_run(oracle_mod, cfg, cfg.nsteps)
+    Ig, Tg, st = gpu_run(cfg, cfg.nsteps)
+    assert_parity(Ig, Tg, Io, To)
+    assert st["steps"] == cfg.nsteps
+    assert To.max() > 300.5  # the hot spot moved heat in
+
+
+@pytest.mark.parametrize("bg", [1, 2, 4, 8])
+@pytest.mark.parametrize("threads", [64, 256])
+def test_c1_launch_configs(bte, oracle_mod, bg, threads):
+    cfg = _cfg("C1", steps=20)
+    Io, To = oracle_run(oracle_mod, cfg, 20)
+    Ig, Tg, st = gpu_run(cfg, 20, band_group=bg, block_threads=threads)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_c2_100_steps(bte, oracle_mod):
+    cfg = _cfg("C2", steps=100)
+    Io, To = oracle_run(oracle_mod, cfg, 100)
+    Ig, Tg, st = gpu_run(cfg, 100)
+    assert_parity(Ig, Tg, Io, To)
+    assert st["newton_iter_max"] >= 2
+
+
+@pytest.mark.parametrize("spare", [1, 3, 5])
+def test_slab_rotation_matches(bte, oracle_mod, spare):
+    """Slab rotation (nb + k slabs, band batches per launch) == oracle."""
+    cfg = _cfg("C2", steps=30)
+    Io, To = oracle_run(oracle_mod, cfg, 30)
+    Ig, Tg, st = gpu_run(cfg, 30, max_spare_slabs=spare, band_group=4)
+    assert st["spare_slabs"] == spare
+    assert_parity(Ig, Tg, Io, To)
+
+
+@pytest.mark.parametrize("shape", [(6, 5, 4), (13, 7, 5), (33, 9, 3)])
+def test_3d_ragged(bte, oracle_mod, shape):
+    cfg = gen.small_3d_config(shape, n_spectral=3, ntheta=4, nphi=8)
+    Io, To = oracle_run(oracle_mod, cfg, 25)
+    Ig, Tg, _ = gpu_run(cfg, 25)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_3d_400_dirs_55_rows_small_mesh(bte, oracle_mod):
+    """The bench's band table and direction set on a small 3-D mesh."""
+    h = 8.2e-6
+    mesh = gen.gen_mesh((7, 6, 5), (h, h, h))
+    bands, dirs = gen.gen_bands_si(40), gen.gen_dirs_product(20, 20)
+    bcs = gen.gen_bcs_fig1(mesh, radius=2 * h)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    cfg = gen.Config("3d55", mesh, bands, dirs, bcs, 300.0, dt, 10, ic_eps=0.1)
+    Io, To = oracle_run(oracle_mod, cfg, 10)
+    Ig, Tg, _ = gpu_run(cfg, 10)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_c3_mesh_scaled_short(bte, oracle_mod):
+    """C3 (paper's 120 x 120, 55 rows) with 24 of the 400 directions, 5 steps."""
+    cfg = _cfg("C3")
+    dirs = gen.gen_dirs_product(4, 6)
+    dt = 0.5 * gen.cartesian_dt_bound(cfg.mesh, cfg.bands, dirs)
+    cfg = dataclasses.replace(cfg, dirs=dirs, dt=dt)
+    Io, To = oracle_run(oracle_mod, cfg, 5)
+    Ig, Tg, _ = gpu_run(cfg, 5)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_c3_paper_faithful_dt(bte, oracle_mod):
+    """Paper regime: IC 300 K, dt = 1 ps (L1328), reduced direction set."""
+    cfg = gen.make_config("C3", variant="paper")
+    dirs = gen.gen_dirs_inplane(20)  # the paper's 2-D set of 20 (L594-595)
+    cfg = dataclasses.replace(cfg, dirs=dirs, bands=gen.select_bands(cfg.bands, np.arange(0, 55, 6)))
+    Io, To = oracle_run(oracle_mod, cfg, 20)
+    Ig, Tg, _ = gpu_run(cfg, 20)
+    assert_parity(Ig, Tg, Io, To)
+
+
+# ------------------------------------------------------------------ edge cases
+def test_single_cell_all_walls(bte, oracle_mod):
+    mesh = gen.gen_mesh((1, 1), (1e-6, 1e-6))
+    bands = gen.gen_bands_si(4)
+    dirs = gen.gen_dirs_product(2, 8)
+    bcs = gen.gen_bcs_walls(mesh, {gen.WALL_XM: (gen.ISOTHERMAL, 320.0), gen.WALL_XP: (gen.SYMMETRY, 0),
+                                   gen.WALL_YM: (gen.ISOTHERMAL, 290.0), gen.WALL_YP: (gen.SYMMETRY, 0)})
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    cfg = gen.Config("1cell", mesh, bands, dirs, bcs, 300.0, dt, 10, ic_eps=0.2)
+    Io, To = oracle_run(oracle_mod, cfg, 10)
+    Ig, Tg, st = gpu_run(cfg, 10)
+    assert st["n_interior_cells"] == 0
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_no_boundary_cells_periodic_like(bte, oracle_mod):
+    """A mesh with no boundary faces at all (a periodic 4 x 3 torus)."""
+    mesh = gen.gen_mesh((4, 3), (1e-6, 1e-6))
+    nbr = mesh["face_nbr"].reshape(-1, 4).copy()
+    c = np.arange(12)
+    i, j = c % 4, c // 4
+    nbr[:, 0] = (i - 1) % 4 + 4 * j
+    nbr[:, 1] = (i + 1) % 4 + 4 * j
+    nbr[:, 2] = i + 4 * ((j - 1) % 3)
+    nbr[:, 3] = i + 4 * ((j + 1) % 3)
+    mesh = dict(mesh, face_nbr=nbr.ravel(), n_bfaces=0)
+    bcs = {"n_bfaces": 0, "kind": np.zeros(0, np.int32), "t_wall": np.zeros(0)}
+    bands, dirs = gen.gen_bands_si(3), gen.gen_dirs_inplane(12)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    cfg = gen.Config("torus", mesh, bands, dirs, bcs, 300.0, dt, 10, ic_eps=0.3)
+    Io, To = oracle_run(oracle_mod, cfg, 15)
+    Ig, Tg, st = gpu_run(cfg, 15)
+    assert st["n_interior_cells"] == 12
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_ballistic_row_with_R1(bte, oracle_mod):
+    """A tau = inf band-row (no scattering) under temp_rule 1 (c_b = 1/v_b)."""
+    mesh = gen.gen_mesh((9, 7), (1e-6, 1e-6))
+    bands = gen.gen_bands_si(3)
+    bands["tau"][1] = np.inf
+    dirs = gen.gen_dirs_inplane(16)
+    bcs = gen.gen_bcs_fig1(mesh, radius=2e-6)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    cfg = gen.Config("ballistic", mesh, bands, dirs, bcs, 300.0, dt, 10, ic_eps=0.1, temp_rule=1)
+    Io, To = oracle_run(oracle_mod, cfg, 30)
+    Ig, Tg, _ = gpu_run(cfg, 30)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_permuted_unstructured_order(bte, oracle_mod):
+    """Random cell labels and face order: the generic connectivity path."""
+    cfg = gen.small_3d_config((7, 5, 4), n_spectral=2)
+    mesh, _ = gen.permute_mesh(cfg.mesh, seed=11)
+    cfg = dataclasses.replace(cfg, mesh=mesh)
+    Io, To = oracle_run(oracle_mod, cfg, 15)
+    Ig, Tg, _ = gpu_run(cfg, 15)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_zero_steps_is_identity_and_dt_bound(bte, oracle_mod):
+    cfg = _cfg("C1")
+    with bte.solver_from_config(cfg) as s:
+        bte.apply_ic(s, cfg)
+        I0 = s.intensity()
+        s.step(cfg.dt, 0)
+        assert np.array_equal(s.intensity(), I0)
+        assert abs(s.dt_bound() / cfg.extra["dt_bound"] - 1) < 1e-12
+        with pytest.raises(bte.BTEError) as e:
+            s.step(s.dt_bound() * 1.01, 1)
+        assert e.value.status == bte.BTE_EINVAL
+        with pytest.raises(bte.BTEError):
+            s.step(-1.0, 1)
+
+
+def test_equilibrium_invariance_full_bench_size(bte):
+    """P1 at the bench size: all walls at T0, uniform IC -> I and T stay put."""
+    cfg = _cfg("C4")
+    bcs = gen.gen_bcs_fig1(cfg.mesh, t_hot=300.0)
+    with bte.Solver(cfg.mesh, cfg.bands, cfg.dirs, bcs, t_init=300.0) as s:
+        I0 = s.intensity(0, 1)
+        s.step(cfg.dt, 3)
+        T = s.temperature()
+        assert np.max(np.abs(T / 300.0 - 1)) < 1e-13
+        assert rel_err(s.intensity(0, 1), I0) < 1e-13
+        last = s.b_hi - 1
+        I_last = s.intensity(last, last + 1)
+    with bte.Solver(cfg.mesh, cfg.bands, cfg.dirs, bcs, t_init=300.0) as s2:
+        assert rel_err(I_last, s2.intensity(last, last + 1)) < 1e-13
+
+
+def test_sampled_full_bench_size(bte, oracle_mod):
+    """C4 at full size in the bench's launch configuration: one step from a
+    non-uniform equilibrium, sampled cells against the oracle cell by cell."""
+    cfg = _cfg("C4")
+    nc = cfg.mesh["n_cells"]
+    rng = np.random.default_rng(5)
+    T0 = 300.0 + 40.0 * rng.random(nc)
+    nx, ny, nz = cfg.mesh["shape"]
+    corners = [0, nx - 1, nx * ny - 1, nc - 1, nx * (ny - 1), nc - nx]
+    cells = np.unique(np.concatenate([corners, rng.integers(0, nc, 40),
+                                      [nx // 2 + nx * (ny // 2) + nx * ny * (nz - 1)]]))
+    p = oracle_mod.problem_from_config(cfg)
+    Io_sel, To_sel = p.step_cells_equilibrium(T0, cells, cfg.dt)
+    with bte.solver_from_config(cfg) as s:
+        s.set_equilibrium(T0)
+        s.step(cfg.dt, 1)
+        Tg = s.temperature()
+        Ig_sel = np.empty((cells.size, s.n_bands, s.n_dirs))
+        buf = np.empty((1, s.n_dirs, nc))
+        for b in range(s.n_bands):
+            s.intensity(b, b + 1, out=buf)
+            Ig_sel[:, b, :] = buf[0][:, cells].T
+    assert rel_err(Ig_sel, Io_sel) <= RTOL_I
+    assert rel_err(Tg[cells], To_sel) <= RTOL_T
+
+
+def test_split_step_band_sharding_emulated(bte, oracle_mod):
+    """Band sharding over 2 'ranks' on one device: each context owns half the
+    rows; the caller sums the energy partials (the all-reduce) and both finish.
+    Must equal the single-context result and the oracle."""
+    cfg = _cfg("C2", steps=10)
+    rng = np.random.default_rng(9)
+    T0 = 300.0 + 20 * rng.random(cfg.mesh["n_cells"])
+    p = oracle_mod.problem_from_config(cfg)
+    Io, To = p.run(p.equilibrium(T0), T0, cfg.dt, 10)
+    ranks = [bte.solver_from_config(cfg, rank=r, world=2) for r in range(2)]
+    try:
+        for s in ranks:
+            s.set_equilibrium(T0)
+        with pytest.raises(bte.BTEError):
+            ranks[0].step(cfg.dt, 1)  # no communicator: split calls only
+        for _ in range(10):
+            for s in ranks:
+                s.step_begin(cfg.dt)
+            E = ranks[0].energy() + ranks[1].energy()
+            for s in ranks:
+                s.set_energy(E)
+                s.step_finish()
+        Ts = [s.temperature() for s in ranks]
+        assert np.array_equal(Ts[0], Ts[1])
+        Ig = np.concatenate([s.intensity() for s in ranks], axis=0)
+        assert [(s.b_lo, s.b_hi) for s in ranks] == [(0, 6), (6, 13)]
+    finally:
+        for s in ranks:
+            s.close()
+    assert_parity(Ig, Ts[0], Io, To)
+
+
+def test_profile_stats(bte):
+    cfg = _cfg("C2")
+    with bte.solver_from_config(cfg, profile=True) as s:
+        s.step(cfg.dt, 3)
+        st = s.stats()
+    assert st["steps"] == 3 and st["kernel_launches"] == 9
+    assert st["ms_flux_interior"] > 0 and st["ms_newton"] > 0 and st["ms_total"] > 0
+    assert st["updates"] == 3 * cfg.n_updates_per_step
+
+
+def test_nan_energy_reports_enoconv(bte):
+    cfg = _cfg("C1")
+    with bte.solver_from_config(cfg) as s:
+        I = s.intensity()
+        I[:, :, 5] = -1.0  # negative energy in one cell: no temperature exists
+        s.set_intensity(I)
+        with pytest.raises(bte.BTEError) as e:
+            s.solve_temperature()
+        assert e.value.status == bte.BTE_ENOCONV
