@@ -79,6 +79,9 @@ typedef struct {
     const double *face_area;     /* [n_faces], > 0 */
     const double *face_normal;   /* [n_faces][3], unit, outward from the owning cell */
     const double *cell_volume;   /* [n_cells], > 0 */
+    const double *cell_centre;   /* [n_cells][3] optional (NULL: keep the caller's order).  A
+                                    locality hint only: cells are stored internally in Morton
+                                    order of these points; results do not depend on it. */
 } bte_mesh;
 
 /* Band-rows: one row per (spectral band, polarization) present (L507-514). */
@@ -109,7 +112,8 @@ typedef struct {
 } bte_bcs;
 
 /* bte_options.flags */
-#define BTE_FLAG_PROFILE 1u /* record CUDA events around every phase (see bte_stats) */
+#define BTE_FLAG_PROFILE 1u       /* record CUDA events around every phase (see bte_stats) */
+#define BTE_FLAG_GENERIC_FACES 2u /* never use the opposite-face-pair layout (testing) */
 
 typedef struct {
     double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */
@@ -128,6 +132,7 @@ typedef struct {
                                  fits, else slab rotation), k > 0 forces at most k */
     int32_t block_threads;    /* 0 auto; else 64..1024, multiple of 32 */
     int32_t band_group;       /* 0 auto; else 1..8 band-rows per thread */
+    int32_t dir_chunk;        /* 0 auto; else directions per thread block */
 } bte_options;
 
 /* Per-context counters since creation / the last bte_reset_stats. Phase

@@ -17,6 +17,7 @@ LIB_PATH = os.path.join(_HERE, "libbte.so")
 
 BTE_OK, BTE_EINVAL, BTE_ENOMEM, BTE_ECUDA, BTE_ENCCL, BTE_ENOCONV, BTE_ESTATE = range(7)
 BTE_FLAG_PROFILE = 1
+BTE_FLAG_GENERIC_FACES = 2
 ISOTHERMAL, SYMMETRY = 0, 1
 
 
@@ -33,7 +34,7 @@ _STATUS = {0: "BTE_OK", 1: "BTE_EINVAL", 2: "BTE_ENOMEM", 3: "BTE_ECUDA", 4: "BT
 class Mesh(C.Structure):
     _fields_ = [("dim", C.c_int32), ("n_cells", C.c_int64), ("face_offsets", C.c_void_p),
                 ("face_nbr", C.c_void_p), ("face_area", C.c_void_p), ("face_normal", C.c_void_p),
-                ("cell_volume", C.c_void_p)]
+                ("cell_volume", C.c_void_p), ("cell_centre", C.c_void_p)]
 
 
 class Bands(C.Structure):
@@ -55,7 +56,7 @@ class Options(C.Structure):
                 ("newton_max_iter", C.c_int32), ("rank", C.c_int32), ("world", C.c_int32),
                 ("device", C.c_int32), ("nccl_unique_id", C.c_void_p), ("stream", C.c_void_p),
                 ("flags", C.c_uint32), ("max_spare_slabs", C.c_int32), ("block_threads", C.c_int32),
-                ("band_group", C.c_int32)]
+                ("band_group", C.c_int32), ("dir_chunk", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -141,17 +142,22 @@ def nccl_unique_id() -> bytes:
 
 
 class Solver:
-    """One bte_ctx.  Arrays in caller cell order; I is [bands][dirs][cells]."""
+    """One bte_ctx.  Arrays in caller cell order; I is [bands][dirs][cells].
+
+    locality: pass the mesh's cell centroids (if the dict has them) as the
+    library's internal-ordering hint; results are identical either way."""
 
     def __init__(self, mesh, bands, dirs, bcs, *, t_init=300.0, temp_rule=0, newton_rtol=1e-12,
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
-                 stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0):
+                 stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
+                 generic_faces=False, locality=True, dir_chunk=0):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
         k = self._keep = dict(
             off=i64(mesh["face_offsets"]), nbr=i64(mesh["face_nbr"]), area=f64(mesh["face_area"]),
             nrm=f64(mesh["face_normal"]), vol=f64(mesh["cell_volume"]),
+            cen=f64(mesh["cell_centre"]) if (locality and mesh.get("cell_centre") is not None) else None,
             omega=f64(bands["omega"]), dw=f64(bands.get("d_omega", np.ones(bands["n_bands"]))),
             vg=f64(bands["vg"]), tau=f64(bands["tau"]),
             pol=i32(bands.get("polarization", np.zeros(bands["n_bands"]))), C=f64(bands["C"]),
@@ -159,7 +165,7 @@ class Solver:
         )
         self.n_cells, self.n_bands, self.n_dirs = int(mesh["n_cells"]), int(bands["n_bands"]), int(dirs["n_dirs"])
         m = Mesh(int(mesh["dim"]), self.n_cells, _p(k["off"]).value, _p(k["nbr"]).value, _p(k["area"]).value,
-                 _p(k["nrm"]).value, _p(k["vol"]).value)
+                 _p(k["nrm"]).value, _p(k["vol"]).value, _p(k["cen"]).value if k["cen"] is not None else None)
         b = Bands(self.n_bands, _p(k["omega"]).value, _p(k["dw"]).value, _p(k["vg"]).value, _p(k["tau"]).value,
                   _p(k["pol"]).value, _p(k["C"]).value)
         d = Dirs(self.n_dirs, _p(k["s"]).value, _p(k["w"]).value)
@@ -176,8 +182,9 @@ class Solver:
             o.nccl_unique_id = C.cast(self._nccl_buf, C.c_void_p).value
         if stream is not None:
             o.stream = int(getattr(stream, "cuda_stream", stream))
-        o.flags = BTE_FLAG_PROFILE if profile else 0
+        o.flags = (BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)
+        o.dir_chunk = int(dir_chunk)
         ctx = C.c_void_p()
         _check(lib.bte_create(C.byref(m), C.byref(b), C.byref(d), C.byref(bc), C.byref(o), C.byref(ctx)))
         self.ctx = ctx

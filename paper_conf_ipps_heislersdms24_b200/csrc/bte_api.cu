@@ -1,9 +1,10 @@
 // bte_api.cu -- host runtime behind include/bte.h.
 //
-// Owns validation, the device layout (cell reorder, padded face slots,
-// reflection maps, slab pool), launch planning, the per-step launch sequence,
-// the NCCL energy all-reduce and the getters.  All arithmetic of the step runs
-// in the kernels of bte_kernels.cuh; the host only moves data and plans.
+// Owns validation, the device layout (face slots, opposite-face pairing,
+// ghost columns for boundary faces, reflection maps, slab pool), launch
+// planning, the per-step launch sequence, the NCCL energy all-reduce and the
+// getters.  All arithmetic of the step runs in the kernels of bte_kernels.cuh;
+// the host only validates, moves data and plans launches.
 #include "../../include/bte.h"
 #include "bte_kernels.cuh"
 #include "bte_nccl.h"
@@ -19,7 +20,7 @@
 
 namespace {
 
-// CODATA 2018 values (library's own copy; theta_b = hbar omega_b / kB).
+// CODATA 2018 values (the library's own copy; theta_b = hbar omega_b / kB).
 constexpr double kHbar = 1.054571817e-34;
 constexpr double kKb = 1.380649e-23;
 constexpr int kMaxFaces = 8;
@@ -40,7 +41,7 @@ struct PhaseEvent {
     int phase;
     cudaEvent_t a, b;
 };
-enum Phase { kPhInterior = 0, kPhBoundary = 1, kPhAllreduce = 2, kPhNewton = 3 };
+enum Phase { kPhFlux = 0, kPhAllreduce = 2, kPhNewton = 3 };
 
 }  // namespace
 
@@ -48,27 +49,34 @@ struct bte_ctx {
     std::string err = "no error";
     bte_options opt{};
     int dim = 0, nd = 0, nb = 0, b_lo = 0, b_hi = 0, nb_loc = 0, mf = 0, mf_t = 0;
-    int32_t nc = 0, n_int = 0;
+    int32_t nc = 0, ps = 0, n_ghost = 0, n_bcells = 0;
     int device = 0;
     int sm_count = 148;
     double W = 0.0, s_max = 0.0, dt_bound = 0.0;
-    // device state
+    // slab pool: nb_loc current slabs + n_spare workspace slabs of nd x ps doubles
     double *pool = nullptr;
     int64_t slab_elems = 0;
     int n_spare = 0;
     std::vector<int32_t> cur_slot, spare_slot;
-    int32_t *d_cur_slot = nullptr;  // for energy/equilibrium kernels
+    int32_t *d_cur_slot = nullptr, *d_band_ids = nullptr, *d_tmp_slot = nullptr;
     double *i0 = nullptr, *T = nullptr, *E = nullptr, *part = nullptr;
     int n_slots_step = 0;
     double *staging = nullptr;
     int64_t staging_elems = 0;
-    int32_t *nbr = nullptr, *aux = nullptr, *refl = nullptr, *pos = nullptr;
+    // face slots [mf_t][nc]
+    int32_t *nbr = nullptr, *nbm = nullptr, *symc = nullptr, *pos = nullptr;
+    uint32_t *symp = nullptr;
     double *gx = nullptr, *gy = nullptr, *gz = nullptr;
-    int8_t *kind = nullptr;
+    bool paired = false;
+    // boundary ghosts
+    int32_t *refl = nullptr;
+    int32_t n_iso = 0, n_sym = 0, n_refl = 0;
+    int32_t *iso_col = nullptr, *sym_col = nullptr, *sym_owner = nullptr, *sym_cls = nullptr;
     double *i0w = nullptr, *twall = nullptr;
-    int32_t n_iso = 0, n_refl = 0;
+    // tables
     double4 *dirs = nullptr;
-    double *inv_tau = nullptr, *vg = nullptr, *cw_loc = nullptr;
+    double *cw_loc = nullptr;
+    std::vector<double> h_inv_tau, h_vg, h_cw;  // local band-rows
     double *Cb = nullptr, *theta = nullptr, *cw_all = nullptr;
     int32_t *d_iter_max = nullptr, *d_fail = nullptr;
     unsigned long long *d_smax = nullptr;
@@ -81,7 +89,6 @@ struct bte_ctx {
     bte::nccl::Comm comm{};
     bool have_comm = false;
     bool begun = false;  // split step in flight
-    double begun_dt = 0.0;
     // stats
     bte_stats st{};
     std::vector<PhaseEvent> ev_live, ev_pool;
@@ -119,32 +126,52 @@ bte_status upload(bte_ctx *ctx, T **p, const std::vector<T> &h) {
 }
 
 // ------------------------------------------------------------- template dispatch
-using FluxLaunch = void (*)(bool, dim3, dim3, cudaStream_t, const bte::FluxParams &);
+using FluxLaunch = void (*)(dim3, dim3, cudaStream_t, const bte::FluxParams &);
 
-template <int DIM, int MF, int BG>
-void flux_launch_t(bool bnd, dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    if (bnd)
-        bte::flux_kernel<DIM, MF, BG, true><<<g, b, 0, s>>>(p);
+template <int DIM, int MF, int BG, bool PAIRED>
+void flux_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    if constexpr (PAIRED)
+        bte::flux_paired_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
     else
-        bte::flux_kernel<DIM, MF, BG, false><<<g, b, 0, s>>>(p);
+        bte::flux_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
 }
 
+// Paired kernels exist for every band group 1..8, generic ones for 1, 2, 4.
 template <int DIM, int MF>
-FluxLaunch pick_bg(int bg) {
+FluxLaunch pick_paired(int bg) {
     switch (bg) {
-        case 1: return flux_launch_t<DIM, MF, 1>;
-        case 2: return flux_launch_t<DIM, MF, 2>;
-        case 4: return flux_launch_t<DIM, MF, 4>;
-        default: return flux_launch_t<DIM, MF, 8>;
+        case 1: return flux_launch_t<DIM, MF, 1, true>;
+        case 2: return flux_launch_t<DIM, MF, 2, true>;
+        case 3: return flux_launch_t<DIM, MF, 3, true>;
+        case 4: return flux_launch_t<DIM, MF, 4, true>;
+        case 5: return flux_launch_t<DIM, MF, 5, true>;
+        case 6: return flux_launch_t<DIM, MF, 6, true>;
+        case 7: return flux_launch_t<DIM, MF, 7, true>;
+        default: return flux_launch_t<DIM, MF, 8, true>;
     }
 }
 
-FluxLaunch pick_flux(int dim, int mf_t, int bg) {
-    if (dim == 2) return mf_t == 4 ? pick_bg<2, 4>(bg) : pick_bg<2, 8>(bg);
-    return mf_t == 6 ? pick_bg<3, 6>(bg) : pick_bg<3, 8>(bg);
+template <int DIM, int MF>
+FluxLaunch pick_generic(int bg) {
+    switch (bg) {
+        case 1: return flux_launch_t<DIM, MF, 1, false>;
+        case 2: return flux_launch_t<DIM, MF, 2, false>;
+        default: return flux_launch_t<DIM, MF, 4, false>;
+    }
 }
 
-int round_bg(int bg) { return bg <= 1 ? 1 : bg <= 2 ? 2 : bg <= 4 ? 4 : 8; }
+// mf_t: padded faces per cell (generic) or face pairs per cell (paired)
+FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired) {
+    if (paired) return dim == 2 ? pick_paired<2, 2>(bg) : pick_paired<3, 3>(bg);
+    if (dim == 2) return mf_t == 4 ? pick_generic<2, 4>(bg) : pick_generic<2, 8>(bg);
+    return mf_t == 6 ? pick_generic<3, 6>(bg) : pick_generic<3, 8>(bg);
+}
+
+int legal_bg(int bg, bool paired) {
+    bg = std::max(1, std::min(8, bg));
+    if (paired) return bg;
+    return bg <= 1 ? 1 : bg <= 3 ? 2 : 4;
+}
 
 // ------------------------------------------------------------- profiling
 void ev_mark(bte_ctx *ctx, int phase, bool begin) {
@@ -174,8 +201,7 @@ void ev_collect(bte_ctx *ctx) {  // after a stream sync
     for (auto &pe : ctx->ev_live) {
         float ms = 0.f;
         cudaEventElapsedTime(&ms, pe.a, pe.b);
-        double *dst = pe.phase == kPhInterior   ? &ctx->st.ms_flux_interior
-                      : pe.phase == kPhBoundary ? &ctx->st.ms_flux_boundary
+        double *dst = pe.phase == kPhFlux ? &ctx->st.ms_flux_interior
                       : pe.phase == kPhAllreduce ? &ctx->st.ms_allreduce
                                                  : &ctx->st.ms_newton;
         *dst += ms;
@@ -189,81 +215,141 @@ struct LaunchPlan {
     int groups, n_dch, dchunk;
 };
 
-LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int cells) {
+// A band batch of nbl rows is launched as segments of full band groups: the
+// largest multiple of bg first, then the remainder as one smaller group
+// (paired kernels: any size 1..8) or as power-of-two groups (generic kernels).
+struct Segment {
+    int off, nbl, bg;
+};
+std::vector<Segment> segments(int nbl, int bg, bool paired) {
+    std::vector<Segment> out;
+    int off = 0;
+    while (off < nbl) {
+        int g = std::min(bg, nbl - off);
+        if (!paired)
+            while (g & (g - 1)) g &= g - 1;  // largest power of two <= g
+        const int n = (nbl - off) / g * g;
+        out.push_back({off, n, g});
+        off += n;
+    }
+    return out;
+}
+
+// Direction chunks so the grid holds ~2 full waves of threads.
+LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int bg) {
     LaunchPlan lp;
-    lp.groups = (nbl + ctx->bg - 1) / ctx->bg;
-    const int64_t target = (int64_t)ctx->sm_count * 2048 * 2;  // ~2 full waves of threads
-    const int64_t have = std::max<int64_t>(1, (int64_t)cells * lp.groups);
-    int n = (int)std::min<int64_t>(ctx->nd, std::max<int64_t>(1, (target + have - 1) / have));
-    if (ctx->opt.flags & 0x100u) n = 1;  // (debug) force one chunk
+    lp.groups = nbl / bg;
+    const int64_t target = (int64_t)ctx->sm_count * 2048 * 2;
+    const int64_t have = std::max<int64_t>(1, (int64_t)ctx->nc * lp.groups);
+    const int n = (int)std::min<int64_t>(ctx->nd, std::max<int64_t>(1, (target + have - 1) / have));
     lp.dchunk = (ctx->nd + n - 1) / n;
+    if (ctx->opt.dir_chunk > 0) lp.dchunk = std::min(lp.dchunk, (int)ctx->opt.dir_chunk);
     lp.n_dch = (ctx->nd + lp.dchunk - 1) / lp.dchunk;
     return lp;
 }
 
-// Flux + relaxation + energy partials for all local band-rows: one launch pair
-// (interior, boundary) per band batch of <= n_spare rows, rotating slabs.
+int count_slots(const bte_ctx *ctx) {
+    int slots = 0;
+    for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare)
+        for (const Segment &sg : segments(std::min(ctx->n_spare, ctx->nb_loc - l0), ctx->bg, ctx->paired)) {
+            const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
+            slots += lp.groups * lp.n_dch;
+        }
+    return slots;
+}
+
+// Isothermal ghost columns of the given slabs (entries: slab slot, local band).
+bte_status fill_iso_ghosts(bte_ctx *ctx, const std::vector<int32_t> &slots, const std::vector<int32_t> &bands) {
+    if (ctx->n_iso == 0 || slots.empty()) return BTE_OK;
+    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_tmp_slot, slots.data(), slots.size() * sizeof(int32_t),
+                                  cudaMemcpyHostToDevice, ctx->stream));
+    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_band_ids, bands.data(), bands.size() * sizeof(int32_t),
+                                  cudaMemcpyHostToDevice, ctx->stream));
+    const int tb = 256;
+    const int64_t n = (int64_t)ctx->nd * ctx->n_iso;
+    dim3 grid((unsigned)std::min<int64_t>(2048, (n + tb - 1) / tb), (unsigned)slots.size());
+    bte::iso_ghost_kernel<<<grid, tb, 0, ctx->stream>>>(ctx->pool, ctx->d_tmp_slot, ctx->d_band_ids,
+                                                        ctx->slab_elems, ctx->ps, ctx->nd, ctx->n_iso,
+                                                        ctx->iso_col, ctx->i0w);
+    CUDA_TRY(ctx, cudaGetLastError());
+    ctx->st.kernel_launches++;
+    return BTE_OK;
+}
+
+// Specular ghost columns of the current slabs from the current state.
+bte_status fill_sym_ghosts(bte_ctx *ctx) {
+    if (ctx->n_sym == 0) return BTE_OK;
+    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_cur_slot, ctx->cur_slot.data(), ctx->nb_loc * sizeof(int32_t),
+                                  cudaMemcpyHostToDevice, ctx->stream));
+    const int tb = 256;
+    const int64_t n = (int64_t)ctx->nd * ctx->n_sym;
+    dim3 grid((unsigned)std::min<int64_t>(2048, (n + tb - 1) / tb), (unsigned)ctx->nb_loc);
+    bte::sym_ghost_kernel<<<grid, tb, 0, ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps,
+                                                        ctx->nd, ctx->n_sym, ctx->sym_col, ctx->sym_owner,
+                                                        ctx->sym_cls, ctx->refl);
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+// Flux + relaxation + energy partials for all local band-rows: per band batch
+// of <= n_spare rows, one launch per segment of full band groups, reading the
+// current slabs and writing the spare ones, which then become current (double
+// buffering when n_spare == nb_loc, slab rotation otherwise).
 bte_status run_flux(bte_ctx *ctx, double dt) {
     bte::FluxParams p{};
     p.nc = ctx->nc;
+    p.ps = ctx->ps;
     p.nd = ctx->nd;
     p.slab_elems = ctx->slab_elems;
     p.pool = ctx->pool;
     p.i0 = ctx->i0;
     p.part = ctx->part;
     p.nbr = ctx->nbr;
+    p.nbm = ctx->nbm;
     p.gx = ctx->gx;
     p.gy = ctx->gy;
     p.gz = ctx->gz;
-    p.kind = ctx->kind;
-    p.aux = ctx->aux;
+    p.symc = ctx->symc;
+    p.symp = ctx->symp;
     p.refl = ctx->refl;
-    p.i0w = ctx->i0w;
-    p.n_iso = ctx->n_iso;
     p.dirs = ctx->dirs;
-    p.inv_tau = ctx->inv_tau;
-    p.vg = ctx->vg;
-    p.cw = ctx->cw_loc;
     p.dt = dt;
-    p.bg = ctx->bg;
-    FluxLaunch fn = pick_flux(ctx->dim, ctx->mf_t, ctx->bg);
     int slot = 0;
-    const int n_bnd = ctx->nc - ctx->n_int;
+    const bool rotating = ctx->n_spare < ctx->nb_loc;
+    const dim3 block(ctx->block);
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
-        const int nbl = std::min(ctx->n_spare, ctx->nb_loc - l0);
-        p.nbl = nbl;
-        p.band0 = l0;
-        p.slot0 = slot;
-        for (int k = 0; k < nbl; ++k) {
-            p.in_slot[k] = ctx->cur_slot[l0 + k];
-            p.out_slot[k] = ctx->spare_slot[k];
+        const int nbl_batch = std::min(ctx->n_spare, ctx->nb_loc - l0);
+        if (rotating) {  // spare slabs change band: give them this batch's isothermal ghosts
+            std::vector<int32_t> sl(ctx->spare_slot.begin(), ctx->spare_slot.begin() + nbl_batch), bl(nbl_batch);
+            for (int k = 0; k < nbl_batch; ++k) bl[k] = l0 + k;
+            STATUS_TRY(fill_iso_ghosts(ctx, sl, bl));
         }
-        LaunchPlan lp = plan_launch(ctx, nbl, ctx->n_int > 0 ? ctx->n_int : n_bnd);
-        p.dchunk = lp.dchunk;
-        p.n_dchunks = lp.n_dch;
-        ctx->dir_chunks = lp.n_dch;
-        const dim3 block(ctx->block);
-        if (ctx->n_int > 0) {
-            p.cell_begin = 0;
-            p.cell_end = ctx->n_int;
-            dim3 grid((ctx->n_int + ctx->block - 1) / ctx->block, lp.groups * lp.n_dch);
-            ev_mark(ctx, kPhInterior, true);
-            fn(false, grid, block, ctx->stream, p);
-            ev_mark(ctx, kPhInterior, false);
+        for (const Segment &sg : segments(nbl_batch, ctx->bg, ctx->paired)) {
+            const FluxLaunch fn = pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired);
+            const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
+            p.nbl = sg.nbl;
+            p.band0 = l0 + sg.off;
+            p.dchunk = lp.dchunk;
+            p.n_dchunks = lp.n_dch;
+            p.slot0 = slot;
+            for (int k = 0; k < sg.nbl; ++k) {
+                const int b = l0 + sg.off + k;  // rank-local band-row
+                p.in_ptr[k] = ctx->pool + (int64_t)ctx->cur_slot[b] * ctx->slab_elems;
+                p.out_ptr[k] = ctx->pool + (int64_t)ctx->spare_slot[sg.off + k] * ctx->slab_elems;
+                p.dtit[k] = dt * ctx->h_inv_tau[b];
+                p.kv[k] = dt * ctx->h_vg[b];
+                p.cw[k] = ctx->h_cw[b];
+            }
+            if (sg.off == 0) ctx->dir_chunks = lp.n_dch;
+            const dim3 grid((ctx->nc + ctx->block - 1) / ctx->block, lp.groups * lp.n_dch);
+            ev_mark(ctx, kPhFlux, true);
+            fn(grid, block, ctx->stream, p);
+            ev_mark(ctx, kPhFlux, false);
             ctx->st.kernel_launches++;
-        }
-        if (n_bnd > 0) {
-            p.cell_begin = ctx->n_int;
-            p.cell_end = ctx->nc;
-            dim3 grid((n_bnd + ctx->block - 1) / ctx->block, lp.groups * lp.n_dch);
-            ev_mark(ctx, kPhBoundary, true);
-            fn(true, grid, block, ctx->stream, p);
-            ev_mark(ctx, kPhBoundary, false);
-            ctx->st.kernel_launches++;
+            slot += lp.groups * lp.n_dch;
         }
         CUDA_TRY(ctx, cudaGetLastError());
-        slot += lp.groups * lp.n_dch;
-        for (int k = 0; k < nbl; ++k) std::swap(ctx->cur_slot[l0 + k], ctx->spare_slot[k]);
+        for (int k = 0; k < nbl_batch; ++k) std::swap(ctx->cur_slot[l0 + k], ctx->spare_slot[k]);
     }
     ctx->n_slots_step = slot;
     return BTE_OK;
@@ -309,8 +395,8 @@ bte_status allreduce_E(bte_ctx *ctx) {
 
 bte_status reduce_slots(bte_ctx *ctx) {
     const int tb = 256;
-    bte::sum_slots_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->part, ctx->n_slots_step,
-                                                                           ctx->nc, ctx->E);
+    bte::sum_slots_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->part, ctx->n_slots_step, ctx->nc,
+                                                                           ctx->E);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
@@ -356,7 +442,7 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
                     const bte_options *o) {
     if (!m || !b || !d || !bc || !o) return set_err(nullptr, "NULL argument"), BTE_EINVAL;
     if (m->dim != 2 && m->dim != 3) return set_err(nullptr, "dim must be 2 or 3 (got %d)", m->dim), BTE_EINVAL;
-    if (m->n_cells <= 0 || m->n_cells >= (int64_t)1 << 31)
+    if (m->n_cells <= 0 || m->n_cells >= (int64_t)1 << 30)
         return set_err(nullptr, "n_cells out of range"), BTE_EINVAL;
     if (!m->face_offsets || !m->face_nbr || !m->face_area || !m->face_normal || !m->cell_volume)
         return set_err(nullptr, "mesh array is NULL"), BTE_EINVAL;
@@ -369,6 +455,7 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
         if (!(m->cell_volume[c] > 0.0)) return set_err(nullptr, "cell %lld volume <= 0", (long long)c), BTE_EINVAL;
     }
     const int64_t nfaces = m->face_offsets[m->n_cells];
+    std::vector<char> seen(bc->n_bfaces > 0 ? bc->n_bfaces : 0, 0);
     for (int64_t f = 0; f < nfaces; ++f) {
         if (!(m->face_area[f] > 0.0)) return set_err(nullptr, "face %lld area <= 0", (long long)f), BTE_EINVAL;
         const double *n = m->face_normal + 3 * f;
@@ -376,8 +463,11 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
         if (m->dim == 2 && n[2] != 0.0) return set_err(nullptr, "2-D mesh with n_z != 0 (face %lld)", (long long)f), BTE_EINVAL;
         const int64_t nb = m->face_nbr[f];
         if (nb >= m->n_cells) return set_err(nullptr, "face %lld neighbour out of range", (long long)f), BTE_EINVAL;
-        if (nb < 0 && -1 - nb >= bc->n_bfaces)
-            return set_err(nullptr, "face %lld boundary id out of range", (long long)f), BTE_EINVAL;
+        if (nb < 0) {
+            const int64_t bf = -1 - nb;
+            if (bf >= bc->n_bfaces) return set_err(nullptr, "face %lld boundary id out of range", (long long)f), BTE_EINVAL;
+            if (seen[bf]++) return set_err(nullptr, "boundary face id %lld used twice", (long long)bf), BTE_EINVAL;
+        }
     }
     if (b->n_bands < 1 || !b->omega || !b->vg || !b->tau)
         return set_err(nullptr, "band table incomplete"), BTE_EINVAL;
@@ -449,10 +539,11 @@ void bte_destroy(bte_ctx *ctx) {
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->have_comm) bte::nccl::destroy(ctx->comm);
-    void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E, ctx->part, ctx->staging,
-                    ctx->nbr, ctx->aux, ctx->refl, ctx->pos, ctx->gx, ctx->gy, ctx->gz, ctx->kind,
-                    ctx->i0w, ctx->twall, ctx->dirs, ctx->inv_tau, ctx->vg, ctx->cw_loc, ctx->Cb,
-                    ctx->theta, ctx->cw_all, ctx->d_iter_max, ctx->d_fail, ctx->d_smax};
+    void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->d_band_ids, ctx->d_tmp_slot, ctx->i0, ctx->T, ctx->E,
+                    ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->symc, ctx->symp, ctx->pos, ctx->gx,
+                    ctx->gy, ctx->gz, ctx->refl, ctx->iso_col, ctx->sym_col, ctx->sym_owner, ctx->sym_cls,
+                    ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
+                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -489,18 +580,52 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     if (nb_loc > bte::kMaxBandsPerLaunch)
         return set_err(nullptr, "%d band-rows on one rank (max %d)", nb_loc, bte::kMaxBandsPerLaunch), BTE_EINVAL;
 
-    // --- reflection classes of symmetric faces and their maps (Eq. 6)
+    // --- internal cell order: Morton order of the optional centroids (tiles of
+    // 256 consecutive cells become compact bricks, so upwind neighbours are
+    // cache hits), else the caller's order.  pos_h: caller -> internal.
+    std::vector<int32_t> user_of(nc), pos_h(nc);
+    for (int32_t c = 0; c < nc; ++c) user_of[c] = c;
+    if (m->cell_centre) {
+        double lo[3] = {INFINITY, INFINITY, INFINITY}, hi[3] = {-INFINITY, -INFINITY, -INFINITY};
+        for (int32_t c = 0; c < nc; ++c)
+            for (int a = 0; a < 3; ++a) {
+                lo[a] = std::min(lo[a], m->cell_centre[3 * c + a]);
+                hi[a] = std::max(hi[a], m->cell_centre[3 * c + a]);
+            }
+        std::vector<uint64_t> key(nc);
+        for (int32_t c = 0; c < nc; ++c) {
+            uint64_t q[3];
+            for (int a = 0; a < 3; ++a) {
+                const double span = hi[a] - lo[a];
+                const double t = span > 0.0 ? (m->cell_centre[3 * c + a] - lo[a]) / span : 0.0;
+                q[a] = (uint64_t)std::min(2097151.0, std::max(0.0, std::floor(t * 2097151.0)));
+            }
+            uint64_t k = 0;
+            for (int bit = 20; bit >= 0; --bit)
+                for (int a = 0; a < 3; ++a) k = (k << 1) | ((q[a] >> bit) & 1u);
+            key[c] = k;
+        }
+        std::stable_sort(user_of.begin(), user_of.end(), [&](int32_t a, int32_t b) { return key[a] < key[b]; });
+    }
+    for (int32_t i = 0; i < nc; ++i) pos_h[user_of[i]] = i;
+
+    // --- boundary faces -> ghost columns (internal cell order); reflection classes (Eq. 6)
     std::map<std::vector<double>, int> cls_of;
-    std::vector<int32_t> refl_h;
-    std::vector<int32_t> bface_aux(bc->n_bfaces, -1);
+    std::vector<int32_t> refl_h, ghost_of(bc->n_bfaces, -1), bcls(bc->n_bfaces, -1);
+    std::vector<int32_t> iso_col_h, sym_col_h, sym_owner_h, sym_cls_h;
     std::vector<double> twall_h;
-    for (int64_t c = 0; c < nc64; ++c) {
+    int32_t n_ghost = 0, n_bcells = 0;
+    for (int32_t i = 0; i < nc; ++i) {
+        const int64_t c = user_of[i];
+        bool bcell = false;
         for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f) {
             if (m->face_nbr[f] >= 0) continue;
+            bcell = true;
             const int64_t bf = -1 - m->face_nbr[f];
-            if (bface_aux[bf] >= 0) continue;
+            const int32_t col = n_ghost++;
+            ghost_of[bf] = col;
             if (bc->kind[bf] == BTE_BC_ISOTHERMAL) {
-                bface_aux[bf] = (int32_t)twall_h.size();
+                iso_col_h.push_back(nc + col);  // plane index of the ghost column
                 twall_h.push_back(bc->t_wall[bf]);
                 continue;
             }
@@ -530,52 +655,83 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                 }
                 it = cls_of.emplace(key, id).first;
             }
-            bface_aux[bf] = it->second;
+            bcls[bf] = it->second;
+            sym_col_h.push_back(nc + col);
+            sym_owner_h.push_back(i);
+            sym_cls_h.push_back(it->second);
+        }
+        n_bcells += bcell;
+    }
+
+    // --- plane stride: cells + ghost columns, padded to 32 doubles (256 B)
+    const int32_t ps = (int32_t)((nc64 + n_ghost + 31) / 32 * 32);
+
+    // --- face pairing: every face of every cell has an exactly opposite partner
+    // (same area, negated normal) -> paired layout, one upwind load per pair.
+    int mf = 0;
+    for (int64_t c = 0; c < nc64; ++c) mf = std::max<int>(mf, (int)(m->face_offsets[c + 1] - m->face_offsets[c]));
+    std::vector<int64_t> partner(m->face_offsets[nc64], -1);
+    // (paired layout packs each side's reflection class in 5 bits: < 31 classes)
+    bool paired = mf <= 2 * m->dim && cls_of.size() < 31 && !(o->flags & BTE_FLAG_GENERIC_FACES);
+    for (int64_t c = 0; c < nc64 && paired; ++c) {
+        const int64_t f0 = m->face_offsets[c], f1 = m->face_offsets[c + 1];
+        for (int64_t f = f0; f < f1 && paired; ++f) {
+            if (partner[f] >= 0) continue;
+            const double *n = m->face_normal + 3 * f;
+            for (int64_t g = f + 1; g < f1; ++g) {
+                const double *q = m->face_normal + 3 * g;
+                if (partner[g] < 0 && m->face_area[g] == m->face_area[f] && q[0] == -n[0] && q[1] == -n[1] &&
+                    q[2] == -n[2]) {
+                    partner[f] = g;
+                    partner[g] = f;
+                    break;
+                }
+            }
+            if (partner[f] < 0) paired = false;
         }
     }
-
-    // --- interior-first cell order
-    std::vector<char> is_bnd(nc, 0);
-    int mf = 0;
-    for (int32_t c = 0; c < nc; ++c) {
-        mf = std::max<int>(mf, (int)(m->face_offsets[c + 1] - m->face_offsets[c]));
-        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f)
-            if (m->face_nbr[f] < 0) is_bnd[c] = 1;
-    }
-    std::vector<int32_t> user_of, pos_h(nc);
-    user_of.reserve(nc);
-    for (int32_t c = 0; c < nc; ++c)
-        if (!is_bnd[c]) user_of.push_back(c);
-    const int32_t n_int = (int32_t)user_of.size();
-    for (int32_t c = 0; c < nc; ++c)
-        if (is_bnd[c]) user_of.push_back(c);
-    for (int32_t i = 0; i < nc; ++i) pos_h[user_of[i]] = i;
-
-    const int mf_t = m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8);
+    const int mf_t = paired ? m->dim : (m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
-    std::vector<int32_t> nbr_h(ell), aux_h(ell, 0);
+    std::vector<int32_t> nbr_h(ell), symc_h(ell, -1), nbm_h(paired ? ell : 1, 0);
+    std::vector<uint32_t> symp_h(paired ? nc : 1, 0xffffffffu);
     std::vector<double> gx_h(ell, 0.0), gy_h(ell, 0.0), gz_h(ell, 0.0);
-    std::vector<int8_t> kind_h(ell, bte::kFaceInterior);
+    // upwind source index of face f: neighbour cell, or the face's ghost column
+    auto face_src = [&](int64_t f, int32_t *nbv, int32_t *cls) {
+        const int64_t v = m->face_nbr[f];
+        if (v >= 0) {
+            *nbv = pos_h[v];
+            *cls = -1;
+        } else {
+            const int64_t bf = -1 - v;
+            *nbv = nc + ghost_of[bf];
+            *cls = bcls[bf];
+        }
+    };
     for (int32_t i = 0; i < nc; ++i) {
-        const int32_t c = user_of[i];
+        const int64_t c = user_of[i];
         int j = 0;
-        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f, ++j) {
+        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f) {
+            if (paired && partner[f] < f) continue;  // "+" face = first of its pair
             const size_t q = (size_t)j * nc + i;
             const double av = m->face_area[f] / m->cell_volume[c];
             gx_h[q] = av * m->face_normal[3 * f + 0];
             gy_h[q] = av * m->face_normal[3 * f + 1];
             gz_h[q] = av * m->face_normal[3 * f + 2];
-            const int64_t nbv = m->face_nbr[f];
-            if (nbv >= 0) {
-                nbr_h[q] = pos_h[nbv];
-            } else {
-                const int64_t bf = -1 - nbv;
-                nbr_h[q] = i;
-                kind_h[q] = bc->kind[bf] == BTE_BC_ISOTHERMAL ? bte::kFaceIso : bte::kFaceSym;
-                aux_h[q] = bface_aux[bf];
+            face_src(f, &nbr_h[q], &symc_h[q]);
+            if (paired) {
+                int32_t cm = -1;
+                face_src(partner[f], &nbm_h[q], &cm);
+                const uint32_t cp5 = symc_h[q] < 0 ? 31u : (uint32_t)symc_h[q];
+                const uint32_t cm5 = cm < 0 ? 31u : (uint32_t)cm;
+                const uint32_t mask = ~(1023u << (10 * j));
+                symp_h[i] = (symp_h[i] & mask) | ((cp5 | (cm5 << 5)) << (10 * j));
             }
+            ++j;
         }
-        for (; j < mf_t; ++j) nbr_h[(size_t)j * nc + i] = i;  // padding: zero geometry
+        for (; j < mf_t; ++j) {  // padding: zero geometry, self neighbour
+            nbr_h[(size_t)j * nc + i] = i;
+            if (paired) nbm_h[(size_t)j * nc + i] = i;
+        }
     }
 
     // --- context
@@ -589,10 +745,14 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     ctx->nb_loc = nb_loc;
     ctx->mf = mf;
     ctx->mf_t = mf_t;
+    ctx->paired = paired;
     ctx->nc = nc;
-    ctx->n_int = n_int;
+    ctx->ps = ps;
+    ctx->n_ghost = n_ghost;
+    ctx->n_bcells = n_bcells;
     ctx->device = o->device;
-    ctx->n_iso = (int32_t)twall_h.size();
+    ctx->n_iso = (int32_t)iso_col_h.size();
+    ctx->n_sym = (int32_t)sym_col_h.size();
     ctx->n_refl = (int32_t)cls_of.size();
     ctx->W = 0.0;
     for (int d = 0; d < nd; ++d) ctx->W += dr->w[d];
@@ -640,19 +800,19 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->have_comm = true;
     }
 
-    // --- launch plan knobs
+    // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
-    ctx->bg = round_bg(o->band_group > 0 ? o->band_group : 4);
+    ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : (paired ? 8 : 2), paired);
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
-    ctx->slab_elems = (int64_t)nd * nc;
+    ctx->slab_elems = (int64_t)nd * ps;
     const size_t slab_bytes = (size_t)ctx->slab_elems * sizeof(double);
     int n_spare = nb_loc;
     if (o->max_spare_slabs > 0) n_spare = std::min(n_spare, (int)o->max_spare_slabs);
     {
         size_t free_b = 0, total_b = 0;
         CREATE_CUDA(cudaMemGetInfo(&free_b, &total_b));
-        const size_t other = (size_t)nc * sizeof(double) * (size_t)(3 * nb_loc + 16) + ell * 40 + (64u << 20);
+        const size_t other = (size_t)nc * sizeof(double) * (size_t)(3 * nb_loc + 16) + ell * 48 + (64u << 20);
         const size_t reserve = (size_t)1 << 30;
         while (n_spare > 1 && (size_t)(nb_loc + n_spare) * slab_bytes + other + reserve > free_b) --n_spare;
         if ((size_t)(nb_loc + n_spare) * slab_bytes + other > free_b) {
@@ -662,7 +822,6 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         }
     }
     ctx->n_spare = n_spare;
-    ctx->bg = std::min(ctx->bg, round_bg(n_spare));
     while (ctx->bg > n_spare) ctx->bg /= 2;
     ctx->cur_slot.resize(nb_loc);
     ctx->spare_slot.resize(n_spare);
@@ -670,38 +829,41 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     for (int k = 0; k < n_spare; ++k) ctx->spare_slot[k] = nb_loc + k;
     CREATE_TRY(dalloc(ctx, &ctx->pool, (size_t)(nb_loc + n_spare) * ctx->slab_elems));
 
-    // --- energy partial slots: worst case over the launch batches
-    int max_slots = 0;
-    for (int l0 = 0; l0 < nb_loc; l0 += n_spare) {
-        const int nbl = std::min(n_spare, nb_loc - l0);
-        LaunchPlan lp = plan_launch(ctx, nbl, n_int > 0 ? n_int : nc - n_int);
-        max_slots += lp.groups * lp.n_dch;
-    }
+    const int max_slots = count_slots(ctx);
     CREATE_TRY(dalloc(ctx, &ctx->part, (size_t)max_slots * nc));
     CREATE_TRY(dalloc(ctx, &ctx->i0, (size_t)nb_loc * nc));
     CREATE_TRY(dalloc(ctx, &ctx->T, (size_t)nc));
     CREATE_TRY(dalloc(ctx, &ctx->E, (size_t)nc));
-    ctx->staging_elems = std::min<int64_t>(ctx->slab_elems, std::max<int64_t>(nc, (int64_t)8 << 20));
+    ctx->staging_elems = std::min<int64_t>((int64_t)nd * nc, std::max<int64_t>(nc, (int64_t)8 << 20));
     CREATE_TRY(dalloc(ctx, &ctx->staging, (size_t)ctx->staging_elems));
     CREATE_TRY(upload(ctx, &ctx->d_cur_slot, ctx->cur_slot));
+    CREATE_TRY(dalloc(ctx, &ctx->d_tmp_slot, (size_t)(nb_loc + n_spare)));
+    CREATE_TRY(dalloc(ctx, &ctx->d_band_ids, (size_t)(nb_loc + n_spare)));
     CREATE_TRY(upload(ctx, &ctx->nbr, nbr_h));
-    CREATE_TRY(upload(ctx, &ctx->aux, aux_h));
-    CREATE_TRY(upload(ctx, &ctx->kind, kind_h));
+    CREATE_TRY(upload(ctx, &ctx->nbm, nbm_h));
+    CREATE_TRY(upload(ctx, &ctx->symc, symc_h));
+    if (paired) {  // sides beyond the cell's pairs stay "31" (none); keep only 10*dim bits
+        const uint32_t keep = m->dim == 2 ? 0xfffffu : 0x3fffffffu;
+        for (auto &v : symp_h) v &= keep;
+    }
+    CREATE_TRY(upload(ctx, &ctx->symp, symp_h));
     CREATE_TRY(upload(ctx, &ctx->gx, gx_h));
     CREATE_TRY(upload(ctx, &ctx->gy, gy_h));
     CREATE_TRY(upload(ctx, &ctx->gz, gz_h));
     CREATE_TRY(upload(ctx, &ctx->pos, pos_h));
     CREATE_TRY(upload(ctx, &ctx->refl, refl_h));
+    CREATE_TRY(upload(ctx, &ctx->iso_col, iso_col_h));
+    CREATE_TRY(upload(ctx, &ctx->sym_col, sym_col_h));
+    CREATE_TRY(upload(ctx, &ctx->sym_owner, sym_owner_h));
+    CREATE_TRY(upload(ctx, &ctx->sym_cls, sym_cls_h));
     CREATE_TRY(upload(ctx, &ctx->twall, twall_h));
     std::vector<double4> dirs_h(nd);
     for (int d = 0; d < nd; ++d) dirs_h[d] = make_double4(dr->s[3 * d], dr->s[3 * d + 1], dr->s[3 * d + 2], dr->w[d]);
     CREATE_TRY(upload(ctx, &ctx->dirs, dirs_h));
-    std::vector<double> it_loc(inv_tau.begin() + b_lo, inv_tau.begin() + b_hi);
-    std::vector<double> vg_loc(bd->vg + b_lo, bd->vg + b_hi);
-    std::vector<double> cw_loc(cw.begin() + b_lo, cw.begin() + b_hi);
-    CREATE_TRY(upload(ctx, &ctx->inv_tau, it_loc));
-    CREATE_TRY(upload(ctx, &ctx->vg, vg_loc));
-    CREATE_TRY(upload(ctx, &ctx->cw_loc, cw_loc));
+    ctx->h_inv_tau.assign(inv_tau.begin() + b_lo, inv_tau.begin() + b_hi);
+    ctx->h_vg.assign(bd->vg + b_lo, bd->vg + b_hi);
+    ctx->h_cw.assign(cw.begin() + b_lo, cw.begin() + b_hi);
+    CREATE_TRY(upload(ctx, &ctx->cw_loc, ctx->h_cw));
     CREATE_TRY(upload(ctx, &ctx->Cb, std::vector<double>(bd->i0_prefactor, bd->i0_prefactor + nb)));
     CREATE_TRY(upload(ctx, &ctx->theta, theta));
     CREATE_TRY(upload(ctx, &ctx->cw_all, cw));
@@ -713,22 +875,32 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_CUDA(cudaMemsetAsync(ctx->d_fail, 0, sizeof(int32_t), ctx->stream));
     CREATE_CUDA(cudaMemsetAsync(ctx->d_smax, 0, sizeof(unsigned long long), ctx->stream));
 
-    // --- initial state: T = t_init, I = I0_b(t_init); ghost table; dt bound
+    // --- initial state: T = t_init, I = I0_b(t_init); ghosts; dt bound
     {
         std::vector<double> T0(nc, o->t_init);
         CREATE_CUDA(cudaMemcpy(ctx->T, T0.data(), nc * sizeof(double), cudaMemcpyHostToDevice));
         const int tb = 256;
         const int gb = (nc + tb - 1) / tb;
         bte::i0_table_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->T, nc, b_lo, nb_loc, ctx->Cb, ctx->theta, ctx->i0);
-        bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, (ctx->slab_elems + tb - 1) / tb), nb_loc), tb, 0,
-                                  ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, nd, nc, ctx->i0);
-        if (ctx->n_iso > 0)
+        bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)nd * nc + tb - 1) / tb), nb_loc), tb, 0,
+                                  ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ps, nd, nc, ctx->i0);
+        if (ctx->n_iso > 0) {
             bte::i0w_kernel<<<(ctx->n_iso + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->twall, ctx->n_iso, b_lo, nb_loc,
                                                                                ctx->Cb, ctx->theta, ctx->i0w);
+            // every slab that will hold a band's state gets that band's isothermal ghosts
+            std::vector<int32_t> sl, bl;
+            for (int k = 0; k < nb_loc; ++k) sl.push_back(ctx->cur_slot[k]), bl.push_back(k);
+            if (n_spare == nb_loc)
+                for (int k = 0; k < nb_loc; ++k) sl.push_back(ctx->spare_slot[k]), bl.push_back(k);
+            CREATE_TRY(fill_iso_ghosts(ctx, sl, bl));
+        }
+        CREATE_TRY(fill_sym_ghosts(ctx));
         if (m->dim == 2)
-            bte::outflow_max_kernel<2><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, nd, ctx->gx, ctx->gy, ctx->gz, ctx->dirs, ctx->d_smax);
+            bte::outflow_max_kernel<2><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, paired, nd, ctx->gx, ctx->gy, ctx->gz,
+                                                                  ctx->dirs, ctx->d_smax);
         else
-            bte::outflow_max_kernel<3><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, nd, ctx->gx, ctx->gy, ctx->gz, ctx->dirs, ctx->d_smax);
+            bte::outflow_max_kernel<3><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, paired, nd, ctx->gx, ctx->gy, ctx->gz,
+                                                                  ctx->dirs, ctx->d_smax);
         CREATE_CUDA(cudaGetLastError());
         unsigned long long bits = 0;
         CREATE_CUDA(cudaMemcpyAsync(&bits, ctx->d_smax, sizeof bits, cudaMemcpyDeviceToHost, ctx->stream));
@@ -738,8 +910,9 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         for (int b = 0; b < nb; ++b) rate = std::max(rate, inv_tau[b] + bd->vg[b] * ctx->s_max);
         ctx->dt_bound = rate > 0.0 ? 1.0 / rate : INFINITY;
     }
+    std::memset(&ctx->st, 0, sizeof ctx->st);
     ctx->st.spare_slabs = n_spare;
-    ctx->st.n_interior_cells = n_int;
+    ctx->st.n_interior_cells = nc - n_bcells;
     ctx->st.band_group = ctx->bg;
     ctx->st.block_threads = ctx->block;
     *out = ctx;
@@ -806,7 +979,6 @@ bte_status bte_step_begin(bte_ctx *ctx, double dt) {
     STATUS_TRY(upload_cur_slots(ctx));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     ctx->begun = true;
-    ctx->begun_dt = dt;
     return BTE_OK;
 }
 
@@ -821,8 +993,8 @@ bte_status bte_step_finish(bte_ctx *ctx) {
     return check_newton(ctx);
 }
 
-// rows of nc doubles between a device array (internal order) and a host array (caller order)
-static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t rows, double *host) {
+// rows of nc doubles (device rows of `stride` elements, internal order) <-> host (caller order)
+static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t stride, int64_t rows, double *host) {
     bte_ctx *ctx = const_cast<bte_ctx *>(cctx);
     const int64_t per = std::max<int64_t>(1, ctx->staging_elems / ctx->nc);
     for (int64_t r0 = 0; r0 < rows; r0 += per) {
@@ -830,7 +1002,8 @@ static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t 
         const int64_t n = nr * ctx->nc;
         const int tb = 256;
         const int gb = (int)std::min<int64_t>(8192, (n + tb - 1) / tb);
-        bte::gather_rows_kernel<<<gb, tb, 0, ctx->stream>>>(dsrc + r0 * ctx->nc, ctx->pos, ctx->nc, nr, ctx->staging);
+        bte::gather_rows_kernel<<<gb, tb, 0, ctx->stream>>>(dsrc + r0 * stride, ctx->pos, ctx->nc, stride, nr,
+                                                            ctx->staging);
         CUDA_TRY(ctx, cudaGetLastError());
         CUDA_TRY(ctx, cudaMemcpyAsync(host + r0 * ctx->nc, ctx->staging, n * sizeof(double), cudaMemcpyDeviceToHost,
                                       ctx->stream));
@@ -839,7 +1012,7 @@ static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t 
     return BTE_OK;
 }
 
-static bte_status rows_from_host(bte_ctx *ctx, const double *host, int64_t rows, double *ddst) {
+static bte_status rows_from_host(bte_ctx *ctx, const double *host, int64_t stride, int64_t rows, double *ddst) {
     const int64_t per = std::max<int64_t>(1, ctx->staging_elems / ctx->nc);
     for (int64_t r0 = 0; r0 < rows; r0 += per) {
         const int64_t nr = std::min(per, rows - r0);
@@ -848,7 +1021,8 @@ static bte_status rows_from_host(bte_ctx *ctx, const double *host, int64_t rows,
                                       ctx->stream));
         const int tb = 256;
         const int gb = (int)std::min<int64_t>(8192, (n + tb - 1) / tb);
-        bte::scatter_rows_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->staging, ctx->pos, ctx->nc, nr, ddst + r0 * ctx->nc);
+        bte::scatter_rows_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->staging, ctx->pos, ctx->nc, stride, nr,
+                                                             ddst + r0 * stride);
         CUDA_TRY(ctx, cudaGetLastError());
         CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     }
@@ -858,19 +1032,19 @@ static bte_status rows_from_host(bte_ctx *ctx, const double *host, int64_t rows,
 bte_status bte_get_temperature(const bte_ctx *ctx, double *T) {
     if (!ctx || !T) return BTE_EINVAL;
     CUDA_TRY(const_cast<bte_ctx *>(ctx), cudaSetDevice(ctx->device));
-    return rows_to_host(ctx, ctx->T, 1, T);
+    return rows_to_host(ctx, ctx->T, ctx->nc, 1, T);
 }
 
 bte_status bte_get_energy(const bte_ctx *ctx, double *E) {
     if (!ctx || !E) return BTE_EINVAL;
     CUDA_TRY(const_cast<bte_ctx *>(ctx), cudaSetDevice(ctx->device));
-    return rows_to_host(ctx, ctx->E, 1, E);
+    return rows_to_host(ctx, ctx->E, ctx->nc, 1, E);
 }
 
 bte_status bte_set_energy(bte_ctx *ctx, const double *E) {
     if (!ctx || !E) return BTE_EINVAL;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
-    return rows_from_host(ctx, E, 1, ctx->E);
+    return rows_from_host(ctx, E, ctx->nc, 1, ctx->E);
 }
 
 static bte_status check_rows(const bte_ctx *ctx, int32_t b_lo, int32_t b_hi) {
@@ -889,7 +1063,7 @@ bte_status bte_get_intensity(const bte_ctx *ctx, int32_t b_lo, int32_t b_hi, dou
     CUDA_TRY(const_cast<bte_ctx *>(ctx), cudaSetDevice(ctx->device));
     for (int32_t b = b_lo; b < b_hi; ++b) {
         const double *slab = ctx->pool + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
-        STATUS_TRY(rows_to_host(ctx, slab, ctx->nd, I + (int64_t)(b - b_lo) * ctx->slab_elems));
+        STATUS_TRY(rows_to_host(ctx, slab, ctx->ps, ctx->nd, I + (int64_t)(b - b_lo) * ctx->nd * ctx->nc));
     }
     return BTE_OK;
 }
@@ -900,8 +1074,10 @@ bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const dou
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int32_t b = b_lo; b < b_hi; ++b) {
         double *slab = ctx->pool + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
-        STATUS_TRY(rows_from_host(ctx, I + (int64_t)(b - b_lo) * ctx->slab_elems, ctx->nd, slab));
+        STATUS_TRY(rows_from_host(ctx, I + (int64_t)(b - b_lo) * ctx->nd * ctx->nc, ctx->ps, ctx->nd, slab));
     }
+    STATUS_TRY(fill_sym_ghosts(ctx));  // specular ghosts follow the new state
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     return BTE_OK;
 }
 
@@ -911,9 +1087,11 @@ bte_status bte_solve_temperature(bte_ctx *ctx) {
     if (ctx->opt.world > 1 && !ctx->have_comm)
         return set_err(&ctx->err, "world > 1 without a communicator: cannot reduce the energy"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    STATUS_TRY(upload_cur_slots(ctx));
     const int tb = 128;
     bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
-        ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc, ctx->E);
+        ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc,
+        ctx->E);
     CUDA_TRY(ctx, cudaGetLastError());
     STATUS_TRY(allreduce_E(ctx));
     STATUS_TRY(run_newton(ctx, ctx->E));
@@ -926,12 +1104,15 @@ bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int32_t c = 0; c < ctx->nc; ++c)
         if (!(T[c] > 0.0) || !std::isfinite(T[c])) return set_err(&ctx->err, "T[%d] must be > 0", c), BTE_EINVAL;
-    STATUS_TRY(rows_from_host(ctx, T, 1, ctx->T));
+    STATUS_TRY(rows_from_host(ctx, T, ctx->nc, 1, ctx->T));
     STATUS_TRY(refresh_i0(ctx));
+    STATUS_TRY(upload_cur_slots(ctx));
     const int tb = 256;
-    bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, (ctx->slab_elems + tb - 1) / tb), ctx->nb_loc), tb, 0,
-                              ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->nd, ctx->nc, ctx->i0);
+    bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)ctx->nd * ctx->nc + tb - 1) / tb), ctx->nb_loc),
+                              tb, 0, ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nd,
+                                                    ctx->nc, ctx->i0);
     CUDA_TRY(ctx, cudaGetLastError());
+    STATUS_TRY(fill_sym_ghosts(ctx));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     return BTE_OK;
 }

@@ -31,131 +31,249 @@ constexpr int kMaxThreads = 256;
 enum : int8_t { kFaceInterior = 0, kFaceIso = 1, kFaceSym = 2 };
 
 struct FluxParams {
-    int32_t nc;          // cells = plane stride
-    int32_t cell_begin;  // cell range of this launch (internal order)
-    int32_t cell_end;
+    int32_t nc;          // cells
+    int32_t ps;          // plane stride: nc cells + ghost columns (boundary faces), padded
     int32_t nd;          // directions
     int32_t dchunk;      // directions per block
     int32_t n_dchunks;
-    int32_t nbl;         // band-rows in this launch
-    int32_t bg;          // band-rows per thread group (<= BG)
+    int32_t nbl;         // band-rows in this launch (a multiple of the template BG)
     int32_t band0;       // rank-local index of the launch's first band-row
     int32_t slot0;       // first energy-partial slot of this launch
-    int64_t slab_elems;  // nd * nc
+    int64_t slab_elems;  // nd * ps
     double *pool;        // slab pool
     const double *i0;    // [nb_loc][nc]  I0_b(T_c) of the current step
     double *part;        // [n_slots][nc] energy partials
-    const int32_t *nbr;  // [MF][nc]
-    const double *gx, *gy, *gz;  // [MF][nc]
-    const int8_t *kind;  // [MF][nc] (boundary cells only are read)
-    const int32_t *aux;  // [MF][nc]
-    const int32_t *refl; // [n_refl_classes][nd]
-    const double *i0w;   // [nb_loc][n_iso]  I0_b(T_wall) per isothermal face
-    int32_t n_iso;
-    const double4 *dirs; // [nd] {s_x, s_y, s_z, w}
-    const double *inv_tau, *vg, *cw;  // [nb_loc]
+    // Face slots, struct-of-arrays [slot][nc].  Generic: one slot per face.
+    // Paired: one slot per opposite face pair; nbr/symc describe the "+" face
+    // (the one whose normal g is stored), nbm the "-" face (g_- = -g_+).
+    // nbr >= nc addresses the face's ghost column in the same plane.
+    const int32_t *nbr, *nbm;
+    const double *gx, *gy, *gz;  // g = (A_f / V_c) n_f
+    const int32_t *symc;         // generic [MF][nc]: reflection class of a specular face, -1 otherwise
+    const uint32_t *symp;        // paired [nc]: 5-bit reflection class per side (pair q: bits 10q / 10q+5), 31 = none
+    const int32_t *refl;         // [n_classes][nd] reflected direction
+    const double4 *dirs;         // [nd] {s_x, s_y, s_z, w}
     double dt;
-    int32_t in_slot[kMaxBandsPerLaunch];
-    int32_t out_slot[kMaxBandsPerLaunch];
+    const double *in_ptr[kMaxBandsPerLaunch];  // per launch-local band-row: input slab (I^n)
+    double *out_ptr[kMaxBandsPerLaunch];       // ... output slab (I^{n+1})
+    double dtit[kMaxBandsPerLaunch];       // dt / tau_b
+    double kv[kMaxBandsPerLaunch];         // dt v_b
+    double cw[kMaxBandsPerLaunch];         // temperature weight c_b
 };
 
-// One thread owns one cell and a (band group, direction chunk) of its unknowns.
-// Per direction it forms alpha_j = s_d . g_j for its faces once and reuses it for
-// every band-row of the group; per band-row it streams I^n[b][d][c] in, reads the
-// upwind neighbours of the inflow faces (L1/L2 hits: same plane), and streams
-// I^{n+1} out.  The energy partial stays in registers until the end.
-template <int DIM, int MF, int BG, bool BND>
-__global__ void __launch_bounds__(kMaxThreads)
+__device__ __forceinline__ double4 load_dir(const double4 *dirs, int d) {
+    const double2 a = __ldg(reinterpret_cast<const double2 *>(dirs + d));
+    const double2 b = __ldg(reinterpret_cast<const double2 *>(dirs + d) + 1);
+    return make_double4(a.x, a.y, b.x, b.y);
+}
+
+// Boundary faces are ghost columns of every (b, d) plane (Eq. 6:
+// "setting the intensity of ghost cells on the outside"):
+//   isothermal face: ghost = I0_b(T_wall), constant in time, written at set-up;
+//   specular face f of cell c: ghost[b][d] = I^n[b][r_f(d)][c].  It is written
+//   by the step that produces I^n: when a thread computes I'[b][d][c] it also
+//   stores it to ghost column f of direction r_f(d) of the output slab (r_f is
+//   an involution), so the flux loop never branches on the face kind.  The
+//   reflected directions of an iteration are fetched with its other loads.
+constexpr uint32_t kNoClass = 31;
+
+// ---------------------------------------------------------------------------
+// Generic connectivity: up to MF faces per cell, each with its own neighbour.
+// One thread owns one cell and a (band group, direction chunk) of its
+// unknowns.  Per direction it forms alpha_j = s_d . g_j once for the BG
+// band-rows, issues every load of the iteration (own value and the inflow
+// faces' upwind values of all BG rows) before using any, then writes
+//   I' = I (1 - dt/tau - dt v out) + (dt/tau) I0 - dt v sum_{alpha<0} alpha I_up
+// (Eq. 3/5, L269-292, L546-553; upwind L264-267) with a streaming store and
+// accumulates c_b w_d I' for the energy partial (L412-418).
+template <int DIM, int MF, int BG>
+__global__ void __launch_bounds__(kMaxThreads, 2)
 flux_kernel(const __grid_constant__ FluxParams p) {
-    const int c = p.cell_begin + blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= p.cell_end) return;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= p.nc) return;
     const int grp = blockIdx.y / p.n_dchunks;
     const int dch = blockIdx.y - grp * p.n_dchunks;
-    const int lg0 = grp * p.bg;  // launch-local first band-row of the group
-    const int nbg = min(p.bg, p.nbl - lg0);
+    const int lg0 = grp * BG;  // launch-local first band-row of the group (groups are full)
     const int d0 = dch * p.dchunk;
     const int d1 = min(p.nd, d0 + p.dchunk);
     const int nc = p.nc;
 
-    int nbr[MF];
+    int nbr[MF], cls[MF];
     double gx[MF], gy[MF], gz[MF];
-    int8_t kind[MF];
-    int aux[MF];
+    bool has_sym = false;
 #pragma unroll
     for (int j = 0; j < MF; ++j) {
-        nbr[j] = __ldg(p.nbr + (size_t)j * nc + c);
-        gx[j] = __ldg(p.gx + (size_t)j * nc + c);
-        gy[j] = __ldg(p.gy + (size_t)j * nc + c);
-        gz[j] = DIM == 3 ? __ldg(p.gz + (size_t)j * nc + c) : 0.0;
-        if (BND) {
-            kind[j] = p.kind[(size_t)j * nc + c];
-            aux[j] = __ldg(p.aux + (size_t)j * nc + c);
-        }
+        const size_t q = (size_t)j * nc + c;
+        nbr[j] = __ldg(p.nbr + q);
+        gx[j] = __ldg(p.gx + q);
+        gy[j] = __ldg(p.gy + q);
+        gz[j] = DIM == 3 ? __ldg(p.gz + q) : 0.0;
+        cls[j] = __ldg(p.symc + q);
+        has_sym |= cls[j] >= 0;
     }
-
-    const double *inb[BG];
-    double *outb[BG];
-    double src[BG], diag[BG], kv[BG], acc[BG];
-    int lb[BG];
+    double src[BG];
 #pragma unroll
-    for (int k = 0; k < BG; ++k) {
-        const int kk = k < nbg ? k : 0;
-        lb[k] = p.band0 + lg0 + kk;
-        inb[k] = p.pool + (int64_t)p.in_slot[lg0 + kk] * p.slab_elems;
-        outb[k] = p.pool + (int64_t)p.out_slot[lg0 + kk] * p.slab_elems;
-        const double dtit = p.dt * __ldg(p.inv_tau + lb[k]);
-        src[k] = dtit * __ldg(p.i0 + (size_t)lb[k] * nc + c);  // dt/tau I0_b(T_c)
-        diag[k] = 1.0 - dtit;
-        kv[k] = p.dt * __ldg(p.vg + lb[k]);
-        acc[k] = 0.0;
-    }
-
+    for (int k = 0; k < BG; ++k)  // dt/tau I0_b(T_c)
+        src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (size_t)(p.band0 + lg0 + k) * nc + c);
+    double e = 0.0;
     for (int d = d0; d < d1; ++d) {
-        const double2 sxy = __ldg(reinterpret_cast<const double2 *>(p.dirs + d));
-        const double2 szw = __ldg(reinterpret_cast<const double2 *>(p.dirs + d) + 1);
-        const double4 sd = make_double4(sxy.x, sxy.y, szw.x, szw.y);
+        const double4 sd = load_dir(p.dirs, d);
         double a[MF];
         double out = 0.0;
 #pragma unroll
         for (int j = 0; j < MF; ++j) {
-            a[j] = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j]))
-                            : fma(sd.y, gy[j], sd.x * gx[j]);
-            out += fmax(a[j], 0.0);  // outflow faces use the cell's own value
+            a[j] = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
+            out += fmax(a[j], 0.0);  // outflow faces carry the cell's own value
         }
-        const size_t po = (size_t)d * nc;
+        const size_t po = (size_t)d * p.ps;
+        int rr[MF];
+#pragma unroll
+        for (int j = 0; j < MF; ++j) rr[j] = (has_sym && cls[j] >= 0) ? __ldg(p.refl + (size_t)cls[j] * p.nd + d) : 0;
+        double ic[BG], nv[BG][MF];
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {  // every load of the iteration first
+            const double *pl = p.in_ptr[lg0 + k] + po;
+            ic[k] = __ldg(pl + c);
+#pragma unroll
+            for (int j = 0; j < MF; ++j) nv[k][j] = a[j] < 0.0 ? __ldg(pl + nbr[j]) : 0.0;
+        }
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
-            if (k < nbg) {
-                const double *pl = inb[k] + po;
-                const double ic = __ldg(pl + c);
-                double infl = 0.0;
+            double infl = 0.0;
 #pragma unroll
-                for (int j = 0; j < MF; ++j) {
-                    if (a[j] < 0.0) {  // inflow: upwind neighbour or ghost
-                        double v;
-                        if (!BND || kind[j] == kFaceInterior) {
-                            v = __ldg(pl + nbr[j]);
-                        } else if (kind[j] == kFaceIso) {
-                            v = __ldg(p.i0w + (size_t)lb[k] * p.n_iso + aux[j]);
-                        } else {  // specular: reflected direction, same cell, old level
-                            const int r = __ldg(p.refl + (size_t)aux[j] * p.nd + d);
-                            v = __ldg(inb[k] + (size_t)r * nc + c);
-                        }
-                        infl = fma(a[j], v, infl);
-                    }
-                }
-                // I' = I (1 - dt/tau - dt v out) + dt/tau I0 - dt v sum_in alpha I_nbr
-                const double inew = fma(ic, diag[k] - kv[k] * out, fma(-kv[k], infl, src[k]));
-                __stcs(outb[k] + po + c, inew);
-                acc[k] = fma(sd.w, inew, acc[k]);
+            for (int j = 0; j < MF; ++j) infl = fma(fmin(a[j], 0.0), nv[k][j], infl);
+            const double kv = p.kv[lg0 + k];
+            const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
+            double *ob = p.out_ptr[lg0 + k];
+            __stcs(ob + po + c, inew);
+            if (has_sym) {
+#pragma unroll
+                for (int j = 0; j < MF; ++j)
+                    if (cls[j] >= 0) __stcs(ob + (size_t)rr[j] * p.ps + nbr[j], inew);
             }
+            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
         }
     }
-    double e = 0.0;
-#pragma unroll
-    for (int k = 0; k < BG; ++k)
-        if (k < nbg) e = fma(__ldg(p.cw + lb[k]), acc[k], e);
     p.part[(size_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
+}
+
+// ---------------------------------------------------------------------------
+// Paired faces (every cell's faces come in exactly opposite pairs, g_- = -g_+,
+// as in the paper's uniform quad/hex grids): for each pair only the face with
+// s_d . g < 0 is an inflow, so one upwind load and one FMA per pair, and
+// out = sum_pairs |s_d . g_+|.  Same arithmetic as the generic kernel.
+template <int DIM, int NP, int BG>
+__global__ void __launch_bounds__(kMaxThreads, 2)
+flux_paired_kernel(const __grid_constant__ FluxParams p) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= p.nc) return;
+    const int grp = blockIdx.y / p.n_dchunks;
+    const int dch = blockIdx.y - grp * p.n_dchunks;
+    const int lg0 = grp * BG;
+    const int d0 = dch * p.dchunk;
+    const int d1 = min(p.nd, d0 + p.dchunk);
+    const int nc = p.nc;
+    const int ps = p.ps;
+
+    int np_[NP], nm_[NP];
+    double gx[NP], gy[NP], gz[NP];
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+        const int o = q * nc + c;
+        np_[q] = __ldg(p.nbr + o);
+        nm_[q] = __ldg(p.nbm + o);
+        gx[q] = __ldg(p.gx + o);
+        gy[q] = __ldg(p.gy + o);
+        gz[q] = DIM == 3 ? __ldg(p.gz + o) : 0.0;
+    }
+    const uint32_t symp = __ldg(p.symp + c);
+    constexpr uint32_t kNone = (1u << (10 * NP)) - 1u;  // every side "31"
+    const bool has_sym = symp != kNone;
+    double src[BG];  // dt/tau I0_b(T_c) per band-row of the group
+#pragma unroll
+    for (int k = 0; k < BG; ++k) src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c);
+    double e = 0.0;
+    for (int d = d0; d < d1; ++d) {
+        const double4 sd = load_dir(p.dirs, d);
+        double amin[NP];  // -|s.g|: alpha of the pair's inflow face
+        int ni[NP];
+        double out = 0.0;
+#pragma unroll
+        for (int q = 0; q < NP; ++q) {
+            const double a = DIM == 3 ? fma(sd.z, gz[q], fma(sd.y, gy[q], sd.x * gx[q])) : fma(sd.y, gy[q], sd.x * gx[q]);
+            out += fabs(a);
+            amin[q] = -fabs(a);
+            ni[q] = a > 0.0 ? nm_[q] : np_[q];  // "+" face outgoing -> inflow through "-"
+        }
+        const int64_t po = (int64_t)d * ps;
+        int gofs[2 * NP];  // specular sides: plane offset of ghost column f in direction r_f(d)
+        if (has_sym) {
+#pragma unroll
+            for (int s = 0; s < 2 * NP; ++s) {
+                const uint32_t cl = (symp >> (5 * s)) & kNoClass;
+                const int col = (s & 1) ? nm_[s >> 1] : np_[s >> 1];
+                gofs[s] = cl != kNoClass ? __ldg(p.refl + cl * p.nd + d) * ps + col : -1;
+            }
+        }
+        double ic[BG], nv[BG][NP];
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {  // every load of the iteration first
+            const double *pl = p.in_ptr[lg0 + k] + po;  // slab bases come from the constant bank
+            ic[k] = __ldg(pl + c);
+#pragma unroll
+            for (int q = 0; q < NP; ++q) nv[k][q] = __ldg(pl + ni[q]);
+        }
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            double infl = 0.0;
+#pragma unroll
+            for (int q = 0; q < NP; ++q) infl = fma(amin[q], nv[k][q], infl);
+            const double kv = p.kv[lg0 + k];
+            const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
+            double *ob = p.out_ptr[lg0 + k];
+            __stcs(ob + po + c, inew);
+            if (has_sym) {
+#pragma unroll
+                for (int s = 0; s < 2 * NP; ++s)
+                    if (gofs[s] >= 0) __stcs(ob + gofs[s], inew);
+            }
+            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
+        }
+    }
+    p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
+}
+
+// ---------------------------------------------------------------- ghost set-up
+// Isothermal ghosts of band-row b in slab s: ghost[d][col] = I0_b(T_wall).
+__global__ void iso_ghost_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,
+                                 const int32_t *__restrict__ band_of_slot_entry, int64_t slab_elems, int ps,
+                                 int nd, int n_iso, const int32_t *__restrict__ iso_col /* plane index */,
+                                 const double *__restrict__ i0w) {
+    const int k = blockIdx.y;  // entry: slab slot[k] holds local band-row band_of_slot_entry[k]
+    double *s = pool + (int64_t)slot[k] * slab_elems;
+    const int b = band_of_slot_entry[k];
+    const int64_t n = (int64_t)nd * n_iso;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int d = (int)(e / n_iso);
+        const int f = (int)(e - (int64_t)d * n_iso);
+        s[(size_t)d * ps + iso_col[f]] = i0w[(size_t)b * n_iso + f];
+    }
+}
+
+// Specular ghosts of the current state: ghost[b][d][col_f] = I[b][r_f(d)][owner_f].
+__global__ void sym_ghost_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot, int64_t slab_elems,
+                                 int ps, int nd, int n_sym, const int32_t *__restrict__ sym_col /* plane index */,
+                                 const int32_t *__restrict__ sym_owner, const int32_t *__restrict__ sym_cls,
+                                 const int32_t *__restrict__ refl) {
+    const int k = blockIdx.y;
+    double *s = pool + (int64_t)slot[k] * slab_elems;
+    const int64_t n = (int64_t)nd * n_sym;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int d = (int)(e / n_sym);
+        const int f = (int)(e - (int64_t)d * n_sym);
+        const int r = refl[(size_t)sym_cls[f] * nd + d];
+        s[(size_t)d * ps + sym_col[f]] = s[(size_t)r * ps + sym_owner[f]];
+    }
 }
 
 // ---------------------------------------------------------------- temperature
@@ -261,8 +379,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
 }
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
-__global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc,
-                                 double *__restrict__ E) {
+__global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= nc) return;
     double e = 0.0;
@@ -272,7 +389,7 @@ __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, i
 
 // E_loc[c] = sum_{local b} c_b sum_d w_d I[b][d][c] of the current state.
 __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__restrict__ slot,
-                              int64_t slab_elems, int nb_loc, int nd, int nc,
+                              int64_t slab_elems, int ps, int nb_loc, int nd, int nc,
                               const double4 *__restrict__ dirs, const double *__restrict__ cw,
                               double *__restrict__ E) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -281,7 +398,7 @@ __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__
     for (int k = 0; k < nb_loc; ++k) {
         const double *s = pool + (int64_t)slot[k] * slab_elems;
         double sb = 0.0;
-        for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * nc + c], sb);
+        for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * ps + c], sb);
         e = fma(cw[k], sb, e);
     }
     E[c] = e;
@@ -300,15 +417,18 @@ __global__ void i0_table_kernel(const double *__restrict__ T, int nc, int b_lo, 
 
 // Equilibrium field I[k][d][c] = i0[k][c] into the current slabs (blockIdx.y = k).
 __global__ void equilibrium_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,
-                                   int64_t slab_elems, int nd, int nc,
+                                   int64_t slab_elems, int ps, int nd, int nc,
                                    const double *__restrict__ i0) {
     const int64_t n = (int64_t)nd * nc;
     const int k = blockIdx.y;
     double *s = pool + (int64_t)slot[k] * slab_elems;
     const double *t = i0 + (size_t)k * nc;
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
-         e += (int64_t)gridDim.x * blockDim.x)
-        s[e] = t[e % nc];
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t d = e / nc;
+        const int c = (int)(e - d * nc);
+        s[d * ps + c] = t[c];
+    }
 }
 
 // Isothermal ghost table i0w[k][f] = I0_{b_lo+k}(T_wall(f)) (Eq. 6, constant in time).
@@ -321,9 +441,10 @@ __global__ void i0w_kernel(const double *__restrict__ twall, int n_iso, int b_lo
         i0w[(size_t)k * n_iso + f] = Cb[b_lo + k] / expm1(theta[b_lo + k] / twall[f]);
 }
 
-// S_max = max_{c,d} sum_j max(s_d . g_j(c), 0) (positivity bound of the step).
+// S_max = max_{c,d} sum_faces max(s_d . g, 0) (positivity bound of the step).
+// Paired layout: g holds the "+" face of each pair and the sum is sum |s.g|.
 template <int DIM>
-__global__ void outflow_max_kernel(int nc, int mf, int nd, const double *__restrict__ gx,
+__global__ void outflow_max_kernel(int nc, int mf, int paired, int nd, const double *__restrict__ gx,
                                    const double *__restrict__ gy, const double *__restrict__ gz,
                                    const double4 *__restrict__ dirs,
                                    unsigned long long *__restrict__ smax_bits) {
@@ -337,34 +458,34 @@ __global__ void outflow_max_kernel(int nc, int mf, int nd, const double *__restr
             const size_t q = (size_t)j * nc + c;
             double a = s.x * gx[q] + s.y * gy[q];
             if (DIM == 3) a += s.z * gz[q];
-            out += fmax(a, 0.0);
+            out += paired ? fabs(a) : fmax(a, 0.0);
         }
         m = fmax(m, out);
     }
     atomicMax(smax_bits, (unsigned long long)__double_as_longlong(m));  // m >= 0: bit order = value order
 }
 
-// dst[d][u] = src[d][pos[u]]  (internal -> caller cell order), rows of nc.
+// dst[r][u] = src[r * stride + pos[u]]  (internal -> caller cell order).
 __global__ void gather_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
-                                   int nc, int64_t rows, double *__restrict__ dst) {
+                                   int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
     const int64_t n = rows * nc;
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
          e += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = e / nc;
         const int u = (int)(e - r * nc);
-        dst[e] = src[r * nc + pos[u]];
+        dst[e] = src[r * stride + pos[u]];
     }
 }
 
-// dst[d][pos[u]] = src[d][u]  (caller -> internal order)
+// dst[r * stride + pos[u]] = src[r][u]  (caller -> internal order)
 __global__ void scatter_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
-                                    int nc, int64_t rows, double *__restrict__ dst) {
+                                    int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
     const int64_t n = rows * nc;
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
          e += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = e / nc;
         const int u = (int)(e - r * nc);
-        dst[r * nc + pos[u]] = src[e];
+        dst[r * stride + pos[u]] = src[e];
     }
 }
 

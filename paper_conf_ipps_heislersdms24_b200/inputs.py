@@ -141,6 +141,32 @@ def permute_mesh(mesh, seed=SEED):
     return out, perm
 
 
+def split_faces(mesh, every=3):
+    """Split the first face of every `every`-th cell into two half-area faces
+    with the same normal and neighbour (a hanging-node style polygon): such
+    cells no longer have opposite-face pairs, which exercises the generic
+    face-slot path.  Boundary faces are not split (ids stay unique)."""
+    off, nbr = mesh["face_offsets"], mesh["face_nbr"]
+    area, nrm = mesh["face_area"], mesh["face_normal"]
+    o_off, o_nbr, o_area, o_nrm = [0], [], [], []
+    for c in range(mesh["n_cells"]):
+        lo, hi = off[c], off[c + 1]
+        for f in range(lo, hi):
+            if f == lo and c % every == 0 and nbr[f] >= 0:
+                o_nbr += [nbr[f], nbr[f]]
+                o_area += [0.5 * area[f], 0.5 * area[f]]
+                o_nrm += [nrm[f], nrm[f]]
+            else:
+                o_nbr.append(nbr[f])
+                o_area.append(area[f])
+                o_nrm.append(nrm[f])
+        o_off.append(len(o_nbr))
+    out = dict(mesh)
+    out.update(face_offsets=np.asarray(o_off, np.int64), face_nbr=np.asarray(o_nbr, np.int64),
+               face_area=np.asarray(o_area), face_normal=np.asarray(o_nrm).reshape(-1, 3))
+    return out
+
+
 # --------------------------------------------------------------------------- bands
 # External Si quadratic dispersion omega = v_s k + c k^2 (SURVEY 8(c) #13, #14).
 SI_LATTICE = 5.431e-10

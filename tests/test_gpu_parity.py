@@ -122,7 +122,7 @@ def test_single_cell_all_walls(bte, oracle_mod):
     cfg = gen.Config("1cell", mesh, bands, dirs, bcs, 300.0, dt, 10, ic_eps=0.2)
     Io, To = oracle_run(oracle_mod, cfg, 10)
     Ig, Tg, st = gpu_run(cfg, 10)
-    assert st["n_interior_cells"] == 0
+    assert st["n_interior_cells"] == 0  # the one cell has four wall faces
     assert_parity(Ig, Tg, Io, To)
 
 
@@ -159,6 +159,31 @@ def test_ballistic_row_with_R1(bte, oracle_mod):
     Io, To = oracle_run(oracle_mod, cfg, 30)
     Ig, Tg, _ = gpu_run(cfg, 30)
     assert_parity(Ig, Tg, Io, To)
+
+
+@pytest.mark.parametrize("bg", [1, 2, 4])
+def test_generic_face_path_2d_3d(bte, oracle_mod, bg):
+    """The generic (unpaired) face-slot kernel: forced on a 3-D Fig.-1 problem,
+    and chosen by the library for a 2-D mesh with split (hanging) faces."""
+    cfg = gen.small_3d_config((9, 5, 4), n_spectral=2)
+    Io, To = oracle_run(oracle_mod, cfg, 12)
+    Ig, Tg, _ = gpu_run(cfg, 12, generic_faces=True, band_group=bg)
+    assert_parity(Ig, Tg, Io, To)
+    c2 = _cfg("C1", steps=12)
+    bands = gen.gen_bands_si(3)
+    c2 = dataclasses.replace(c2, mesh=gen.split_faces(c2.mesh), bands=bands,
+                             dt=0.5 * gen.cartesian_dt_bound(c2.mesh, bands, c2.dirs))
+    Io, To = oracle_run(oracle_mod, c2, 12)
+    Ig, Tg, _ = gpu_run(c2, 12, band_group=bg)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_locality_order_is_invisible(bte):
+    """The Morton-order hint changes only the internal layout: bitwise equal."""
+    cfg = gen.small_3d_config((11, 6, 5), n_spectral=3)
+    a = gpu_run(cfg, 8, locality=True)
+    b = gpu_run(cfg, 8, locality=False)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
 
 
 def test_permuted_unstructured_order(bte, oracle_mod):
@@ -265,7 +290,7 @@ def test_profile_stats(bte):
     with bte.solver_from_config(cfg, profile=True) as s:
         s.step(cfg.dt, 3)
         st = s.stats()
-    assert st["steps"] == 3 and st["kernel_launches"] == 9
+    assert st["steps"] == 3 and st["kernel_launches"] >= 6 and st["kernel_launches"] % 3 == 0
     assert st["ms_flux_interior"] > 0 and st["ms_newton"] > 0 and st["ms_total"] > 0
     assert st["updates"] == 3 * cfg.n_updates_per_step
 
