@@ -114,6 +114,8 @@ typedef struct {
 /* bte_options.flags */
 #define BTE_FLAG_PROFILE 1u       /* record CUDA events around every phase (see bte_stats) */
 #define BTE_FLAG_GENERIC_FACES 2u /* never use the opposite-face-pair layout (testing) */
+#define BTE_FLAG_NO_TMA 4u        /* paired meshes: register-pipelined kernel instead of the
+                                     TMA-staged one (testing / comparison) */
 
 typedef struct {
     double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */
@@ -125,7 +127,9 @@ typedef struct {
     const void *nccl_unique_id; /* world > 1: 128-byte ncclUniqueId from bte_nccl_unique_id()
                                    on rank 0, broadcast by the caller.  NULL with world > 1:
                                    no communicator; the caller reduces the energy itself
-                                   through the split-step calls (bte_step returns ESTATE) */
+                                   through the split-step calls (bte_step returns ESTATE).
+                                   An id with world == 1 builds a one-rank communicator and
+                                   runs the all-reduce path (testing) */
     void *stream;             /* cudaStream_t to launch on (NULL: library-owned stream) */
     uint32_t flags;           /* BTE_FLAG_* */
     int32_t max_spare_slabs;  /* band slabs of workspace: <= 0 auto (double buffer when it

@@ -13,11 +13,13 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbte.so")
+# BTE_LIB selects an experiment build of the same library (tools/); default in-tree libbte.so
+LIB_PATH = os.environ.get("BTE_LIB") or os.path.join(_HERE, "libbte.so")
 
 BTE_OK, BTE_EINVAL, BTE_ENOMEM, BTE_ECUDA, BTE_ENCCL, BTE_ENOCONV, BTE_ESTATE = range(7)
 BTE_FLAG_PROFILE = 1
 BTE_FLAG_GENERIC_FACES = 2
+BTE_FLAG_NO_TMA = 4
 ISOTHERMAL, SYMMETRY = 0, 1
 
 
@@ -150,7 +152,7 @@ class Solver:
     def __init__(self, mesh, bands, dirs, bcs, *, t_init=300.0, temp_rule=0, newton_rtol=1e-12,
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
                  stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
-                 generic_faces=False, locality=True, dir_chunk=0):
+                 generic_faces=False, locality=True, dir_chunk=0, tma=True):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -175,14 +177,15 @@ class Solver:
         o.t_init, o.temp_rule, o.newton_rtol, o.newton_max_iter = float(t_init), int(temp_rule), float(newton_rtol), int(newton_max_iter)
         o.rank, o.world, o.device = int(rank), int(world), int(device)
         self._nccl_buf = None
-        if world > 1 and nccl_id is not None:  # None: caller reduces E (split-step calls)
+        if nccl_id is not None:  # world > 1 and None: the caller reduces E (split-step calls)
             if len(nccl_id) != 128:
                 raise ValueError("the NCCL id is 128 bytes (from nccl_unique_id() on rank 0)")
             self._nccl_buf = C.create_string_buffer(bytes(nccl_id), 128)
             o.nccl_unique_id = C.cast(self._nccl_buf, C.c_void_p).value
         if stream is not None:
             o.stream = int(getattr(stream, "cuda_stream", stream))
-        o.flags = (BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
+        o.flags = ((BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
+                   | (0 if tma else BTE_FLAG_NO_TMA))
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)
         o.dir_chunk = int(dir_chunk)
         ctx = C.c_void_p()

@@ -52,19 +52,21 @@ def stale():
     return any(os.path.getmtime(p) > t for p in deps())
 
 
-def build(force=False, verbose=False, extra=()):
-    if not force and not stale():
+def build(force=False, verbose=False, extra=(), out=None):
+    """Compile libbte.so (or `out`, an experiment variant with `extra` flags)."""
+    lib = out or LIB
+    if not force and out is None and not stale():
         return LIB
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
            "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
            "-I", os.path.join(ROOT, "include"), "-I", _nccl_include(),
-           "-DBTE_BUILD", *extra, *sources(), "-o", LIB + ".tmp", "-ldl"]
+           "-DBTE_BUILD", *extra, *sources(), "-o", lib + ".tmp", "-ldl"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(lib + ".tmp", lib)
+    return lib
 
 
 if __name__ == "__main__":

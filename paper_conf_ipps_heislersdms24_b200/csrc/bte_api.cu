@@ -1,7 +1,7 @@
 // bte_api.cu -- host runtime behind include/bte.h.
 //
 // Owns validation, the device layout (face slots, opposite-face pairing,
-// ghost columns for boundary faces, reflection maps, slab pool), launch
+// boundary-face codes, reflection maps, isothermal table, slab pool), launch
 // planning, the per-step launch sequence, the NCCL energy all-reduce and the
 // getters.  All arithmetic of the step runs in the kernels of bte_kernels.cuh;
 // the host only validates, moves data and plans launches.
@@ -49,7 +49,7 @@ struct bte_ctx {
     std::string err = "no error";
     bte_options opt{};
     int dim = 0, nd = 0, nb = 0, b_lo = 0, b_hi = 0, nb_loc = 0, mf = 0, mf_t = 0;
-    int32_t nc = 0, ps = 0, n_ghost = 0, n_bcells = 0;
+    int32_t nc = 0, ps = 0, n_bcells = 0;
     int device = 0;
     int sm_count = 148;
     double W = 0.0, s_max = 0.0, dt_bound = 0.0;
@@ -58,20 +58,23 @@ struct bte_ctx {
     int64_t slab_elems = 0;
     int n_spare = 0;
     std::vector<int32_t> cur_slot, spare_slot;
-    int32_t *d_cur_slot = nullptr, *d_band_ids = nullptr, *d_tmp_slot = nullptr;
+    int32_t *d_cur_slot = nullptr;
     double *i0 = nullptr, *T = nullptr, *E = nullptr, *part = nullptr;
     int n_slots_step = 0;
     double *staging = nullptr;
     int64_t staging_elems = 0;
     // face slots [mf_t][nc]
-    int32_t *nbr = nullptr, *nbm = nullptr, *symc = nullptr, *pos = nullptr;
-    uint32_t *symp = nullptr;
+    int32_t *nbr = nullptr, *nbm = nullptr, *pos = nullptr;
+    uint32_t *fcode = nullptr;  // paired: 5-bit face codes per cell
+    uint8_t *fcode8 = nullptr;  // generic: 8-bit face codes per face slot
     double *gx = nullptr, *gy = nullptr, *gz = nullptr;
-    bool paired = false;
-    // boundary ghosts
+    bool paired = false;     // every cell's faces are exact opposite pairs
+    bool uniform_g = false;  // ... and every cell has the same g per pair
+    bool tma = false;        // paired + 256-thread blocks: the TMA-staged kernel
+    double gu[3][3] = {};
+    // boundary faces: reflection maps of specular classes, isothermal table
     int32_t *refl = nullptr;
-    int32_t n_iso = 0, n_sym = 0, n_refl = 0;
-    int32_t *iso_col = nullptr, *sym_col = nullptr, *sym_owner = nullptr, *sym_cls = nullptr;
+    int32_t n_iso = 0, n_refl = 0;
     double *i0w = nullptr, *twall = nullptr;
     // tables
     double4 *dirs = nullptr;
@@ -128,26 +131,54 @@ bte_status upload(bte_ctx *ctx, T **p, const std::vector<T> &h) {
 // ------------------------------------------------------------- template dispatch
 using FluxLaunch = void (*)(dim3, dim3, cudaStream_t, const bte::FluxParams &);
 
-template <int DIM, int MF, int BG, bool PAIRED>
+template <int DIM, int MF, int BG, bool PAIRED, bool UG = false>
 void flux_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
     if constexpr (PAIRED)
-        bte::flux_paired_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
+        bte::flux_paired_kernel<DIM, MF, BG, UG><<<g, b, 0, s>>>(p);
     else
         bte::flux_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
 }
 
-// Paired kernels exist for every band group 1..8, generic ones for 1, 2, 4.
-template <int DIM, int MF>
+// TMA-staged paired kernel: one 256-cell tile per block, kStages x BG x 2 KB ring.
+template <int DIM, int NP, int BG, bool UG>
+void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    constexpr size_t smem = (size_t)bte::kStages * BG * bte::kTile * sizeof(double);
+    static bool attr = false;  // > 48 KB of dynamic shared memory needs an opt-in
+    if (!attr) {
+        cudaFuncSetAttribute(bte::flux_tma_kernel<DIM, NP, BG, UG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smem);
+        attr = true;
+    }
+    bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTile), smem, s>>>(p);
+}
+
+template <int DIM, int NP, bool UG>
+FluxLaunch pick_tma(int bg) {
+    switch (bg) {
+        case 1: return flux_tma_launch_t<DIM, NP, 1, UG>;
+        case 2: return flux_tma_launch_t<DIM, NP, 2, UG>;
+        case 3: return flux_tma_launch_t<DIM, NP, 3, UG>;
+        case 4: return flux_tma_launch_t<DIM, NP, 4, UG>;
+        case 5: return flux_tma_launch_t<DIM, NP, 5, UG>;
+        case 6: return flux_tma_launch_t<DIM, NP, 6, UG>;
+        case 7: return flux_tma_launch_t<DIM, NP, 7, UG>;
+        default: return flux_tma_launch_t<DIM, NP, 8, UG>;
+    }
+}
+
+// Paired kernels exist for every band group 1..8 (per-cell or uniform geometry),
+// generic ones for 1, 2, 4.
+template <int DIM, int MF, bool UG>
 FluxLaunch pick_paired(int bg) {
     switch (bg) {
-        case 1: return flux_launch_t<DIM, MF, 1, true>;
-        case 2: return flux_launch_t<DIM, MF, 2, true>;
-        case 3: return flux_launch_t<DIM, MF, 3, true>;
-        case 4: return flux_launch_t<DIM, MF, 4, true>;
-        case 5: return flux_launch_t<DIM, MF, 5, true>;
-        case 6: return flux_launch_t<DIM, MF, 6, true>;
-        case 7: return flux_launch_t<DIM, MF, 7, true>;
-        default: return flux_launch_t<DIM, MF, 8, true>;
+        case 1: return flux_launch_t<DIM, MF, 1, true, UG>;
+        case 2: return flux_launch_t<DIM, MF, 2, true, UG>;
+        case 3: return flux_launch_t<DIM, MF, 3, true, UG>;
+        case 4: return flux_launch_t<DIM, MF, 4, true, UG>;
+        case 5: return flux_launch_t<DIM, MF, 5, true, UG>;
+        case 6: return flux_launch_t<DIM, MF, 6, true, UG>;
+        case 7: return flux_launch_t<DIM, MF, 7, true, UG>;
+        default: return flux_launch_t<DIM, MF, 8, true, UG>;
     }
 }
 
@@ -161,8 +192,13 @@ FluxLaunch pick_generic(int bg) {
 }
 
 // mf_t: padded faces per cell (generic) or face pairs per cell (paired)
-FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired) {
-    if (paired) return dim == 2 ? pick_paired<2, 2>(bg) : pick_paired<3, 3>(bg);
+FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, bool tma) {
+    if (paired && tma) {
+        if (uniform_g) return dim == 2 ? pick_tma<2, 2, true>(bg) : pick_tma<3, 3, true>(bg);
+        return dim == 2 ? pick_tma<2, 2, false>(bg) : pick_tma<3, 3, false>(bg);
+    }
+    if (paired && uniform_g) return dim == 2 ? pick_paired<2, 2, true>(bg) : pick_paired<3, 3, true>(bg);
+    if (paired) return dim == 2 ? pick_paired<2, 2, false>(bg) : pick_paired<3, 3, false>(bg);
     if (dim == 2) return mf_t == 4 ? pick_generic<2, 4>(bg) : pick_generic<2, 8>(bg);
     return mf_t == 6 ? pick_generic<3, 6>(bg) : pick_generic<3, 8>(bg);
 }
@@ -258,39 +294,6 @@ int count_slots(const bte_ctx *ctx) {
     return slots;
 }
 
-// Isothermal ghost columns of the given slabs (entries: slab slot, local band).
-bte_status fill_iso_ghosts(bte_ctx *ctx, const std::vector<int32_t> &slots, const std::vector<int32_t> &bands) {
-    if (ctx->n_iso == 0 || slots.empty()) return BTE_OK;
-    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_tmp_slot, slots.data(), slots.size() * sizeof(int32_t),
-                                  cudaMemcpyHostToDevice, ctx->stream));
-    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_band_ids, bands.data(), bands.size() * sizeof(int32_t),
-                                  cudaMemcpyHostToDevice, ctx->stream));
-    const int tb = 256;
-    const int64_t n = (int64_t)ctx->nd * ctx->n_iso;
-    dim3 grid((unsigned)std::min<int64_t>(2048, (n + tb - 1) / tb), (unsigned)slots.size());
-    bte::iso_ghost_kernel<<<grid, tb, 0, ctx->stream>>>(ctx->pool, ctx->d_tmp_slot, ctx->d_band_ids,
-                                                        ctx->slab_elems, ctx->ps, ctx->nd, ctx->n_iso,
-                                                        ctx->iso_col, ctx->i0w);
-    CUDA_TRY(ctx, cudaGetLastError());
-    ctx->st.kernel_launches++;
-    return BTE_OK;
-}
-
-// Specular ghost columns of the current slabs from the current state.
-bte_status fill_sym_ghosts(bte_ctx *ctx) {
-    if (ctx->n_sym == 0) return BTE_OK;
-    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_cur_slot, ctx->cur_slot.data(), ctx->nb_loc * sizeof(int32_t),
-                                  cudaMemcpyHostToDevice, ctx->stream));
-    const int tb = 256;
-    const int64_t n = (int64_t)ctx->nd * ctx->n_sym;
-    dim3 grid((unsigned)std::min<int64_t>(2048, (n + tb - 1) / tb), (unsigned)ctx->nb_loc);
-    bte::sym_ghost_kernel<<<grid, tb, 0, ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps,
-                                                        ctx->nd, ctx->n_sym, ctx->sym_col, ctx->sym_owner,
-                                                        ctx->sym_cls, ctx->refl);
-    CUDA_TRY(ctx, cudaGetLastError());
-    return BTE_OK;
-}
-
 // Flux + relaxation + energy partials for all local band-rows: per band batch
 // of <= n_spare rows, one launch per segment of full band groups, reading the
 // current slabs and writing the spare ones, which then become current (double
@@ -300,8 +303,6 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.nc = ctx->nc;
     p.ps = ctx->ps;
     p.nd = ctx->nd;
-    p.slab_elems = ctx->slab_elems;
-    p.pool = ctx->pool;
     p.i0 = ctx->i0;
     p.part = ctx->part;
     p.nbr = ctx->nbr;
@@ -309,23 +310,20 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.gx = ctx->gx;
     p.gy = ctx->gy;
     p.gz = ctx->gz;
-    p.symc = ctx->symc;
-    p.symp = ctx->symp;
+    std::memcpy(p.gu, ctx->gu, sizeof p.gu);
+    p.fcode = ctx->fcode;
+    p.fcode8 = ctx->fcode8;
+    p.i0w = ctx->i0w;
+    p.n_iso = ctx->n_iso;
     p.refl = ctx->refl;
     p.dirs = ctx->dirs;
     p.dt = dt;
     int slot = 0;
-    const bool rotating = ctx->n_spare < ctx->nb_loc;
     const dim3 block(ctx->block);
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
         const int nbl_batch = std::min(ctx->n_spare, ctx->nb_loc - l0);
-        if (rotating) {  // spare slabs change band: give them this batch's isothermal ghosts
-            std::vector<int32_t> sl(ctx->spare_slot.begin(), ctx->spare_slot.begin() + nbl_batch), bl(nbl_batch);
-            for (int k = 0; k < nbl_batch; ++k) bl[k] = l0 + k;
-            STATUS_TRY(fill_iso_ghosts(ctx, sl, bl));
-        }
         for (const Segment &sg : segments(nbl_batch, ctx->bg, ctx->paired)) {
-            const FluxLaunch fn = pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired);
+            const FluxLaunch fn = pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma);
             const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
             p.nbl = sg.nbl;
             p.band0 = l0 + sg.off;
@@ -384,7 +382,7 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null) {
 }
 
 bte_status allreduce_E(bte_ctx *ctx) {
-    if (ctx->opt.world <= 1) return BTE_OK;
+    if (!ctx->have_comm) return BTE_OK;
     std::string e;
     if (!bte::nccl::allreduce_sum_f64(ctx->comm, ctx->E, ctx->nc, ctx->stream, &e)) {
         set_err(&ctx->err, "NCCL all-reduce failed: %s", e.c_str());
@@ -539,10 +537,9 @@ void bte_destroy(bte_ctx *ctx) {
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->have_comm) bte::nccl::destroy(ctx->comm);
-    void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->d_band_ids, ctx->d_tmp_slot, ctx->i0, ctx->T, ctx->E,
-                    ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->symc, ctx->symp, ctx->pos, ctx->gx,
-                    ctx->gy, ctx->gz, ctx->refl, ctx->iso_col, ctx->sym_col, ctx->sym_owner, ctx->sym_cls,
-                    ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
+    void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
+                    ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
+                    ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_fail, ctx->d_smax};
     for (void *p : ptrs)
         if (p) cudaFree(p);
@@ -609,12 +606,12 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     for (int32_t i = 0; i < nc; ++i) pos_h[user_of[i]] = i;
 
-    // --- boundary faces -> ghost columns (internal cell order); reflection classes (Eq. 6)
+    // --- boundary faces: isothermal table columns (internal cell order) and
+    // reflection classes of specular faces with their maps (Eq. 6)
     std::map<std::vector<double>, int> cls_of;
-    std::vector<int32_t> refl_h, ghost_of(bc->n_bfaces, -1), bcls(bc->n_bfaces, -1);
-    std::vector<int32_t> iso_col_h, sym_col_h, sym_owner_h, sym_cls_h;
+    std::vector<int32_t> refl_h, iso_of(bc->n_bfaces, -1), bcls(bc->n_bfaces, -1);
     std::vector<double> twall_h;
-    int32_t n_ghost = 0, n_bcells = 0;
+    int32_t n_bcells = 0;
     for (int32_t i = 0; i < nc; ++i) {
         const int64_t c = user_of[i];
         bool bcell = false;
@@ -622,10 +619,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             if (m->face_nbr[f] >= 0) continue;
             bcell = true;
             const int64_t bf = -1 - m->face_nbr[f];
-            const int32_t col = n_ghost++;
-            ghost_of[bf] = col;
             if (bc->kind[bf] == BTE_BC_ISOTHERMAL) {
-                iso_col_h.push_back(nc + col);  // plane index of the ghost column
+                iso_of[bf] = (int32_t)twall_h.size();
                 twall_h.push_back(bc->t_wall[bf]);
                 continue;
             }
@@ -656,23 +651,25 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                 it = cls_of.emplace(key, id).first;
             }
             bcls[bf] = it->second;
-            sym_col_h.push_back(nc + col);
-            sym_owner_h.push_back(i);
-            sym_cls_h.push_back(it->second);
         }
         n_bcells += bcell;
     }
 
-    // --- plane stride: cells + ghost columns, padded to 32 doubles (256 B)
-    const int32_t ps = (int32_t)((nc64 + n_ghost + 31) / 32 * 32);
+    if ((int)cls_of.size() > bte::kMaxGenericClasses)
+        return set_err(nullptr, "%d distinct specular wall normals (max %d)", (int)cls_of.size(),
+                       bte::kMaxGenericClasses), BTE_EINVAL;
+
+    // --- plane stride: cells padded to a whole 256-cell tile (2 KB)
+    const int32_t ps = (int32_t)((nc64 + bte::kTile - 1) / bte::kTile * bte::kTile);
 
     // --- face pairing: every face of every cell has an exactly opposite partner
     // (same area, negated normal) -> paired layout, one upwind load per pair.
     int mf = 0;
     for (int64_t c = 0; c < nc64; ++c) mf = std::max<int>(mf, (int)(m->face_offsets[c + 1] - m->face_offsets[c]));
     std::vector<int64_t> partner(m->face_offsets[nc64], -1);
-    // (paired layout packs each side's reflection class in 5 bits: < 31 classes)
-    bool paired = mf <= 2 * m->dim && cls_of.size() < 31 && !(o->flags & BTE_FLAG_GENERIC_FACES);
+    // (the paired layout's 5-bit face codes hold up to 16 specular classes)
+    bool paired = mf <= 2 * m->dim && (int)cls_of.size() <= bte::kMaxPairedClasses &&
+                  !(o->flags & BTE_FLAG_GENERIC_FACES);
     for (int64_t c = 0; c < nc64 && paired; ++c) {
         const int64_t f0 = m->face_offsets[c], f1 = m->face_offsets[c + 1];
         for (int64_t f = f0; f < f1 && paired; ++f) {
@@ -692,21 +689,26 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     const int mf_t = paired ? m->dim : (m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
-    std::vector<int32_t> nbr_h(ell), symc_h(ell, -1), nbm_h(paired ? ell : 1, 0);
-    std::vector<uint32_t> symp_h(paired ? nc : 1, 0xffffffffu);
+    std::vector<int32_t> nbr_h(ell), nbm_h(paired ? ell : 1, 0);
+    std::vector<uint32_t> fcode_h(paired ? nc : 1, (1u << (10 * m->dim)) - 1u);  // all interior
+    std::vector<uint8_t> fcode8_h(paired ? 1 : ell, (uint8_t)bte::kCode8Interior);
     std::vector<double> gx_h(ell, 0.0), gy_h(ell, 0.0), gz_h(ell, 0.0);
-    // upwind source index of face f: neighbour cell, or the face's ghost column
-    auto face_src = [&](int64_t f, int32_t *nbv, int32_t *cls) {
+    // upwind source of face f: (index, kind) with kind -1 interior (index =
+    // neighbour cell), -2 isothermal (index = table column), >= 0 specular class
+    auto face_src = [&](int64_t f, int32_t *idx, int32_t *kind) {
         const int64_t v = m->face_nbr[f];
         if (v >= 0) {
-            *nbv = pos_h[v];
-            *cls = -1;
+            *idx = pos_h[v];
+            *kind = -1;
         } else {
             const int64_t bf = -1 - v;
-            *nbv = nc + ghost_of[bf];
-            *cls = bcls[bf];
+            const bool iso = bc->kind[bf] == BTE_BC_ISOTHERMAL;
+            *idx = iso ? iso_of[bf] : 0;
+            *kind = iso ? -2 : bcls[bf];
         }
     };
+    auto code5 = [](int32_t kind) { return kind == -1 ? bte::kCodeInterior : kind == -2 ? bte::kCodeIso : (uint32_t)kind; };
+    auto code8 = [](int32_t kind) { return (uint8_t)(kind == -1 ? bte::kCode8Interior : kind == -2 ? bte::kCode8Iso : kind); };
     for (int32_t i = 0; i < nc; ++i) {
         const int64_t c = user_of[i];
         int j = 0;
@@ -717,14 +719,14 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             gx_h[q] = av * m->face_normal[3 * f + 0];
             gy_h[q] = av * m->face_normal[3 * f + 1];
             gz_h[q] = av * m->face_normal[3 * f + 2];
-            face_src(f, &nbr_h[q], &symc_h[q]);
+            int32_t kp = -1, km = -1;
+            face_src(f, &nbr_h[q], &kp);
             if (paired) {
-                int32_t cm = -1;
-                face_src(partner[f], &nbm_h[q], &cm);
-                const uint32_t cp5 = symc_h[q] < 0 ? 31u : (uint32_t)symc_h[q];
-                const uint32_t cm5 = cm < 0 ? 31u : (uint32_t)cm;
-                const uint32_t mask = ~(1023u << (10 * j));
-                symp_h[i] = (symp_h[i] & mask) | ((cp5 | (cm5 << 5)) << (10 * j));
+                face_src(partner[f], &nbm_h[q], &km);
+                const uint32_t bits = code5(kp) | (code5(km) << 5);
+                fcode_h[i] = (fcode_h[i] & ~(1023u << (10 * j))) | (bits << (10 * j));
+            } else {
+                fcode8_h[q] = code8(kp);
             }
             ++j;
         }
@@ -746,13 +748,25 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     ctx->mf = mf;
     ctx->mf_t = mf_t;
     ctx->paired = paired;
+    if (paired) {  // uniform geometry: g of pair j identical (bitwise) in every cell
+        bool uni = true;
+        for (int j = 0; j < mf_t && uni; ++j)
+            for (int32_t i = 1; i < nc && uni; ++i) {
+                const size_t q0 = (size_t)j * nc, q = q0 + i;
+                uni = gx_h[q] == gx_h[q0] && gy_h[q] == gy_h[q0] && gz_h[q] == gz_h[q0];
+            }
+        ctx->uniform_g = uni && !(o->flags & BTE_FLAG_GENERIC_FACES);
+        for (int j = 0; j < mf_t; ++j) {
+            ctx->gu[j][0] = gx_h[(size_t)j * nc];
+            ctx->gu[j][1] = gy_h[(size_t)j * nc];
+            ctx->gu[j][2] = gz_h[(size_t)j * nc];
+        }
+    }
     ctx->nc = nc;
     ctx->ps = ps;
-    ctx->n_ghost = n_ghost;
     ctx->n_bcells = n_bcells;
     ctx->device = o->device;
-    ctx->n_iso = (int32_t)iso_col_h.size();
-    ctx->n_sym = (int32_t)sym_col_h.size();
+    ctx->n_iso = (int32_t)twall_h.size();
     ctx->n_refl = (int32_t)cls_of.size();
     ctx->W = 0.0;
     for (int d = 0; d < nd; ++d) ctx->W += dr->w[d];
@@ -791,7 +805,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         CREATE_CUDA(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
         ctx->own_stream = true;
     }
-    if (o->world > 1 && o->nccl_unique_id) {
+    if (o->nccl_unique_id) {  // (world == 1 with an id: a one-rank communicator, same code path)
         std::string e;
         if (!bte::nccl::init(&ctx->comm, o->nccl_unique_id, o->rank, o->world, &e)) {
             set_err(&ctx->err, "NCCL init failed: %s", e.c_str());
@@ -802,6 +816,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
 
     // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
+    ctx->tma = paired && ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);
     ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : (paired ? 8 : 2), paired);
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
@@ -837,25 +852,15 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     ctx->staging_elems = std::min<int64_t>((int64_t)nd * nc, std::max<int64_t>(nc, (int64_t)8 << 20));
     CREATE_TRY(dalloc(ctx, &ctx->staging, (size_t)ctx->staging_elems));
     CREATE_TRY(upload(ctx, &ctx->d_cur_slot, ctx->cur_slot));
-    CREATE_TRY(dalloc(ctx, &ctx->d_tmp_slot, (size_t)(nb_loc + n_spare)));
-    CREATE_TRY(dalloc(ctx, &ctx->d_band_ids, (size_t)(nb_loc + n_spare)));
     CREATE_TRY(upload(ctx, &ctx->nbr, nbr_h));
     CREATE_TRY(upload(ctx, &ctx->nbm, nbm_h));
-    CREATE_TRY(upload(ctx, &ctx->symc, symc_h));
-    if (paired) {  // sides beyond the cell's pairs stay "31" (none); keep only 10*dim bits
-        const uint32_t keep = m->dim == 2 ? 0xfffffu : 0x3fffffffu;
-        for (auto &v : symp_h) v &= keep;
-    }
-    CREATE_TRY(upload(ctx, &ctx->symp, symp_h));
+    CREATE_TRY(upload(ctx, &ctx->fcode, fcode_h));
+    CREATE_TRY(upload(ctx, &ctx->fcode8, fcode8_h));
     CREATE_TRY(upload(ctx, &ctx->gx, gx_h));
     CREATE_TRY(upload(ctx, &ctx->gy, gy_h));
     CREATE_TRY(upload(ctx, &ctx->gz, gz_h));
     CREATE_TRY(upload(ctx, &ctx->pos, pos_h));
     CREATE_TRY(upload(ctx, &ctx->refl, refl_h));
-    CREATE_TRY(upload(ctx, &ctx->iso_col, iso_col_h));
-    CREATE_TRY(upload(ctx, &ctx->sym_col, sym_col_h));
-    CREATE_TRY(upload(ctx, &ctx->sym_owner, sym_owner_h));
-    CREATE_TRY(upload(ctx, &ctx->sym_cls, sym_cls_h));
     CREATE_TRY(upload(ctx, &ctx->twall, twall_h));
     std::vector<double4> dirs_h(nd);
     for (int d = 0; d < nd; ++d) dirs_h[d] = make_double4(dr->s[3 * d], dr->s[3 * d + 1], dr->s[3 * d + 2], dr->w[d]);
@@ -875,7 +880,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_CUDA(cudaMemsetAsync(ctx->d_fail, 0, sizeof(int32_t), ctx->stream));
     CREATE_CUDA(cudaMemsetAsync(ctx->d_smax, 0, sizeof(unsigned long long), ctx->stream));
 
-    // --- initial state: T = t_init, I = I0_b(t_init); ghosts; dt bound
+    // --- initial state: T = t_init, I = I0_b(t_init); isothermal table; dt bound
     {
         std::vector<double> T0(nc, o->t_init);
         CREATE_CUDA(cudaMemcpy(ctx->T, T0.data(), nc * sizeof(double), cudaMemcpyHostToDevice));
@@ -884,17 +889,9 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         bte::i0_table_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->T, nc, b_lo, nb_loc, ctx->Cb, ctx->theta, ctx->i0);
         bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)nd * nc + tb - 1) / tb), nb_loc), tb, 0,
                                   ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ps, nd, nc, ctx->i0);
-        if (ctx->n_iso > 0) {
+        if (ctx->n_iso > 0)
             bte::i0w_kernel<<<(ctx->n_iso + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->twall, ctx->n_iso, b_lo, nb_loc,
                                                                                ctx->Cb, ctx->theta, ctx->i0w);
-            // every slab that will hold a band's state gets that band's isothermal ghosts
-            std::vector<int32_t> sl, bl;
-            for (int k = 0; k < nb_loc; ++k) sl.push_back(ctx->cur_slot[k]), bl.push_back(k);
-            if (n_spare == nb_loc)
-                for (int k = 0; k < nb_loc; ++k) sl.push_back(ctx->spare_slot[k]), bl.push_back(k);
-            CREATE_TRY(fill_iso_ghosts(ctx, sl, bl));
-        }
-        CREATE_TRY(fill_sym_ghosts(ctx));
         if (m->dim == 2)
             bte::outflow_max_kernel<2><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, paired, nd, ctx->gx, ctx->gy, ctx->gz,
                                                                   ctx->dirs, ctx->d_smax);
@@ -953,7 +950,7 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int64_t s = 0; s < n; ++s) {
         STATUS_TRY(run_flux(ctx, dt));
-        if (ctx->opt.world > 1) {
+        if (ctx->have_comm) {
             ev_mark(ctx, kPhAllreduce, true);
             STATUS_TRY(reduce_slots(ctx));
             STATUS_TRY(allreduce_E(ctx));
@@ -1076,7 +1073,6 @@ bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const dou
         double *slab = ctx->pool + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
         STATUS_TRY(rows_from_host(ctx, I + (int64_t)(b - b_lo) * ctx->nd * ctx->nc, ctx->ps, ctx->nd, slab));
     }
-    STATUS_TRY(fill_sym_ghosts(ctx));  // specular ghosts follow the new state
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     return BTE_OK;
 }
@@ -1112,7 +1108,6 @@ bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
                               tb, 0, ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nd,
                                                     ctx->nc, ctx->i0);
     CUDA_TRY(ctx, cudaGetLastError());
-    STATUS_TRY(fill_sym_ghosts(ctx));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     return BTE_OK;
 }

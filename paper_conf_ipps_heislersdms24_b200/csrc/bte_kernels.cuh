@@ -27,39 +27,56 @@ namespace bte {
 
 constexpr int kMaxBandsPerLaunch = 128;
 constexpr int kMaxThreads = 256;
+#ifndef BTE_MIN_BLOCKS
+#define BTE_MIN_BLOCKS 2  // resident 256-thread blocks per SM the flux kernels are compiled for
+#endif
 
 enum : int8_t { kFaceInterior = 0, kFaceIso = 1, kFaceSym = 2 };
 
 struct FluxParams {
     int32_t nc;          // cells
-    int32_t ps;          // plane stride: nc cells + ghost columns (boundary faces), padded
+    int32_t ps;          // plane stride (nc padded to 32)
     int32_t nd;          // directions
     int32_t dchunk;      // directions per block
     int32_t n_dchunks;
     int32_t nbl;         // band-rows in this launch (a multiple of the template BG)
     int32_t band0;       // rank-local index of the launch's first band-row
     int32_t slot0;       // first energy-partial slot of this launch
-    int64_t slab_elems;  // nd * ps
-    double *pool;        // slab pool
     const double *i0;    // [nb_loc][nc]  I0_b(T_c) of the current step
     double *part;        // [n_slots][nc] energy partials
     // Face slots, struct-of-arrays [slot][nc].  Generic: one slot per face.
-    // Paired: one slot per opposite face pair; nbr/symc describe the "+" face
-    // (the one whose normal g is stored), nbm the "-" face (g_- = -g_+).
-    // nbr >= nc addresses the face's ghost column in the same plane.
+    // Paired: one slot per opposite face pair; nbr describes the "+" face (the
+    // one whose g is stored), nbm the "-" face (g_- = -g_+).  For a boundary
+    // face nbr holds its isothermal-table column (isothermal) or is unused
+    // (specular); the face kind is in fcode.
     const int32_t *nbr, *nbm;
     const double *gx, *gy, *gz;  // g = (A_f / V_c) n_f
-    const int32_t *symc;         // generic [MF][nc]: reflection class of a specular face, -1 otherwise
-    const uint32_t *symp;        // paired [nc]: 5-bit reflection class per side (pair q: bits 10q / 10q+5), 31 = none
-    const int32_t *refl;         // [n_classes][nd] reflected direction
+    double gu[3][3];             // uniform-geometry meshes: g of pair q (same for every cell)
+    const uint32_t *fcode;       // paired [nc]: 5-bit code per side (pair q: bits 10q "+", 10q+5 "-")
+    const uint8_t *fcode8;       // generic [MF][nc]: code per face
+    const int32_t *refl;         // [n_classes][nd] reflected direction of a specular class
+    const double *i0w;           // [nb_loc][n_iso]  I0_b(T_wall) per isothermal face
+    int32_t n_iso;
     const double4 *dirs;         // [nd] {s_x, s_y, s_z, w}
     double dt;
     const double *in_ptr[kMaxBandsPerLaunch];  // per launch-local band-row: input slab (I^n)
     double *out_ptr[kMaxBandsPerLaunch];       // ... output slab (I^{n+1})
-    double dtit[kMaxBandsPerLaunch];       // dt / tau_b
-    double kv[kMaxBandsPerLaunch];         // dt v_b
-    double cw[kMaxBandsPerLaunch];         // temperature weight c_b
+    double dtit[kMaxBandsPerLaunch];           // dt / tau_b
+    double kv[kMaxBandsPerLaunch];             // dt v_b
+    double cw[kMaxBandsPerLaunch];             // temperature weight c_b
 };
+
+// L2 eviction-priority policies (createpolicy) for the streamed intensity planes.
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ double ldg_hint(const double *ptr, uint64_t pol) {
+    double v;
+    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(ptr), "l"(pol));
+    return v;
+}
 
 __device__ __forceinline__ double4 load_dir(const double4 *dirs, int d) {
     const double2 a = __ldg(reinterpret_cast<const double2 *>(dirs + d));
@@ -67,27 +84,33 @@ __device__ __forceinline__ double4 load_dir(const double4 *dirs, int d) {
     return make_double4(a.x, a.y, b.x, b.y);
 }
 
-// Boundary faces are ghost columns of every (b, d) plane (Eq. 6:
-// "setting the intensity of ghost cells on the outside"):
-//   isothermal face: ghost = I0_b(T_wall), constant in time, written at set-up;
-//   specular face f of cell c: ghost[b][d] = I^n[b][r_f(d)][c].  It is written
-//   by the step that produces I^n: when a thread computes I'[b][d][c] it also
-//   stores it to ghost column f of direction r_f(d) of the output slab (r_f is
-//   an involution), so the flux loop never branches on the face kind.  The
-//   reflected directions of an iteration are fetched with its other loads.
-constexpr uint32_t kNoClass = 31;
+// Face codes (Eq. 6: the upwind value entering through a face):
+//   kCodeInterior  I^n[b][d][nbr]            (same plane)
+//   kCodeIso       I0_b(T_wall) = I0w[b][nbr] (isothermal table column)
+//   0..15          specular class k: I^n[b][r_k(d)][c] (reflected direction,
+//                  same cell, old level) = same plane + (r_k(d) - d) * ps + c - c
+// Paired layout: 5-bit codes; generic layout: 8-bit codes.
+constexpr uint32_t kCodeInterior = 31;
+constexpr uint32_t kCodeIso = 16;
+constexpr int kMaxPairedClasses = 16;
+constexpr uint32_t kCode8Interior = 255;
+constexpr uint32_t kCode8Iso = 254;
+constexpr int kMaxGenericClasses = 254;
 
 // ---------------------------------------------------------------------------
-// Generic connectivity: up to MF faces per cell, each with its own neighbour.
 // One thread owns one cell and a (band group, direction chunk) of its
-// unknowns.  Per direction it forms alpha_j = s_d . g_j once for the BG
-// band-rows, issues every load of the iteration (own value and the inflow
-// faces' upwind values of all BG rows) before using any, then writes
+// unknowns.  Per direction it forms alpha_j = s_d . g_j (g_j = A_j/V n_j) once
+// for the BG band-rows, issues every load of the iteration (own value and the
+// inflow faces' upwind values of all BG rows) before using any, then writes
 //   I' = I (1 - dt/tau - dt v out) + (dt/tau) I0 - dt v sum_{alpha<0} alpha I_up
 // (Eq. 3/5, L269-292, L546-553; upwind L264-267) with a streaming store and
-// accumulates c_b w_d I' for the energy partial (L412-418).
+// accumulates c_b w_d I' for the energy partial (L412-418).  Cells with a
+// boundary face (has_bnd) take the face-kind path; for the others it is a
+// warp-uniform skip.
+//
+// Generic connectivity: up to MF faces per cell, each with its own neighbour.
 template <int DIM, int MF, int BG>
-__global__ void __launch_bounds__(kMaxThreads, 2)
+__global__ void __launch_bounds__(kMaxThreads, BTE_MIN_BLOCKS)
 flux_kernel(const __grid_constant__ FluxParams p) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= p.nc) return;
@@ -97,45 +120,58 @@ flux_kernel(const __grid_constant__ FluxParams p) {
     const int d0 = dch * p.dchunk;
     const int d1 = min(p.nd, d0 + p.dchunk);
     const int nc = p.nc;
+    const int ps = p.ps;
 
-    int nbr[MF], cls[MF];
+    int nbr[MF];
+    uint32_t code[MF];
     double gx[MF], gy[MF], gz[MF];
-    bool has_sym = false;
+    bool has_bnd = false;
 #pragma unroll
     for (int j = 0; j < MF; ++j) {
-        const size_t q = (size_t)j * nc + c;
+        const int q = j * nc + c;
         nbr[j] = __ldg(p.nbr + q);
         gx[j] = __ldg(p.gx + q);
         gy[j] = __ldg(p.gy + q);
         gz[j] = DIM == 3 ? __ldg(p.gz + q) : 0.0;
-        cls[j] = __ldg(p.symc + q);
-        has_sym |= cls[j] >= 0;
+        code[j] = __ldg(p.fcode8 + q);
+        has_bnd |= code[j] != kCode8Interior;
     }
     double src[BG];
 #pragma unroll
     for (int k = 0; k < BG; ++k)  // dt/tau I0_b(T_c)
-        src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (size_t)(p.band0 + lg0 + k) * nc + c);
+        src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c);
     double e = 0.0;
     for (int d = d0; d < d1; ++d) {
         const double4 sd = load_dir(p.dirs, d);
         double a[MF];
+        int idx[MF];
         double out = 0.0;
 #pragma unroll
         for (int j = 0; j < MF; ++j) {
             a[j] = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
             out += fmax(a[j], 0.0);  // outflow faces carry the cell's own value
+            idx[j] = nbr[j];
         }
-        const size_t po = (size_t)d * p.ps;
-        int rr[MF];
+        if (has_bnd) {
 #pragma unroll
-        for (int j = 0; j < MF; ++j) rr[j] = (has_sym && cls[j] >= 0) ? __ldg(p.refl + (size_t)cls[j] * p.nd + d) : 0;
+            for (int j = 0; j < MF; ++j)
+                if (code[j] < kCode8Iso) idx[j] = (__ldg(p.refl + code[j] * p.nd + d) - d) * ps + c;
+        }
+        const int64_t po = (int64_t)d * ps;
         double ic[BG], nv[BG][MF];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {  // every load of the iteration first
             const double *pl = p.in_ptr[lg0 + k] + po;
             ic[k] = __ldg(pl + c);
+            if (!has_bnd) {
 #pragma unroll
-            for (int j = 0; j < MF; ++j) nv[k][j] = a[j] < 0.0 ? __ldg(pl + nbr[j]) : 0.0;
+                for (int j = 0; j < MF; ++j) nv[k][j] = a[j] < 0.0 ? __ldg(pl + idx[j]) : 0.0;
+            } else {
+                const double *iso = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
+#pragma unroll
+                for (int j = 0; j < MF; ++j)
+                    nv[k][j] = a[j] < 0.0 ? __ldg((code[j] == kCode8Iso ? iso : pl) + idx[j]) : 0.0;
+            }
         }
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
@@ -144,17 +180,11 @@ flux_kernel(const __grid_constant__ FluxParams p) {
             for (int j = 0; j < MF; ++j) infl = fma(fmin(a[j], 0.0), nv[k][j], infl);
             const double kv = p.kv[lg0 + k];
             const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
-            double *ob = p.out_ptr[lg0 + k];
-            __stcs(ob + po + c, inew);
-            if (has_sym) {
-#pragma unroll
-                for (int j = 0; j < MF; ++j)
-                    if (cls[j] >= 0) __stcs(ob + (size_t)rr[j] * p.ps + nbr[j], inew);
-            }
+            __stcs(p.out_ptr[lg0 + k] + po + c, inew);
             e = fma(p.cw[lg0 + k] * sd.w, inew, e);
         }
     }
-    p.part[(size_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
+    p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
 }
 
 // ---------------------------------------------------------------------------
@@ -162,8 +192,10 @@ flux_kernel(const __grid_constant__ FluxParams p) {
 // as in the paper's uniform quad/hex grids): for each pair only the face with
 // s_d . g < 0 is an inflow, so one upwind load and one FMA per pair, and
 // out = sum_pairs |s_d . g_+|.  Same arithmetic as the generic kernel.
-template <int DIM, int NP, int BG>
-__global__ void __launch_bounds__(kMaxThreads, 2)
+// UG (uniform geometry, e.g. the paper's uniform grids): every cell has the
+// same g per pair, read from the constant bank instead of per-thread registers.
+template <int DIM, int NP, int BG, bool UG>
+__global__ void __launch_bounds__(kMaxThreads, BTE_MIN_BLOCKS)
 flux_paired_kernel(const __grid_constant__ FluxParams p) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= p.nc) return;
@@ -182,13 +214,18 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
         const int o = q * nc + c;
         np_[q] = __ldg(p.nbr + o);
         nm_[q] = __ldg(p.nbm + o);
-        gx[q] = __ldg(p.gx + o);
-        gy[q] = __ldg(p.gy + o);
-        gz[q] = DIM == 3 ? __ldg(p.gz + o) : 0.0;
+        if (!UG) {
+            gx[q] = __ldg(p.gx + o);
+            gy[q] = __ldg(p.gy + o);
+            gz[q] = DIM == 3 ? __ldg(p.gz + o) : 0.0;
+        }
     }
-    const uint32_t symp = __ldg(p.symp + c);
-    constexpr uint32_t kNone = (1u << (10 * NP)) - 1u;  // every side "31"
-    const bool has_sym = symp != kNone;
+    const uint32_t codes = __ldg(p.fcode + c);
+#ifdef BTE_EXP_KEEP
+    const uint64_t pol = l2_policy_evict_last();
+#endif
+    constexpr uint32_t kAllInterior = (1u << (10 * NP)) - 1u;
+    const bool has_bnd = codes != kAllInterior;
     double src[BG];  // dt/tau I0_b(T_c) per band-row of the group
 #pragma unroll
     for (int k = 0; k < BG; ++k) src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c);
@@ -196,32 +233,46 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
     for (int d = d0; d < d1; ++d) {
         const double4 sd = load_dir(p.dirs, d);
         double amin[NP];  // -|s.g|: alpha of the pair's inflow face
-        int ni[NP];
+        int idx[NP];
+        bool iso[NP];
         double out = 0.0;
 #pragma unroll
         for (int q = 0; q < NP; ++q) {
-            const double a = DIM == 3 ? fma(sd.z, gz[q], fma(sd.y, gy[q], sd.x * gx[q])) : fma(sd.y, gy[q], sd.x * gx[q]);
+            const double ggx = UG ? p.gu[q][0] : gx[q], ggy = UG ? p.gu[q][1] : gy[q];
+            const double ggz = UG ? p.gu[q][2] : gz[q];
+            const double a = DIM == 3 ? fma(sd.z, ggz, fma(sd.y, ggy, sd.x * ggx)) : fma(sd.y, ggy, sd.x * ggx);
             out += fabs(a);
             amin[q] = -fabs(a);
-            ni[q] = a > 0.0 ? nm_[q] : np_[q];  // "+" face outgoing -> inflow through "-"
-        }
-        const int64_t po = (int64_t)d * ps;
-        int gofs[2 * NP];  // specular sides: plane offset of ghost column f in direction r_f(d)
-        if (has_sym) {
-#pragma unroll
-            for (int s = 0; s < 2 * NP; ++s) {
-                const uint32_t cl = (symp >> (5 * s)) & kNoClass;
-                const int col = (s & 1) ? nm_[s >> 1] : np_[s >> 1];
-                gofs[s] = cl != kNoClass ? __ldg(p.refl + cl * p.nd + d) * ps + col : -1;
+            idx[q] = a > 0.0 ? nm_[q] : np_[q];  // "+" face outgoing -> inflow through "-"
+            iso[q] = false;
+            if (has_bnd) {
+                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
+                iso[q] = cd == kCodeIso;
+                if (cd < kCodeIso) idx[q] = (__ldg(p.refl + cd * p.nd + d) - d) * ps + c;
             }
         }
+        const int64_t po = (int64_t)d * ps;
         double ic[BG], nv[BG][NP];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {  // every load of the iteration first
             const double *pl = p.in_ptr[lg0 + k] + po;  // slab bases come from the constant bank
+#ifdef BTE_EXP_KEEP
+            ic[k] = ldg_hint(pl + c, pol);
+#else
             ic[k] = __ldg(pl + c);
+#endif
+            if (!has_bnd) {
 #pragma unroll
-            for (int q = 0; q < NP; ++q) nv[k][q] = __ldg(pl + ni[q]);
+#ifdef BTE_EXP_NO_NBR
+                for (int q = 0; q < NP; ++q) nv[k][q] = ic[k];
+#else
+                for (int q = 0; q < NP; ++q) nv[k][q] = __ldg(pl + idx[q]);
+#endif
+            } else {
+                const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
+#pragma unroll
+                for (int q = 0; q < NP; ++q) nv[k][q] = __ldg((iso[q] ? isot : pl) + idx[q]);
+            }
         }
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
@@ -230,50 +281,174 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
             for (int q = 0; q < NP; ++q) infl = fma(amin[q], nv[k][q], infl);
             const double kv = p.kv[lg0 + k];
             const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
-            double *ob = p.out_ptr[lg0 + k];
-            __stcs(ob + po + c, inew);
-            if (has_sym) {
-#pragma unroll
-                for (int s = 0; s < 2 * NP; ++s)
-                    if (gofs[s] >= 0) __stcs(ob + gofs[s], inew);
-            }
+            __stcs(p.out_ptr[lg0 + k] + po + c, inew);
             e = fma(p.cw[lg0 + k] * sd.w, inew, e);
         }
     }
     p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
 }
 
-// ---------------------------------------------------------------- ghost set-up
-// Isothermal ghosts of band-row b in slab s: ghost[d][col] = I0_b(T_wall).
-__global__ void iso_ghost_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,
-                                 const int32_t *__restrict__ band_of_slot_entry, int64_t slab_elems, int ps,
-                                 int nd, int n_iso, const int32_t *__restrict__ iso_col /* plane index */,
-                                 const double *__restrict__ i0w) {
-    const int k = blockIdx.y;  // entry: slab slot[k] holds local band-row band_of_slot_entry[k]
-    double *s = pool + (int64_t)slot[k] * slab_elems;
-    const int b = band_of_slot_entry[k];
-    const int64_t n = (int64_t)nd * n_iso;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        const int d = (int)(e / n_iso);
-        const int f = (int)(e - (int64_t)d * n_iso);
-        s[(size_t)d * ps + iso_col[f]] = i0w[(size_t)b * n_iso + f];
-    }
+// ---------------------------------------------------------------------------
+// TMA-staged paired kernel (sm_100a bulk-copy engine + mbarriers).
+//
+// A block is one tile of kTile = 256 consecutive cells (with the Morton hint:
+// an 8x8x4 brick).  For every (band-row, direction) plane the tile's own
+// values are one contiguous 2 KB segment, so one elected thread streams them
+// into a kStages-deep shared-memory ring with cp.async.bulk (completion counted
+// on an mbarrier), kStages iterations ahead of the compute.  Upwind neighbours
+// inside the tile are read from the staged segment; only halo neighbours,
+// specular faces (another direction's plane) and isothermal faces (the I0w
+// table) are global loads, issued at the top of the iteration.  Arithmetic is
+// identical to flux_paired_kernel.
+constexpr int kTile = 256;
+constexpr int kStages = 4;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *ptr) {
+    return (uint32_t)__cvta_generic_to_shared(ptr);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t phase) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(phase)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
 }
 
-// Specular ghosts of the current state: ghost[b][d][col_f] = I[b][r_f(d)][owner_f].
-__global__ void sym_ghost_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot, int64_t slab_elems,
-                                 int ps, int nd, int n_sym, const int32_t *__restrict__ sym_col /* plane index */,
-                                 const int32_t *__restrict__ sym_owner, const int32_t *__restrict__ sym_cls,
-                                 const int32_t *__restrict__ refl) {
-    const int k = blockIdx.y;
-    double *s = pool + (int64_t)slot[k] * slab_elems;
-    const int64_t n = (int64_t)nd * n_sym;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        const int d = (int)(e / n_sym);
-        const int f = (int)(e - (int64_t)d * n_sym);
-        const int r = refl[(size_t)sym_cls[f] * nd + d];
-        s[(size_t)d * ps + sym_col[f]] = s[(size_t)r * ps + sym_owner[f]];
+template <int DIM, int NP, int BG, bool UG>
+__global__ void __launch_bounds__(kTile, BTE_MIN_BLOCKS)
+flux_tma_kernel(const __grid_constant__ FluxParams p) {
+    extern __shared__ __align__(128) double ring[];  // [kStages][BG][kTile]
+    __shared__ __align__(8) uint64_t full[kStages];
+    const int tid = threadIdx.x;
+    const int tile0 = blockIdx.x * kTile;
+    const int c = tile0 + tid;
+    const bool valid = c < p.nc;
+    const int grp = blockIdx.y / p.n_dchunks;
+    const int dch = blockIdx.y - grp * p.n_dchunks;
+    const int lg0 = grp * BG;
+    const int d0 = dch * p.dchunk;
+    const int nit = min(p.nd, d0 + p.dchunk) - d0;
+    const int nc = p.nc;
+    const int ps = p.ps;
+    constexpr uint32_t kBytes = BG * kTile * sizeof(double);
+
+    if (tid == 0) {
+#pragma unroll
+        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    __syncthreads();
+    auto issue = [&](int i) {  // stage i % kStages <- planes (band-rows of the group, direction d0 + i)
+        uint64_t *bar = &full[i % kStages];
+        mbar_arrive_expect_tx(bar, kBytes);
+        const int64_t off = (int64_t)(d0 + i) * ps + tile0;
+#pragma unroll
+        for (int k = 0; k < BG; ++k)
+            bulk_g2s(ring + ((i % kStages) * BG + k) * kTile, p.in_ptr[lg0 + k] + off, kTile * sizeof(double), bar);
+    };
+    if (tid == 0)
+        for (int i = 0; i < min(kStages, nit); ++i) issue(i);
+
+    int np_[NP], nm_[NP];
+    double gx[NP], gy[NP], gz[NP];
+    uint32_t codes = (1u << (10 * NP)) - 1u;
+    double src[BG];
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+        const int o = q * nc + c;
+        np_[q] = valid ? __ldg(p.nbr + o) : c;
+        nm_[q] = valid ? __ldg(p.nbm + o) : c;
+        if (!UG) {
+            gx[q] = valid ? __ldg(p.gx + o) : 0.0;
+            gy[q] = valid ? __ldg(p.gy + o) : 0.0;
+            gz[q] = (DIM == 3 && valid) ? __ldg(p.gz + o) : 0.0;
+        }
+    }
+    if (valid) codes = __ldg(p.fcode + c);
+    const bool has_bnd = codes != (1u << (10 * NP)) - 1u;
+#pragma unroll
+    for (int k = 0; k < BG; ++k)
+        src[k] = valid ? p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c) : 0.0;
+
+    double e = 0.0;
+    for (int i = 0; i < nit; ++i) {
+        const int d = d0 + i;
+        const double4 sd = load_dir(p.dirs, d);
+        double amin[NP];
+        int idx[NP];
+        bool glob[NP], iso[NP];
+        double out = 0.0;
+#pragma unroll
+        for (int q = 0; q < NP; ++q) {
+            const double ggx = UG ? p.gu[q][0] : gx[q], ggy = UG ? p.gu[q][1] : gy[q];
+            const double ggz = UG ? p.gu[q][2] : gz[q];
+            const double a = DIM == 3 ? fma(sd.z, ggz, fma(sd.y, ggy, sd.x * ggx)) : fma(sd.y, ggy, sd.x * ggx);
+            out += fabs(a);
+            amin[q] = -fabs(a);
+            idx[q] = a > 0.0 ? nm_[q] : np_[q];
+            iso[q] = false;
+            if (has_bnd) {
+                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
+                iso[q] = cd == kCodeIso;
+                if (cd < kCodeIso) idx[q] = (__ldg(p.refl + cd * p.nd + d) - d) * ps + c;
+            }
+            glob[q] = iso[q] || (unsigned)(idx[q] - tile0) >= (unsigned)kTile;
+        }
+        // halo / boundary values: global loads first (overlap the stage wait)
+        const int64_t po = (int64_t)d * ps;
+        double nv[BG][NP];
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            const double *pl = p.in_ptr[lg0 + k] + po;
+            const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
+#pragma unroll
+            for (int q = 0; q < NP; ++q)
+                nv[k][q] = (valid && glob[q]) ? __ldg((iso[q] ? isot : pl) + idx[q]) : 0.0;
+        }
+        const int st = i % kStages;
+        while (!mbar_try_wait(&full[st], (i / kStages) & 1)) {
+        }
+        const double *stage = ring + st * BG * kTile;
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            const double *sk = stage + k * kTile;
+            const double ic = sk[tid];
+            double infl = 0.0;
+#pragma unroll
+            for (int q = 0; q < NP; ++q) {
+                const double v = glob[q] ? nv[k][q] : sk[idx[q] - tile0];
+                infl = fma(amin[q], v, infl);
+            }
+            const double kv = p.kv[lg0 + k];
+            const double inew = fma(ic, (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
+            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew);
+            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
+        }
+        __syncthreads();  // every thread is done with stage st
+        if (tid == 0 && i + kStages < nit) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            issue(i + kStages);
+        }
+    }
+    if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
 }
 
 // ---------------------------------------------------------------- temperature

@@ -178,6 +178,34 @@ def test_generic_face_path_2d_3d(bte, oracle_mod, bg):
     assert_parity(Ig, Tg, Io, To)
 
 
+@pytest.mark.parametrize("bg", [1, 3, 4, 8])
+def test_register_pipelined_kernel(bte, oracle_mod, bg):
+    """The non-TMA paired kernel (BTE_FLAG_NO_TMA), uniform and per-cell geometry."""
+    cfg = gen.small_3d_config((13, 7, 5), n_spectral=3, ntheta=4, nphi=8)
+    Io, To = oracle_run(oracle_mod, cfg, 10)
+    Ig, Tg, _ = gpu_run(cfg, 10, tma=False, band_group=bg)
+    assert_parity(Ig, Tg, Io, To)
+    c2 = _cfg("C2", steps=10)
+    Io, To = oracle_run(oracle_mod, c2, 10)
+    Ig, Tg, _ = gpu_run(c2, 10, tma=False, band_group=bg)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_graded_mesh_per_cell_geometry(bte, oracle_mod):
+    """Non-uniform (graded) cell sizes: paired but not uniform geometry, on the
+    TMA kernel and the register kernel."""
+    cfg = gen.small_3d_config((9, 8, 5), n_spectral=2)
+    m = dict(cfg.mesh)
+    scale = np.repeat(1.0 + 0.5 * (np.arange(m["n_cells"]) % 3), 6)
+    m["face_area"] = m["face_area"] * scale
+    m["cell_volume"] = m["cell_volume"] * (1.0 + 0.5 * (np.arange(m["n_cells"]) % 3)) * 1.7
+    cfg = dataclasses.replace(cfg, mesh=m, dt=0.25 * cfg.dt)
+    Io, To = oracle_run(oracle_mod, cfg, 10)
+    for tma in (True, False):
+        Ig, Tg, _ = gpu_run(cfg, 10, tma=tma)
+        assert_parity(Ig, Tg, Io, To)
+
+
 def test_locality_order_is_invisible(bte):
     """The Morton-order hint changes only the internal layout: bitwise equal."""
     cfg = gen.small_3d_config((11, 6, 5), n_spectral=3)
@@ -283,6 +311,16 @@ def test_split_step_band_sharding_emulated(bte, oracle_mod):
         for s in ranks:
             s.close()
     assert_parity(Ig, Ts[0], Io, To)
+
+
+def test_nccl_allreduce_path_one_rank(bte):
+    """The NCCL code path (dlopen, ncclCommInitRank, per-step ncclAllReduce of E)
+    on a one-rank communicator: bitwise equal to the fused single-GPU path."""
+    cfg = _cfg("C2", steps=5)
+    a = gpu_run(cfg, 5)
+    b = gpu_run(cfg, 5, nccl_id=bte.nccl_unique_id(), profile=True)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    assert b[2]["ms_allreduce"] > 0.0
 
 
 def test_profile_stats(bte):

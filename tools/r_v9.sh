@@ -1,0 +1,8 @@
+cd $GRAFT_REPO_ROOT
+OUT=gpurun_out/v9; mkdir -p $OUT
+timeout 900 python -m pytest tests -m gpu -q -x --timeout 600 > $OUT/pytest_gpu.log 2>&1; tail -3 $OUT/pytest_gpu.log
+L=paper_conf_ipps_heislersdms24_b200/libbte.so
+bash tools/gpu_libsweep.sh v9 $L "--band-group 4 --dir-chunk 40" "--band-group 6 --dir-chunk 40" "--band-group 8 --dir-chunk 40" "--band-group 8 --dir-chunk 100"
+bash tools/gpu_libsweep.sh v9 build_exp/libbte_mb3.so "--band-group 2 --dir-chunk 40" "--band-group 3 --dir-chunk 40" "--band-group 4 --dir-chunk 40" "--band-group 4 --dir-chunk 100" "--band-group 4 --dir-chunk 40 --no-tma"
+bash tools/gpu_libsweep.sh v9 build_exp/libbte_mb4.so "--band-group 2 --dir-chunk 40" "--band-group 3 --dir-chunk 40"
+cat $OUT/sweep.txt
