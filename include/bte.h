@@ -157,6 +157,9 @@ typedef struct {
     int32_t band_group;
     int32_t block_threads;
     int32_t dir_chunks;        /* direction chunks per launch (grid.y factor) */
+    int32_t flux_variant;      /* flux kernel in use: 0 generic faces, 1 paired, 2 paired +
+                                  uniform geometry, 3 TMA-staged, 4 TMA-staged + uniform
+                                  geometry, 5 stencil-staged (structured order) */
 } bte_stats;
 
 /* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,

@@ -67,11 +67,13 @@ class Stats(C.Structure):
                 ("ms_allreduce", C.c_double), ("ms_newton", C.c_double), ("ms_total", C.c_double),
                 ("newton_iter_max", C.c_int32), ("spare_slabs", C.c_int32),
                 ("n_interior_cells", C.c_int32), ("band_group", C.c_int32),
-                ("block_threads", C.c_int32), ("dir_chunks", C.c_int32)]
+                ("block_threads", C.c_int32), ("dir_chunks", C.c_int32), ("flux_variant", C.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
+
+FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil"}
 
 EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte_get_temperature",
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",

@@ -71,6 +71,8 @@ struct bte_ctx {
     bool paired = false;     // every cell's faces are exact opposite pairs
     bool uniform_g = false;  // ... and every cell has the same g per pair
     bool tma = false;        // paired + 256-thread blocks: the TMA-staged kernel
+    bool stencil = false;    // ... + constant neighbour offsets: the stencil-staged kernel
+    int32_t so[3] = {0, 0, 0}, halo = 0, wmain = 0, nfar = 0, farq[3] = {0, 0, 0};
     double gu[3][3] = {};
     // boundary faces: reflection maps of specular classes, isothermal table
     int32_t *refl = nullptr;
@@ -152,6 +154,33 @@ void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p)
     bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTile), smem, s>>>(p);
 }
 
+// Stencil-staged kernel (structured meshes): near + far windows per plane.
+template <int DIM, int NP, int BG>
+void flux_stencil_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    const size_t smem = (size_t)bte::kStages * BG * (p.wmain + p.nfar * bte::kFarWin) * sizeof(double);
+    static size_t attr = 0;
+    if (attr < smem) {
+        cudaFuncSetAttribute(bte::flux_stencil_kernel<DIM, NP, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smem);
+        attr = smem;
+    }
+    bte::flux_stencil_kernel<DIM, NP, BG><<<g, dim3(bte::kTile), smem, s>>>(p);
+}
+
+template <int DIM, int NP>
+FluxLaunch pick_stencil(int bg) {
+    switch (bg) {
+        case 1: return flux_stencil_launch_t<DIM, NP, 1>;
+        case 2: return flux_stencil_launch_t<DIM, NP, 2>;
+        case 3: return flux_stencil_launch_t<DIM, NP, 3>;
+        case 4: return flux_stencil_launch_t<DIM, NP, 4>;
+        case 5: return flux_stencil_launch_t<DIM, NP, 5>;
+        case 6: return flux_stencil_launch_t<DIM, NP, 6>;
+        case 7: return flux_stencil_launch_t<DIM, NP, 7>;
+        default: return flux_stencil_launch_t<DIM, NP, 8>;
+    }
+}
+
 template <int DIM, int NP, bool UG>
 FluxLaunch pick_tma(int bg) {
     switch (bg) {
@@ -192,7 +221,8 @@ FluxLaunch pick_generic(int bg) {
 }
 
 // mf_t: padded faces per cell (generic) or face pairs per cell (paired)
-FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, bool tma) {
+FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, bool tma, bool stencil) {
+    if (stencil) return dim == 2 ? pick_stencil<2, 2>(bg) : pick_stencil<3, 3>(bg);
     if (paired && tma) {
         if (uniform_g) return dim == 2 ? pick_tma<2, 2, true>(bg) : pick_tma<3, 3, true>(bg);
         return dim == 2 ? pick_tma<2, 2, false>(bg) : pick_tma<3, 3, false>(bg);
@@ -271,7 +301,11 @@ std::vector<Segment> segments(int nbl, int bg, bool paired) {
     return out;
 }
 
-// Direction chunks so the grid holds ~2 full waves of threads.
+// Direction chunks: at most kAutoDirChunk directions per block (short blocks
+// keep the tiles that share halo data resident at the same time, so upwind
+// reads hit L2; measured best on B200) and enough chunks for the
+// grid to hold ~2 full waves of threads.
+constexpr int kAutoDirChunk = 40;
 LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int bg) {
     LaunchPlan lp;
     lp.groups = nbl / bg;
@@ -279,7 +313,7 @@ LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int bg) {
     const int64_t have = std::max<int64_t>(1, (int64_t)ctx->nc * lp.groups);
     const int n = (int)std::min<int64_t>(ctx->nd, std::max<int64_t>(1, (target + have - 1) / have));
     lp.dchunk = (ctx->nd + n - 1) / n;
-    if (ctx->opt.dir_chunk > 0) lp.dchunk = std::min(lp.dchunk, (int)ctx->opt.dir_chunk);
+    lp.dchunk = std::min(lp.dchunk, ctx->opt.dir_chunk > 0 ? (int)ctx->opt.dir_chunk : kAutoDirChunk);
     lp.n_dch = (ctx->nd + lp.dchunk - 1) / lp.dchunk;
     return lp;
 }
@@ -311,6 +345,11 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.gy = ctx->gy;
     p.gz = ctx->gz;
     std::memcpy(p.gu, ctx->gu, sizeof p.gu);
+    std::memcpy(p.so, ctx->so, sizeof p.so);
+    std::memcpy(p.farq, ctx->farq, sizeof p.farq);
+    p.halo = ctx->halo;
+    p.wmain = ctx->wmain;
+    p.nfar = ctx->nfar;
     p.fcode = ctx->fcode;
     p.fcode8 = ctx->fcode8;
     p.i0w = ctx->i0w;
@@ -323,7 +362,8 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
         const int nbl_batch = std::min(ctx->n_spare, ctx->nb_loc - l0);
         for (const Segment &sg : segments(nbl_batch, ctx->bg, ctx->paired)) {
-            const FluxLaunch fn = pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma);
+            const FluxLaunch fn =
+                pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma, ctx->stencil);
             const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
             p.nbl = sg.nbl;
             p.band0 = l0 + sg.off;
@@ -577,12 +617,58 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     if (nb_loc > bte::kMaxBandsPerLaunch)
         return set_err(nullptr, "%d band-rows on one rank (max %d)", nb_loc, bte::kMaxBandsPerLaunch), BTE_EINVAL;
 
+    // --- face pairing: every face of every cell has an exactly opposite partner
+    // (same area, negated normal) -> paired layout, one upwind load per pair.
+    int mf = 0;
+    for (int64_t c = 0; c < nc64; ++c) mf = std::max<int>(mf, (int)(m->face_offsets[c + 1] - m->face_offsets[c]));
+    std::vector<int64_t> partner(m->face_offsets[nc64], -1);
+    bool paired_geom = mf <= 2 * m->dim && !(o->flags & BTE_FLAG_GENERIC_FACES);
+    for (int64_t c = 0; c < nc64 && paired_geom; ++c) {
+        const int64_t f0 = m->face_offsets[c], f1 = m->face_offsets[c + 1];
+        for (int64_t f = f0; f < f1 && paired_geom; ++f) {
+            if (partner[f] >= 0) continue;
+            const double *n = m->face_normal + 3 * f;
+            for (int64_t g = f + 1; g < f1; ++g) {
+                const double *q = m->face_normal + 3 * g;
+                if (partner[g] < 0 && m->face_area[g] == m->face_area[f] && q[0] == -n[0] && q[1] == -n[1] &&
+                    q[2] == -n[2]) {
+                    partner[f] = g;
+                    partner[g] = f;
+                    break;
+                }
+            }
+            if (partner[f] < 0) paired_geom = false;
+        }
+    }
+    // --- stencil: every cell has dim pairs, and pair j of every cell neighbours
+    // c + so[j] ("+") and c - so[j] ("-") in the caller's order (structured grids)
+    int32_t so[3] = {0, 0, 0};
+    bool stencil_order = paired_geom && mf == 2 * m->dim && nc64 >= 2 * bte::kTile;
+    for (int64_t c = 0; c < nc64 && stencil_order; ++c) {
+        int j = 0;
+        if (m->face_offsets[c + 1] - m->face_offsets[c] != 2 * m->dim) stencil_order = false;
+        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1] && stencil_order; ++f) {
+            if (partner[f] < f) continue;
+            const int64_t vp = m->face_nbr[f], vm = m->face_nbr[partner[f]];
+            if (vp >= 0) {
+                if (so[j] == 0) so[j] = (int32_t)(vp - c);
+                stencil_order &= vp - c == so[j];
+            }
+            if (vm >= 0) {
+                if (so[j] == 0) so[j] = (int32_t)(c - vm);
+                stencil_order &= c - vm == so[j];
+            }
+            ++j;
+        }
+    }
+    for (int j = 0; j < m->dim; ++j) stencil_order &= so[j] != 0;
+
     // --- internal cell order: Morton order of the optional centroids (tiles of
     // 256 consecutive cells become compact bricks, so upwind neighbours are
     // cache hits), else the caller's order.  pos_h: caller -> internal.
     std::vector<int32_t> user_of(nc), pos_h(nc);
     for (int32_t c = 0; c < nc; ++c) user_of[c] = c;
-    if (m->cell_centre) {
+    if (m->cell_centre && !stencil_order) {  // (a structured index order is kept: stencil kernel)
         double lo[3] = {INFINITY, INFINITY, INFINITY}, hi[3] = {-INFINITY, -INFINITY, -INFINITY};
         for (int32_t c = 0; c < nc; ++c)
             for (int a = 0; a < 3; ++a) {
@@ -662,31 +748,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- plane stride: cells padded to a whole 256-cell tile (2 KB)
     const int32_t ps = (int32_t)((nc64 + bte::kTile - 1) / bte::kTile * bte::kTile);
 
-    // --- face pairing: every face of every cell has an exactly opposite partner
-    // (same area, negated normal) -> paired layout, one upwind load per pair.
-    int mf = 0;
-    for (int64_t c = 0; c < nc64; ++c) mf = std::max<int>(mf, (int)(m->face_offsets[c + 1] - m->face_offsets[c]));
-    std::vector<int64_t> partner(m->face_offsets[nc64], -1);
     // (the paired layout's 5-bit face codes hold up to 16 specular classes)
-    bool paired = mf <= 2 * m->dim && (int)cls_of.size() <= bte::kMaxPairedClasses &&
-                  !(o->flags & BTE_FLAG_GENERIC_FACES);
-    for (int64_t c = 0; c < nc64 && paired; ++c) {
-        const int64_t f0 = m->face_offsets[c], f1 = m->face_offsets[c + 1];
-        for (int64_t f = f0; f < f1 && paired; ++f) {
-            if (partner[f] >= 0) continue;
-            const double *n = m->face_normal + 3 * f;
-            for (int64_t g = f + 1; g < f1; ++g) {
-                const double *q = m->face_normal + 3 * g;
-                if (partner[g] < 0 && m->face_area[g] == m->face_area[f] && q[0] == -n[0] && q[1] == -n[1] &&
-                    q[2] == -n[2]) {
-                    partner[f] = g;
-                    partner[g] = f;
-                    break;
-                }
-            }
-            if (partner[f] < 0) paired = false;
-        }
-    }
+    const bool paired = paired_geom && (int)cls_of.size() <= bte::kMaxPairedClasses;
     const int mf_t = paired ? m->dim : (m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
     std::vector<int32_t> nbr_h(ell), nbm_h(paired ? ell : 1, 0);
@@ -817,6 +880,22 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
     ctx->tma = paired && ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);
+    if (ctx->tma && ctx->uniform_g && stencil_order) {  // near / far staging windows
+        int32_t halo = 0, nfar = 0;
+        for (int j = 0; j < m->dim; ++j) {
+            const int32_t a = std::abs(so[j]);
+            if (a <= bte::kTile) halo = std::max(halo, a);
+            else ctx->farq[nfar++] = j;
+        }
+        const int32_t wmain = bte::kTile + 2 * halo + 2;
+        if (ps >= wmain && ps >= bte::kFarWin) {
+            ctx->stencil = true;
+            ctx->halo = halo;
+            ctx->wmain = wmain;
+            ctx->nfar = nfar;
+            for (int j = 0; j < 3; ++j) ctx->so[j] = so[j];
+        }
+    }
     ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : (paired ? 8 : 2), paired);
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
@@ -1116,6 +1195,7 @@ bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st) {
     if (!ctx || !st) return BTE_EINVAL;
     *st = ctx->st;
     st->dir_chunks = ctx->dir_chunks;
+    st->flux_variant = ctx->stencil ? 5 : ctx->tma ? (ctx->uniform_g ? 4 : 3) : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
     return BTE_OK;
 }
 

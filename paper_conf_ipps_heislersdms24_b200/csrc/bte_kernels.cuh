@@ -52,6 +52,13 @@ struct FluxParams {
     const int32_t *nbr, *nbm;
     const double *gx, *gy, *gz;  // g = (A_f / V_c) n_f
     double gu[3][3];             // uniform-geometry meshes: g of pair q (same for every cell)
+    // stencil meshes (structured index order): the "+" face of pair q of every
+    // cell neighbours cell c + so[q], the "-" face c - so[q]; staging windows
+    int32_t so[3];
+    int32_t halo;                // near window: [t0 - halo, t0 + kTile + halo)
+    int32_t wmain;               // cells staged for the near window (even)
+    int32_t nfar;                // pairs with so > halo: one far window each
+    int32_t farq[3];             // ... which pairs
     const uint32_t *fcode;       // paired [nc]: 5-bit code per side (pair q: bits 10q "+", 10q+5 "-")
     const uint8_t *fcode8;       // generic [MF][nc]: code per face
     const int32_t *refl;         // [n_classes][nd] reflected direction of a specular class
@@ -443,6 +450,179 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
             e = fma(p.cw[lg0 + k] * sd.w, inew, e);
         }
         __syncthreads();  // every thread is done with stage st
+        if (tid == 0 && i + kStages < nit) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            issue(i + kStages);
+        }
+    }
+    if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
+}
+
+// ---------------------------------------------------------------------------
+// Stencil-staged kernel for structured meshes (uniform geometry, constant
+// neighbour offsets so[q] in the stored cell order: +-1, +-nx, +-nx*ny).  For
+// every (band-row, direction) plane one elected thread bulk-copies (TMA) a
+// near window [t0 - halo, t0 + 256 + halo) that holds the tile and every
+// upwind neighbour with |offset| <= halo, plus one 256-cell far window per
+// remaining pair on its upwind side (e.g. the tile shifted by -+nx*ny), into a
+// kStages-deep ring.  All interior upwind values then come from shared memory;
+// only boundary faces (specular: another direction's plane; isothermal: the
+// I0w table) are global loads.  A plane's values are read from DRAM once (by
+// the tile that owns them) and from L2 by its neighbours.  Same arithmetic as
+// flux_paired_kernel.
+constexpr int kFarWin = kTile + 2;  // far window cells (even; 1 cell of alignment slack)
+
+template <int DIM, int NP, int BG>
+__global__ void __launch_bounds__(kTile, BTE_MIN_BLOCKS)
+flux_stencil_kernel(const __grid_constant__ FluxParams p) {
+    extern __shared__ __align__(128) double ring[];  // [kStages][BG][wmain + nfar * kFarWin]
+    __shared__ __align__(8) uint64_t full[kStages];
+    __shared__ int32_t wstart[kStages][1 + NP];       // window start cells of each stage
+    const int tid = threadIdx.x;
+    const int tile0 = blockIdx.x * kTile;
+    const int c = tile0 + tid;
+    const bool valid = c < p.nc;
+    const int grp = blockIdx.y / p.n_dchunks;
+    const int dch = blockIdx.y - grp * p.n_dchunks;
+    const int lg0 = grp * BG;
+    const int d0 = dch * p.dchunk;
+    const int nit = min(p.nd, d0 + p.dchunk) - d0;
+    const int nc = p.nc;
+    const int ps = p.ps;
+    const int plane = p.wmain + p.nfar * kFarWin;  // staged cells per (band-row, direction)
+
+    if (tid == 0) {
+#pragma unroll
+        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    // upwind offset of pair q in direction d: a = s_d . g_q > 0 -> inflow through "-" (c - so)
+    auto upwind = [&](const double4 &sd, int q) {
+        const double a = DIM == 3 ? fma(sd.z, p.gu[q][2], fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]))
+                                  : fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]);
+        return a > 0.0 ? -p.so[q] : p.so[q];
+    };
+    auto clamp_start = [&](int st, int cells) {  // even (16 B aligned), inside the plane
+        st &= ~1;
+        return max(0, min(st, ps - cells));
+    };
+    auto issue = [&](int i) {
+        const int slot = i % kStages;
+        const int d = d0 + i;
+        const double4 sd = load_dir(p.dirs, d);
+        uint64_t *bar = &full[slot];
+        mbar_arrive_expect_tx(bar, (uint32_t)(BG * plane * sizeof(double)));
+        const int wm = clamp_start(tile0 - p.halo, p.wmain);
+        wstart[slot][0] = wm;
+        int wf[NP];
+#pragma unroll
+        for (int f = 0; f < NP; ++f)
+            if (f < p.nfar) {
+                const int q = p.farq[f];
+                wf[f] = clamp_start(tile0 + upwind(sd, q), kFarWin);
+                wstart[slot][1 + f] = wf[f];
+            }
+        const int64_t po = (int64_t)d * ps;
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            double *dst = ring + ((int64_t)slot * BG + k) * plane;
+            const double *pl = p.in_ptr[lg0 + k] + po;
+            bulk_g2s(dst, pl + wm, (uint32_t)(p.wmain * sizeof(double)), bar);
+#pragma unroll
+            for (int f = 0; f < NP; ++f)
+                if (f < p.nfar) bulk_g2s(dst + p.wmain + f * kFarWin, pl + wf[f], kFarWin * sizeof(double), bar);
+        }
+    };
+    if (tid == 0)
+        for (int i = 0; i < min(kStages, nit); ++i) issue(i);
+
+    uint32_t codes = (1u << (10 * NP)) - 1u;
+    int np_[NP], nm_[NP];
+    if (valid) codes = __ldg(p.fcode + c);
+    const bool has_bnd = codes != (1u << (10 * NP)) - 1u;
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {  // boundary cells only: isothermal table columns
+        np_[q] = has_bnd ? __ldg(p.nbr + q * nc + c) : 0;
+        nm_[q] = has_bnd ? __ldg(p.nbm + q * nc + c) : 0;
+    }
+    int farslot[NP];  // far-window index of pair q (-1: near window)
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+        farslot[q] = -1;
+#pragma unroll
+        for (int f = 0; f < NP; ++f)
+            if (f < p.nfar && p.farq[f] == q) farslot[q] = f;
+    }
+    double src[BG];
+#pragma unroll
+    for (int k = 0; k < BG; ++k)
+        src[k] = valid ? p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c) : 0.0;
+
+    double e = 0.0;
+    for (int i = 0; i < nit; ++i) {
+        const int d = d0 + i;
+        const int slot = i % kStages;
+        const double4 sd = load_dir(p.dirs, d);
+        double amin[NP];
+        int up[NP];     // upwind offset
+        int gidx[NP];   // boundary faces: global index (plane-relative or table column)
+        bool glob[NP], iso[NP];
+        double out = 0.0;
+#pragma unroll
+        for (int q = 0; q < NP; ++q) {
+            const double a = DIM == 3 ? fma(sd.z, p.gu[q][2], fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]))
+                                      : fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]);
+            out += fabs(a);
+            amin[q] = -fabs(a);
+            up[q] = a > 0.0 ? -p.so[q] : p.so[q];
+            glob[q] = false;
+            iso[q] = false;
+            gidx[q] = 0;
+            if (has_bnd) {
+                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
+                iso[q] = cd == kCodeIso;
+                glob[q] = cd != kCodeInterior;
+                gidx[q] = iso[q] ? (a > 0.0 ? nm_[q] : np_[q])
+                                 : (glob[q] ? (__ldg(p.refl + cd * p.nd + d) - d) * ps + c : 0);
+            }
+        }
+        const int64_t po = (int64_t)d * ps;
+        double nv[BG][NP];
+        if (has_bnd) {
+#pragma unroll
+            for (int k = 0; k < BG; ++k) {
+                const double *pl = p.in_ptr[lg0 + k] + po;
+                const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
+#pragma unroll
+                for (int q = 0; q < NP; ++q) nv[k][q] = (valid && glob[q]) ? __ldg((iso[q] ? isot : pl) + gidx[q]) : 0.0;
+            }
+        }
+        while (!mbar_try_wait(&full[slot], (i / kStages) & 1)) {
+        }
+        const int wm = wstart[slot][0];
+        int loc[NP];  // position of the upwind neighbour in the staged plane
+#pragma unroll
+        for (int q = 0; q < NP; ++q) {
+            const int nb = c + up[q];
+            loc[q] = glob[q] ? 0
+                     : farslot[q] < 0 ? nb - wm
+                                      : p.wmain + farslot[q] * kFarWin + (nb - wstart[slot][1 + farslot[q]]);
+        }
+        const double *stage = ring + (int64_t)slot * BG * plane;
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            const double *sk = stage + k * plane;
+            const double ic = sk[c - wm];
+            double infl = 0.0;
+#pragma unroll
+            for (int q = 0; q < NP; ++q) infl = fma(amin[q], glob[q] ? nv[k][q] : sk[loc[q]], infl);
+            const double kv = p.kv[lg0 + k];
+            const double inew = fma(ic, (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
+            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew);
+            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
+        }
+        __syncthreads();  // every thread is done with this stage
         if (tid == 0 && i + kStages < nit) {
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             issue(i + kStages);

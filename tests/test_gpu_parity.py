@@ -38,6 +38,7 @@ def test_c1_full_50_steps(bte, oracle_mod):
     Io, To = oracle_run(oracle_mod, cfg, cfg.nsteps)
     Ig, Tg, st = gpu_run(cfg, cfg.nsteps)
     assert_parity(Ig, Tg, Io, To)
+    assert st["flux_variant"] == 4  # 256 cells: too small for the stencil windows
     assert st["steps"] == cfg.nsteps
     assert To.max() > 300.5  # the hot spot moved heat in
 
@@ -204,6 +205,24 @@ def test_graded_mesh_per_cell_geometry(bte, oracle_mod):
     for tma in (True, False):
         Ig, Tg, _ = gpu_run(cfg, 10, tma=tma)
         assert_parity(Ig, Tg, Io, To)
+
+
+@pytest.mark.parametrize("shape", [(40, 24), (33, 20, 6), (64, 64, 3)])
+@pytest.mark.parametrize("bg", [1, 3, 8])
+def test_stencil_kernel(bte, oracle_mod, shape, bg):
+    """Structured index order -> the stencil-staged kernel (near/far TMA windows),
+    incl. odd row lengths (unaligned windows) and far windows in 2-D and 3-D."""
+    h = 1e-6
+    mesh = gen.gen_mesh(shape, (h,) * len(shape))
+    bands = gen.gen_bands_si(3)
+    dirs = gen.gen_dirs_product(4, 8)
+    bcs = gen.gen_bcs_fig1(mesh, radius=3 * h)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    cfg = gen.Config("st", mesh, bands, dirs, bcs, 300.0, dt, 8, ic_eps=0.2)
+    Io, To = oracle_run(oracle_mod, cfg, 8)
+    Ig, Tg, st = gpu_run(cfg, 8, band_group=bg)
+    assert st["flux_variant"] == 5
+    assert_parity(Ig, Tg, Io, To)
 
 
 def test_locality_order_is_invisible(bte):

@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Summarise ncu captures into profiles/ (run here, on the CPU box).
 
-    python tools/ncu_summary.py full  <rep.ncu-rep> <out.json> [--config C4]
+    python tools/ncu_summary.py full  <rep.ncu-rep> <out.json> [--config C4] [--bands-in-launch 48 --bands 55]
     python tools/ncu_summary.py launches <launches.csv> <out.json>
 
 `full`: per captured kernel the duration, DRAM bytes read/written, achieved
@@ -43,7 +43,7 @@ def _num(v, unit):
     return x * UNIT.get(unit, 1.0)
 
 
-def full(rep, out, config=None):
+def full(rep, out, config=None, bands_in_launch=None, bands=None):
     raw = subprocess.check_output(["ncu", "-i", rep, "--page", "raw", "--csv"], text=True)
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
@@ -67,10 +67,13 @@ def full(rep, out, config=None):
             k["dram_GBs"] = k["dram_bytes"] / k["duration"] / 1e9
         kernels.append(k)
     res = {"source": rep, "config": config, "kernels": kernels}
-    flux = [k for k in kernels if "flux" in k["name"] and ", false>" in k["name"]]
+    flux = [k for k in kernels if "flux" in k["name"]]
     if flux:
         res["dram_bytes_per_launch"] = flux[0]["dram_bytes"]
-        res["interior_kernel"] = flux[0]["name"]
+        res["flux_kernel"] = flux[0]["name"]
+        if bands_in_launch and bands:  # the captured launch covers bands_in_launch of the step's rows
+            res["dram_bytes_per_step"] = flux[0]["dram_bytes"] * bands / bands_in_launch
+            res["bands_in_launch"], res["bands_per_step"] = bands_in_launch, bands
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
     for k in kernels:
@@ -98,18 +101,26 @@ def launches(path, out):
         a[0] += 1
         a[1] += t
     tot = sum(v[1] for v in agg.values())
-    res = {k: {"launches": v[0], "total_ms": v[1] * 1e3, "mean_ms": v[1] * 1e3 / v[0], "share": v[1] / tot}
+    step = {k: v for k, v in agg.items() if any(t in k for t in ("flux", "newton", "sum_slots"))}
+    tot_step = sum(v[1] for v in step.values()) or 1.0
+    res = {k: {"launches": v[0], "total_ms": v[1] * 1e3, "mean_ms": v[1] * 1e3 / v[0], "share": v[1] / tot,
+               "share_of_step_kernels": (v[1] / tot_step) if k in step else None}
            for k, v in sorted(agg.items(), key=lambda kv: -kv[1][1])}
     with open(out, "w") as f:
-        json.dump({"source": path, "kernels": res}, f, indent=1)
+        json.dump({"source": path, "kernels": res,
+                   "note": "cold-cache serialised ncu times; share_of_step_kernels = share among the step's kernels"},
+                  f, indent=1)
     for k, v in res.items():
-        print(f"{k[:70]:70s} n={v['launches']:4d} mean {v['mean_ms']:9.3f} ms share {v['share']*100:5.1f}%")
+        ss = v["share_of_step_kernels"]
+        print(f"{k[:60]:60s} n={v['launches']:4d} mean {v['mean_ms']:9.3f} ms share {v['share']*100:5.1f}%"
+              + (f"  step-share {ss*100:5.1f}%" if ss is not None else ""))
 
 
 if __name__ == "__main__":
     mode = sys.argv[1]
     if mode == "full":
-        cfg = sys.argv[sys.argv.index("--config") + 1] if "--config" in sys.argv else "C4"
-        full(sys.argv[2], sys.argv[3], cfg)
+        arg = lambda k, d=None: sys.argv[sys.argv.index(k) + 1] if k in sys.argv else d
+        bil, nb = arg("--bands-in-launch"), arg("--bands")
+        full(sys.argv[2], sys.argv[3], arg("--config", "C4"), int(bil) if bil else None, int(nb) if nb else None)
     else:
         launches(sys.argv[2], sys.argv[3])
