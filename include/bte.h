@@ -80,7 +80,7 @@ typedef struct {
     const double *face_normal;   /* [n_faces][3], unit, outward from the owning cell */
     const double *cell_volume;   /* [n_cells], > 0 */
     const double *cell_centre;   /* [n_cells][3] optional (NULL: keep the caller's order).  A
-                                    locality hint only: cells are stored internally in Morton
+                                    locality hint only: cells are stored internally in brick
                                     order of these points; results do not depend on it. */
 } bte_mesh;
 
@@ -116,6 +116,8 @@ typedef struct {
 #define BTE_FLAG_GENERIC_FACES 2u /* never use the opposite-face-pair layout (testing) */
 #define BTE_FLAG_NO_TMA 4u        /* paired meshes: register-pipelined kernel instead of the
                                      TMA-staged one (testing / comparison) */
+#define BTE_FLAG_STENCIL 8u       /* structured index order: stencil-staged kernel (near/far
+                                     TMA windows; L2-bandwidth-heavy, opt-in) */
 
 typedef struct {
     double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */

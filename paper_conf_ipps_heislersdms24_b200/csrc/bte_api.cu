@@ -151,7 +151,7 @@ void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p)
                              (int)smem);
         attr = true;
     }
-    bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTile), smem, s>>>(p);
+    bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
 }
 
 // Stencil-staged kernel (structured meshes): near + far windows per plane.
@@ -663,30 +663,48 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     for (int j = 0; j < m->dim; ++j) stencil_order &= so[j] != 0;
 
-    // --- internal cell order: Morton order of the optional centroids (tiles of
-    // 256 consecutive cells become compact bricks, so upwind neighbours are
-    // cache hits), else the caller's order.  pos_h: caller -> internal.
+    // --- internal cell order from the optional centroids: cells are grouped
+    // into bricks of 8 x 8 x 4 (2-D: 16 x 16) typical cell sizes, Morton order
+    // inside a brick (a 256-cell thread block is one brick), bricks in
+    // row-major order with the axis of most bricks slowest, so every face
+    // neighbour of a brick is at most (bricks per slab) blocks away and its
+    // upwind data is still in L2 when needed.  Else: the caller's order.
+    // pos_h: caller -> internal.
     std::vector<int32_t> user_of(nc), pos_h(nc);
     for (int32_t c = 0; c < nc; ++c) user_of[c] = c;
-    if (m->cell_centre && !stencil_order) {  // (a structured index order is kept: stencil kernel)
+    const bool use_locality = m->cell_centre && !(stencil_order && (o->flags & BTE_FLAG_STENCIL));
+    if (use_locality) {
+        const int D = m->dim;
         double lo[3] = {INFINITY, INFINITY, INFINITY}, hi[3] = {-INFINITY, -INFINITY, -INFINITY};
         for (int32_t c = 0; c < nc; ++c)
-            for (int a = 0; a < 3; ++a) {
+            for (int a = 0; a < D; ++a) {
                 lo[a] = std::min(lo[a], m->cell_centre[3 * c + a]);
                 hi[a] = std::max(hi[a], m->cell_centre[3 * c + a]);
             }
+        double vol = 1.0;
+        for (int a = 0; a < D; ++a) vol *= std::max(hi[a] - lo[a], 1e-300);
+        const double h = std::pow(vol / (double)nc, 1.0 / D);  // typical cell size
+        const double bsz[3] = {8.0 * h, 8.0 * h, (D == 3 ? 4.0 : 16.0) * h};
+        const double bsz2[3] = {16.0 * h, 16.0 * h, 1.0};
+        const double *B = D == 3 ? bsz : bsz2;
+        int64_t nbk[3] = {1, 1, 1};
+        for (int a = 0; a < D; ++a) nbk[a] = (int64_t)std::floor((hi[a] - lo[a]) / B[a]) + 1;
+        int ax[3] = {0, 1, 2};  // brick axes, slowest first: the axis with the most bricks
+        std::sort(ax, ax + D, [&](int a, int b) { return nbk[a] > nbk[b]; });
         std::vector<uint64_t> key(nc);
         for (int32_t c = 0; c < nc; ++c) {
-            uint64_t q[3];
-            for (int a = 0; a < 3; ++a) {
-                const double span = hi[a] - lo[a];
-                const double t = span > 0.0 ? (m->cell_centre[3 * c + a] - lo[a]) / span : 0.0;
-                q[a] = (uint64_t)std::min(2097151.0, std::max(0.0, std::floor(t * 2097151.0)));
+            uint64_t bidx = 0, loc[3] = {0, 0, 0};
+            for (int t = 0; t < D; ++t) {
+                const int a = ax[t];
+                const double r = (m->cell_centre[3 * c + a] - lo[a]) / B[a];
+                const int64_t bi = std::min<int64_t>(nbk[a] - 1, std::max<int64_t>(0, (int64_t)std::floor(r)));
+                bidx = bidx * (uint64_t)nbk[a] + (uint64_t)bi;
+                loc[a] = (uint64_t)std::min(1023.0, std::max(0.0, std::floor((r - bi) * 1024.0)));
             }
-            uint64_t k = 0;
-            for (int bit = 20; bit >= 0; --bit)
-                for (int a = 0; a < 3; ++a) k = (k << 1) | ((q[a] >> bit) & 1u);
-            key[c] = k;
+            uint64_t mort = 0;  // Morton code of the position inside the brick (10 bits per axis)
+            for (int bit = 9; bit >= 0; --bit)
+                for (int a = 0; a < D; ++a) mort = (mort << 1) | ((loc[a] >> bit) & 1u);
+            key[c] = (bidx << 30) | mort;
         }
         std::stable_sort(user_of.begin(), user_of.end(), [&](int32_t a, int32_t b) { return key[a] < key[b]; });
     }
@@ -880,7 +898,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
     ctx->tma = paired && ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);
-    if (ctx->tma && ctx->uniform_g && stencil_order) {  // near / far staging windows
+    if (ctx->tma && ctx->uniform_g && stencil_order && (o->flags & BTE_FLAG_STENCIL)) {  // near / far windows
         int32_t halo = 0, nfar = 0;
         for (int j = 0; j < m->dim; ++j) {
             const int32_t a = std::abs(so[j]);
@@ -896,7 +914,10 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             for (int j = 0; j < 3; ++j) ctx->so[j] = so[j];
         }
     }
-    ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : (paired ? 8 : 2), paired);
+    // auto band group (measured on B200): the largest group that
+    // compiles without spills for the chosen kernel
+    const int auto_bg = !paired ? 2 : ctx->stencil ? 4 : ctx->tma ? (ctx->uniform_g ? 5 : 3) : 8;
+    ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : auto_bg, paired);
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
     ctx->slab_elems = (int64_t)nd * ps;

@@ -339,15 +339,24 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
         : "memory");
 }
 
+// Warp-specialised: warps 0..7 compute (one cell each), warp 8 is the producer.
+// full[s] completes when stage s has landed (tx bytes); empty[s] completes when
+// all 8 compute warps are done with it -- no block-wide barrier in the loop.
+constexpr int kComputeWarps = kTile / 32;
+constexpr int kTmaThreads = kTile + 32;
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
 template <int DIM, int NP, int BG, bool UG>
-__global__ void __launch_bounds__(kTile, BTE_MIN_BLOCKS)
+__global__ void __launch_bounds__(kTmaThreads, BTE_MIN_BLOCKS)
 flux_tma_kernel(const __grid_constant__ FluxParams p) {
     extern __shared__ __align__(128) double ring[];  // [kStages][BG][kTile]
     __shared__ __align__(8) uint64_t full[kStages];
+    __shared__ __align__(8) uint64_t empty[kStages];
     const int tid = threadIdx.x;
     const int tile0 = blockIdx.x * kTile;
-    const int c = tile0 + tid;
-    const bool valid = c < p.nc;
     const int grp = blockIdx.y / p.n_dchunks;
     const int dch = blockIdx.y - grp * p.n_dchunks;
     const int lg0 = grp * BG;
@@ -359,21 +368,35 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
 
     if (tid == 0) {
 #pragma unroll
-        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kComputeWarps);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    auto issue = [&](int i) {  // stage i % kStages <- planes (band-rows of the group, direction d0 + i)
-        uint64_t *bar = &full[i % kStages];
-        mbar_arrive_expect_tx(bar, kBytes);
-        const int64_t off = (int64_t)(d0 + i) * ps + tile0;
-#pragma unroll
-        for (int k = 0; k < BG; ++k)
-            bulk_g2s(ring + ((i % kStages) * BG + k) * kTile, p.in_ptr[lg0 + k] + off, kTile * sizeof(double), bar);
-    };
-    if (tid == 0)
-        for (int i = 0; i < min(kStages, nit); ++i) issue(i);
 
+    if (tid >= kTile) {  // ------------------------------------------ producer warp
+        if (tid == kTile) {
+            for (int i = 0; i < nit; ++i) {
+                const int st = i % kStages;
+                if (i >= kStages)
+                    while (!mbar_try_wait(&empty[st], ((i / kStages) - 1) & 1)) {
+                    }
+                mbar_arrive_expect_tx(&full[st], kBytes);
+                const int64_t off = (int64_t)(d0 + i) * ps + tile0;
+#pragma unroll
+                for (int k = 0; k < BG; ++k)
+                    bulk_g2s(ring + (st * BG + k) * kTile, p.in_ptr[lg0 + k] + off, kTile * sizeof(double), &full[st]);
+            }
+        }
+        return;
+    }
+
+    // --------------------------------------------------------------- compute warps
+    const int c = tile0 + tid;
+    const bool valid = c < nc;
+    const int lane = tid & 31;
     int np_[NP], nm_[NP];
     double gx[NP], gy[NP], gz[NP];
     uint32_t codes = (1u << (10 * NP)) - 1u;
@@ -434,25 +457,23 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
         while (!mbar_try_wait(&full[st], (i / kStages) & 1)) {
         }
         const double *stage = ring + st * BG * kTile;
+        double inew[BG];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
             const double *sk = stage + k * kTile;
             const double ic = sk[tid];
             double infl = 0.0;
 #pragma unroll
-            for (int q = 0; q < NP; ++q) {
-                const double v = glob[q] ? nv[k][q] : sk[idx[q] - tile0];
-                infl = fma(amin[q], v, infl);
-            }
+            for (int q = 0; q < NP; ++q) infl = fma(amin[q], glob[q] ? nv[k][q] : sk[idx[q] - tile0], infl);
             const double kv = p.kv[lg0 + k];
-            const double inew = fma(ic, (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
-            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew);
-            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
+            inew[k] = fma(ic, (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
         }
-        __syncthreads();  // every thread is done with stage st
-        if (tid == 0 && i + kStages < nit) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            issue(i + kStages);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done with the stage
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew[k]);
+            e = fma(p.cw[lg0 + k] * sd.w, inew[k], e);
         }
     }
     if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;

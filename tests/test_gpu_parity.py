@@ -210,7 +210,7 @@ def test_graded_mesh_per_cell_geometry(bte, oracle_mod):
 @pytest.mark.parametrize("shape", [(40, 24), (33, 20, 6), (64, 64, 3)])
 @pytest.mark.parametrize("bg", [1, 3, 8])
 def test_stencil_kernel(bte, oracle_mod, shape, bg):
-    """Structured index order -> the stencil-staged kernel (near/far TMA windows),
+    """Structured index order + BTE_FLAG_STENCIL -> the stencil-staged kernel (near/far TMA windows),
     incl. odd row lengths (unaligned windows) and far windows in 2-D and 3-D."""
     h = 1e-6
     mesh = gen.gen_mesh(shape, (h,) * len(shape))
@@ -220,7 +220,7 @@ def test_stencil_kernel(bte, oracle_mod, shape, bg):
     dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
     cfg = gen.Config("st", mesh, bands, dirs, bcs, 300.0, dt, 8, ic_eps=0.2)
     Io, To = oracle_run(oracle_mod, cfg, 8)
-    Ig, Tg, st = gpu_run(cfg, 8, band_group=bg)
+    Ig, Tg, st = gpu_run(cfg, 8, band_group=bg, stencil=True)
     assert st["flux_variant"] == 5
     assert_parity(Ig, Tg, Io, To)
 
