@@ -194,6 +194,9 @@ def run_ours(args):
     from paper_conf_ipps_heislersdms24_b200 import inputs as gen
 
     cfg = gen.make_config(args.config)
+    if args.ic_eps is not None:
+        import dataclasses
+        cfg = dataclasses.replace(cfg, ic_eps=args.ic_eps)
     nccl_id = None
     if world > 1:
         from paper_conf_ipps_heislersdms24_b200.dist import share_nccl_id
@@ -313,8 +316,7 @@ def _emit(v):
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOADS[args.config], "name": args.config, "n_cells": nc, "n_dirs": nd,
                        "n_band_rows": nb, "dt": dt, "parallelism": f"band-shard x{world}",
-                       "l2": "state 23 GB/copy >> 126 MB L2 (no flush needed)" if args.config != "C3"
-                             else "state 2.5 GB/copy >> L2"},
+                       "l2": f"state {nc * nd * nb * 8 / 1e9:.1f} GB per copy >> 126 MB L2 (no flush needed)"},
             "roofline": roof, "cpu_baseline": cb, "e2e": e2e, "clocks": clocks,
             "gpu_launches": st["kernel_launches"], "phases_ms_per_step": phases,
             "newton_iter_max": st["newton_iter_max"], "band_group": st["band_group"],
@@ -341,6 +343,7 @@ def main():
     ap.add_argument("--no-locality", action="store_true", help="keep row-major cell order (no Morton hint)")
     ap.add_argument("--no-tma", action="store_true", help="register-pipelined flux kernel instead of TMA-staged")
     ap.add_argument("--stencil", action="store_true", help="stencil-staged kernel (structured order, opt-in)")
+    ap.add_argument("--ic-eps", type=float, default=None, help="override the IC perturbation (0: equilibrium IC)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")
     args = ap.parse_args()

@@ -144,12 +144,13 @@ void flux_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
 // TMA-staged paired kernel: one 256-cell tile per block, kStages x BG x 2 KB ring.
 template <int DIM, int NP, int BG, bool UG>
 void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    constexpr size_t smem = (size_t)bte::kStages * BG * bte::kTile * sizeof(double);
-    static bool attr = false;  // > 48 KB of dynamic shared memory needs an opt-in
-    if (!attr) {
+    const size_t smem = (size_t)bte::kStages * BG * bte::kTile * sizeof(double) +
+                        (UG ? (size_t)p.dchunk * sizeof(bte::DirEntry<NP>) : 0);
+    static size_t attr = 0;  // > 48 KB of dynamic shared memory needs an opt-in
+    if (attr < smem) {
         cudaFuncSetAttribute(bte::flux_tma_kernel<DIM, NP, BG, UG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)smem);
-        attr = true;
+        attr = smem;
     }
     bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
 }
@@ -936,8 +937,11 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             return fail(BTE_ENOMEM);
         }
     }
+    // slab rotation: batches of whole band groups (a batch of 11 at group 5 would
+    // launch 5 + 5 + 1, and the 1-row tail launch is slow)
+    if (n_spare < nb_loc && n_spare >= ctx->bg && o->max_spare_slabs <= 0) n_spare -= n_spare % ctx->bg;
     ctx->n_spare = n_spare;
-    while (ctx->bg > n_spare) ctx->bg /= 2;
+    while (ctx->bg > n_spare) ctx->bg = std::max(1, legal_bg(ctx->bg - 1, paired));
     ctx->cur_slot.resize(nb_loc);
     ctx->spare_slot.resize(n_spare);
     for (int k = 0; k < nb_loc; ++k) ctx->cur_slot[k] = k;

@@ -349,10 +349,36 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// Shared-memory direction table of a block's chunk (uniform geometry): per
+// direction out = sum |s.g_q|, -|s.g_q| per pair, w_d, and the upwind side bits.
+template <int NP>
+struct DirEntry {
+    double out, amin[NP], w;
+    uint32_t up;  // bit q: s.g_q > 0 (inflow through the "-" face)
+};
+
+template <int DIM, int NP>
+__device__ __forceinline__ DirEntry<NP> dir_entry(const FluxParams &p, int d) {
+    const double4 sd = load_dir(p.dirs, d);
+    DirEntry<NP> t;
+    t.out = 0.0;
+    t.up = 0;
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+        const double a = DIM == 3 ? fma(sd.z, p.gu[q][2], fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]))
+                                  : fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]);
+        t.out += fabs(a);
+        t.amin[q] = -fabs(a);
+        t.up |= (a > 0.0 ? 1u : 0u) << q;
+    }
+    t.w = sd.w;
+    return t;
+}
+
 template <int DIM, int NP, int BG, bool UG>
 __global__ void __launch_bounds__(kTmaThreads, BTE_MIN_BLOCKS)
 flux_tma_kernel(const __grid_constant__ FluxParams p) {
-    extern __shared__ __align__(128) double ring[];  // [kStages][BG][kTile]
+    extern __shared__ __align__(128) double ring[];  // [kStages][BG][kTile], then (UG) DirEntry[dchunk]
     __shared__ __align__(8) uint64_t full[kStages];
     __shared__ __align__(8) uint64_t empty[kStages];
     const int tid = threadIdx.x;
@@ -366,6 +392,7 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
     const int ps = p.ps;
     constexpr uint32_t kBytes = BG * kTile * sizeof(double);
 
+    DirEntry<NP> *dtab = reinterpret_cast<DirEntry<NP> *>(ring + kStages * BG * kTile);
     if (tid == 0) {
 #pragma unroll
         for (int s = 0; s < kStages; ++s) {
@@ -374,6 +401,8 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    if (UG)
+        for (int i = tid; i < nit; i += kTmaThreads) dtab[i] = dir_entry<DIM, NP>(p, d0 + i);
     __syncthreads();
 
     if (tid >= kTile) {  // ------------------------------------------ producer warp
@@ -421,22 +450,36 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
     double e = 0.0;
     for (int i = 0; i < nit; ++i) {
         const int d = d0 + i;
-        const double4 sd = load_dir(p.dirs, d);
-        double amin[NP];
+        double amin[NP], out, wd;
+        uint32_t up = 0;
+        if (UG) {  // block-uniform: from the shared-memory direction table
+            const DirEntry<NP> &t = dtab[i];
+            out = t.out;
+            wd = t.w;
+            up = t.up;
+#pragma unroll
+            for (int q = 0; q < NP; ++q) amin[q] = t.amin[q];
+        } else {
+            const double4 sd = load_dir(p.dirs, d);
+            out = 0.0;
+            wd = sd.w;
+#pragma unroll
+            for (int q = 0; q < NP; ++q) {
+                const double a = DIM == 3 ? fma(sd.z, gz[q], fma(sd.y, gy[q], sd.x * gx[q])) : fma(sd.y, gy[q], sd.x * gx[q]);
+                out += fabs(a);
+                amin[q] = -fabs(a);
+                up |= (a > 0.0 ? 1u : 0u) << q;
+            }
+        }
         int idx[NP];
         bool glob[NP], iso[NP];
-        double out = 0.0;
 #pragma unroll
         for (int q = 0; q < NP; ++q) {
-            const double ggx = UG ? p.gu[q][0] : gx[q], ggy = UG ? p.gu[q][1] : gy[q];
-            const double ggz = UG ? p.gu[q][2] : gz[q];
-            const double a = DIM == 3 ? fma(sd.z, ggz, fma(sd.y, ggy, sd.x * ggx)) : fma(sd.y, ggy, sd.x * ggx);
-            out += fabs(a);
-            amin[q] = -fabs(a);
-            idx[q] = a > 0.0 ? nm_[q] : np_[q];
+            const bool plus_out = (up >> q) & 1u;
+            idx[q] = plus_out ? nm_[q] : np_[q];
             iso[q] = false;
             if (has_bnd) {
-                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
+                const uint32_t cd = (codes >> (10 * q + (plus_out ? 5 : 0))) & kCodeInterior;
                 iso[q] = cd == kCodeIso;
                 if (cd < kCodeIso) idx[q] = (__ldg(p.refl + cd * p.nd + d) - d) * ps + c;
             }
@@ -473,7 +516,7 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
             if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew[k]);
-            e = fma(p.cw[lg0 + k] * sd.w, inew[k], e);
+            e = fma(p.cw[lg0 + k] * wd, inew[k], e);
         }
     }
     if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
