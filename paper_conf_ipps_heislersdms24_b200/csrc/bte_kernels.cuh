@@ -308,7 +308,10 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
 // table) are global loads, issued at the top of the iteration.  Arithmetic is
 // identical to flux_paired_kernel.
 constexpr int kTile = 256;
-constexpr int kStages = 4;
+#ifndef BTE_TMA_STAGES
+#define BTE_TMA_STAGES 4
+#endif
+constexpr int kStages = BTE_TMA_STAGES;  // shared-memory ring depth (iterations in flight)
 
 __device__ __forceinline__ uint32_t smem_u32(const void *ptr) {
     return (uint32_t)__cvta_generic_to_shared(ptr);
