@@ -118,6 +118,8 @@ typedef struct {
                                      TMA-staged one (testing / comparison) */
 #define BTE_FLAG_STENCIL 8u       /* structured index order: stencil-staged kernel (near/far
                                      TMA windows; L2-bandwidth-heavy, opt-in) */
+#define BTE_FLAG_NO_BOX 16u       /* structured 3-D box grids: do not use the box kernel
+                                     (tensor-copy z-marching tiles, the default there) */
 
 typedef struct {
     double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */
@@ -137,8 +139,10 @@ typedef struct {
     int32_t max_spare_slabs;  /* band slabs of workspace: <= 0 auto (double buffer when it
                                  fits, else slab rotation), k > 0 forces at most k */
     int32_t block_threads;    /* 0 auto; else 64..1024, multiple of 32 */
-    int32_t band_group;       /* 0 auto; else 1..8 band-rows per thread */
-    int32_t dir_chunk;        /* 0 auto; else directions per thread block */
+    int32_t band_group;       /* 0 auto; else 1..8 band-rows per thread (box kernel: band-rows
+                                 per thread block, any >= 1) */
+    int32_t dir_chunk;        /* 0 auto; else directions per thread block (box kernel: rounded
+                                 down to whole 4-direction orbits) */
 } bte_options;
 
 /* Per-context counters since creation / the last bte_reset_stats. Phase
@@ -161,7 +165,8 @@ typedef struct {
     int32_t dir_chunks;        /* direction chunks per launch (grid.y factor) */
     int32_t flux_variant;      /* flux kernel in use: 0 generic faces, 1 paired, 2 paired +
                                   uniform geometry, 3 TMA-staged, 4 TMA-staged + uniform
-                                  geometry, 5 stencil-staged (structured order) */
+                                  geometry, 5 stencil-staged (structured order), 6 box
+                                  (structured 3-D grid, tensor copies, z-marching) */
 } bte_stats;
 
 /* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,

@@ -21,6 +21,7 @@ BTE_FLAG_PROFILE = 1
 BTE_FLAG_GENERIC_FACES = 2
 BTE_FLAG_NO_TMA = 4
 BTE_FLAG_STENCIL = 8
+BTE_FLAG_NO_BOX = 16
 ISOTHERMAL, SYMMETRY = 0, 1
 
 
@@ -74,7 +75,7 @@ class Stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
-FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil"}
+FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil", 6: "box"}
 
 EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte_get_temperature",
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",
@@ -155,7 +156,7 @@ class Solver:
     def __init__(self, mesh, bands, dirs, bcs, *, t_init=300.0, temp_rule=0, newton_rtol=1e-12,
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
                  stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
-                 generic_faces=False, locality=True, dir_chunk=0, tma=True, stencil=False):
+                 generic_faces=False, locality=True, dir_chunk=0, tma=True, stencil=False, box=True):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -188,7 +189,8 @@ class Solver:
         if stream is not None:
             o.stream = int(getattr(stream, "cuda_stream", stream))
         o.flags = ((BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
-                   | (0 if tma else BTE_FLAG_NO_TMA) | (BTE_FLAG_STENCIL if stencil else 0))
+                   | (0 if tma else BTE_FLAG_NO_TMA) | (BTE_FLAG_STENCIL if stencil else 0)
+                   | (0 if box else BTE_FLAG_NO_BOX))
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)
         o.dir_chunk = int(dir_chunk)
         ctx = C.c_void_p()

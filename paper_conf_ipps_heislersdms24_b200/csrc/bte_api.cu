@@ -9,6 +9,8 @@
 #include "bte_kernels.cuh"
 #include "bte_nccl.h"
 
+#include <cudaTypedefs.h>  // PFN_cuTensorMapEncodeTiled (driver entry point, no -lcuda)
+
 #include <algorithm>
 #include <cmath>
 #include <cstdarg>
@@ -74,6 +76,16 @@ struct bte_ctx {
     bool stencil = false;    // ... + constant neighbour offsets: the stencil-staged kernel
     int32_t so[3] = {0, 0, 0}, halo = 0, wmain = 0, nfar = 0, farq[3] = {0, 0, 0};
     double gu[3][3] = {};
+    // box path (structured hex grid in lexicographic order, flux_box_kernel)
+    bool box = false;
+    int32_t bn[3] = {0, 0, 0}, bzside[2] = {0, 0};
+    double bgeo[3] = {0, 0, 0};
+    int n_orb = 0, box_L = 8, box_nbb = 5, box_oc = 25;
+    bte::BoxOrbit *orb = nullptr;
+    double4 *dirs_box = nullptr;
+    double *side_tab = nullptr;
+    int32_t *side_col = nullptr;
+    CUtensorMap tm_in{}, tm_out{}, tm_i0{}, tm_side{};
     // boundary faces: reflection maps of specular classes, isothermal table
     int32_t *refl = nullptr;
     int32_t n_iso = 0, n_refl = 0;
@@ -277,6 +289,224 @@ void ev_collect(bte_ctx *ctx) {  // after a stream sync
     ctx->ev_live.clear();
 }
 
+// ------------------------------------------------------------- box path
+// Structured hexahedral grid detection (flux_box_kernel): every cell has six
+// faces with normals exactly +-e_a, the face graph is an n_0 x n_1 x n_2
+// lattice (walked from the corner cell), A_f / V_c is the same for every cell
+// per axis, and each of the six sides is uniformly isothermal or specular with
+// isothermal faces on at most one axis.  That axis (else mesh z) becomes grid
+// axis 2 (the marching axis); grid axis 0 (contiguous) is a remaining axis of
+// even extent (16-byte tensor strides).  cell_at lists the user cells in grid
+// lexicographic order.
+struct BoxDetect {
+    bool ok = false;
+    int ax[3] = {0, 1, 2};      // grid axis -> mesh axis
+    int32_t n[3] = {0, 0, 0};   // extents along grid axes
+    double g[3] = {0, 0, 0};    // A / V along grid axes
+    int zside[2] = {1, 1};      // grid axis-2 low / high side: 0 isothermal, 1 specular
+    std::vector<int32_t> cell_at;
+    std::vector<int64_t> zbface[2];  // [n1][n0] boundary face id of the axis-2 side faces
+};
+
+BoxDetect detect_box(const bte_mesh *m, const bte_bcs *bc) {
+    BoxDetect r;
+    if (m->dim != 3) return r;
+    const int64_t nc = m->n_cells;
+    std::vector<int64_t> fa((size_t)nc * 6, -1);  // [cell][2 axis + (normal > 0)] -> face
+    for (int64_t c = 0; c < nc; ++c) {
+        if (m->face_offsets[c + 1] - m->face_offsets[c] != 6) return r;
+        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f) {
+            const double *nv = m->face_normal + 3 * f;
+            int a = -1;
+            for (int t = 0; t < 3; ++t)
+                if (nv[t] == 1.0 || nv[t] == -1.0) a = t;
+            if (a < 0 || nv[(a + 1) % 3] != 0.0 || nv[(a + 2) % 3] != 0.0) return r;
+            int64_t &slot = fa[(size_t)c * 6 + 2 * a + (nv[a] > 0.0)];
+            if (slot >= 0) return r;
+            slot = f;
+        }
+    }
+    auto nbr = [&](int64_t c, int a, int sd) { return m->face_nbr[fa[(size_t)c * 6 + 2 * a + sd]]; };
+    int64_t corner = -1;
+    for (int64_t c = 0; c < nc && corner < 0; ++c)
+        if (nbr(c, 0, 0) < 0 && nbr(c, 1, 0) < 0 && nbr(c, 2, 0) < 0) corner = c;
+    if (corner < 0) return r;
+    int64_t n[3];
+    for (int a = 0; a < 3; ++a) {
+        n[a] = 1;
+        for (int64_t c = corner; nbr(c, a, 1) >= 0; c = nbr(c, a, 1))
+            if (++n[a] > nc) return r;
+    }
+    if (n[0] * n[1] * n[2] != nc) return r;
+    std::vector<int32_t> at(nc, -1);  // mesh-axis lexicographic position -> cell
+    std::vector<char> seen(nc, 0);
+    int64_t zs = corner;
+    for (int64_t z = 0; z < n[2]; ++z) {
+        if (z > 0 && (zs = nbr(zs, 2, 1)) < 0) return r;
+        int64_t ys = zs;
+        for (int64_t y = 0; y < n[1]; ++y) {
+            if (y > 0 && (ys = nbr(ys, 1, 1)) < 0) return r;
+            int64_t c = ys;
+            for (int64_t x = 0; x < n[0]; ++x) {
+                if (x > 0 && (c = nbr(c, 0, 1)) < 0) return r;
+                if (seen[c]) return r;
+                seen[c] = 1;
+                at[(z * n[1] + y) * n[0] + x] = (int32_t)c;
+            }
+        }
+    }
+    int kind[3][2] = {{-1, -1}, {-1, -1}, {-1, -1}};  // -1 none yet, 0 iso, 1 sym, 2 mixed
+    double g[3];
+    for (int a = 0; a < 3; ++a) g[a] = m->face_area[fa[(size_t)at[0] * 6 + 2 * a + 1]] / m->cell_volume[at[0]];
+    for (int64_t z = 0; z < n[2]; ++z)
+        for (int64_t y = 0; y < n[1]; ++y)
+            for (int64_t x = 0; x < n[0]; ++x) {
+                const int64_t p[3] = {x, y, z};
+                const int64_t c = at[(z * n[1] + y) * n[0] + x];
+                for (int a = 0; a < 3; ++a)
+                    for (int sd = 0; sd < 2; ++sd) {
+                        const int64_t f = fa[(size_t)c * 6 + 2 * a + sd];
+                        if (m->face_area[f] / m->cell_volume[c] != g[a]) return r;
+                        int64_t q[3] = {p[0], p[1], p[2]};
+                        q[a] += sd ? 1 : -1;
+                        const int64_t v = m->face_nbr[f];
+                        if (q[a] >= 0 && q[a] < n[a]) {
+                            if (v != at[(q[2] * n[1] + q[1]) * n[0] + q[0]]) return r;
+                        } else {
+                            if (v >= 0) return r;
+                            const int k = bc->kind[-1 - v] == BTE_BC_ISOTHERMAL ? 0 : 1;
+                            int &s = kind[a][sd];
+                            s = s < 0 ? k : (s == k ? k : 2);
+                        }
+                    }
+            }
+    int isoax = -1;
+    for (int a = 0; a < 3; ++a) {
+        if (kind[a][0] == 2 || kind[a][1] == 2) return r;
+        if (kind[a][0] == 0 || kind[a][1] == 0) {
+            if (isoax >= 0) return r;
+            isoax = a;
+        }
+    }
+    r.ax[2] = isoax >= 0 ? isoax : 2;
+    int rest[2], nr = 0;
+    for (int a = 0; a < 3; ++a)
+        if (a != r.ax[2]) rest[nr++] = a;
+    if (n[rest[0]] % 2 == 0) r.ax[0] = rest[0], r.ax[1] = rest[1];
+    else if (n[rest[1]] % 2 == 0) r.ax[0] = rest[1], r.ax[1] = rest[0];
+    else return r;
+    for (int t = 0; t < 3; ++t) r.n[t] = (int32_t)n[r.ax[t]], r.g[t] = g[r.ax[t]];
+    for (int sd = 0; sd < 2; ++sd) r.zside[sd] = kind[r.ax[2]][sd];
+    r.cell_at.resize(nc);
+    for (int sd = 0; sd < 2; ++sd) r.zbface[sd].assign((size_t)r.n[0] * r.n[1], -1);
+    for (int64_t i2 = 0; i2 < r.n[2]; ++i2)
+        for (int64_t i1 = 0; i1 < r.n[1]; ++i1)
+            for (int64_t i0 = 0; i0 < r.n[0]; ++i0) {
+                int64_t p[3];
+                p[r.ax[0]] = i0, p[r.ax[1]] = i1, p[r.ax[2]] = i2;
+                const int32_t c = at[(p[2] * n[1] + p[1]) * n[0] + p[0]];
+                r.cell_at[(i2 * r.n[1] + i1) * r.n[0] + i0] = c;
+                for (int sd = 0; sd < 2; ++sd)
+                    if (i2 == (sd ? r.n[2] - 1 : 0))
+                        r.zbface[sd][i1 * r.n[0] + i0] = -1 - nbr(c, r.ax[2], sd);
+            }
+    r.ok = true;
+    return r;
+}
+
+// Orbits of the direction set under the grid axis-0 and axis-1 mirrors (both
+// pairs of sides are specular, so the set is closed under them; Eq. 6).  Every
+// orbit must have four members (no direction with s_0 = 0 or s_1 = 0).  rz:
+// axis-2 mirror, needed when an axis-2 side is specular.
+bool box_orbits(const bte_dirs *dr, const int ax[3], bool need_rz, std::vector<bte::BoxOrbit> *out) {
+    const int nd = dr->n_dirs;
+    auto mirror = [&](int d, int a) {
+        const double *s = dr->s + 3 * d;
+        double r[3] = {s[0], s[1], s[2]};
+        r[a] = -r[a];
+        for (int e = 0; e < nd; ++e) {
+            const double *t = dr->s + 3 * e;
+            if (std::fabs(t[0] - r[0]) <= 1e-10 && std::fabs(t[1] - r[1]) <= 1e-10 && std::fabs(t[2] - r[2]) <= 1e-10)
+                return e;
+        }
+        return -1;
+    };
+    std::vector<int> m0(nd), m1(nd), m2(nd, -1);
+    for (int d = 0; d < nd; ++d) {
+        if (dr->s[3 * d + ax[0]] == 0.0 || dr->s[3 * d + ax[1]] == 0.0) return false;
+        m0[d] = mirror(d, ax[0]);
+        m1[d] = mirror(d, ax[1]);
+        if (need_rz) m2[d] = mirror(d, ax[2]);
+        if (m0[d] < 0 || m1[d] < 0 || (need_rz && m2[d] < 0)) return false;
+    }
+    std::vector<char> used(nd, 0);
+    out->clear();
+    for (int d = 0; d < nd; ++d) {
+        if (used[d]) continue;
+        int b = dr->s[3 * d + ax[0]] > 0.0 ? d : m0[d];
+        b = dr->s[3 * b + ax[1]] > 0.0 ? b : m1[b];
+        const int q[4] = {b, m0[b], m1[b], m0[m1[b]]};
+        if (m1[m0[b]] != q[3]) return false;
+        bte::BoxOrbit o;
+        for (int j = 0; j < 4; ++j) {
+            if (used[q[j]]) return false;
+            used[q[j]] = 1;
+            o.d[j] = q[j];
+            o.rz[j] = need_rz ? m2[q[j]] : -1;
+        }
+        out->push_back(o);
+    }
+    return true;
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q{};
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    }
+    return fn;
+}
+
+// FP64 tiled tensor map; dims/box innermost first, strides in bytes for dims 1..rank-1.
+bool encode_map(CUtensorMap *tm, void *base, int rank, const uint64_t *dims, const uint64_t *strides,
+                const uint32_t *box) {
+    auto fn = tensor_map_encoder();
+    if (!fn) return false;
+    cuuint64_t gd[5], gs[4];
+    cuuint32_t bx[5], es[5];
+    for (int i = 0; i < rank; ++i) gd[i] = dims[i], bx[i] = box[i], es[i] = 1;
+    for (int i = 0; i + 1 < rank; ++i) gs[i] = strides[i];
+    return fn(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, (cuuint32_t)rank, base, gd, gs, bx, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Launch geometry of the box kernel: layers per CTA, band-rows per CTA,
+// orbits per CTA (options: band_group = band-rows per CTA, dir_chunk =
+// directions per CTA).
+struct BoxPlan {
+    int tiles0, tiles1, zranges, n_batches, n_chunks;
+};
+BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
+    BoxPlan b;
+    b.tiles0 = (ctx->bn[0] + bte::kBoxTX - 1) / bte::kBoxTX;
+    b.tiles1 = (ctx->bn[1] + bte::kBoxTY - 1) / bte::kBoxTY;
+    b.zranges = (ctx->bn[2] + ctx->box_L - 1) / ctx->box_L;
+    b.n_batches = (nbl + ctx->box_nbb - 1) / ctx->box_nbb;
+    b.n_chunks = (ctx->n_orb + ctx->box_oc - 1) / ctx->box_oc;
+    return b;
+}
+
+size_t box_smem(const bte_ctx *ctx) {
+    return ((size_t)bte::kBoxStages * bte::kBoxStage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
+               sizeof(double) +
+           (size_t)ctx->box_oc * sizeof(bte::BoxOrbit);
+}
+
 // ------------------------------------------------------------- launch plan
 struct LaunchPlan {
     int groups, n_dch, dchunk;
@@ -321,6 +551,13 @@ LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int bg) {
 
 int count_slots(const bte_ctx *ctx) {
     int slots = 0;
+    if (ctx->box) {
+        for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
+            const BoxPlan bp = plan_box(ctx, std::min(ctx->n_spare, ctx->nb_loc - l0));
+            slots += bp.n_batches * bp.n_chunks;
+        }
+        return slots;
+    }
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare)
         for (const Segment &sg : segments(std::min(ctx->n_spare, ctx->nb_loc - l0), ctx->bg, ctx->paired)) {
             const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
@@ -333,7 +570,66 @@ int count_slots(const bte_ctx *ctx) {
 // of <= n_spare rows, one launch per segment of full band groups, reading the
 // current slabs and writing the spare ones, which then become current (double
 // buffering when n_spare == nb_loc, slab rotation otherwise).
+// Box path: one launch per band batch; a CTA = (32 x 8 x L cell block,
+// nbb band-rows, box_oc orbits), one energy slot per (band batch, orbit chunk).
+bte_status run_flux_box(bte_ctx *ctx, double dt) {
+    bte::BoxParams p{};
+    p.n0 = ctx->bn[0];
+    p.n1 = ctx->bn[1];
+    p.n2 = ctx->bn[2];
+    p.L = ctx->box_L;
+    p.n_orb = ctx->n_orb;
+    p.orb_chunk = ctx->box_oc;
+    p.nbb = ctx->box_nbb;
+    p.nc = ctx->nc;
+    p.zside[0] = ctx->bzside[0];
+    p.zside[1] = ctx->bzside[1];
+    for (int a = 0; a < 3; ++a) p.g[a] = ctx->bgeo[a];
+    p.orb = ctx->orb;
+    p.dirs = ctx->dirs_box;
+    p.part = ctx->part;
+    const size_t smem = box_smem(ctx);
+    static size_t attr = 0;  // > 48 KB of dynamic shared memory needs an opt-in
+    if (attr < smem) {
+        CUDA_TRY(ctx, cudaFuncSetAttribute(bte::flux_box_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        attr = smem;
+    }
+    int slot = 0;
+    for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
+        const int nbl = std::min(ctx->n_spare, ctx->nb_loc - l0);
+        const BoxPlan bp = plan_box(ctx, nbl);
+        p.tiles0 = bp.tiles0;
+        p.tiles1 = bp.tiles1;
+        p.zranges = bp.zranges;
+        p.n_chunks = bp.n_chunks;
+        p.nbl = nbl;
+        p.band0 = l0;
+        p.slot0 = slot;
+        for (int k = 0; k < nbl; ++k) {
+            const int b = l0 + k;
+            p.in_slab[k] = ctx->cur_slot[b];
+            p.out_slab[k] = ctx->spare_slot[k];
+            p.dtit[k] = dt * ctx->h_inv_tau[b];
+            p.kv[k] = dt * ctx->h_vg[b];
+            p.cw[k] = ctx->h_cw[b];
+        }
+        ctx->dir_chunks = bp.n_chunks;
+        const dim3 grid(bp.tiles0 * bp.tiles1 * bp.zranges, bp.n_batches * bp.n_chunks);
+        ev_mark(ctx, kPhFlux, true);
+        bte::flux_box_kernel<<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(p, ctx->tm_in, ctx->tm_out,
+                                                                                 ctx->tm_i0, ctx->tm_side);
+        ev_mark(ctx, kPhFlux, false);
+        ctx->st.kernel_launches++;
+        slot += bp.n_batches * bp.n_chunks;
+        CUDA_TRY(ctx, cudaGetLastError());
+        for (int k = 0; k < nbl; ++k) std::swap(ctx->cur_slot[l0 + k], ctx->spare_slot[k]);
+    }
+    ctx->n_slots_step = slot;
+    return BTE_OK;
+}
+
 bte_status run_flux(bte_ctx *ctx, double dt) {
+    if (ctx->box) return run_flux_box(ctx, dt);
     bte::FluxParams p{};
     p.nc = ctx->nc;
     p.ps = ctx->ps;
@@ -581,7 +877,7 @@ void bte_destroy(bte_ctx *ctx) {
     void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
-                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax};
+                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -664,6 +960,13 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     for (int j = 0; j < m->dim; ++j) stencil_order &= so[j] != 0;
 
+    // --- structured box grid -> the box kernel (grid lexicographic order)
+    BoxDetect bx;
+    std::vector<bte::BoxOrbit> orbs;
+    if (paired_geom && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
+        bx = detect_box(m, bc);
+    const bool use_box = bx.ok && box_orbits(dr, bx.ax, bx.zside[0] == 1 || bx.zside[1] == 1, &orbs);
+
     // --- internal cell order from the optional centroids: cells are grouped
     // into bricks of 8 x 8 x 4 (2-D: 16 x 16) typical cell sizes, Morton order
     // inside a brick (a 256-cell thread block is one brick), bricks in
@@ -673,8 +976,10 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // pos_h: caller -> internal.
     std::vector<int32_t> user_of(nc), pos_h(nc);
     for (int32_t c = 0; c < nc; ++c) user_of[c] = c;
-    const bool use_locality = m->cell_centre && !(stencil_order && (o->flags & BTE_FLAG_STENCIL));
-    if (use_locality) {
+    const bool use_locality = !use_box && m->cell_centre && !(stencil_order && (o->flags & BTE_FLAG_STENCIL));
+    if (use_box) {
+        user_of = bx.cell_at;
+    } else if (use_locality) {
         const int D = m->dim;
         double lo[3] = {INFINITY, INFINITY, INFINITY}, hi[3] = {-INFINITY, -INFINITY, -INFINITY};
         for (int32_t c = 0; c < nc; ++c)
@@ -919,6 +1224,17 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // compiles without spills for the chosen kernel
     const int auto_bg = !paired ? 2 : ctx->stencil ? 4 : ctx->tma ? (ctx->uniform_g ? 5 : 3) : 8;
     ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : auto_bg, paired);
+    if (use_box) {  // one band-row per stage; band_group / dir_chunk size the CTA's work instead
+        ctx->box = true;
+        ctx->bg = 1;
+        for (int a = 0; a < 3; ++a) ctx->bn[a] = bx.n[a], ctx->bgeo[a] = bx.g[a];
+        ctx->bzside[0] = bx.zside[0];
+        ctx->bzside[1] = bx.zside[1];
+        ctx->n_orb = (int)orbs.size();
+        ctx->box_nbb = o->band_group > 0 ? o->band_group : 5;
+        ctx->box_oc = std::min(ctx->n_orb, o->dir_chunk > 0 ? std::max(1, (int)o->dir_chunk / 4) : 25);
+        ctx->box_L = std::min<int>(8, bx.n[2]);
+    }
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
     ctx->slab_elems = (int64_t)nd * ps;
@@ -1011,11 +1327,44 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         for (int b = 0; b < nb; ++b) rate = std::max(rate, inv_tau[b] + bd->vg[b] * ctx->s_max);
         ctx->dt_bound = rate > 0.0 ? 1.0 / rate : INFINITY;
     }
+    if (ctx->box) {  // orbit table, grid-axis directions, isothermal side tables, tensor maps
+        CREATE_TRY(upload(ctx, &ctx->orb, orbs));
+        std::vector<double4> db(nd);
+        for (int d = 0; d < nd; ++d) {
+            const double *sd = dr->s + 3 * d;
+            db[d] = make_double4(sd[bx.ax[0]], sd[bx.ax[1]], sd[bx.ax[2]], dr->w[d]);
+        }
+        CREATE_TRY(upload(ctx, &ctx->dirs_box, db));
+        const int64_t nside = (int64_t)bx.n[0] * bx.n[1];
+        std::vector<int32_t> col(2 * nside, -1);
+        for (int sd = 0; sd < 2; ++sd)
+            if (bx.zside[sd] == 0)
+                for (int64_t i = 0; i < nside; ++i) col[sd * nside + i] = iso_of[bx.zbface[sd][i]];
+        CREATE_TRY(upload(ctx, &ctx->side_col, col));
+        CREATE_TRY(dalloc(ctx, &ctx->side_tab, (size_t)nb_loc * 2 * nside));
+        bte::side_table_kernel<<<256, 256, 0, ctx->stream>>>(ctx->i0w, ctx->n_iso, ctx->side_col, (int)(2 * nside),
+                                                            nb_loc, ctx->side_tab);
+        CREATE_CUDA(cudaGetLastError());
+        const uint64_t n0 = bx.n[0], n1 = bx.n[1], n2 = bx.n[2];
+        const uint64_t dpool[5] = {n0, n1, n2, (uint64_t)nd, (uint64_t)(nb_loc + n_spare)};
+        const uint64_t spool[4] = {n0 * 8, n0 * n1 * 8, (uint64_t)ps * 8, (uint64_t)ctx->slab_elems * 8};
+        const uint32_t bin[5] = {bte::kBoxBX, bte::kBoxBY, 1, 1, 1}, bout[5] = {bte::kBoxTX, bte::kBoxTY, 1, 1, 1};
+        const uint64_t di0[4] = {n0, n1, n2, (uint64_t)nb_loc}, si0[3] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8};
+        const uint64_t dsd[4] = {n0, n1, 2, (uint64_t)nb_loc}, ssd[3] = {n0 * 8, n0 * n1 * 8, 2 * n0 * n1 * 8};
+        if (!encode_map(&ctx->tm_in, ctx->pool, 5, dpool, spool, bin) ||
+            !encode_map(&ctx->tm_out, ctx->pool, 5, dpool, spool, bout) ||
+            !encode_map(&ctx->tm_i0, ctx->i0, 4, di0, si0, bout) ||
+            !encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin)) {
+            set_err(&ctx->err, "cuTensorMapEncodeTiled failed for the box kernel maps");
+            return fail(BTE_ECUDA);
+        }
+        CREATE_CUDA(cudaStreamSynchronize(ctx->stream));
+    }
     std::memset(&ctx->st, 0, sizeof ctx->st);
     ctx->st.spare_slabs = n_spare;
     ctx->st.n_interior_cells = nc - n_bcells;
-    ctx->st.band_group = ctx->bg;
-    ctx->st.block_threads = ctx->block;
+    ctx->st.band_group = ctx->box ? ctx->box_nbb : ctx->bg;
+    ctx->st.block_threads = ctx->box ? bte::kBoxThreads : ctx->block;
     *out = ctx;
     return BTE_OK;
 #undef CREATE_TRY
@@ -1220,7 +1569,7 @@ bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st) {
     if (!ctx || !st) return BTE_EINVAL;
     *st = ctx->st;
     st->dir_chunks = ctx->dir_chunks;
-    st->flux_variant = ctx->stencil ? 5 : ctx->tma ? (ctx->uniform_g ? 4 : 3) : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
+    st->flux_variant = ctx->box ? 6 : ctx->stencil ? 5 : ctx->tma ? (ctx->uniform_g ? 4 : 3) : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
     return BTE_OK;
 }
 

@@ -21,6 +21,7 @@
 //   and aux[j][c] (isothermal ghost column / reflection-class row).
 #pragma once
 #include <cstdint>
+#include <cuda.h>  // CUtensorMap (box kernel tensor maps)
 #include <cuda_runtime.h>
 
 namespace bte {
@@ -698,6 +699,277 @@ flux_stencil_kernel(const __grid_constant__ FluxParams p) {
     if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
 }
 
+// ---------------------------------------------------------------------------
+// Box kernel: structured hexahedral grids (the paper's uniform meshes, Fig. 1
+// L617-621) stored in lexicographic order (axis 0 fastest), axis-0 and axis-1
+// sides specular, axis-2 sides isothermal or specular (each side uniform).
+//
+// Same update as flux_paired_kernel (Eq. 3/5 with the Eq. 6 ghosts, L269-292,
+// L546-576), organised for the bulk-copy tensor engine:
+//  * a CTA owns a tile of 32 x 8 cells (axes 0, 1) and a range of L layers
+//    along axis 2, and marches through the layers in the upwind order of the
+//    direction, so the axis-2 upwind value of layer z is the previous layer's
+//    staged box (no reload);
+//  * one stage = the 4 directions of an orbit {d, m0(d), m1(d), m0 m1(d)} under
+//    the axis-0 / axis-1 mirrors, each a (32+2) x (8+1) box of I^n (own cells
+//    plus the upwind halo row/column), and the I0 row of the layer.  The
+//    specular ghost of an axis-0/1 wall face, I^n[b][m(d)][c] (Eq. 6 at the old
+//    level), is then the own value of the partner slot in the same stage: no
+//    global load and no boundary branch.  The axis-2 ghost layer is a tensor
+//    copy too: the isothermal side table I0_b(T_wall) or, for a specular side,
+//    the wall layer of the z-mirrored direction;
+//  * a producer warp issues every copy (cp.async.bulk.tensor, mbarrier
+//    complete_tx) S stages ahead; results go to shared memory and leave with
+//    tensor stores; the per-cell energy partial sum_b c_b sum_d w_d I'
+//    (L412-418) accumulates in shared memory per layer.
+// HBM-bound, 16 B per update; every other byte is an L2 hit (halo boxes,
+// I0 rows, the ghost layer).
+constexpr int kBoxTX = 32, kBoxTY = 8;
+constexpr int kBoxBX = kBoxTX + 2;           // staged box row (own cells + 2: 16-byte rows)
+constexpr int kBoxBY = kBoxTY + 1;           // own rows + the upwind halo row
+constexpr int kBoxBoxElems = kBoxBX * kBoxBY;  // 306 doubles copied per plane
+constexpr int kBoxPlane = 320;               // doubles per staged plane (128-byte aligned)
+constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
+constexpr int kBoxStage = 4 * kBoxPlane + kBoxCells;  // 4 direction planes + the I0 row
+constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
+#ifndef BTE_BOX_STAGES
+#define BTE_BOX_STAGES 6
+#endif
+#ifndef BTE_BOX_MIN_BLOCKS
+#define BTE_BOX_MIN_BLOCKS 2
+#endif
+constexpr int kBoxStages = BTE_BOX_STAGES;
+
+// One orbit of directions under the two in-plane mirrors.  Slot j has
+// s_0 > 0 for even j, s_0 < 0 for odd j; s_1 > 0 for j < 2, s_1 < 0 for j >= 2;
+// slot j ^ 1 is the axis-0 mirror of slot j, slot j ^ 2 the axis-1 mirror.
+struct BoxOrbit {
+    int32_t d[4];
+    int32_t rz[4];  // axis-2 mirror of d[j] (specular axis-2 sides), else -1
+};
+
+struct BoxParams {
+    int32_t n0, n1, n2;        // grid extents, axis 0 contiguous
+    int32_t tiles0, tiles1;    // 32-cell tiles along axis 0, 8-cell tiles along axis 1
+    int32_t L, zranges;        // layers per CTA, ranges along axis 2
+    int32_t n_orb, orb_chunk, n_chunks;  // orbits, orbits per CTA, chunks
+    int32_t nbl, nbb;          // band-rows in this launch, band-rows per CTA
+    int32_t band0, slot0;      // rank-local first band-row; first energy slot
+    int32_t nc;
+    int32_t zside[2];          // axis-2 low / high side: 0 isothermal, 1 specular
+    double g[3];               // A_f / V_c per axis (uniform grid)
+    const BoxOrbit *orb;       // [n_orb]
+    const double4 *dirs;       // [nd] {s_0, s_1, s_2, w} in grid axes
+    double *part;              // [n_slots][nc] energy partials
+    int32_t in_slab[kMaxBandsPerLaunch];   // launch-local band-row -> slab of I^n
+    int32_t out_slab[kMaxBandsPerLaunch];  // ... slab of I^{n+1}
+    double dtit[kMaxBandsPerLaunch];       // dt / tau_b
+    double kv[kMaxBandsPerLaunch];         // dt v_b
+    double cw[kMaxBandsPerLaunch];         // temperature weight c_b
+};
+
+__device__ __forceinline__ void tma_load_5d(void *dst, const void *tmap, int c0, int c1, int c2, int c3, int c4,
+                                            uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(void *dst, const void *tmap, int c0, int c1, int c2, int c3,
+                                            uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(smem_u32(bar))
+        : "memory");
+}
+__device__ __forceinline__ void tma_store_5d(const void *tmap, const void *src, int c0, int c1, int c2, int c3,
+                                             int c4) {
+    asm volatile("cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
+                     reinterpret_cast<uint64_t>(tmap)),
+                 "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read_all() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_smem_to_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void bar_compute() { asm volatile("bar.sync 1, %0;" ::"n"(kBoxCells) : "memory"); }
+
+// Tensor maps (host-encoded, see bte_api.cu box_maps):
+//   tm_in   the slab pool as {n0, n1, n2, nd, n_slabs}, box {34, 9, 1, 1, 1}
+//   tm_out  same tensor, box {32, 8, 1, 1, 1} (stores)
+//   tm_i0   I0 table as {n0, n1, n2, nb_loc}, box {32, 8, 1, 1}
+//   tm_side isothermal axis-2 side tables as {n0, n1, 2, nb_loc}, box {34, 9, 1, 1}
+// Box origin of slot j: axis 0 at x0 - 2 (s_0 > 0: upwind is x - 1) or x0
+// (s_0 < 0: x + 1); axis 1 at y0 - 1 (s_1 > 0) or y0.
+__device__ __forceinline__ int box_xs(int j) { return (j & 1) ? 0 : 2; }
+__device__ __forceinline__ int box_hy(int j) { return (j & 2) ? 0 : 1; }
+
+__global__ void __launch_bounds__(kBoxThreads, BTE_BOX_MIN_BLOCKS)
+flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUtensorMap tm_in,
+                const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_i0,
+                const __grid_constant__ CUtensorMap tm_side) {
+    extern __shared__ __align__(128) double bsm[];
+    double *ring = bsm;                                  // [kBoxStages][kBoxStage]
+    double *obuf = ring + kBoxStages * kBoxStage;        // [2][4][256]
+    double *eacc = obuf + 2 * 4 * kBoxCells;             // [L][256]
+    BoxOrbit *sorb = reinterpret_cast<BoxOrbit *>(eacc + p.L * kBoxCells);  // [orb_chunk]
+    __shared__ __align__(8) uint64_t full[kBoxStages];
+    __shared__ __align__(8) uint64_t empty[kBoxStages];
+
+    const int tid = threadIdx.x;
+    int t = blockIdx.x;
+    const int t0 = t % p.tiles0;
+    t /= p.tiles0;
+    const int t1 = t % p.tiles1;
+    const int zr = t / p.tiles1;
+    const int x0 = t0 * kBoxTX, y0 = t1 * kBoxTY, z0 = zr * p.L;
+    const int Lc = min(p.L, p.n2 - z0);
+    const int chunk = blockIdx.y % p.n_chunks;
+    const int batch = blockIdx.y / p.n_chunks;
+    const int k0 = batch * p.nbb, k1 = min(p.nbl, k0 + p.nbb);
+    const int o0 = chunk * p.orb_chunk, o1 = min(p.n_orb, o0 + p.orb_chunk);
+
+    if (tid == 0) {
+        for (int s = 0; s < kBoxStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kBoxCells / 32);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    for (int i = tid; i < o1 - o0; i += kBoxThreads) sorb[i] = p.orb[o0 + i];
+    __syncthreads();
+
+    if (tid >= kBoxCells) {  // ------------------------------------------- producer warp
+        if (tid == kBoxCells) {
+            uint32_t it = 0;
+            for (int k = k0; k < k1; ++k) {
+                const int slab = p.in_slab[k], bl = p.band0 + k;
+                for (int o = o0; o < o1; ++o) {
+                    const BoxOrbit ob = sorb[o - o0];
+                    const bool asc = __ldg(&p.dirs[ob.d[0]].z) >= 0.0;
+                    for (int j = 0; j <= Lc; ++j, ++it) {
+                        const int s = it % kBoxStages;
+                        if (it >= kBoxStages)
+                            while (!mbar_try_wait(&empty[s], ((it / kBoxStages) - 1) & 1)) {
+                            }
+                        double *st = ring + s * kBoxStage;
+                        if (j == 0) {  // the upwind layer of the range: neighbour range or ghost layer
+                            const int zh = asc ? z0 - 1 : z0 + Lc;
+                            mbar_arrive_expect_tx(&full[s], 4 * kBoxBoxElems * sizeof(double));
+                            for (int q = 0; q < 4; ++q) {
+                                const int xs = x0 - box_xs(q), ys = y0 - box_hy(q);
+                                if (zh >= 0 && zh < p.n2)
+                                    tma_load_5d(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
+                                else if (p.zside[asc ? 0 : 1] == 0)  // isothermal: I0_b(T_wall) side table
+                                    tma_load_4d(st + q * kBoxPlane, &tm_side, xs, ys, asc ? 0 : 1, bl, &full[s]);
+                                else  // specular: the wall layer of the z-mirrored direction (old level)
+                                    tma_load_5d(st + q * kBoxPlane, &tm_in, xs, ys, asc ? 0 : p.n2 - 1, ob.rz[q],
+                                                slab, &full[s]);
+                            }
+                        } else {
+                            const int z = asc ? z0 + j - 1 : z0 + Lc - j;
+                            mbar_arrive_expect_tx(&full[s], (4 * kBoxBoxElems + kBoxCells) * sizeof(double));
+                            for (int q = 0; q < 4; ++q)
+                                tma_load_5d(st + q * kBoxPlane, &tm_in, x0 - box_xs(q), y0 - box_hy(q), z, ob.d[q],
+                                            slab, &full[s]);
+                            tma_load_4d(st + 4 * kBoxPlane, &tm_i0, x0, y0, z, bl, &full[s]);
+                        }
+                    }
+                }
+            }
+        }
+        return;
+    }
+
+    // ------------------------------------------------------------------ compute warps
+    const int tx = tid & 31, ty = tid >> 5;
+    const int gx = x0 + tx, gy = y0 + ty;
+    const bool valid = gx < p.n0 && gy < p.n1;
+    // staged-plane offsets of this thread: own value, axis-0 and axis-1 upwind
+    // values per slot (walls: the mirrored slot's own value, Eq. 6 specular)
+    int own[4], ux[4], uy[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) own[q] = q * kBoxPlane + (ty + box_hy(q)) * kBoxBX + tx + box_xs(q);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const bool wall0 = (q & 1) ? gx == p.n0 - 1 : gx == 0;
+        const bool wall1 = (q & 2) ? gy == p.n1 - 1 : gy == 0;
+        ux[q] = wall0 ? own[q ^ 1] : own[q] + ((q & 1) ? 1 : -1);
+        uy[q] = wall1 ? own[q ^ 2] : own[q] + ((q & 2) ? kBoxBX : -kBoxBX);
+    }
+    for (int l = 0; l < Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
+
+    uint32_t it = 0, ob = 0;
+    int sp = 0;
+    const int lane = tid & 31;
+    for (int k = k0; k < k1; ++k) {
+        const double dtit = p.dtit[k], kv = p.kv[k], cw = p.cw[k];
+        for (int o = o0; o < o1; ++o) {
+            const BoxOrbit orb = sorb[o - o0];
+            double w[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) w[q] = __ldg(&p.dirs[orb.d[q]].w);
+            const double4 s0 = load_dir(p.dirs, orb.d[0]);
+            const bool asc = s0.z >= 0.0;
+            // -|s . g| per axis and the outflow sum: the same for the 4 slots
+            const double a0 = fabs(s0.x * p.g[0]), a1 = fabs(s0.y * p.g[1]), a2 = fabs(s0.z * p.g[2]);
+            const double coef = (1.0 - dtit) - kv * ((a0 + a1) + a2);
+            const double m0 = -a0, m1 = -a1, m2 = -a2;
+            for (int j = 0; j <= Lc; ++j, ++it) {
+                const int s = it % kBoxStages;
+                while (!mbar_try_wait(&full[s], (it / kBoxStages) & 1)) {
+                }
+                if (j == 0) {
+                    sp = s;
+                    continue;
+                }
+                const int z = asc ? z0 + j - 1 : z0 + Lc - j;
+                const double *cur = ring + s * kBoxStage;
+                const double *prv = ring + sp * kBoxStage;
+                const double src = dtit * cur[4 * kBoxPlane + tid];
+                double *out = obuf + ob * (4 * kBoxCells);
+                double acc = 0.0;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const double ic = cur[own[q]];
+                    double infl = m0 * cur[ux[q]];
+                    infl = fma(m1, cur[uy[q]], infl);
+                    infl = fma(m2, prv[own[q]], infl);
+                    const double inew = fma(ic, coef, fma(-kv, infl, src));
+                    out[q * kBoxCells + tid] = inew;
+                    acc = fma(w[q], inew, acc);
+                }
+                double *ea = eacc + (z - z0) * kBoxCells + tid;
+                *ea = fma(cw, acc, *ea);
+                __syncwarp();
+                if (lane == 0) {  // the previous layer's stage is no longer needed
+                    mbar_arrive(&empty[sp]);
+                    if (j == Lc) mbar_arrive(&empty[s]);
+                }
+                sp = s;
+                fence_smem_to_async();
+                if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
+                bar_compute();
+                if (tid == 0) {
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        tma_store_5d(&tm_out, out + q * kBoxCells, x0, y0, z, orb.d[q], p.out_slab[k]);
+                    bulk_commit();
+                }
+                ob ^= 1u;
+            }
+        }
+    }
+    if (valid) {
+        double *part = p.part + (int64_t)(p.slot0 + blockIdx.y) * p.nc;
+        for (int l = 0; l < Lc; ++l) part[((int64_t)(z0 + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
+    }
+    if (tid == 0) bulk_wait_all();
+}
+
 // ---------------------------------------------------------------- temperature
 
 struct NewtonParams {
@@ -885,6 +1157,18 @@ __global__ void outflow_max_kernel(int nc, int mf, int paired, int nd, const dou
         m = fmax(m, out);
     }
     atomicMax(smax_bits, (unsigned long long)__double_as_longlong(m));  // m >= 0: bit order = value order
+}
+
+// Isothermal axis-2 side tables of the box kernel: out[k][i] = I0w[k][col[i]]
+// (Eq. 6 ghost I0_b(T_wall), already evaluated by i0w_kernel); 0 where no column.
+__global__ void side_table_kernel(const double *__restrict__ i0w, int n_iso, const int32_t *__restrict__ col,
+                                  int n_side, int nb_loc, double *__restrict__ out) {
+    const int64_t n = (int64_t)n_side * nb_loc;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t k = e / n_side;
+        const int c = col[e - k * n_side];
+        out[e] = c >= 0 ? i0w[k * n_iso + c] : 0.0;
+    }
 }
 
 // dst[r][u] = src[r * stride + pos[u]]  (internal -> caller cell order).
