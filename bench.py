@@ -205,7 +205,8 @@ def run_ours(args):
     s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream,
                                profile=True, band_group=args.band_group, block_threads=args.block_threads,
                                max_spare_slabs=args.max_spare, dir_chunk=args.dir_chunk,
-                               locality=not args.no_locality, tma=not args.no_tma, stencil=args.stencil)
+                               locality=not args.no_locality, tma=not args.no_tma, stencil=args.stencil,
+                               box=not args.no_box)
     bte.apply_ic(s, cfg)
     nb_loc = s.b_hi - s.b_lo
     nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
@@ -343,6 +344,7 @@ def main():
     ap.add_argument("--no-locality", action="store_true", help="keep row-major cell order (no Morton hint)")
     ap.add_argument("--no-tma", action="store_true", help="register-pipelined flux kernel instead of TMA-staged")
     ap.add_argument("--stencil", action="store_true", help="stencil-staged kernel (structured order, opt-in)")
+    ap.add_argument("--no-box", action="store_true", help="structured grids: TMA-staged kernel instead of the box kernel")
     ap.add_argument("--ic-eps", type=float, default=None, help="override the IC perturbation (0: equilibrium IC)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")

@@ -16,6 +16,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <map>
 #include <string>
 #include <vector>
@@ -80,7 +81,8 @@ struct bte_ctx {
     bool box = false;
     int32_t bn[3] = {0, 0, 0}, bzside[2] = {0, 0};
     double bgeo[3] = {0, 0, 0};
-    int n_orb = 0, box_L = 8, box_nbb = 5, box_oc = 25;
+    int n_orb = 0, box_L = 8, box_ctas_per_sm = 2;
+    std::map<int, std::pair<int, int>> box_plans;  // launch band-rows -> (band-rows, orbits) per CTA
     bte::BoxOrbit *orb = nullptr;
     double4 *dirs_box = nullptr;
     double *side_tab = nullptr;
@@ -485,26 +487,81 @@ bool encode_map(CUtensorMap *tm, void *base, int rank, const uint64_t *dims, con
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-// Launch geometry of the box kernel: layers per CTA, band-rows per CTA,
-// orbits per CTA (options: band_group = band-rows per CTA, dir_chunk =
-// directions per CTA).
+// Launch geometry of the box kernel: a CTA = one 32 x 8 x L cell block x nbb
+// band-rows x oc orbits.  Unless the options fix them (band_group = band-rows
+// per CTA, dir_chunk = directions per CTA), nbb and oc are chosen per launch
+// size by simulating the in-order dispatch of the CTAs onto the resident CTA
+// slots (work per CTA ~ band-rows x orbits x (layers + 1) stages, plus the
+// energy-partial traffic of each slot), so that the last wave is not mostly
+// empty.
 struct BoxPlan {
-    int tiles0, tiles1, zranges, n_batches, n_chunks;
+    int tiles0, tiles1, zranges, n_batches, n_chunks, nbb, oc;
 };
+constexpr int kBoxMaxOrbChunk = 64;  // orbits per CTA (shared-memory orbit table)
+
+double box_makespan(const bte_ctx *ctx, int tiles0, int tiles1, int zranges, int nbl, int nbb, int oc) {
+    const int nbat = (nbl + nbb - 1) / nbb, nch = (ctx->n_orb + oc - 1) / oc;
+    const int slots = std::max(1, ctx->sm_count * ctx->box_ctas_per_sm);
+    std::vector<double> busy(slots, 0.0);  // min-heap of slot finish times
+    const double fixed = 2.0;               // prologue / epilogue, in stage units
+    for (int y = 0; y < nbat * nch; ++y) {
+        const int ch = y % nch, bt = y / nch;
+        const int nb_c = std::min(nbb, nbl - bt * nbb), no_c = std::min(oc, ctx->n_orb - ch * oc);
+        for (int zr = 0; zr < zranges; ++zr) {
+            const int lc = std::min(ctx->box_L, ctx->bn[2] - zr * ctx->box_L);
+            const double w = fixed + (double)nb_c * no_c * (lc + 1);
+            for (int t = 0; t < tiles0 * tiles1; ++t) {
+                std::pop_heap(busy.begin(), busy.end(), std::greater<double>());
+                busy.back() += w;
+                std::push_heap(busy.begin(), busy.end(), std::greater<double>());
+            }
+        }
+    }
+    const double span = *std::max_element(busy.begin(), busy.end());
+    // energy partials: n_slots x nc x 16 B (write + read), a stage moves ~16 KB
+    const double slot_cost = (double)nbat * nch * ctx->nc * 16.0 / 16384.0 / slots;
+    return span + slot_cost;
+}
+
 BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
     BoxPlan b;
     b.tiles0 = (ctx->bn[0] + bte::kBoxTX - 1) / bte::kBoxTX;
     b.tiles1 = (ctx->bn[1] + bte::kBoxTY - 1) / bte::kBoxTY;
     b.zranges = (ctx->bn[2] + ctx->box_L - 1) / ctx->box_L;
-    b.n_batches = (nbl + ctx->box_nbb - 1) / ctx->box_nbb;
-    b.n_chunks = (ctx->n_orb + ctx->box_oc - 1) / ctx->box_oc;
+    const int omax = std::min(ctx->n_orb, kBoxMaxOrbChunk);
+    b.nbb = ctx->opt.band_group > 0 ? std::min<int>(ctx->opt.band_group, nbl) : 0;
+    b.oc = ctx->opt.dir_chunk > 0 ? std::max(1, std::min(omax, (int)ctx->opt.dir_chunk / 4)) : 0;
+    if (b.nbb == 0 || b.oc == 0) {
+        auto it = ctx->box_plans.find(nbl);
+        if (it != ctx->box_plans.end()) {
+            if (b.nbb == 0) b.nbb = it->second.first;
+            if (b.oc == 0) b.oc = it->second.second;
+        } else {
+            double best = 1e300;
+            int bn = 1, bo = 1;
+            for (int nbb = 1; nbb <= std::min(nbl, 8); ++nbb) {
+                if (b.nbb && nbb != b.nbb) continue;
+                for (int k = 1; k <= 16; ++k) {  // oc = ceil(n_orb / k), at most kBoxMaxOrbChunk
+                    const int oc = std::min(omax, (ctx->n_orb + k - 1) / k);
+                    if (b.oc && oc != b.oc) continue;
+                    const double t = box_makespan(ctx, b.tiles0, b.tiles1, b.zranges, nbl, nbb, oc);
+                    if (t < best * (1.0 - 1e-9)) best = t, bn = nbb, bo = oc;
+                }
+            }
+            const_cast<bte_ctx *>(ctx)->box_plans[nbl] = {bn, bo};
+            if (b.nbb == 0) b.nbb = bn;
+            if (b.oc == 0) b.oc = bo;
+        }
+    }
+    b.n_batches = (nbl + b.nbb - 1) / b.nbb;
+    b.n_chunks = (ctx->n_orb + b.oc - 1) / b.oc;
     return b;
 }
 
 size_t box_smem(const bte_ctx *ctx) {
     return ((size_t)bte::kBoxStages * bte::kBoxStage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
                sizeof(double) +
-           (size_t)ctx->box_oc * sizeof(bte::BoxOrbit);
+           (size_t)std::min(ctx->n_orb, kBoxMaxOrbChunk) * sizeof(bte::BoxOrbit);
 }
 
 // ------------------------------------------------------------- launch plan
@@ -579,8 +636,6 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     p.n2 = ctx->bn[2];
     p.L = ctx->box_L;
     p.n_orb = ctx->n_orb;
-    p.orb_chunk = ctx->box_oc;
-    p.nbb = ctx->box_nbb;
     p.nc = ctx->nc;
     p.zside[0] = ctx->bzside[0];
     p.zside[1] = ctx->bzside[1];
@@ -602,6 +657,8 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
         p.tiles1 = bp.tiles1;
         p.zranges = bp.zranges;
         p.n_chunks = bp.n_chunks;
+        p.orb_chunk = bp.oc;
+        p.nbb = bp.nbb;
         p.nbl = nbl;
         p.band0 = l0;
         p.slot0 = slot;
@@ -614,6 +671,7 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
             p.cw[k] = ctx->h_cw[b];
         }
         ctx->dir_chunks = bp.n_chunks;
+        ctx->st.band_group = bp.nbb;
         const dim3 grid(bp.tiles0 * bp.tiles1 * bp.zranges, bp.n_batches * bp.n_chunks);
         ev_mark(ctx, kPhFlux, true);
         bte::flux_box_kernel<<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(p, ctx->tm_in, ctx->tm_out,
@@ -1231,9 +1289,13 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->bzside[0] = bx.zside[0];
         ctx->bzside[1] = bx.zside[1];
         ctx->n_orb = (int)orbs.size();
-        ctx->box_nbb = o->band_group > 0 ? o->band_group : 5;
-        ctx->box_oc = std::min(ctx->n_orb, o->dir_chunk > 0 ? std::max(1, (int)o->dir_chunk / 4) : 25);
         ctx->box_L = std::min<int>(8, bx.n[2]);
+        int occ = 0;
+        CREATE_CUDA(cudaFuncSetAttribute(bte::flux_box_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)box_smem(ctx)));
+        CREATE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bte::flux_box_kernel, bte::kBoxThreads,
+                                                                  box_smem(ctx)));
+        ctx->box_ctas_per_sm = std::max(1, occ);
     }
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
@@ -1363,7 +1425,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     std::memset(&ctx->st, 0, sizeof ctx->st);
     ctx->st.spare_slabs = n_spare;
     ctx->st.n_interior_cells = nc - n_bcells;
-    ctx->st.band_group = ctx->box ? ctx->box_nbb : ctx->bg;
+    ctx->st.band_group = ctx->box ? plan_box(ctx, std::min(ctx->n_spare, nb_loc)).nbb : ctx->bg;
     ctx->st.block_threads = ctx->box ? bte::kBoxThreads : ctx->block;
     *out = ctx;
     return BTE_OK;
