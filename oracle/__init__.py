@@ -41,6 +41,7 @@ class _Problem(C.Structure):
         ("n_dirs", C.c_int32), ("s", C.c_void_p), ("w", C.c_void_p),
         ("n_bfaces", C.c_int64), ("bkind", C.c_void_p), ("t_wall", C.c_void_p),
         ("temp_rule", C.c_int32), ("newton_rtol", C.c_double), ("newton_maxit", C.c_int32),
+        ("rate_a", C.c_void_p), ("rate_b", C.c_void_p), ("rate_theta", C.c_void_p),
     ]
 
 
@@ -57,21 +58,34 @@ def lib():
         _lib.oracle_I0.restype = dbl
         _lib.oracle_weight.argtypes = [P, i32]
         _lib.oracle_weight.restype = dbl
+        _lib.oracle_weight_at.argtypes = [P, i32, dbl]
+        _lib.oracle_weight_at.restype = dbl
+        _lib.oracle_rate.argtypes = [P, i32, dbl]
+        _lib.oracle_rate.restype = dbl
         _lib.oracle_reflection_map.argtypes = [P, vp]
-        _lib.oracle_update_intensity.argtypes = [P, vp, vp, vp, vp, dbl, i32, i32]
+        _lib.oracle_update_intensity.argtypes = [P, vp, vp, vp, vp, vp, dbl, i32, i32]
         _lib.oracle_update_intensity.restype = None
-        _lib.oracle_energy.argtypes = [P, vp, i32, i32, vp]
+        _lib.oracle_energy.argtypes = [P, vp, vp, i32, i32, vp]
         _lib.oracle_energy.restype = None
-        _lib.oracle_newton.argtypes = [P, vp, vp, vp]
+        _lib.oracle_newton.argtypes = [P, vp, vp, vp, vp]
         _lib.oracle_equilibrium.argtypes = [P, vp, i32, i32, vp]
         _lib.oracle_equilibrium.restype = None
-        _lib.oracle_run.argtypes = [P, dbl, i64, vp, vp]
+        _lib.oracle_run.argtypes = [P, dbl, i64, vp, vp, vp]
         _lib.oracle_step_cells_equilibrium.argtypes = [P, vp, vp, vp, i64, dbl, vp, vp]
     return _lib
 
 
 def _ptr(a):
     return a.ctypes.data_as(C.c_void_p)
+
+
+def _optr(a):
+    """Pointer of an optional per-cell array (None -> NULL)."""
+    return None if a is None else _ptr(a)
+
+
+def _cells(x, nc):
+    return None if x is None else np.ascontiguousarray(np.broadcast_to(np.asarray(x, np.float64), (nc,)))
 
 
 class Problem:
@@ -89,6 +103,11 @@ class Problem:
             s=f64(dirs["s"]), w=f64(dirs["w"]),
             bkind=i32(bcs["kind"]), t_wall=f64(bcs["t_wall"]),
         )
+        # temperature-dependent relaxation times (N1): 1/tau_b(T) = a + b T exp(-theta/T)
+        self.has_rates = bands.get("rate_a") is not None
+        if self.has_rates:
+            self.keep.update(rate_a=f64(bands["rate_a"]), rate_b=f64(bands["rate_b"]),
+                             rate_theta=f64(bands["rate_theta"]))
         k = self.keep
         self.nc, self.nb, self.nd = int(mesh["n_cells"]), int(bands["n_bands"]), int(dirs["n_dirs"])
         self.nbf = int(bcs["n_bfaces"])
@@ -102,6 +121,9 @@ class Problem:
             n_dirs=self.nd, s=_ptr(k["s"]).value, w=_ptr(k["w"]).value,
             n_bfaces=self.nbf, bkind=_ptr(k["bkind"]).value, t_wall=_ptr(k["t_wall"]).value,
             temp_rule=int(temp_rule), newton_rtol=float(rtol), newton_maxit=int(maxit),
+            rate_a=_ptr(k["rate_a"]).value if self.has_rates else None,
+            rate_b=_ptr(k["rate_b"]).value if self.has_rates else None,
+            rate_theta=_ptr(k["rate_theta"]).value if self.has_rates else None,
         )
         self._r = None
 
@@ -119,6 +141,18 @@ class Problem:
     def weights(self):
         return np.array([self.weight(b) for b in range(self.nb)])
 
+    def weight_at(self, b, Tr):
+        return lib().oracle_weight_at(self.ref, int(b), float(Tr))
+
+    def rate(self, b, Tr):
+        """1/tau_b at rate temperature Tr (constant rates ignore Tr)."""
+        return lib().oracle_rate(self.ref, int(b), float(Tr))
+
+    def _need_tr(self, Tr):
+        if self.has_rates and Tr is None:
+            raise ValueError("temperature-dependent rates need the rate temperature Tr")
+        return _cells(Tr, self.nc)
+
     def reflection_map(self):
         if self._r is None:
             r = np.empty((max(self.nbf, 1), self.nd), dtype=np.int32)
@@ -135,41 +169,49 @@ class Problem:
         lib().oracle_equilibrium(self.ref, _ptr(T), int(b_lo), int(b_hi), _ptr(I))
         return I
 
-    def update_intensity(self, T, I, dt, b_lo=0, b_hi=None):
+    def update_intensity(self, T, I, dt, b_lo=0, b_hi=None, Tr=None):
         b_hi = self.nb if b_hi is None else b_hi
         T = np.ascontiguousarray(T, np.float64)
         I = np.ascontiguousarray(I, np.float64)
+        Tr = self._need_tr(Tr)
         out = np.zeros_like(I)
-        lib().oracle_update_intensity(self.ref, _ptr(self.reflection_map()), _ptr(T), _ptr(I),
+        lib().oracle_update_intensity(self.ref, _ptr(self.reflection_map()), _ptr(T), _optr(Tr), _ptr(I),
                                       _ptr(out), float(dt), int(b_lo), int(b_hi))
         return out
 
-    def energy(self, I, b_lo=0, b_hi=None):
+    def energy(self, I, b_lo=0, b_hi=None, Tr=None):
         b_hi = self.nb if b_hi is None else b_hi
         I = np.ascontiguousarray(I, np.float64)
+        Tr = self._need_tr(Tr)
         E = np.empty(self.nc)
-        lib().oracle_energy(self.ref, _ptr(I), int(b_lo), int(b_hi), _ptr(E))
+        lib().oracle_energy(self.ref, _ptr(I), _optr(Tr), int(b_lo), int(b_hi), _ptr(E))
         return E
 
-    def newton(self, E, T_guess):
+    def newton(self, E, T_guess, Tr=None):
         E = np.ascontiguousarray(E, np.float64)
+        Tr = self._need_tr(Tr)
         T = np.array(np.broadcast_to(np.asarray(T_guess, np.float64), (self.nc,)))
         iters = np.zeros(self.nc, dtype=np.int32)
-        rc = lib().oracle_newton(self.ref, _ptr(E), _ptr(T), _ptr(iters))
+        rc = lib().oracle_newton(self.ref, _ptr(E), _optr(Tr), _ptr(T), _ptr(iters))
         if rc != OK:
             raise RuntimeError(f"oracle newton failed rc={rc}")
         return T, iters
 
-    def run(self, I, T, dt, nsteps):
-        """nsteps explicit steps from (I, T); returns new copies."""
+    def run(self, I, T, dt, nsteps, Tr=None):
+        """nsteps explicit steps from (I, T); returns new copies.  With a rate
+        law the state also carries the rate temperature Tr: pass it and get
+        (I, T, Tr) back."""
         I = np.array(I, dtype=np.float64, order="C")
         T = np.array(T, dtype=np.float64, order="C")
+        Tr_in = Tr
+        Tr = None if Tr is None else np.array(np.broadcast_to(np.asarray(Tr, np.float64), (self.nc,)))
+        self._need_tr(Tr)
         assert I.shape == (self.nb, self.nd, self.nc)
         self.reflection_map()  # raise early on an unclosed map
-        rc = lib().oracle_run(self.ref, float(dt), int(nsteps), _ptr(I), _ptr(T))
+        rc = lib().oracle_run(self.ref, float(dt), int(nsteps), _ptr(I), _ptr(T), _optr(Tr))
         if rc != OK:
             raise RuntimeError(f"oracle run failed rc={rc}")
-        return I, T
+        return (I, T) if Tr_in is None else (I, T, Tr)
 
     def step_cells_equilibrium(self, T0, cells, dt):
         T0 = np.ascontiguousarray(T0, np.float64)
@@ -184,17 +226,19 @@ class Problem:
         return out, T1
 
     # -- initial state ----------------------------------------------------------
-    def initial_state(self, t_init, ic_eps=0.0, seed=None, mult_fn=None):
+    def initial_state(self, t_init, ic_eps=0.0, seed=None, mult_fn=None, with_tr=False):
         """IC of the synthetic configs: I = I0_b(t_init) * multiplier, then
-        T = temperature of that field (Newton from t_init)."""
+        T = temperature of that field (Newton from t_init, weights at the rate
+        temperature Tr = t_init).  with_tr: also return Tr."""
         T = np.full(self.nc, float(t_init))
+        Tr = np.full(self.nc, float(t_init)) if (with_tr or self.has_rates) else None
         I = self.equilibrium(T)
         if ic_eps:
             from paper_conf_ipps_heislersdms24_b200.inputs import ic_multiplier, SEED
             for b in range(self.nb):
                 I[b] *= ic_multiplier(self.nd, self.nc, b, ic_eps, SEED if seed is None else seed)
-            T, _ = self.newton(self.energy(I), T)
-        return I, T
+            T, _ = self.newton(self.energy(I, Tr=Tr), T, Tr=Tr)
+        return (I, T, Tr) if with_tr else (I, T)
 
 
 def problem_from_config(cfg, **kw):

@@ -35,14 +35,30 @@ static double oracle_dI0dT(double C, double omega, double T) {
     return (C / em1) * (x / T) * (1.0 + 1.0 / em1);
 }
 
-/* Temperature weight c_b (SURVEY 8(c) #5, #7):
- * R2 (default): c_b = 1/(v_b tau_b)  -- tau = +inf gives 0;
- * R1:           c_b = 1/v_b. */
-double oracle_weight(const oracle_problem *p, int32_t b) {
-    if (p->temp_rule == 1) return 1.0 / p->vg[b];
+/* Scattering rate 1/tau_b (Eq. 5's 1/tau_b, L549).  Constant: 1/tau_b (tau =
+ * +inf gives 0).  Temperature-dependent (N1, L666-669): the law
+ *   1/tau_b(T) = a_b + b_b T exp(-theta_b / T)
+ * (impurity-like + Umklapp-like terms; the form is external)
+ * at the rate temperature Tr. */
+double oracle_rate(const oracle_problem *p, int32_t b, double Tr) {
+    if (p->rate_a) return p->rate_a[b] + p->rate_b[b] * Tr * exp(-p->rate_theta[b] / Tr);
     if (isinf(p->tau[b])) return 0.0;
-    return 1.0 / (p->vg[b] * p->tau[b]);
+    return 1.0 / p->tau[b];
 }
+
+/* Temperature weight c_b (SURVEY 8(c) #5, #7):
+ * R2 (default): c_b = (1/tau_b) / v_b  -- tau = +inf gives 0;
+ * R1:           c_b = 1/v_b. */
+double oracle_weight_at(const oracle_problem *p, int32_t b, double Tr) {
+    if (p->temp_rule == 1) return 1.0 / p->vg[b];
+    if (!p->rate_a) {
+        if (isinf(p->tau[b])) return 0.0;
+        return 1.0 / (p->vg[b] * p->tau[b]);
+    }
+    return oracle_rate(p, b, Tr) / p->vg[b];
+}
+
+double oracle_weight(const oracle_problem *p, int32_t b) { return oracle_weight_at(p, b, NAN); }
 
 /* ------------------------------------------------------------------ Eq. 6 map */
 
@@ -103,7 +119,7 @@ static double field_in(const void *vctx, int32_t b, int32_t d, int64_t c) {
  *           = I0_b(T_wall)     isothermal boundary face      Eq. 6
  *           = I_{r,b} (c)      symmetric boundary face       Eq. 6 (old level)
  */
-static double update_one(const oracle_problem *p, const int32_t *r, const double *T,
+static double update_one(const oracle_problem *p, const int32_t *r, const double *T, const double *Tr,
                          oracle_in_fn In, const void *ctx, double dt, int32_t b, int32_t d,
                          int64_t c) {
     const double *s = &p->s[3 * d];
@@ -126,12 +142,12 @@ static double update_one(const oracle_problem *p, const int32_t *r, const double
         }
         F += p->face_area[f] * mu * Ihat;
     }
-    double inv_tau = isinf(p->tau[b]) ? 0.0 : 1.0 / p->tau[b];
+    double inv_tau = oracle_rate(p, b, Tr ? Tr[c] : NAN);
     double I0 = oracle_I0(p->C[b], p->omega[b], T[c]);
     return Ic + dt * ((I0 - Ic) * inv_tau - p->vg[b] * F / p->cell_volume[c]);
 }
 
-void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const double *T,
+void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const double *T, const double *Tr,
                              const double *I, double *Inew, double dt, int32_t b_lo, int32_t b_hi) {
     field_ctx ctx = {I, p->n_dirs, p->n_cells};
     const int64_t nc = p->n_cells;
@@ -140,7 +156,7 @@ void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const do
             double *out = &Inew[((int64_t)b * p->n_dirs + d) * nc];
 #pragma omp parallel for schedule(static)
             for (int64_t c = 0; c < nc; ++c)
-                out[c] = update_one(p, r, T, field_in, &ctx, dt, b, d, c);
+                out[c] = update_one(p, r, T, Tr, field_in, &ctx, dt, b, d, c);
         }
 }
 
@@ -148,7 +164,8 @@ void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const do
 
 /* E_c = sum_b c_b sum_d w_d I_{d,b}(c): "integrating the phonon intensity over
  * all directions and bands" (L415-418), weights per SURVEY 8(c) #5. */
-void oracle_energy(const oracle_problem *p, const double *I, int32_t b_lo, int32_t b_hi, double *E) {
+void oracle_energy(const oracle_problem *p, const double *I, const double *Tr, int32_t b_lo, int32_t b_hi,
+                   double *E) {
     const int64_t nc = p->n_cells;
     const int32_t nd = p->n_dirs;
 #pragma omp parallel for schedule(static)
@@ -157,7 +174,7 @@ void oracle_energy(const oracle_problem *p, const double *I, int32_t b_lo, int32
         for (int32_t b = b_lo; b < b_hi; ++b) {
             double sb = 0.0;
             for (int32_t d = 0; d < nd; ++d) sb += p->w[d] * I[((int64_t)b * nd + d) * nc + c];
-            e += oracle_weight(p, b) * sb;
+            e += oracle_weight_at(p, b, Tr ? Tr[c] : NAN) * sb;
         }
         E[c] = e;
     }
@@ -165,30 +182,32 @@ void oracle_energy(const oracle_problem *p, const double *I, int32_t b_lo, int32
 
 /* ------------------------------------------------------------------ temperature */
 
-/* g(T) = W sum_b c_b I0_b(T) - E, strictly increasing in T. */
-static double g_of(const oracle_problem *p, double W, double E, double T) {
+/* g(T) = W sum_b c_b I0_b(T) - E, strictly increasing in T;
+ * the weights are taken at the cell's rate temperature Tr (fixed in the solve). */
+static double g_of(const oracle_problem *p, double W, double E, double Tr, double T) {
     double g = 0.0;
-    for (int32_t b = 0; b < p->n_bands; ++b) g += oracle_weight(p, b) * oracle_I0(p->C[b], p->omega[b], T);
+    for (int32_t b = 0; b < p->n_bands; ++b) g += oracle_weight_at(p, b, Tr) * oracle_I0(p->C[b], p->omega[b], T);
     return W * g - E;
 }
 
-static double gprime_of(const oracle_problem *p, double W, double T) {
+static double gprime_of(const oracle_problem *p, double W, double Tr, double T) {
     double g = 0.0;
-    for (int32_t b = 0; b < p->n_bands; ++b) g += oracle_weight(p, b) * oracle_dI0dT(p->C[b], p->omega[b], T);
+    for (int32_t b = 0; b < p->n_bands; ++b)
+        g += oracle_weight_at(p, b, Tr) * oracle_dI0dT(p->C[b], p->omega[b], T);
     return W * g;
 }
 
 /* Bisection on a bracket grown from T0 by halving/doubling. */
-static int bisect(const oracle_problem *p, double W, double E, double T0, double *T) {
+static int bisect(const oracle_problem *p, double W, double E, double Tr, double T0, double *T) {
     double lo = T0, hi = T0;
     int k = 0;
-    while (g_of(p, W, E, lo) > 0.0 && k++ < 2000) lo *= 0.5;
+    while (g_of(p, W, E, Tr, lo) > 0.0 && k++ < 2000) lo *= 0.5;
     k = 0;
-    while (g_of(p, W, E, hi) < 0.0 && k++ < 2000) hi *= 2.0;
-    if (!(g_of(p, W, E, lo) <= 0.0 && g_of(p, W, E, hi) >= 0.0)) return ORACLE_ENOCONV;
+    while (g_of(p, W, E, Tr, hi) < 0.0 && k++ < 2000) hi *= 2.0;
+    if (!(g_of(p, W, E, Tr, lo) <= 0.0 && g_of(p, W, E, Tr, hi) >= 0.0)) return ORACLE_ENOCONV;
     for (k = 0; k < 400 && (hi - lo) > p->newton_rtol * hi; ++k) {
         double mid = 0.5 * (lo + hi);
-        if (g_of(p, W, E, mid) < 0.0) lo = mid; else hi = mid;
+        if (g_of(p, W, E, Tr, mid) < 0.0) lo = mid; else hi = mid;
     }
     *T = 0.5 * (lo + hi);
     return ORACLE_OK;
@@ -198,11 +217,11 @@ static int bisect(const oracle_problem *p, double W, double E, double T0, double
  *   T <- T - g(T)/g'(T) until |dT| <= rtol T, at most maxit iterations;
  *   a non-positive or non-finite iterate, or no convergence, falls back to
  *   bisection. */
-static int solve_cell(const oracle_problem *p, double W, double E, double *T, int32_t *iters) {
+static int solve_cell(const oracle_problem *p, double W, double E, double Tr, double *T, int32_t *iters) {
     double Tc = *T;
     if (!(E > 0.0) || !isfinite(E)) return ORACLE_ENOCONV;
     for (int32_t it = 1; it <= p->newton_maxit; ++it) {
-        double delta = g_of(p, W, E, Tc) / gprime_of(p, W, Tc);
+        double delta = g_of(p, W, E, Tr, Tc) / gprime_of(p, W, Tr, Tc);
         double Tn = Tc - delta;
         if (!(Tn > 0.0) || !isfinite(Tn)) break;
         Tc = Tn;
@@ -213,17 +232,17 @@ static int solve_cell(const oracle_problem *p, double W, double E, double *T, in
         }
     }
     if (iters) *iters = -1;
-    return bisect(p, W, E, *T, T);
+    return bisect(p, W, E, Tr, *T, T);
 }
 
-int oracle_newton(const oracle_problem *p, const double *E, double *T, int32_t *iters) {
+int oracle_newton(const oracle_problem *p, const double *E, const double *Tr, double *T, int32_t *iters) {
     double W = 0.0;
     for (int32_t d = 0; d < p->n_dirs; ++d) W += p->w[d];
     int status = ORACLE_OK;
 #pragma omp parallel for schedule(static)
     for (int64_t c = 0; c < p->n_cells; ++c) {
         int32_t it = 0;
-        int rc = solve_cell(p, W, E[c], &T[c], &it);
+        int rc = solve_cell(p, W, E[c], Tr ? Tr[c] : NAN, &T[c], &it);
         if (iters) iters[c] = it;
         if (rc != ORACLE_OK) {
 #pragma omp critical
@@ -245,18 +264,21 @@ void oracle_equilibrium(const oracle_problem *p, const double *T, int32_t b_lo, 
 
 /* ------------------------------------------------------------------ steps */
 
-int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, double *T) {
+int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, double *T, double *Tr) {
     const int64_t n = (int64_t)p->n_bands * p->n_dirs * p->n_cells;
     int32_t *r = (int32_t *)malloc(sizeof(int32_t) * (size_t)(p->n_bfaces * p->n_dirs + 1));
     double *Inew = (double *)malloc(sizeof(double) * (size_t)(n + 1));
     double *E = (double *)malloc(sizeof(double) * (size_t)(p->n_cells + 1));
     int rc = (r && Inew && E) ? oracle_reflection_map(p, r) : ORACLE_EINVAL;
+    if (p->rate_a && !Tr) rc = ORACLE_EINVAL;
     for (int64_t step = 0; step < nsteps && rc == ORACLE_OK; ++step) {
         /* Finch loop (L357-372): u_new from u; then the post-step temperature
-         * update (L707-716); then u = u_new. */
-        oracle_update_intensity(p, r, T, I, Inew, dt, 0, p->n_bands);
-        oracle_energy(p, Inew, 0, p->n_bands, E);
-        rc = oracle_newton(p, E, T, NULL);
+         * update (L707-716), where I0 and tau become those of the new state
+         * (L666-669; tau one step behind, reading 22); then u = u_new. */
+        oracle_update_intensity(p, r, T, Tr, I, Inew, dt, 0, p->n_bands);
+        if (Tr) memcpy(Tr, T, sizeof(double) * (size_t)p->n_cells);
+        oracle_energy(p, Inew, Tr, 0, p->n_bands, E);
+        rc = oracle_newton(p, E, Tr, T, NULL);
         memcpy(I, Inew, sizeof(double) * (size_t)n);
     }
     free(r);
@@ -292,15 +314,15 @@ int oracle_step_cells_equilibrium(const oracle_problem *p, const int32_t *r, con
         double *out = &Inew_sel[k * nb * nd];
         for (int32_t b = 0; b < nb; ++b)
             for (int32_t d = 0; d < nd; ++d)
-                out[b * nd + d] = update_one(p, r, T0, eq_in, &ctx, dt, b, d, c);
+                out[b * nd + d] = update_one(p, r, T0, T0, eq_in, &ctx, dt, b, d, c);
         double e = 0.0;
         for (int32_t b = 0; b < nb; ++b) {
             double sb = 0.0;
             for (int32_t d = 0; d < nd; ++d) sb += p->w[d] * out[b * nd + d];
-            e += oracle_weight(p, b) * sb;
+            e += oracle_weight_at(p, b, T0[c]) * sb;
         }
         double Tc = T0[c];
-        int rc = solve_cell(p, W, e, &Tc, NULL);
+        int rc = solve_cell(p, W, e, T0[c], &Tc, NULL);
         T1_sel[k] = Tc;
         if (rc != ORACLE_OK) {
 #pragma omp critical

@@ -55,6 +55,14 @@ typedef struct {
     int32_t temp_rule;     /* 0: c_b = 1/(v_b tau_b) (R2), 1: c_b = 1/v_b (R1) */
     double newton_rtol;    /* stop when |dT| <= rtol T */
     int32_t newton_maxit;
+    /* Temperature-dependent relaxation times ("tau ... dependent
+     * on temperature ... mutable values for each cell", L666-669, beta[b] per
+     * cell L1352-1353).  NULL rate_a: constant tau above.  Else
+     *   1/tau_b(T) = rate_a[b] + rate_b[b] T exp(-rate_theta[b] / T)
+     * evaluated per cell at the rate temperature Tr (reading 22:
+     * the rates of step n are those of the temperature of step n-1, so the
+     * R2 temperature equation and the relaxation use the same rates). */
+    const double *rate_a, *rate_b, *rate_theta;
 } oracle_problem;
 
 /* return codes */
@@ -64,8 +72,12 @@ typedef struct {
 
 /* I0_b(T) = C / expm1(theta/T), theta = hbar omega / kB. */
 double oracle_I0(double C, double omega, double T);
-/* c_b, the temperature weight of band-row b under temp_rule. */
+/* c_b, the temperature weight of band-row b under temp_rule (constant rates). */
 double oracle_weight(const oracle_problem *p, int32_t b);
+/* 1/tau_b at rate temperature Tr (the law, or the constant 1/tau_b; +inf -> 0). */
+double oracle_rate(const oracle_problem *p, int32_t b, double Tr);
+/* c_b at rate temperature Tr: R2 rate/v_b, R1 1/v_b. */
+double oracle_weight_at(const oracle_problem *p, int32_t b, double Tr);
 
 /* Specular map (Eq. 6): r[f][d] = d' with s_d' = s_d - 2 (s_d.n_f) n_f within
  * 1e-10, for every symmetric boundary face f; -1 for isothermal faces.
@@ -73,30 +85,36 @@ double oracle_weight(const oracle_problem *p, int32_t b);
 int oracle_reflection_map(const oracle_problem *p, int32_t *r);
 
 /* Intensity update of Eq. 3/5 with the Eq. 6 ghosts for band-rows [b_lo, b_hi):
- * Inew = I + dt ((I0_b(T_c) - I)/tau_b - (v_b/V_c) sum_f A_f (s_d.n_f) I_hat_f). */
-void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const double *T,
+ * Inew = I + dt ((I0_b(T_c) - I)/tau_b - (v_b/V_c) sum_f A_f (s_d.n_f) I_hat_f),
+ * 1/tau_b = oracle_rate(p, b, Tr_c) (Tr may be NULL with constant rates). */
+void oracle_update_intensity(const oracle_problem *p, const int32_t *r, const double *T, const double *Tr,
                              const double *I, double *Inew, double dt, int32_t b_lo, int32_t b_hi);
 
-/* E_c += sum_{b in [b_lo,b_hi)} c_b sum_d w_d I[b][d][c]  (L412-418). E is
- * overwritten (not accumulated). */
-void oracle_energy(const oracle_problem *p, const double *I, int32_t b_lo, int32_t b_hi, double *E);
+/* E_c = sum_{b in [b_lo,b_hi)} c_b(Tr_c) sum_d w_d I[b][d][c]  (L412-418). E is
+ * overwritten (not accumulated).  Tr may be NULL with constant rates. */
+void oracle_energy(const oracle_problem *p, const double *I, const double *Tr, int32_t b_lo, int32_t b_hi,
+                   double *E);
 
-/* Per-cell temperature: solve W sum_b c_b I0_b(T) = E_c by Newton from T_c
- * (bisection safeguard).  T is in/out; iters (may be NULL) gets the per-cell
- * Newton iteration count.  Returns ORACLE_ENOCONV if any cell fails. */
-int oracle_newton(const oracle_problem *p, const double *E, double *T, int32_t *iters);
+/* Per-cell temperature: solve W sum_b c_b(Tr_c) I0_b(T) = E_c by Newton from
+ * T_c (bisection safeguard).  T is in/out; iters (may be NULL) gets the
+ * per-cell Newton iteration count.  Returns ORACLE_ENOCONV if any cell fails. */
+int oracle_newton(const oracle_problem *p, const double *E, const double *Tr, double *T, int32_t *iters);
 
 /* Equilibrium field: I[b-b_lo][d][c] = I0_b(T_c) for b in [b_lo, b_hi) (the IC
  * "equilibrium intensity for a uniform temperature", L678-684). */
 void oracle_equilibrium(const oracle_problem *p, const double *T, int32_t b_lo, int32_t b_hi, double *I);
 
-/* Whole explicit steps: I (all bands) and T in/out.  Returns 0 or an error. */
-int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, double *T);
+/* Whole explicit steps: I (all bands), T and the rate temperature Tr in/out
+ * (Tr may be NULL with constant rates).  Per step: Inew from (I, T, Tr);
+ * Tr <- T; E and the Newton solve with the weights at the new Tr; I <- Inew.
+ * Returns 0 or an error. */
+int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, double *T, double *Tr);
 
 /* One step at selected cells when I^n is the equilibrium of the temperature
- * field T0 (I^n[b][d][c] = I0_b(T0_c)).  Writes Inew_sel[k][b][d] and the
- * Newton temperature T1_sel[k] of cell cells[k] (initial guess T0).  Used for
- * sampled checks at sizes where the full field does not fit on the host. */
+ * field T0 (I^n[b][d][c] = I0_b(T0_c)) and the rate temperature is T0 too.
+ * Writes Inew_sel[k][b][d] and the Newton temperature T1_sel[k] of cell
+ * cells[k] (initial guess T0).  Used for sampled checks at sizes where the
+ * full field does not fit on the host. */
 int oracle_step_cells_equilibrium(const oracle_problem *p, const int32_t *r, const double *T0,
                                   const int64_t *cells, int64_t n_sel, double dt,
                                   double *Inew_sel, double *T1_sel);

@@ -16,6 +16,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <functional>
 #include <map>
 #include <string>
@@ -81,13 +82,14 @@ struct bte_ctx {
     bool box = false;
     int32_t bn[3] = {0, 0, 0}, bzside[2] = {0, 0};
     double bgeo[3] = {0, 0, 0};
-    int n_orb = 0, box_L = 8, box_ctas_per_sm = 2;
-    std::map<int, std::pair<int, int>> box_plans;  // launch band-rows -> (band-rows, orbits) per CTA
+    int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
+    bool td = false;  // temperature-dependent relaxation times (rate tables)
     bte::BoxOrbit *orb = nullptr;
     double4 *dirs_box = nullptr;
     double *side_tab = nullptr;
     int32_t *side_col = nullptr;
-    CUtensorMap tm_in{}, tm_out{}, tm_i0{}, tm_side{};
+    CUtensorMap tm_in{}, tm_out{}, tm_i0{}, tm_side{}, tm_rate{};
+    int rsel = 0;  // rate tables: which half holds the current rates
     // boundary faces: reflection maps of specular classes, isothermal table
     int32_t *refl = nullptr;
     int32_t n_iso = 0, n_refl = 0;
@@ -487,71 +489,38 @@ bool encode_map(CUtensorMap *tm, void *base, int rank, const uint64_t *dims, con
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-// Launch geometry of the box kernel: a CTA = one 32 x 8 x L cell block x nbb
-// band-rows x oc orbits.  Unless the options fix them (band_group = band-rows
-// per CTA, dir_chunk = directions per CTA), nbb and oc are chosen per launch
-// size by simulating the in-order dispatch of the CTAs onto the resident CTA
-// slots (work per CTA ~ band-rows x orbits x (layers + 1) stages, plus the
-// energy-partial traffic of each slot), so that the last wave is not mostly
-// empty.
+// Launch geometry of the box kernel.  Work item = one 32 x 8 x L cell block x
+// nbb band-rows x oc orbits; persistent CTAs (sm_count x resident CTAs per
+// SM) take the items round-robin, tile fastest.  Defaults (measured on B200,
+// DESIGN.md 10): nbb = 5 band-rows, oc = the largest divisor of n_orb <= 20
+// (whole chunks: a ragged last chunk idles part of the grid); the options
+// band_group / dir_chunk override them.  One energy slot per (band batch,
+// orbit chunk).
 struct BoxPlan {
     int tiles0, tiles1, zranges, n_batches, n_chunks, nbb, oc;
 };
-constexpr int kBoxMaxOrbChunk = 64;  // orbits per CTA (shared-memory orbit table)
-
-double box_makespan(const bte_ctx *ctx, int tiles0, int tiles1, int zranges, int nbl, int nbb, int oc) {
-    const int nbat = (nbl + nbb - 1) / nbb, nch = (ctx->n_orb + oc - 1) / oc;
-    const int slots = std::max(1, ctx->sm_count * ctx->box_ctas_per_sm);
-    std::vector<double> busy(slots, 0.0);  // min-heap of slot finish times
-    const double fixed = 2.0;               // prologue / epilogue, in stage units
-    for (int y = 0; y < nbat * nch; ++y) {
-        const int ch = y % nch, bt = y / nch;
-        const int nb_c = std::min(nbb, nbl - bt * nbb), no_c = std::min(oc, ctx->n_orb - ch * oc);
-        for (int zr = 0; zr < zranges; ++zr) {
-            const int lc = std::min(ctx->box_L, ctx->bn[2] - zr * ctx->box_L);
-            const double w = fixed + (double)nb_c * no_c * (lc + 1);
-            for (int t = 0; t < tiles0 * tiles1; ++t) {
-                std::pop_heap(busy.begin(), busy.end(), std::greater<double>());
-                busy.back() += w;
-                std::push_heap(busy.begin(), busy.end(), std::greater<double>());
-            }
-        }
-    }
-    const double span = *std::max_element(busy.begin(), busy.end());
-    // energy partials: n_slots x nc x 16 B (write + read), a stage moves ~16 KB
-    const double slot_cost = (double)nbat * nch * ctx->nc * 16.0 / 16384.0 / slots;
-    return span + slot_cost;
-}
+constexpr int kBoxMaxOrbChunk = 32;  // orbits per item (shared-memory orbit table)
 
 BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
     BoxPlan b;
     b.tiles0 = (ctx->bn[0] + bte::kBoxTX - 1) / bte::kBoxTX;
     b.tiles1 = (ctx->bn[1] + bte::kBoxTY - 1) / bte::kBoxTY;
     b.zranges = (ctx->bn[2] + ctx->box_L - 1) / ctx->box_L;
-    const int omax = std::min(ctx->n_orb, kBoxMaxOrbChunk);
-    b.nbb = ctx->opt.band_group > 0 ? std::min<int>(ctx->opt.band_group, nbl) : 0;
-    b.oc = ctx->opt.dir_chunk > 0 ? std::max(1, std::min(omax, (int)ctx->opt.dir_chunk / 4)) : 0;
-    if (b.nbb == 0 || b.oc == 0) {
-        auto it = ctx->box_plans.find(nbl);
-        if (it != ctx->box_plans.end()) {
-            if (b.nbb == 0) b.nbb = it->second.first;
-            if (b.oc == 0) b.oc = it->second.second;
-        } else {
-            double best = 1e300;
-            int bn = 1, bo = 1;
-            for (int nbb = 1; nbb <= std::min(nbl, 8); ++nbb) {
-                if (b.nbb && nbb != b.nbb) continue;
-                for (int k = 1; k <= 16; ++k) {  // oc = ceil(n_orb / k), at most kBoxMaxOrbChunk
-                    const int oc = std::min(omax, (ctx->n_orb + k - 1) / k);
-                    if (b.oc && oc != b.oc) continue;
-                    const double t = box_makespan(ctx, b.tiles0, b.tiles1, b.zranges, nbl, nbb, oc);
-                    if (t < best * (1.0 - 1e-9)) best = t, bn = nbb, bo = oc;
-                }
+    // band-rows per item: 5 when a slice's tiles all fit in the resident CTAs
+    // (C4), else 1 so that a slice is swept quickly and neighbouring tiles stay
+    // close in time (C5); measured on B200, DESIGN.md 10
+    const int tiles = b.tiles0 * b.tiles1 * b.zranges;
+    const int auto_nbb = tiles <= ctx->sm_count * ctx->box_ctas_per_sm ? ctx->box_nbb : 1;
+    b.nbb = std::min(nbl, ctx->opt.band_group > 0 ? (int)ctx->opt.band_group : auto_nbb);
+    if (ctx->opt.dir_chunk > 0) {
+        b.oc = std::max(1, std::min({ctx->n_orb, kBoxMaxOrbChunk, (int)ctx->opt.dir_chunk / 4}));
+    } else {
+        b.oc = 1;
+        for (int c = std::min({ctx->n_orb, kBoxMaxOrbChunk, ctx->box_oc}); c >= 1; --c)
+            if (ctx->n_orb % c == 0) {
+                b.oc = c;
+                break;
             }
-            const_cast<bte_ctx *>(ctx)->box_plans[nbl] = {bn, bo};
-            if (b.nbb == 0) b.nbb = bn;
-            if (b.oc == 0) b.oc = bo;
-        }
     }
     b.n_batches = (nbl + b.nbb - 1) / b.nbb;
     b.n_chunks = (ctx->n_orb + b.oc - 1) / b.oc;
@@ -559,9 +528,22 @@ BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
 }
 
 size_t box_smem(const bte_ctx *ctx) {
-    return ((size_t)bte::kBoxStages * bte::kBoxStage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
+    const int stage = ctx->td ? bte::box_stage_elems<true>() : bte::box_stage_elems<false>();
+    return ((size_t)ctx->box_stages * stage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
                sizeof(double) +
-           (size_t)std::min(ctx->n_orb, kBoxMaxOrbChunk) * sizeof(bte::BoxOrbit);
+           (size_t)kBoxMaxOrbChunk * sizeof(bte::BoxOrbitC);
+}
+
+template <bool TD>
+bte_status box_setup_kernel(bte_ctx *ctx) {
+    const size_t smem = box_smem(ctx);
+    CUDA_TRY(ctx, cudaFuncSetAttribute(bte::flux_box_kernel<TD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem));
+    int occ = 0;
+    CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bte::flux_box_kernel<TD>, bte::kBoxThreads,
+                                                                smem));
+    ctx->box_ctas_per_sm = std::max(1, occ);
+    return BTE_OK;
 }
 
 // ------------------------------------------------------------- launch plan
@@ -637,18 +619,17 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     p.L = ctx->box_L;
     p.n_orb = ctx->n_orb;
     p.nc = ctx->nc;
+    p.stages = ctx->box_stages;
     p.zside[0] = ctx->bzside[0];
     p.zside[1] = ctx->bzside[1];
+    p.rsel_cur = ctx->rsel;
+    p.rsel_next = 1 - ctx->rsel;
+    p.dt = dt;
     for (int a = 0; a < 3; ++a) p.g[a] = ctx->bgeo[a];
     p.orb = ctx->orb;
     p.dirs = ctx->dirs_box;
     p.part = ctx->part;
     const size_t smem = box_smem(ctx);
-    static size_t attr = 0;  // > 48 KB of dynamic shared memory needs an opt-in
-    if (attr < smem) {
-        CUDA_TRY(ctx, cudaFuncSetAttribute(bte::flux_box_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr = smem;
-    }
     int slot = 0;
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
         const int nbl = std::min(ctx->n_spare, ctx->nb_loc - l0);
@@ -659,6 +640,7 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
         p.n_chunks = bp.n_chunks;
         p.orb_chunk = bp.oc;
         p.nbb = bp.nbb;
+        p.n_slices = bp.n_batches * bp.n_chunks;
         p.nbl = nbl;
         p.band0 = l0;
         p.slot0 = slot;
@@ -669,16 +651,23 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
             p.dtit[k] = dt * ctx->h_inv_tau[b];
             p.kv[k] = dt * ctx->h_vg[b];
             p.cw[k] = ctx->h_cw[b];
+            p.inv_v[k] = 1.0 / ctx->h_vg[b];
         }
         ctx->dir_chunks = bp.n_chunks;
         ctx->st.band_group = bp.nbb;
-        const dim3 grid(bp.tiles0 * bp.tiles1 * bp.zranges, bp.n_batches * bp.n_chunks);
+        const int64_t items = (int64_t)bp.tiles0 * bp.tiles1 * bp.zranges * p.n_slices;
+        if (items > INT32_MAX) return set_err(&ctx->err, "box kernel: %lld work items", (long long)items), BTE_EINVAL;
+        const dim3 grid((unsigned)items);
         ev_mark(ctx, kPhFlux, true);
-        bte::flux_box_kernel<<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(p, ctx->tm_in, ctx->tm_out,
-                                                                                 ctx->tm_i0, ctx->tm_side);
+        if (ctx->td)
+            bte::flux_box_kernel<true><<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(
+                p, ctx->tm_in, ctx->tm_out, ctx->tm_i0, ctx->tm_side, ctx->tm_rate);
+        else
+            bte::flux_box_kernel<false><<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(
+                p, ctx->tm_in, ctx->tm_out, ctx->tm_i0, ctx->tm_side, ctx->tm_rate);
         ev_mark(ctx, kPhFlux, false);
         ctx->st.kernel_launches++;
-        slot += bp.n_batches * bp.n_chunks;
+        slot += p.n_slices;
         CUDA_TRY(ctx, cudaGetLastError());
         for (int k = 0; k < nbl; ++k) std::swap(ctx->cur_slot[l0 + k], ctx->spare_slot[k]);
     }
@@ -1289,13 +1278,16 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->bzside[0] = bx.zside[0];
         ctx->bzside[1] = bx.zside[1];
         ctx->n_orb = (int)orbs.size();
-        ctx->box_L = std::min<int>(8, bx.n[2]);
-        int occ = 0;
-        CREATE_CUDA(cudaFuncSetAttribute(bte::flux_box_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)box_smem(ctx)));
-        CREATE_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bte::flux_box_kernel, bte::kBoxThreads,
-                                                                  box_smem(ctx)));
-        ctx->box_ctas_per_sm = std::max(1, occ);
+        // shared memory for 2 CTAs per SM: ring stages x 12 KB + 16 KB output + L x 2 KB energy
+        const char *ev = std::getenv("BTE_BOX_STAGES");
+        ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : 6));
+        ev = std::getenv("BTE_BOX_L");
+        ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : 8));
+        ev = std::getenv("BTE_BOX_NBB");
+        if (ev) ctx->box_nbb = std::max(1, std::atoi(ev));
+        ev = std::getenv("BTE_BOX_OC");
+        if (ev) ctx->box_oc = std::max(1, std::atoi(ev));
+        CREATE_TRY(ctx->td ? box_setup_kernel<true>(ctx) : box_setup_kernel<false>(ctx));
     }
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
@@ -1416,7 +1408,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         if (!encode_map(&ctx->tm_in, ctx->pool, 5, dpool, spool, bin) ||
             !encode_map(&ctx->tm_out, ctx->pool, 5, dpool, spool, bout) ||
             !encode_map(&ctx->tm_i0, ctx->i0, 4, di0, si0, bout) ||
-            !encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin)) {
+            !encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin) ||
+            !encode_map(&ctx->tm_rate, ctx->i0, 4, di0, si0, bout)) {  // (rate tables: N1, below)
             set_err(&ctx->err, "cuTensorMapEncodeTiled failed for the box kernel maps");
             return fail(BTE_ECUDA);
         }

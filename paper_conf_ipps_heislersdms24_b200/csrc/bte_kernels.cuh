@@ -730,15 +730,15 @@ constexpr int kBoxBY = kBoxTY + 1;           // own rows + the upwind halo row
 constexpr int kBoxBoxElems = kBoxBX * kBoxBY;  // 306 doubles copied per plane
 constexpr int kBoxPlane = 320;               // doubles per staged plane (128-byte aligned)
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
-constexpr int kBoxStage = 4 * kBoxPlane + kBoxCells;  // 4 direction planes + the I0 row
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
-#ifndef BTE_BOX_STAGES
-#define BTE_BOX_STAGES 6
-#endif
+constexpr int kBoxMaxStages = 12;
 #ifndef BTE_BOX_MIN_BLOCKS
 #define BTE_BOX_MIN_BLOCKS 2
 #endif
-constexpr int kBoxStages = BTE_BOX_STAGES;
+// doubles per stage: 4 direction planes + the I0 row (+ the two rate rows with
+// temperature-dependent relaxation times)
+template <bool TD>
+constexpr int box_stage_elems() { return 4 * kBoxPlane + (TD ? 3 : 1) * kBoxCells; }
 
 // One orbit of directions under the two in-plane mirrors.  Slot j has
 // s_0 > 0 for even j, s_0 < 0 for odd j; s_1 > 0 for j < 2, s_1 < 0 for j >= 2;
@@ -751,21 +751,25 @@ struct BoxOrbit {
 struct BoxParams {
     int32_t n0, n1, n2;        // grid extents, axis 0 contiguous
     int32_t tiles0, tiles1;    // 32-cell tiles along axis 0, 8-cell tiles along axis 1
-    int32_t L, zranges;        // layers per CTA, ranges along axis 2
-    int32_t n_orb, orb_chunk, n_chunks;  // orbits, orbits per CTA, chunks
-    int32_t nbl, nbb;          // band-rows in this launch, band-rows per CTA
+    int32_t L, zranges;        // layers per work item, ranges along axis 2
+    int32_t n_orb, orb_chunk, n_chunks;  // orbits, orbits per item, chunks
+    int32_t nbl, nbb, n_slices;  // band-rows in this launch, band-rows per item, band batches x chunks
     int32_t band0, slot0;      // rank-local first band-row; first energy slot
     int32_t nc;
+    int32_t stages;            // shared-memory ring depth
     int32_t zside[2];          // axis-2 low / high side: 0 isothermal, 1 specular
+    int32_t rsel_cur, rsel_next;  // temperature-dependent rates: table halves (current, next)
+    double dt;
     double g[3];               // A_f / V_c per axis (uniform grid)
     const BoxOrbit *orb;       // [n_orb]
     const double4 *dirs;       // [nd] {s_0, s_1, s_2, w} in grid axes
     double *part;              // [n_slots][nc] energy partials
     int32_t in_slab[kMaxBandsPerLaunch];   // launch-local band-row -> slab of I^n
     int32_t out_slab[kMaxBandsPerLaunch];  // ... slab of I^{n+1}
-    double dtit[kMaxBandsPerLaunch];       // dt / tau_b
+    double dtit[kMaxBandsPerLaunch];       // dt / tau_b (constant rates)
     double kv[kMaxBandsPerLaunch];         // dt v_b
-    double cw[kMaxBandsPerLaunch];         // temperature weight c_b
+    double cw[kMaxBandsPerLaunch];         // temperature weight c_b (constant rates)
+    double inv_v[kMaxBandsPerLaunch];      // 1 / v_b (R2 weight rate / v_b with rate tables)
 };
 
 __device__ __forceinline__ void tma_load_5d(void *dst, const void *tmap, int c0, int c1, int c2, int c3, int c4,
@@ -797,70 +801,122 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ void fence_smem_to_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void bar_compute() { asm volatile("bar.sync 1, %0;" ::"n"(kBoxCells) : "memory"); }
 
-// Tensor maps (host-encoded, see bte_api.cu box_maps):
+// Tensor maps (host-encoded, see bte_api.cu):
 //   tm_in   the slab pool as {n0, n1, n2, nd, n_slabs}, box {34, 9, 1, 1, 1}
 //   tm_out  same tensor, box {32, 8, 1, 1, 1} (stores)
 //   tm_i0   I0 table as {n0, n1, n2, nb_loc}, box {32, 8, 1, 1}
 //   tm_side isothermal axis-2 side tables as {n0, n1, 2, nb_loc}, box {34, 9, 1, 1}
+//   tm_rate rate tables 1/tau_b(T) as {n0, n1, n2, nb_loc, 2}, box {32, 8, 1, 1, 1}
 // Box origin of slot j: axis 0 at x0 - 2 (s_0 > 0: upwind is x - 1) or x0
 // (s_0 < 0: x + 1); axis 1 at y0 - 1 (s_1 > 0) or y0.
 __device__ __forceinline__ int box_xs(int j) { return (j & 1) ? 0 : 2; }
 __device__ __forceinline__ int box_hy(int j) { return (j & 2) ? 0 : 1; }
 
-__global__ void __launch_bounds__(kBoxThreads, BTE_BOX_MIN_BLOCKS)
-flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUtensorMap tm_in,
-                const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_i0,
-                const __grid_constant__ CUtensorMap tm_side) {
-    extern __shared__ __align__(128) double bsm[];
-    double *ring = bsm;                                  // [kBoxStages][kBoxStage]
-    double *obuf = ring + kBoxStages * kBoxStage;        // [2][4][256]
-    double *eacc = obuf + 2 * 4 * kBoxCells;             // [L][256]
-    BoxOrbit *sorb = reinterpret_cast<BoxOrbit *>(eacc + p.L * kBoxCells);  // [orb_chunk]
-    __shared__ __align__(8) uint64_t full[kBoxStages];
-    __shared__ __align__(8) uint64_t empty[kBoxStages];
-
-    const int tid = threadIdx.x;
-    int t = blockIdx.x;
+// Work item = (band batch x orbit chunk "slice", 32 x 8 x L cell block "tile"),
+// tile fastest, one CTA per item: the hardware block scheduler balances the
+// SMs (measured better on B200 than persistent CTAs with static or
+// counter-based item assignment) and the resident CTAs work on
+// neighbouring tiles of the same slice, so their halo boxes are L2 hits.
+struct BoxItem {
+    int x0, y0, z0, Lc, k0, k1, o0, o1, slice;
+};
+__device__ __forceinline__ BoxItem box_item(const BoxParams &p, int item) {
+    const int n_tiles = p.tiles0 * p.tiles1 * p.zranges;
+    BoxItem w;
+    w.slice = item / n_tiles;
+    int t = item - w.slice * n_tiles;
     const int t0 = t % p.tiles0;
     t /= p.tiles0;
     const int t1 = t % p.tiles1;
     const int zr = t / p.tiles1;
-    const int x0 = t0 * kBoxTX, y0 = t1 * kBoxTY, z0 = zr * p.L;
-    const int Lc = min(p.L, p.n2 - z0);
-    const int chunk = blockIdx.y % p.n_chunks;
-    const int batch = blockIdx.y / p.n_chunks;
-    const int k0 = batch * p.nbb, k1 = min(p.nbl, k0 + p.nbb);
-    const int o0 = chunk * p.orb_chunk, o1 = min(p.n_orb, o0 + p.orb_chunk);
+    w.x0 = t0 * kBoxTX;
+    w.y0 = t1 * kBoxTY;
+    w.z0 = zr * p.L;
+    w.Lc = min(p.L, p.n2 - w.z0);
+    const int chunk = w.slice % p.n_chunks, batch = w.slice / p.n_chunks;
+    w.k0 = batch * p.nbb;
+    w.k1 = min(p.nbl, w.k0 + p.nbb);
+    w.o0 = chunk * p.orb_chunk;
+    w.o1 = min(p.n_orb, w.o0 + p.orb_chunk);
+    return w;
+}
 
+// Per-orbit constants of a CTA's chunk, formed once in the prologue: the four
+// direction ids and weights, the axis-2 mirrors, |s . g| per axis (the same
+// for the 4 slots) and the marching order along axis 2.
+struct BoxOrbitC {
+    int32_t d[4], rz[4];
+    double w[4];
+    double a[3];
+    int32_t asc;
+    int32_t pad;
+};
+
+template <bool TD>
+__global__ void __launch_bounds__(kBoxThreads, BTE_BOX_MIN_BLOCKS)
+flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUtensorMap tm_in,
+                const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_i0,
+                const __grid_constant__ CUtensorMap tm_side, const __grid_constant__ CUtensorMap tm_rate) {
+    constexpr int kStage = box_stage_elems<TD>();
+    extern __shared__ __align__(128) double bsm[];
+#ifdef BTE_BOX_FIXED_S
+    constexpr int S = BTE_BOX_FIXED_S;
+#else
+    const int S = p.stages;
+#endif
+    double *ring = bsm;                          // [S][kStage]
+    double *obuf = ring + S * kStage;            // [2][4][256]
+    double *eacc = obuf + 2 * 4 * kBoxCells;     // [L][256]
+    BoxOrbitC *sorb = reinterpret_cast<BoxOrbitC *>(eacc + p.L * kBoxCells);  // [orb_chunk]
+    __shared__ __align__(8) uint64_t full[kBoxMaxStages];
+    __shared__ __align__(8) uint64_t empty[kBoxMaxStages];
+
+    const int tid = threadIdx.x;
+    const BoxItem w = box_item(p, blockIdx.x);
     if (tid == 0) {
-        for (int s = 0; s < kBoxStages; ++s) {
+        for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], kBoxCells / 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    for (int i = tid; i < o1 - o0; i += kBoxThreads) sorb[i] = p.orb[o0 + i];
+    for (int i = tid; i < w.o1 - w.o0; i += kBoxThreads) {
+        const BoxOrbit ob = p.orb[w.o0 + i];
+        BoxOrbitC c;
+        for (int q = 0; q < 4; ++q) {
+            c.d[q] = ob.d[q];
+            c.rz[q] = ob.rz[q];
+            c.w[q] = load_dir(p.dirs, ob.d[q]).w;
+        }
+        const double4 s0 = load_dir(p.dirs, ob.d[0]);
+        c.a[0] = fabs(s0.x * p.g[0]);
+        c.a[1] = fabs(s0.y * p.g[1]);
+        c.a[2] = fabs(s0.z * p.g[2]);
+        c.asc = s0.z >= 0.0;
+        c.pad = 0;
+        sorb[i] = c;
+    }
     __syncthreads();
 
     if (tid >= kBoxCells) {  // ------------------------------------------- producer warp
         if (tid == kBoxCells) {
-            uint32_t it = 0;
-            for (int k = k0; k < k1; ++k) {
+            int s = 0;
+            uint32_t ph = 0, wrapped = 0;  // ring slot, its use parity, ring wrapped once
+            for (int k = w.k0; k < w.k1; ++k) {
                 const int slab = p.in_slab[k], bl = p.band0 + k;
-                for (int o = o0; o < o1; ++o) {
-                    const BoxOrbit ob = sorb[o - o0];
-                    const bool asc = __ldg(&p.dirs[ob.d[0]].z) >= 0.0;
-                    for (int j = 0; j <= Lc; ++j, ++it) {
-                        const int s = it % kBoxStages;
-                        if (it >= kBoxStages)
-                            while (!mbar_try_wait(&empty[s], ((it / kBoxStages) - 1) & 1)) {
+                for (int o = w.o0; o < w.o1; ++o) {
+                    const BoxOrbitC &ob = sorb[o - w.o0];
+                    const bool asc = ob.asc;
+                    for (int j = 0; j <= w.Lc; ++j) {
+                        if (wrapped)
+                            while (!mbar_try_wait(&empty[s], ph ^ 1u)) {
                             }
-                        double *st = ring + s * kBoxStage;
+                        double *st = ring + s * kStage;
                         if (j == 0) {  // the upwind layer of the range: neighbour range or ghost layer
-                            const int zh = asc ? z0 - 1 : z0 + Lc;
+                            const int zh = asc ? w.z0 - 1 : w.z0 + w.Lc;
                             mbar_arrive_expect_tx(&full[s], 4 * kBoxBoxElems * sizeof(double));
                             for (int q = 0; q < 4; ++q) {
-                                const int xs = x0 - box_xs(q), ys = y0 - box_hy(q);
+                                const int xs = w.x0 - box_xs(q), ys = w.y0 - box_hy(q);
                                 if (zh >= 0 && zh < p.n2)
                                     tma_load_5d(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
                                 else if (p.zside[asc ? 0 : 1] == 0)  // isothermal: I0_b(T_wall) side table
@@ -870,12 +926,24 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                                                 slab, &full[s]);
                             }
                         } else {
-                            const int z = asc ? z0 + j - 1 : z0 + Lc - j;
-                            mbar_arrive_expect_tx(&full[s], (4 * kBoxBoxElems + kBoxCells) * sizeof(double));
+                            const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
+                            mbar_arrive_expect_tx(&full[s],
+                                                  (4 * kBoxBoxElems + (TD ? 3 : 1) * kBoxCells) * sizeof(double));
                             for (int q = 0; q < 4; ++q)
-                                tma_load_5d(st + q * kBoxPlane, &tm_in, x0 - box_xs(q), y0 - box_hy(q), z, ob.d[q],
-                                            slab, &full[s]);
-                            tma_load_4d(st + 4 * kBoxPlane, &tm_i0, x0, y0, z, bl, &full[s]);
+                                tma_load_5d(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
+                                            ob.d[q], slab, &full[s]);
+                            tma_load_4d(st + 4 * kBoxPlane, &tm_i0, w.x0, w.y0, z, bl, &full[s]);
+                            if (TD) {
+                                tma_load_5d(st + 4 * kBoxPlane + kBoxCells, &tm_rate, w.x0, w.y0, z, bl,
+                                            p.rsel_cur, &full[s]);
+                                tma_load_5d(st + 4 * kBoxPlane + 2 * kBoxCells, &tm_rate, w.x0, w.y0, z, bl,
+                                            p.rsel_next, &full[s]);
+                            }
+                        }
+                        if (++s == S) {
+                            s = 0;
+                            ph ^= 1u;
+                            wrapped = 1;
                         }
                     }
                 }
@@ -885,8 +953,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     }
 
     // ------------------------------------------------------------------ compute warps
-    const int tx = tid & 31, ty = tid >> 5;
-    const int gx = x0 + tx, gy = y0 + ty;
+    const int tx = tid & 31, ty = tid >> 5, lane = tid & 31;
+    const int gx = w.x0 + tx, gy = w.y0 + ty;
     const bool valid = gx < p.n0 && gy < p.n1;
     // staged-plane offsets of this thread: own value, axis-0 and axis-1 upwind
     // values per slot (walls: the mirrored slot's own value, Eq. 6 specular)
@@ -900,72 +968,83 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         ux[q] = wall0 ? own[q ^ 1] : own[q] + ((q & 1) ? 1 : -1);
         uy[q] = wall1 ? own[q ^ 2] : own[q] + ((q & 2) ? kBoxBX : -kBoxBX);
     }
-    for (int l = 0; l < Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
+    for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
 
-    uint32_t it = 0, ob = 0;
-    int sp = 0;
-    const int lane = tid & 31;
-    for (int k = k0; k < k1; ++k) {
-        const double dtit = p.dtit[k], kv = p.kv[k], cw = p.cw[k];
-        for (int o = o0; o < o1; ++o) {
-            const BoxOrbit orb = sorb[o - o0];
-            double w[4];
+    int s = 0, sp = 0;
+    uint32_t ph = 0, ob = 0;
+    for (int k = w.k0; k < w.k1; ++k) {
+        const double kv = p.kv[k];
+        for (int o = w.o0; o < w.o1; ++o) {
+            const BoxOrbitC &orb = sorb[o - w.o0];
+            const bool asc = orb.asc;
+            double wq[4];
 #pragma unroll
-            for (int q = 0; q < 4; ++q) w[q] = __ldg(&p.dirs[orb.d[q]].w);
-            const double4 s0 = load_dir(p.dirs, orb.d[0]);
-            const bool asc = s0.z >= 0.0;
-            // -|s . g| per axis and the outflow sum: the same for the 4 slots
-            const double a0 = fabs(s0.x * p.g[0]), a1 = fabs(s0.y * p.g[1]), a2 = fabs(s0.z * p.g[2]);
-            const double coef = (1.0 - dtit) - kv * ((a0 + a1) + a2);
-            const double m0 = -a0, m1 = -a1, m2 = -a2;
-            for (int j = 0; j <= Lc; ++j, ++it) {
-                const int s = it % kBoxStages;
-                while (!mbar_try_wait(&full[s], (it / kBoxStages) & 1)) {
+            for (int q = 0; q < 4; ++q) wq[q] = orb.w[q];
+            const double kvout = kv * ((orb.a[0] + orb.a[1]) + orb.a[2]);
+            const double coef_c = (1.0 - p.dtit[k]) - kvout;  // constant rates
+            const double m0 = -orb.a[0], m1 = -orb.a[1], m2 = -orb.a[2];
+            for (int j = 0; j <= w.Lc; ++j) {
+                while (!mbar_try_wait(&full[s], ph)) {
                 }
                 if (j == 0) {
                     sp = s;
-                    continue;
-                }
-                const int z = asc ? z0 + j - 1 : z0 + Lc - j;
-                const double *cur = ring + s * kBoxStage;
-                const double *prv = ring + sp * kBoxStage;
-                const double src = dtit * cur[4 * kBoxPlane + tid];
-                double *out = obuf + ob * (4 * kBoxCells);
-                double acc = 0.0;
+                } else {
+                    const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
+                    const double *cur = ring + s * kStage;
+                    const double *prv = ring + sp * kStage;
+                    double dtit, coef, cw;
+                    if (TD) {  // 1/tau_b of this cell at the rate temperature; R2 weight at the next one
+                        dtit = p.dt * cur[4 * kBoxPlane + kBoxCells + tid];
+                        coef = (1.0 - dtit) - kvout;
+                        cw = cur[4 * kBoxPlane + 2 * kBoxCells + tid] * p.inv_v[k];
+                    } else {
+                        dtit = p.dtit[k];
+                        coef = coef_c;
+                        cw = p.cw[k];
+                    }
+                    const double src = dtit * cur[4 * kBoxPlane + tid];
+                    double *out = obuf + ob * (4 * kBoxCells);
+                    double acc = 0.0;
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const double ic = cur[own[q]];
-                    double infl = m0 * cur[ux[q]];
-                    infl = fma(m1, cur[uy[q]], infl);
-                    infl = fma(m2, prv[own[q]], infl);
-                    const double inew = fma(ic, coef, fma(-kv, infl, src));
-                    out[q * kBoxCells + tid] = inew;
-                    acc = fma(w[q], inew, acc);
-                }
-                double *ea = eacc + (z - z0) * kBoxCells + tid;
-                *ea = fma(cw, acc, *ea);
-                __syncwarp();
-                if (lane == 0) {  // the previous layer's stage is no longer needed
-                    mbar_arrive(&empty[sp]);
-                    if (j == Lc) mbar_arrive(&empty[s]);
-                }
-                sp = s;
-                fence_smem_to_async();
-                if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
-                bar_compute();
-                if (tid == 0) {
+                    for (int q = 0; q < 4; ++q) {
+                        const double ic = cur[own[q]];
+                        double infl = m0 * cur[ux[q]];
+                        infl = fma(m1, cur[uy[q]], infl);
+                        infl = fma(m2, prv[own[q]], infl);
+                        const double inew = fma(ic, coef, fma(-kv, infl, src));
+                        out[q * kBoxCells + tid] = inew;
+                        acc = fma(wq[q], inew, acc);
+                    }
+                    double *ea = eacc + (z - w.z0) * kBoxCells + tid;
+                    *ea = fma(cw, acc, *ea);
+                    __syncwarp();
+                    if (lane == 0) {  // the previous layer's stage is no longer needed
+                        mbar_arrive(&empty[sp]);
+                        if (j == w.Lc) mbar_arrive(&empty[s]);
+                    }
+                    sp = s;
+                    fence_smem_to_async();
+                    if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
+                    bar_compute();
+                    if (tid == 0) {
 #pragma unroll
-                    for (int q = 0; q < 4; ++q)
-                        tma_store_5d(&tm_out, out + q * kBoxCells, x0, y0, z, orb.d[q], p.out_slab[k]);
-                    bulk_commit();
+                        for (int q = 0; q < 4; ++q)
+                            tma_store_5d(&tm_out, out + q * kBoxCells, w.x0, w.y0, z, orb.d[q], p.out_slab[k]);
+                        bulk_commit();
+                    }
+                    ob ^= 1u;
                 }
-                ob ^= 1u;
+                if (++s == S) {
+                    s = 0;
+                    ph ^= 1u;
+                }
             }
         }
     }
     if (valid) {
-        double *part = p.part + (int64_t)(p.slot0 + blockIdx.y) * p.nc;
-        for (int l = 0; l < Lc; ++l) part[((int64_t)(z0 + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
+        double *part = p.part + (int64_t)(p.slot0 + w.slice) * p.nc;
+        for (int l = 0; l < w.Lc; ++l)
+            part[((int64_t)(w.z0 + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
     if (tid == 0) bulk_wait_all();
 }

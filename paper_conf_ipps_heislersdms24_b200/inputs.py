@@ -235,10 +235,25 @@ def gen_bands_custom(omega, vg, tau, C, polarization=None, d_omega=None):
     }
 
 
+def with_rate_law(bands, a=TAU_A, b=TAU_B, theta=TAU_THETA):
+    """Temperature-dependent relaxation times: the same
+    placeholder law as gen_bands_si's constant tau, kept as a function of the
+    cell temperature, 1/tau_b(T) = a w^4 + b w^2 T exp(-theta/T), i.e. per row
+    rate_a = a w^4, rate_b = b w^2, rate_theta = theta (external, Si-like)."""
+    w = np.asarray(bands["omega"], dtype=np.float64)
+    out = dict(bands)
+    out["rate_a"] = a * w ** 4
+    out["rate_b"] = b * w ** 2
+    out["rate_theta"] = np.full(w.size, float(theta))
+    return out
+
+
 def select_bands(bands, rows):
     rows = np.asarray(rows)
     out = dict(bands)
-    for key in ("omega", "d_omega", "vg", "tau", "polarization", "C"):
+    keys = ["omega", "d_omega", "vg", "tau", "polarization", "C"]
+    keys += [k for k in ("rate_a", "rate_b", "rate_theta") if bands.get(k) is not None]
+    for key in keys:
         out[key] = bands[key][rows].copy()
     out["n_bands"] = int(rows.size)
     return out
@@ -336,16 +351,21 @@ def ic_multiplier(nd, nc, band, eps, seed=SEED):
     return 1.0 + eps * rng.uniform(-1.0, 1.0, size=(nd, nc))
 
 
-def cartesian_dt_bound(mesh, bands, dirs):
+def cartesian_dt_bound(mesh, bands, dirs, t_max=None):
     """Positivity bound of the explicit step on a uniform Cartesian mesh.
 
     1 / max_b (1/tau_b + v_b S), S = max_d sum_axis |s_axis| / h_axis (one face
     per axis is outgoing; A/V = 1/h).  Only used to choose dt for the synthetic
-    configs ("dt = 0.5 x positivity bound").
+    configs ("dt = 0.5 x positivity bound").  With a rate law
+    (with_rate_law) the rates are taken at t_max (default 350 K, the hot wall).
     """
     h = np.asarray(mesh["spacing"], dtype=np.float64)
     s = np.abs(dirs["s"][:, : mesh["dim"]])
     smax = float(np.max(np.sum(s / h[None, :], axis=1)))
+    if bands.get("rate_a") is not None:
+        t = 350.0 if t_max is None else float(t_max)
+        inv_tau = bands["rate_a"] + bands["rate_b"] * t * np.exp(-bands["rate_theta"] / t)
+        return 1.0 / float(np.max(inv_tau + bands["vg"] * smax))
     inv_tau = np.where(np.isinf(bands["tau"]), 0.0, 1.0 / bands["tau"])
     return 1.0 / float(np.max(inv_tau + bands["vg"] * smax))
 

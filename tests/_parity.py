@@ -11,9 +11,9 @@ RTOL_T = 1e-9   # north star: relative 1e-9 on T
 
 def oracle_run(oracle_mod, cfg, nsteps, ic_eps=None):
     p = oracle_mod.problem_from_config(cfg)
-    I, T = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps if ic_eps is None else ic_eps)
+    I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps if ic_eps is None else ic_eps, with_tr=True)
     if nsteps:
-        I, T = p.run(I, T, cfg.dt, nsteps)
+        I, T, Tr = p.run(I, T, cfg.dt, nsteps, Tr=Tr)
     return I, T
 
 
