@@ -139,7 +139,7 @@ def cpu_baseline(cfg, budget_s=15.0, max_rows=16):
         I = p.equilibrium(T)
         p.reflection_map()
         t0 = time.perf_counter()
-        p.run(I, T, cfg.dt, steps)
+        p.run(I, T, cfg.dt, steps, Tr=T.copy() if p.has_rates else None)
         return time.perf_counter() - t0
 
     t1 = run(1, 1)
@@ -153,13 +153,25 @@ def cpu_baseline(cfg, budget_s=15.0, max_rows=16):
                       f"of {cfg.bands['n_bands']} band-rows, {steps} step(s), {t:.2f} s, OMP_NUM_THREADS={os.environ['OMP_NUM_THREADS']}"}
 
 
+def _bench_config(args):
+    import dataclasses
+    from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+    cfg = gen.make_config(args.config)
+    if args.ic_eps is not None:
+        cfg = dataclasses.replace(cfg, ic_eps=args.ic_eps)
+    if args.rate_law:  # N1: temperature-dependent tau, dt = 0.5 x the bound at the hot wall
+        bands = gen.with_rate_law(cfg.bands)
+        cfg = dataclasses.replace(cfg, bands=bands,
+                                  dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, bands, cfg.dirs, t_max=350.0))
+    return cfg
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle on the same workload/metric (rank 0 only)."""
     rank, world, _ = _dist()
     if rank != 0:
         return
-    from paper_conf_ipps_heislersdms24_b200 import inputs as gen
-    cfg = gen.make_config(args.config)
+    cfg = _bench_config(args)
     vals = []
     cb = None
     for i in range(args.warmup + args.steps):
@@ -172,7 +184,8 @@ def run_reference(args):
     line = {"metric": METRIC, "value": v, "unit": "updates/s", "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "higher_is_better": True, "impl": "reference", "dtype": "f64",
             "data": "synthetic", "scaling": "strong",
-            "config": {"workload": WORKLOADS[args.config], "name": args.config},
+            "config": {"workload": WORKLOADS[args.config], "name": args.config,
+                       "relaxation": "tau(T) law" if args.rate_law else "constant tau"},
             "vs_baseline": None, "cpu_baseline": cb,
             "e2e": {"value": v, "unit": "updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -193,10 +206,7 @@ def run_ours(args):
     from paper_conf_ipps_heislersdms24_b200 import bte
     from paper_conf_ipps_heislersdms24_b200 import inputs as gen
 
-    cfg = gen.make_config(args.config)
-    if args.ic_eps is not None:
-        import dataclasses
-        cfg = dataclasses.replace(cfg, ic_eps=args.ic_eps)
+    cfg = _bench_config(args)
     nccl_id = None
     if world > 1:
         from paper_conf_ipps_heislersdms24_b200.dist import share_nccl_id
@@ -317,6 +327,7 @@ def _emit(v):
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOADS[args.config], "name": args.config, "n_cells": nc, "n_dirs": nd,
                        "n_band_rows": nb, "dt": dt, "parallelism": f"band-shard x{world}",
+                       "relaxation": "tau(T) law" if args.rate_law else "constant tau",
                        "l2": f"state {nc * nd * nb * 8 / 1e9:.1f} GB per copy >> 126 MB L2 (no flush needed)"},
             "roofline": roof, "cpu_baseline": cb, "e2e": e2e, "clocks": clocks,
             "gpu_launches": st["kernel_launches"], "phases_ms_per_step": phases,
@@ -345,6 +356,8 @@ def main():
     ap.add_argument("--no-tma", action="store_true", help="register-pipelined flux kernel instead of TMA-staged")
     ap.add_argument("--stencil", action="store_true", help="stencil-staged kernel (structured order, opt-in)")
     ap.add_argument("--no-box", action="store_true", help="structured grids: TMA-staged kernel instead of the box kernel")
+    ap.add_argument("--rate-law", action="store_true",
+                    help="temperature-dependent relaxation times (SURVEY 8(f) N1) instead of constant tau")
     ap.add_argument("--ic-eps", type=float, default=None, help="override the IC perturbation (0: equilibrium IC)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")

@@ -90,9 +90,21 @@ typedef struct {
     const double *omega;         /* [n_bands] centre angular frequency, rad/s, > 0 */
     const double *d_omega;       /* [n_bands] width, rad/s (metadata; may be NULL) */
     const double *vg;            /* [n_bands] group velocity |v_g|_b, m/s, > 0 */
-    const double *tau;           /* [n_bands] relaxation time, s, in (0, +inf] */
+    const double *tau;           /* [n_bands] relaxation time, s, in (0, +inf]; ignored (may be
+                                    NULL) with the rate law below */
     const int32_t *polarization; /* [n_bands] 0 = LA, 1 = TA (metadata; may be NULL) */
     const double *i0_prefactor;  /* [n_bands] C_b > 0; required */
+    /* Optional temperature-dependent relaxation times (the paper
+     * keeps tau as a per-cell variable that depends on T, L666-669, `beta` per
+     * cell L1352-1353).  NULL rate_a: constant tau.  Else, per band-row and cell,
+     *     1/tau_b(T) = rate_a[b] + rate_b[b] T exp(-rate_theta[b] / T)   (1/s)
+     * with all three arrays >= 0 and finite.  The rates of step n are those of
+     * the cell temperature of step n-1 (reading 22): the relaxation
+     * of a step and the R2 weights 1/(v tau) of the temperature solve that
+     * ends the previous step use the same rates, so the RTA energy balance is
+     * exact.  The library keeps that rate temperature per cell: t_init at
+     * bte_create, T at bte_set_equilibrium, T^n after step n. */
+    const double *rate_a, *rate_b, *rate_theta;
 } bte_bands;
 
 /* Discrete directions (L514-518, L654-664): unit vectors and solid-angle weights. */
@@ -189,7 +201,9 @@ BTE_API bte_status bte_create(const bte_mesh *mesh, const bte_bands *bands, cons
  * (see bte_dt_bound).  ENOCONV if a cell's temperature solve failed. */
 BTE_API bte_status bte_step(bte_ctx *ctx, double dt, int64_t n);
 
-/* Largest admissible dt (the positivity bound above, over all bands). */
+/* Largest admissible dt (the positivity bound above, over all bands; with the
+ * rate law, rates at the highest temperature the state can reach: the max of
+ * t_init, the wall temperatures and the last set / solved T, P10). */
 BTE_API bte_status bte_dt_bound(const bte_ctx *ctx, double *dt_max);
 
 /* T[n_cells] (host, caller order).  T is replicated on every rank. */

@@ -44,7 +44,8 @@ class Mesh(C.Structure):
 class Bands(C.Structure):
     _fields_ = [("n_bands", C.c_int32), ("omega", C.c_void_p), ("d_omega", C.c_void_p),
                 ("vg", C.c_void_p), ("tau", C.c_void_p), ("polarization", C.c_void_p),
-                ("i0_prefactor", C.c_void_p)]
+                ("i0_prefactor", C.c_void_p), ("rate_a", C.c_void_p), ("rate_b", C.c_void_p),
+                ("rate_theta", C.c_void_p)]
 
 
 class Dirs(C.Structure):
@@ -169,11 +170,16 @@ class Solver:
             pol=i32(bands.get("polarization", np.zeros(bands["n_bands"]))), C=f64(bands["C"]),
             s=f64(dirs["s"]), w=f64(dirs["w"]), kind=i32(bcs["kind"]), tw=f64(bcs["t_wall"]),
         )
+        law = bands.get("rate_a") is not None  # temperature-dependent relaxation times (N1)
+        if law:
+            k.update(ra=f64(bands["rate_a"]), rb=f64(bands["rate_b"]), rth=f64(bands["rate_theta"]))
         self.n_cells, self.n_bands, self.n_dirs = int(mesh["n_cells"]), int(bands["n_bands"]), int(dirs["n_dirs"])
         m = Mesh(int(mesh["dim"]), self.n_cells, _p(k["off"]).value, _p(k["nbr"]).value, _p(k["area"]).value,
                  _p(k["nrm"]).value, _p(k["vol"]).value, _p(k["cen"]).value if k["cen"] is not None else None)
         b = Bands(self.n_bands, _p(k["omega"]).value, _p(k["dw"]).value, _p(k["vg"]).value, _p(k["tau"]).value,
-                  _p(k["pol"]).value, _p(k["C"]).value)
+                  _p(k["pol"]).value, _p(k["C"]).value,
+                  _p(k["ra"]).value if law else None, _p(k["rb"]).value if law else None,
+                  _p(k["rth"]).value if law else None)
         d = Dirs(self.n_dirs, _p(k["s"]).value, _p(k["w"]).value)
         bc = Bcs(int(bcs["n_bfaces"]), _p(k["kind"]).value, _p(k["tw"]).value)
         o = Options()

@@ -84,6 +84,11 @@ struct bte_ctx {
     double bgeo[3] = {0, 0, 0};
     int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
     bool td = false;  // temperature-dependent relaxation times (rate tables)
+    std::vector<double> h_ra, h_rb, h_rth, h_vg_all, h_inv_tau_all;  // rate law, constants (global rows)
+    double *d_ra = nullptr, *d_rb = nullptr, *d_rth = nullptr, *d_inv_v = nullptr;
+    double *rates = nullptr;  // [2][nb_loc][nc]: 1/tau at the rate temperature / at the current T
+    double *Tr = nullptr;     // [nc] rate temperature
+    double t_hi = 0.0;        // highest temperature the state can reach (dt bound with the law)
     bte::BoxOrbit *orb = nullptr;
     double4 *dirs_box = nullptr;
     double *side_tab = nullptr;
@@ -546,6 +551,9 @@ bte_status box_setup_kernel(bte_ctx *ctx) {
     return BTE_OK;
 }
 
+// Rate tables (N1): half `sel` of ctx->rates.
+double *rate_half(bte_ctx *ctx, int sel) { return ctx->rates + (size_t)sel * ctx->nb_loc * ctx->nc; }
+
 // ------------------------------------------------------------- launch plan
 struct LaunchPlan {
     int groups, n_dch, dchunk;
@@ -624,6 +632,7 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     p.zside[1] = ctx->bzside[1];
     p.rsel_cur = ctx->rsel;
     p.rsel_next = 1 - ctx->rsel;
+    p.rate_r2 = ctx->opt.temp_rule == 0;
     p.dt = dt;
     for (int a = 0; a < 3; ++a) p.g[a] = ctx->bgeo[a];
     p.orb = ctx->orb;
@@ -701,6 +710,11 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.refl = ctx->refl;
     p.dirs = ctx->dirs;
     p.dt = dt;
+    if (ctx->td) {
+        p.rate_cur = rate_half(ctx, ctx->rsel);
+        p.rate_next = rate_half(ctx, 1 - ctx->rsel);
+        p.rate_r2 = ctx->opt.temp_rule == 0;
+    }
     int slot = 0;
     const dim3 block(ctx->block);
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
@@ -721,6 +735,7 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
                 p.dtit[k] = dt * ctx->h_inv_tau[b];
                 p.kv[k] = dt * ctx->h_vg[b];
                 p.cw[k] = ctx->h_cw[b];
+                p.inv_v[k] = 1.0 / ctx->h_vg[b];
             }
             if (sg.off == 0) ctx->dir_chunks = lp.n_dch;
             const dim3 grid((ctx->nc + ctx->block - 1) / ctx->block, lp.groups * lp.n_dch);
@@ -737,8 +752,23 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     return BTE_OK;
 }
 
-bte_status run_newton(bte_ctx *ctx, const double *E_or_null) {
+// step: the solve that ends a step (rate temperature <- T^n, weights at T^n,
+// the new rates go to the current half, which the caller then swaps); else a
+// re-solve of the current state (weights at the kept rate temperature, the
+// new rates go to the "next" half).
+bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
     bte::NewtonParams q{};
+    if (ctx->td) {
+        q.td = 1;
+        q.tr_step = step;
+        q.r2 = ctx->opt.temp_rule == 0;
+        q.ra = ctx->d_ra;
+        q.rb = ctx->d_rb;
+        q.rth = ctx->d_rth;
+        q.inv_v = ctx->d_inv_v;
+        q.Tr = ctx->Tr;
+        q.rate_out = rate_half(ctx, step ? ctx->rsel : 1 - ctx->rsel);
+    }
     q.nc = ctx->nc;
     q.nb = ctx->nb;
     q.n_slots = ctx->n_slots_step;
@@ -758,7 +788,8 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null) {
     q.fail = ctx->d_fail;
     const int tb = 128;
     ev_mark(ctx, kPhNewton, true);
-    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, 3 * ctx->nb * sizeof(double), ctx->stream>>>(q);
+    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
+    if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
     ev_mark(ctx, kPhNewton, false);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
@@ -799,13 +830,34 @@ bte_status check_newton(bte_ctx *ctx) {
     return BTE_OK;
 }
 
+// I0 of the current T; with the rate law also Tr = T and both rate halves at T
+// (a state set to local equilibrium, bte_create / bte_set_equilibrium).
 bte_status refresh_i0(bte_ctx *ctx) {
     const int tb = 256;
-    bte::i0_table_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->T, ctx->nc, ctx->b_lo,
-                                                                          ctx->nb_loc, ctx->Cb, ctx->theta,
-                                                                          ctx->i0);
+    const int gb = (ctx->nc + tb - 1) / tb;
+    bte::i0_table_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta,
+                                                    ctx->i0);
+    if (ctx->td) {
+        CUDA_TRY(ctx, cudaMemcpyAsync(ctx->Tr, ctx->T, ctx->nc * sizeof(double), cudaMemcpyDeviceToDevice,
+                                      ctx->stream));
+        for (int h = 0; h < 2; ++h)
+            bte::rate_table_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->d_ra,
+                                                              ctx->d_rb, ctx->d_rth, rate_half(ctx, h));
+    }
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
+}
+
+// Positivity bound 1 / max_b (1/tau_b + v_b S_max); with the rate law the rates
+// at t_hi (the max principle keeps T below it, P10).
+void update_dt_bound(bte_ctx *ctx) {
+    double rate = 0.0;
+    for (int b = 0; b < ctx->nb; ++b) {
+        const double r = ctx->td ? ctx->h_ra[b] + ctx->h_rb[b] * ctx->t_hi * std::exp(-ctx->h_rth[b] / ctx->t_hi)
+                                 : ctx->h_inv_tau_all[b];
+        rate = std::max(rate, r + ctx->h_vg_all[b] * ctx->s_max);
+    }
+    ctx->dt_bound = rate > 0.0 ? 1.0 / rate : INFINITY;
 }
 
 bte_status upload_cur_slots(bte_ctx *ctx) {
@@ -851,11 +903,18 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
             if (seen[bf]++) return set_err(nullptr, "boundary face id %lld used twice", (long long)bf), BTE_EINVAL;
         }
     }
-    if (b->n_bands < 1 || !b->omega || !b->vg || !b->tau)
+    const bool law = b->rate_a != nullptr;
+    if (b->n_bands < 1 || !b->omega || !b->vg || (!b->tau && !law))
         return set_err(nullptr, "band table incomplete"), BTE_EINVAL;
+    if (law && (!b->rate_b || !b->rate_theta))
+        return set_err(nullptr, "rate law needs rate_a, rate_b and rate_theta"), BTE_EINVAL;
+    for (int i = 0; law && i < b->n_bands; ++i)
+        if (!(b->rate_a[i] >= 0.0) || !(b->rate_b[i] >= 0.0) || !(b->rate_theta[i] >= 0.0) ||
+            !std::isfinite(b->rate_a[i]) || !std::isfinite(b->rate_b[i]) || !std::isfinite(b->rate_theta[i]))
+            return set_err(nullptr, "band-row %d: rate law coefficients must be finite and >= 0", i), BTE_EINVAL;
     if (!b->i0_prefactor) return set_err(nullptr, "i0_prefactor (C_b) is required"), BTE_EINVAL;
     for (int i = 0; i < b->n_bands; ++i) {
-        if (!(b->omega[i] > 0.0) || !(b->vg[i] > 0.0) || !(b->tau[i] > 0.0) || !(b->i0_prefactor[i] > 0.0))
+        if (!(b->omega[i] > 0.0) || !(b->vg[i] > 0.0) || !(law || b->tau[i] > 0.0) || !(b->i0_prefactor[i] > 0.0))
             return set_err(nullptr, "band-row %d: omega, vg, tau, C must be > 0", i), BTE_EINVAL;
     }
     if (d->n_dirs < 1 || !d->s || !d->w) return set_err(nullptr, "direction set incomplete"), BTE_EINVAL;
@@ -924,7 +983,8 @@ void bte_destroy(bte_ctx *ctx) {
     void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
-                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col};
+                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
+                    ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -945,11 +1005,14 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- temperature weights c_b and band constants
     std::vector<double> cw(nb), theta(nb), inv_tau(nb);
     bool any_w = false;
+    const bool td = bd->rate_a != nullptr;  // rate law (N1): the constants below at t_init
     for (int b = 0; b < nb; ++b) {
-        inv_tau[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / bd->tau[b];
-        cw[b] = o->temp_rule == 1 ? 1.0 / bd->vg[b] : (std::isinf(bd->tau[b]) ? 0.0 : 1.0 / (bd->vg[b] * bd->tau[b]));
+        if (td) inv_tau[b] = bd->rate_a[b] + bd->rate_b[b] * o->t_init * std::exp(-bd->rate_theta[b] / o->t_init);
+        else inv_tau[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / bd->tau[b];
+        cw[b] = o->temp_rule == 1 ? 1.0 / bd->vg[b] : inv_tau[b] / bd->vg[b];
+        if (!td && o->temp_rule != 1) cw[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / (bd->vg[b] * bd->tau[b]);
         theta[b] = kHbar * bd->omega[b] / kKb;
-        any_w |= cw[b] > 0.0;
+        any_w |= cw[b] > 0.0 || (td && o->temp_rule == 0 && bd->rate_b[b] > 0.0);
     }
     if (!any_w) return set_err(nullptr, "all temperature weights are zero (temp_rule 0 with every tau = inf)"), BTE_EINVAL;
 
@@ -1120,7 +1183,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     const int32_t ps = (int32_t)((nc64 + bte::kTile - 1) / bte::kTile * bte::kTile);
 
     // (the paired layout's 5-bit face codes hold up to 16 specular classes)
-    const bool paired = paired_geom && (int)cls_of.size() <= bte::kMaxPairedClasses;
+    // (with the rate law only the box kernel and the generic-face kernel read rate tables)
+    const bool paired = paired_geom && (int)cls_of.size() <= bte::kMaxPairedClasses && !(td && !use_box);
     const int mf_t = paired ? m->dim : (m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
     std::vector<int32_t> nbr_h(ell), nbm_h(paired ? ell : 1, 0);
@@ -1173,6 +1237,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- context
     bte_ctx *ctx = new bte_ctx();
     ctx->opt = *o;
+    ctx->td = td;
     ctx->dim = m->dim;
     ctx->nd = nd;
     ctx->nb = nb;
@@ -1279,10 +1344,11 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->bzside[1] = bx.zside[1];
         ctx->n_orb = (int)orbs.size();
         // shared memory for 2 CTAs per SM: ring stages x 12 KB + 16 KB output + L x 2 KB energy
+        // (rate law: 16 KB stages; 5 stages x 4 layers fit twice per SM, measured best)
         const char *ev = std::getenv("BTE_BOX_STAGES");
-        ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : 6));
+        ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : (td ? 5 : 6)));
         ev = std::getenv("BTE_BOX_L");
-        ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : 8));
+        ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : (td ? 4 : 8)));
         ev = std::getenv("BTE_BOX_NBB");
         if (ev) ctx->box_nbb = std::max(1, std::atoi(ev));
         ev = std::getenv("BTE_BOX_OC");
@@ -1377,9 +1443,26 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         CREATE_CUDA(cudaMemcpyAsync(&bits, ctx->d_smax, sizeof bits, cudaMemcpyDeviceToHost, ctx->stream));
         CREATE_CUDA(cudaStreamSynchronize(ctx->stream));
         std::memcpy(&ctx->s_max, &bits, sizeof(double));
-        double rate = 0.0;
-        for (int b = 0; b < nb; ++b) rate = std::max(rate, inv_tau[b] + bd->vg[b] * ctx->s_max);
-        ctx->dt_bound = rate > 0.0 ? 1.0 / rate : INFINITY;
+        ctx->h_inv_tau_all = inv_tau;
+        ctx->h_vg_all.assign(bd->vg, bd->vg + nb);
+        ctx->t_hi = o->t_init;
+        for (int64_t f = 0; f < bc->n_bfaces; ++f)
+            if (bc->kind[f] == BTE_BC_ISOTHERMAL) ctx->t_hi = std::max(ctx->t_hi, bc->t_wall[f]);
+        if (td) {  // rate law tables: Tr = T = t_init, both halves at t_init
+            ctx->h_ra.assign(bd->rate_a, bd->rate_a + nb);
+            ctx->h_rb.assign(bd->rate_b, bd->rate_b + nb);
+            ctx->h_rth.assign(bd->rate_theta, bd->rate_theta + nb);
+            std::vector<double> iv(nb);
+            for (int b = 0; b < nb; ++b) iv[b] = 1.0 / bd->vg[b];
+            CREATE_TRY(upload(ctx, &ctx->d_ra, ctx->h_ra));
+            CREATE_TRY(upload(ctx, &ctx->d_rb, ctx->h_rb));
+            CREATE_TRY(upload(ctx, &ctx->d_rth, ctx->h_rth));
+            CREATE_TRY(upload(ctx, &ctx->d_inv_v, iv));
+            CREATE_TRY(dalloc(ctx, &ctx->rates, (size_t)2 * nb_loc * nc));
+            CREATE_TRY(dalloc(ctx, &ctx->Tr, (size_t)nc));
+            CREATE_TRY(refresh_i0(ctx));
+        }
+        update_dt_bound(ctx);
     }
     if (ctx->box) {  // orbit table, grid-axis directions, isothermal side tables, tensor maps
         CREATE_TRY(upload(ctx, &ctx->orb, orbs));
@@ -1405,11 +1488,14 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         const uint32_t bin[5] = {bte::kBoxBX, bte::kBoxBY, 1, 1, 1}, bout[5] = {bte::kBoxTX, bte::kBoxTY, 1, 1, 1};
         const uint64_t di0[4] = {n0, n1, n2, (uint64_t)nb_loc}, si0[3] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8};
         const uint64_t dsd[4] = {n0, n1, 2, (uint64_t)nb_loc}, ssd[3] = {n0 * 8, n0 * n1 * 8, 2 * n0 * n1 * 8};
+        const uint64_t drt[5] = {n0, n1, n2, (uint64_t)nb_loc, 2},
+                       srt[4] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8, (uint64_t)nb_loc * nc * 8};
         if (!encode_map(&ctx->tm_in, ctx->pool, 5, dpool, spool, bin) ||
             !encode_map(&ctx->tm_out, ctx->pool, 5, dpool, spool, bout) ||
             !encode_map(&ctx->tm_i0, ctx->i0, 4, di0, si0, bout) ||
             !encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin) ||
-            !encode_map(&ctx->tm_rate, ctx->i0, 4, di0, si0, bout)) {  // (rate tables: N1, below)
+            !encode_map(&ctx->tm_rate, ctx->td ? ctx->rates : ctx->i0, ctx->td ? 5 : 4, ctx->td ? drt : di0,
+                        ctx->td ? srt : si0, bout)) {
             set_err(&ctx->err, "cuTensorMapEncodeTiled failed for the box kernel maps");
             return fail(BTE_ECUDA);
         }
@@ -1593,13 +1679,21 @@ bte_status bte_solve_temperature(bte_ctx *ctx) {
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     STATUS_TRY(upload_cur_slots(ctx));
     const int tb = 128;
+    const bool law_r2 = ctx->td && ctx->opt.temp_rule == 0;  // weights at the kept rate temperature
     bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
         ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc,
-        ctx->E);
+        law_r2 ? rate_half(ctx, ctx->rsel) : nullptr, ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E);
     CUDA_TRY(ctx, cudaGetLastError());
     STATUS_TRY(allreduce_E(ctx));
-    STATUS_TRY(run_newton(ctx, ctx->E));
-    return check_newton(ctx);
+    STATUS_TRY(run_newton(ctx, ctx->E, /*step=*/false));
+    STATUS_TRY(check_newton(ctx));
+    if (ctx->td) {  // the dt bound follows the hottest cell of a state set from outside
+        std::vector<double> T(ctx->nc);
+        CUDA_TRY(ctx, cudaMemcpy(T.data(), ctx->T, ctx->nc * sizeof(double), cudaMemcpyDeviceToHost));
+        for (double t : T) ctx->t_hi = std::max(ctx->t_hi, t);
+        update_dt_bound(ctx);
+    }
+    return BTE_OK;
 }
 
 bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
@@ -1610,6 +1704,10 @@ bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
         if (!(T[c] > 0.0) || !std::isfinite(T[c])) return set_err(&ctx->err, "T[%d] must be > 0", c), BTE_EINVAL;
     STATUS_TRY(rows_from_host(ctx, T, ctx->nc, 1, ctx->T));
     STATUS_TRY(refresh_i0(ctx));
+    if (ctx->td) {
+        for (int32_t c = 0; c < ctx->nc; ++c) ctx->t_hi = std::max(ctx->t_hi, T[c]);
+        update_dt_bound(ctx);
+    }
     STATUS_TRY(upload_cur_slots(ctx));
     const int tb = 256;
     bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)ctx->nd * ctx->nc + tb - 1) / tb), ctx->nb_loc),

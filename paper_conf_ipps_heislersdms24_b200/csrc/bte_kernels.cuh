@@ -67,6 +67,12 @@ struct FluxParams {
     int32_t n_iso;
     const double4 *dirs;         // [nd] {s_x, s_y, s_z, w}
     double dt;
+    // temperature-dependent relaxation times (N1, generic kernel only):
+    // rate_cur / rate_next [nb_loc][nc] = 1/tau at the rate temperature of this
+    // step / at T^n (the R2 energy weight rate_next / v_b); nullptr: constants
+    const double *rate_cur, *rate_next;
+    int32_t rate_r2;                           // R2 weights from rate_next (else cw)
+    double inv_v[kMaxBandsPerLaunch];          // 1 / v_b
     const double *in_ptr[kMaxBandsPerLaunch];  // per launch-local band-row: input slab (I^n)
     double *out_ptr[kMaxBandsPerLaunch];       // ... output slab (I^{n+1})
     double dtit[kMaxBandsPerLaunch];           // dt / tau_b
@@ -144,10 +150,14 @@ flux_kernel(const __grid_constant__ FluxParams p) {
         code[j] = __ldg(p.fcode8 + q);
         has_bnd |= code[j] != kCode8Interior;
     }
-    double src[BG];
+    double src[BG], dtk[BG], cwk[BG];
 #pragma unroll
-    for (int k = 0; k < BG; ++k)  // dt/tau I0_b(T_c)
-        src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c);
+    for (int k = 0; k < BG; ++k) {  // dt/tau I0_b(T_c); the cell's rates with the rate law
+        const int64_t row = (int64_t)(p.band0 + lg0 + k) * nc + c;
+        dtk[k] = p.rate_cur ? p.dt * __ldg(p.rate_cur + row) : p.dtit[lg0 + k];
+        cwk[k] = (p.rate_cur && p.rate_r2) ? __ldg(p.rate_next + row) * p.inv_v[lg0 + k] : p.cw[lg0 + k];
+        src[k] = dtk[k] * __ldg(p.i0 + row);
+    }
     double e = 0.0;
     for (int d = d0; d < d1; ++d) {
         const double4 sd = load_dir(p.dirs, d);
@@ -187,9 +197,9 @@ flux_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
             for (int j = 0; j < MF; ++j) infl = fma(fmin(a[j], 0.0), nv[k][j], infl);
             const double kv = p.kv[lg0 + k];
-            const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
+            const double inew = fma(ic[k], (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
             __stcs(p.out_ptr[lg0 + k] + po + c, inew);
-            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
+            e = fma(cwk[k] * sd.w, inew, e);
         }
     }
     p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
@@ -759,6 +769,7 @@ struct BoxParams {
     int32_t stages;            // shared-memory ring depth
     int32_t zside[2];          // axis-2 low / high side: 0 isothermal, 1 specular
     int32_t rsel_cur, rsel_next;  // temperature-dependent rates: table halves (current, next)
+    int32_t rate_r2;           // ... R2 weights rate_next / v_b (else the constant cw)
     double dt;
     double g[3];               // A_f / V_c per axis (uniform grid)
     const BoxOrbit *orb;       // [n_orb]
@@ -996,7 +1007,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                     if (TD) {  // 1/tau_b of this cell at the rate temperature; R2 weight at the next one
                         dtit = p.dt * cur[4 * kBoxPlane + kBoxCells + tid];
                         coef = (1.0 - dtit) - kvout;
-                        cw = cur[4 * kBoxPlane + 2 * kBoxCells + tid] * p.inv_v[k];
+                        cw = p.rate_r2 ? cur[4 * kBoxPlane + 2 * kBoxCells + tid] * p.inv_v[k] : p.cw[k];
                     } else {
                         dtit = p.dtit[k];
                         coef = coef_c;
@@ -1065,13 +1076,36 @@ struct NewtonParams {
     int32_t maxit;
     int32_t *iter_max;
     int32_t *fail;
+    // temperature-dependent relaxation times (N1): 1/tau_b(T) = ra + rb T exp(-rth / T)
+    int32_t td;            // 0: constant rates (cw); 1: rate law
+    int32_t tr_step;       // 1: a step's solve (rate temperature <- T^n, weights at T^n); 0: weights at Tr
+    int32_t r2;            // R2 weights rate / v_b (else R1 cw = 1 / v_b)
+    const double *ra, *rb, *rth, *inv_v;  // [nb] global
+    double *Tr;            // [nc] rate temperature
+    double *rate_out;      // [nb_loc][nc] rates of the local rows at the new T
 };
+
+// 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
+__device__ __forceinline__ double tau_rate(double a, double b, double th, double T) {
+    return a + b * T * exp(-th / T);
+}
 
 struct Gsum { double g, gp; };
 
 // g(T) = W sum_b c_b I0_b(T) - E and g'(T), I0 = C / expm1(theta/T),
 // I0' = I0 (x/T) (1 + 1/expm1(x)), x = theta/T.
-__device__ __forceinline__ Gsum g_eval(const double *sC, const double *sTh, const double *sW,
+// Band weights of the temperature equation: the constant c_b (sW), or with the
+// rate law under R2, rate_b(Tw) / v_b at the cell's rate temperature Tw.
+struct Weights {
+    const double *sW, *ra, *rb, *rth, *iv;
+    bool law;
+    double Tw;
+    __device__ __forceinline__ double operator()(int b) const {
+        return law ? tau_rate(ra[b], rb[b], rth[b], Tw) * iv[b] : sW[b];
+    }
+};
+
+__device__ __forceinline__ Gsum g_eval(const double *sC, const double *sTh, const Weights &wt,
                                        int nb, double W, double E, double T) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
@@ -1079,26 +1113,34 @@ __device__ __forceinline__ Gsum g_eval(const double *sC, const double *sTh, cons
         const double x = sTh[b] * it;
         const double em1 = expm1(x);
         const double i0 = sC[b] / em1;
-        g = fma(sW[b], i0, g);
-        gp = fma(sW[b], i0 * (x * it) * (1.0 + 1.0 / em1), gp);
+        const double wb = wt(b);
+        g = fma(wb, i0, g);
+        gp = fma(wb, i0 * (x * it) * (1.0 + 1.0 / em1), gp);
     }
     return {W * g - E, W * gp};
 }
 
-__device__ __forceinline__ double g_only(const double *sC, const double *sTh, const double *sW,
+__device__ __forceinline__ double g_only(const double *sC, const double *sTh, const Weights &wt,
                                          int nb, double W, double E, double T) {
     double g = 0.0;
-    for (int b = 0; b < nb; ++b) g = fma(sW[b], sC[b] / expm1(sTh[b] / T), g);
+    for (int b = 0; b < nb; ++b) g = fma(wt(b), sC[b] / expm1(sTh[b] / T), g);
     return W * g - E;
 }
 
 __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
+    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
     for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
         sC[b] = p.Cb[b];
         sTh[b] = p.theta[b];
         sW[b] = p.cw[b];
+        if (p.td) {
+            sA[b] = p.ra[b];
+            sB[b] = p.rb[b];
+            sR[b] = p.rth[b];
+            sV[b] = p.inv_v[b];
+        }
     }
     __syncthreads();
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1111,12 +1153,17 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
     }
     const double T0 = p.T[c];
+    Weights wt{sW, sA, sB, sR, sV, p.td && p.r2, 0.0};
+    if (p.td) {
+        wt.Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
+        if (p.tr_step) p.Tr[c] = T0;
+    }
     double T = T0;
     bool ok = false;
     int it = 0;
     if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval(sC, sTh, sW, p.nb, p.W, E, T);
+            const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -1125,12 +1172,12 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, sW, p.nb, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, sW, p.nb, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
-            if (g_only(sC, sTh, sW, p.nb, p.W, E, lo) <= 0.0 && g_only(sC, sTh, sW, p.nb, p.W, E, hi) >= 0.0) {
+            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
+            if (g_only(sC, sTh, wt, p.nb, p.W, E, lo) <= 0.0 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) >= 0.0) {
                 for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
                     const double mid = 0.5 * (lo + hi);
-                    if (g_only(sC, sTh, sW, p.nb, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
+                    if (g_only(sC, sTh, wt, p.nb, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
                 }
                 T = 0.5 * (lo + hi);
                 ok = true;
@@ -1148,7 +1195,18 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     for (int k = 0; k < p.nb_loc; ++k) {
         const int b = p.b_lo + k;
         p.i0[(size_t)k * p.nc + c] = sC[b] / expm1(sTh[b] * iT);
+        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(sA[b], sB[b], sR[b], T);
     }
+}
+
+// Rate table of the local rows at temperature T: out[k][c] = 1/tau_{b_lo+k}(T_c).
+__global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
+                                  const double *__restrict__ ra, const double *__restrict__ rb,
+                                  const double *__restrict__ rth, double *__restrict__ out) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    const double t = T[c];
+    for (int k = 0; k < nb_loc; ++k) out[(size_t)k * nc + c] = tau_rate(ra[b_lo + k], rb[b_lo + k], rth[b_lo + k], t);
 }
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
@@ -1161,9 +1219,11 @@ __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, i
 }
 
 // E_loc[c] = sum_{local b} c_b sum_d w_d I[b][d][c] of the current state.
+// (rate: R2 with the rate law: c_b = rate[k][c] inv_v[k] at the rate temperature)
 __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__restrict__ slot,
                               int64_t slab_elems, int ps, int nb_loc, int nd, int nc,
                               const double4 *__restrict__ dirs, const double *__restrict__ cw,
+                              const double *__restrict__ rate, const double *__restrict__ inv_v,
                               double *__restrict__ E) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= nc) return;
@@ -1172,7 +1232,7 @@ __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__
         const double *s = pool + (int64_t)slot[k] * slab_elems;
         double sb = 0.0;
         for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * ps + c], sb);
-        e = fma(cw[k], sb, e);
+        e = fma(rate ? rate[(size_t)k * nc + c] * inv_v[k] : cw[k], sb, e);
     }
     E[c] = e;
 }
