@@ -801,10 +801,20 @@ __device__ __forceinline__ void tma_load_4d(void *dst, const void *tmap, int c0,
 }
 __device__ __forceinline__ void tma_store_5d(const void *tmap, const void *src, int c0, int c1, int c2, int c3,
                                              int c4) {
+#ifndef BTE_BOX_STORE_NO_HINT
+    uint64_t pol;  // I^{n+1} is not read again this step: keep L2 for the halo boxes (C5 +1.7 %)
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    asm volatile(
+        "cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group.L2::cache_hint [%0, {%2, %3, %4, %5, %6}], [%1], "
+        "%7;" ::"l"(reinterpret_cast<uint64_t>(tmap)),
+        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "l"(pol)
+        : "memory");
+#else
     asm volatile("cp.async.bulk.tensor.5d.global.shared::cta.tile.bulk_group [%0, {%2, %3, %4, %5, %6}], [%1];" ::"l"(
                      reinterpret_cast<uint64_t>(tmap)),
                  "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
                  : "memory");
+#endif
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read_all() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
