@@ -105,6 +105,96 @@ def gen_mesh(shape, spacing):
     }
 
 
+def gen_mesh_tri(shape, spacing, seed=SEED):
+    """Unstructured 2-D triangle mesh: the nx x ny quad grid
+    with every quad split along a seeded random diagonal, stored face-based
+    like gen_mesh (3 faces per cell, unit depth, outward unit normals, boundary
+    faces on the rectangle's sides with the same wall codes).  Cell 2 q is the
+    triangle holding the quad's bottom edge, 2 q + 1 the one holding its top
+    edge (q = i + nx j)."""
+    nx, ny = (int(v) for v in shape)
+    dx, dy = (float(h) for h in spacing)
+    rng = np.random.default_rng([seed, 7])
+    diag = rng.integers(0, 2, size=(ny, nx))  # 0: v00-v11, 1: v10-v01
+    dl = math.hypot(dx, dy)
+    cid = lambda i, j, t: 2 * (i + nx * j) + t
+    off, nbr, area, nrm, cen = [0], [], [], [], []
+    bcent, bwall = [], []
+
+    def owner_left(i, j):   # triangle of quad (i, j) holding its left edge
+        return cid(i, j, 1 if diag[j, i] == 0 else 0)
+
+    def owner_right(i, j):
+        return cid(i, j, 0 if diag[j, i] == 0 else 1)
+
+    for j in range(ny):
+        for i in range(nx):
+            x0, y0 = i * dx, j * dy
+            v00, v10, v01, v11 = (x0, y0), (x0 + dx, y0), (x0, y0 + dy), (x0 + dx, y0 + dy)
+            d = diag[j, i]
+            for t in (0, 1):
+                faces = []  # (neighbour or ('wall', code), area, normal, face centre)
+                if t == 0:  # holds the bottom edge
+                    faces.append((cid(i, j - 1, 1) if j > 0 else ("w", WALL_YM), dx, (0.0, -1.0), (x0 + dx / 2, y0)))
+                else:       # holds the top edge
+                    faces.append((cid(i, j + 1, 0) if j < ny - 1 else ("w", WALL_YP), dx, (0.0, 1.0),
+                                  (x0 + dx / 2, y0 + dy)))
+                holds_left = (d == 0 and t == 1) or (d == 1 and t == 0)
+                if holds_left:
+                    faces.append((owner_right(i - 1, j) if i > 0 else ("w", WALL_XM), dy, (-1.0, 0.0),
+                                  (x0, y0 + dy / 2)))
+                else:
+                    faces.append((owner_left(i + 1, j) if i < nx - 1 else ("w", WALL_XP), dy, (1.0, 0.0),
+                                  (x0 + dx, y0 + dy / 2)))
+                if d == 0:  # diagonal v00 - v11: lower-right triangle's outward normal points up-left
+                    n = (-dy / dl, dx / dl) if t == 0 else (dy / dl, -dx / dl)
+                else:       # diagonal v10 - v01: lower-left triangle's outward normal points up-right
+                    n = (dy / dl, dx / dl) if t == 0 else (-dy / dl, -dx / dl)
+                faces.append((cid(i, j, 1 - t), dl, n, (x0 + dx / 2, y0 + dy / 2)))
+                verts = {(0, 0): (v00, v10, v11), (0, 1): (v00, v11, v01),
+                         (1, 0): (v00, v10, v01), (1, 1): (v10, v11, v01)}[(d, t)]
+                cen.append((sum(v[0] for v in verts) / 3, sum(v[1] for v in verts) / 3, 0.5))
+                for nb, a, nn, fc in faces:
+                    if isinstance(nb, tuple):
+                        bwall.append(nb[1])
+                        bcent.append((fc[0], fc[1], 0.5))
+                        nbr.append(-len(bwall))
+                    else:
+                        nbr.append(nb)
+                    area.append(a)
+                    nrm.append((nn[0], nn[1], 0.0))
+                off.append(len(nbr))
+    nc = 2 * nx * ny
+    return {
+        "dim": 2, "n_cells": nc,
+        "face_offsets": np.asarray(off, np.int64), "face_nbr": np.asarray(nbr, np.int64),
+        "face_area": np.asarray(area, np.float64), "face_normal": np.asarray(nrm, np.float64),
+        "cell_volume": np.full(nc, 0.5 * dx * dy),
+        "shape": (nx, ny), "spacing": (dx, dy), "cell_centre": np.asarray(cen, np.float64),
+        "bface_centre": np.asarray(bcent, np.float64), "bface_wall": np.asarray(bwall, np.int64),
+        "n_bfaces": len(bwall), "triangles": True,
+    }
+
+
+def general_dt_bound(mesh, bands, dirs, t_max=None):
+    """Positivity bound on any face-based mesh: 1 / max_b (1/tau_b + v_b S),
+    S = max_{c,d} sum_f (A_f / V_c) max(s_d . n_f, 0) (used to pick
+    dt for the synthetic configs, as cartesian_dt_bound on Cartesian grids)."""
+    off = mesh["face_offsets"]
+    owner = np.repeat(np.arange(mesh["n_cells"]), np.diff(off))
+    g = (mesh["face_area"] / mesh["cell_volume"][owner])[:, None] * mesh["face_normal"]
+    mu = np.maximum(g @ dirs["s"].T, 0.0)  # [faces][dirs]
+    per_cell = np.zeros((mesh["n_cells"], dirs["n_dirs"]))
+    np.add.at(per_cell, owner, mu)
+    smax = float(per_cell.max())
+    if bands.get("rate_a") is not None:
+        t = 350.0 if t_max is None else float(t_max)
+        inv_tau = bands["rate_a"] + bands["rate_b"] * t * np.exp(-bands["rate_theta"] / t)
+    else:
+        inv_tau = np.where(np.isinf(bands["tau"]), 0.0, 1.0 / bands["tau"])
+    return 1.0 / float(np.max(inv_tau + bands["vg"] * smax))
+
+
 def permute_mesh(mesh, seed=SEED):
     """Random relabelling of cells and of each cell's face order (pin P11).
 
@@ -424,15 +514,31 @@ def make_config(name, variant="scaled"):
         dirs = gen_dirs_product(20, 20)
         bcs = gen_bcs_fig1(mesh, radius=4 * h)
         nsteps, eps = (100, 0.10) if name == "C4" else (20, 0.10)
+    elif name in ("C6", "C6t"):
+        # Fig. 10 (L1169-1178): a smaller, elongated material,
+        # heat source in one corner, specular left/right, isothermal bottom;
+        # colour scale 100-150 K.  Reading: 40 x 160 um (1:4), the top wall
+        # isothermal 100 K with a 150 K Gaussian (1/e^2 radius 10 um) centred on
+        # the top-left corner, bottom 100 K, IC 100 K; 10 spectral bands (13
+        # rows), the paper's 2-D set of 20 directions (L594-595).  C6t: the same
+        # domain as an unstructured triangle mesh (each quad split on a seeded
+        # random diagonal).
+        shape, h = (20, 80), 2e-6
+        mesh = gen_mesh(shape, (h, h)) if name == "C6" else gen_mesh_tri(shape, (h, h))
+        bands = gen_bands_si(10)
+        dirs = gen_dirs_inplane(20)
+        bcs = gen_bcs_fig1(mesh, t_cold=100.0, t_hot=150.0, radius=10e-6, centre=(0.0, shape[1] * h))
+        nsteps, eps = 200, 0.10
     else:
         raise ValueError(f"unknown config {name}")
-    bound = cartesian_dt_bound(mesh, bands, dirs)
+    t_init = 100.0 if name in ("C6", "C6t") else 300.0
+    bound = general_dt_bound(mesh, bands, dirs) if mesh.get("triangles") else cartesian_dt_bound(mesh, bands, dirs)
     if variant == "paper":
-        assert name == "C3"
-        dt, eps = 1e-12, 0.0
+        assert name in ("C3", "C6", "C6t")
+        dt, eps = (1e-12 if name == "C3" else 0.5 * bound), 0.0
     else:
         dt = 0.5 * bound
-    return Config(name=name, mesh=mesh, bands=bands, dirs=dirs, bcs=bcs, t_init=300.0,
+    return Config(name=name, mesh=mesh, bands=bands, dirs=dirs, bcs=bcs, t_init=t_init,
                   dt=dt, nsteps=nsteps, ic_eps=eps, extra={"dt_bound": bound})
 
 
