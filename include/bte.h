@@ -135,7 +135,10 @@ typedef struct {
 
 typedef struct {
     double t_init;            /* IC: T = t_init, I = I0_b(t_init) (L585-588, L678-684) */
-    int32_t temp_rule;        /* 0: c_b = 1/(v_b tau_b) (default); 1: c_b = 1/v_b */
+    int32_t temp_rule;        /* 0: R2, c_b = 1/(v_b tau_b) (default); 1: R1, c_b = 1/v_b (the
+                                 energy-equivalent temperature); 2: R3, one linearised
+                                 "first-law" step T + dE / C(T) with the R1 weights per step
+                                 (L413-415; reading 5) */
     double newton_rtol;       /* stop when |dT| <= rtol T (default 1e-12) */
     int32_t newton_max_iter;  /* default 50; bisection fallback after that */
     int32_t rank, world;      /* band sharding; world == 1: single GPU, no NCCL */
@@ -205,6 +208,15 @@ BTE_API bte_status bte_step(bte_ctx *ctx, double dt, int64_t n);
  * rate law, rates at the highest temperature the state can reach: the max of
  * t_init, the wall temperatures and the last set / solved T, P10). */
 BTE_API bte_status bte_dt_bound(const bte_ctx *ctx, double *dt_max);
+
+/* Temperature of the CURRENT state under `rule` (0 R2, 1 R1 energy-equivalent,
+ * 2 R3 one linearised step from the current T), without changing the state:
+ * energy reduction with that rule's weights, all-reduce (collective when
+ * world > 1), Newton from the current T.  T[n_cells] host, caller order.
+ * the paper's temperature relation is under-specified
+ * (L413-418), so the other readings are offered as outputs.  ENOCONV if a
+ * cell's solve fails; ESTATE with world > 1 and no communicator. */
+BTE_API bte_status bte_get_temperature_rule(const bte_ctx *ctx, int32_t rule, double *T);
 
 /* T[n_cells] (host, caller order).  T is replicated on every rank. */
 BTE_API bte_status bte_get_temperature(const bte_ctx *ctx, double *T);

@@ -50,7 +50,7 @@ double oracle_rate(const oracle_problem *p, int32_t b, double Tr) {
  * R2 (default): c_b = (1/tau_b) / v_b  -- tau = +inf gives 0;
  * R1:           c_b = 1/v_b. */
 double oracle_weight_at(const oracle_problem *p, int32_t b, double Tr) {
-    if (p->temp_rule == 1) return 1.0 / p->vg[b];
+    if (p->temp_rule == 1 || p->temp_rule == 2) return 1.0 / p->vg[b];
     if (!p->rate_a) {
         if (isinf(p->tau[b])) return 0.0;
         return 1.0 / (p->vg[b] * p->tau[b]);
@@ -220,6 +220,15 @@ static int bisect(const oracle_problem *p, double W, double E, double Tr, double
 static int solve_cell(const oracle_problem *p, double W, double E, double Tr, double *T, int32_t *iters) {
     double Tc = *T;
     if (!(E > 0.0) || !isfinite(E)) return ORACLE_ENOCONV;
+    if (p->temp_rule == 2) {
+        /* R3: T' = T + (E - E_eq(T)) / C(T), C = dE_eq/dT -- one linearised
+         * "first law" step from the previous temperature (L413-415). */
+        double Tn = Tc - g_of(p, W, E, Tr, Tc) / gprime_of(p, W, Tr, Tc);
+        if (!(Tn > 0.0) || !isfinite(Tn)) return ORACLE_ENOCONV;
+        *T = Tn;
+        if (iters) *iters = 1;
+        return ORACLE_OK;
+    }
     for (int32_t it = 1; it <= p->newton_maxit; ++it) {
         double delta = g_of(p, W, E, Tr, Tc) / gprime_of(p, W, Tr, Tc);
         double Tn = Tc - delta;

@@ -52,7 +52,10 @@ typedef struct {
     const int32_t *bkind;  /* 0 isothermal, 1 symmetric */
     const double *t_wall;  /* K, isothermal faces */
     /* temperature rule and Newton controls */
-    int32_t temp_rule;     /* 0: c_b = 1/(v_b tau_b) (R2), 1: c_b = 1/v_b (R1) */
+    int32_t temp_rule;     /* 0: c_b = 1/(v_b tau_b) (R2), 1: c_b = 1/v_b (R1), 2: R3 = one
+                              linearised first-law step dT = dE / C(T) with the R1 weights
+                              (L413-415 "can be approximated ... using the first law";
+                              SURVEY 8(c) #5, 8(f) N4) */
     double newton_rtol;    /* stop when |dT| <= rtol T */
     int32_t newton_maxit;
     /* Temperature-dependent relaxation times ("tau ... dependent

@@ -82,7 +82,7 @@ EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",
            "bte_band_range", "bte_step_begin", "bte_get_energy", "bte_set_energy", "bte_step_finish",
            "bte_get_stats", "bte_reset_stats", "bte_nccl_unique_id", "bte_last_error",
-           "bte_status_string", "bte_destroy"]
+           "bte_status_string", "bte_destroy", "bte_get_temperature_rule"]
 
 
 def _load():
@@ -106,6 +106,7 @@ def _load():
         "bte_step": ([vp, dbl, i64], i32),
         "bte_dt_bound": ([vp, P(dbl)], i32),
         "bte_get_temperature": ([vp, vp], i32),
+        "bte_get_temperature_rule": ([vp, i32, vp], i32),
         "bte_get_intensity": ([vp, i32, i32, vp], i32),
         "bte_set_intensity": ([vp, i32, i32, vp], i32),
         "bte_solve_temperature": ([vp], i32),
@@ -246,6 +247,12 @@ class Solver:
     def temperature(self, out=None):
         out = np.empty(self.n_cells) if out is None else out
         _check(lib.bte_get_temperature(self.ctx, _ptr_any(out)), self.ctx)
+        return out
+
+    def temperature_rule(self, rule, out=None):
+        """T of the current state under rule 0 (R2), 1 (R1) or 2 (R3), state untouched."""
+        out = np.empty(self.n_cells) if out is None else out
+        _check(lib.bte_get_temperature_rule(self.ctx, int(rule), _ptr_any(out)), self.ctx)
         return out
 
     def energy(self):

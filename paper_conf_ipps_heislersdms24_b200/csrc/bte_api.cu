@@ -85,6 +85,7 @@ struct bte_ctx {
     int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
     bool td = false;  // temperature-dependent relaxation times (rate tables)
     std::vector<double> h_ra, h_rb, h_rth, h_vg_all, h_inv_tau_all;  // rate law, constants (global rows)
+    double *E2 = nullptr, *T2 = nullptr, *cw_diag = nullptr;  // bte_get_temperature_rule scratch
     double *d_ra = nullptr, *d_rb = nullptr, *d_rth = nullptr, *d_inv_v = nullptr;
     double *rates = nullptr;  // [2][nb_loc][nc]: 1/tau at the rate temperature / at the current T
     double *Tr = nullptr;     // [nc] rate temperature
@@ -786,6 +787,7 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
+    q.single = ctx->opt.temp_rule == 2;
     const int tb = 128;
     ev_mark(ctx, kPhNewton, true);
     bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
@@ -796,10 +798,10 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
     return BTE_OK;
 }
 
-bte_status allreduce_E(bte_ctx *ctx) {
+bte_status allreduce_E(bte_ctx *ctx, double *E = nullptr) {
     if (!ctx->have_comm) return BTE_OK;
     std::string e;
-    if (!bte::nccl::allreduce_sum_f64(ctx->comm, ctx->E, ctx->nc, ctx->stream, &e)) {
+    if (!bte::nccl::allreduce_sum_f64(ctx->comm, E ? E : ctx->E, ctx->nc, ctx->stream, &e)) {
         set_err(&ctx->err, "NCCL all-reduce failed: %s", e.c_str());
         return BTE_ENCCL;
     }
@@ -928,7 +930,7 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
         if (bc->kind[f] == BTE_BC_ISOTHERMAL && !(bc->t_wall[f] > 0.0))
             return set_err(nullptr, "boundary face %lld: wall temperature <= 0", (long long)f), BTE_EINVAL;
     }
-    if (o->temp_rule != 0 && o->temp_rule != 1) return set_err(nullptr, "temp_rule must be 0 or 1"), BTE_EINVAL;
+    if (o->temp_rule < 0 || o->temp_rule > 2) return set_err(nullptr, "temp_rule must be 0, 1 or 2"), BTE_EINVAL;
     if (!(o->t_init > 0.0)) return set_err(nullptr, "t_init must be > 0"), BTE_EINVAL;
     if (o->world < 1 || o->rank < 0 || o->rank >= o->world) return set_err(nullptr, "bad rank/world"), BTE_EINVAL;
     if (!(o->newton_rtol > 0.0) || o->newton_max_iter < 1) return set_err(nullptr, "bad Newton controls"), BTE_EINVAL;
@@ -984,7 +986,8 @@ void bte_destroy(bte_ctx *ctx) {
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
-                    ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr};
+                    ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
+                    ctx->E2, ctx->T2, ctx->cw_diag};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -1009,8 +1012,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     for (int b = 0; b < nb; ++b) {
         if (td) inv_tau[b] = bd->rate_a[b] + bd->rate_b[b] * o->t_init * std::exp(-bd->rate_theta[b] / o->t_init);
         else inv_tau[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / bd->tau[b];
-        cw[b] = o->temp_rule == 1 ? 1.0 / bd->vg[b] : inv_tau[b] / bd->vg[b];
-        if (!td && o->temp_rule != 1) cw[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / (bd->vg[b] * bd->tau[b]);
+        cw[b] = o->temp_rule != 0 ? 1.0 / bd->vg[b] : inv_tau[b] / bd->vg[b];  // R1 / R3: 1/v_b
+        if (!td && o->temp_rule == 0) cw[b] = std::isinf(bd->tau[b]) ? 0.0 : 1.0 / (bd->vg[b] * bd->tau[b]);
         theta[b] = kHbar * bd->omega[b] / kKb;
         any_w |= cw[b] > 0.0 || (td && o->temp_rule == 0 && bd->rate_b[b] > 0.0);
     }
@@ -1694,6 +1697,71 @@ bte_status bte_solve_temperature(bte_ctx *ctx) {
         update_dt_bound(ctx);
     }
     return BTE_OK;
+}
+
+// Temperature of the current state under another rule (N4): energy reduction
+// with that rule's weights, all-reduce, Newton (R3: one step) from the current
+// T into scratch; the state (T, I0, rates) is not touched.
+bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T) {
+    if (!cctx || !T) return BTE_EINVAL;
+    bte_ctx *ctx = const_cast<bte_ctx *>(cctx);
+    if (rule < 0 || rule > 2) return set_err(&ctx->err, "rule must be 0, 1 or 2"), BTE_EINVAL;
+    if (ctx->begun) return BTE_ESTATE;
+    if (ctx->opt.world > 1 && !ctx->have_comm)
+        return set_err(&ctx->err, "world > 1 without a communicator: cannot reduce the energy"), BTE_ESTATE;
+    CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    if (!ctx->E2) {
+        STATUS_TRY(dalloc(ctx, &ctx->E2, (size_t)ctx->nc));
+        STATUS_TRY(dalloc(ctx, &ctx->T2, (size_t)ctx->nc));
+        STATUS_TRY(dalloc(ctx, &ctx->cw_diag, (size_t)ctx->nb));
+    }
+    std::vector<double> w(ctx->nb);
+    bool any = false;
+    for (int b = 0; b < ctx->nb; ++b) {
+        w[b] = rule != 0 ? 1.0 / ctx->h_vg_all[b] : ctx->h_inv_tau_all[b] / ctx->h_vg_all[b];
+        any |= w[b] > 0.0 || (ctx->td && ctx->h_rb[b] > 0.0);
+    }
+    if (!any) return set_err(&ctx->err, "all temperature weights are zero under rule %d", rule), BTE_EINVAL;
+    CUDA_TRY(ctx, cudaMemcpyAsync(ctx->cw_diag, w.data(), ctx->nb * sizeof(double), cudaMemcpyHostToDevice,
+                                  ctx->stream));
+    STATUS_TRY(upload_cur_slots(ctx));
+    const bool law_r2 = ctx->td && rule == 0;
+    const int tb = 128;
+    bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
+        ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs,
+        ctx->cw_diag + ctx->b_lo, law_r2 ? rate_half(ctx, ctx->rsel) : nullptr,
+        ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E2);
+    CUDA_TRY(ctx, cudaGetLastError());
+    STATUS_TRY(allreduce_E(ctx, ctx->E2));
+    bte::NewtonParams q{};
+    q.nc = ctx->nc;
+    q.nb = ctx->nb;
+    q.E = ctx->E2;
+    q.T = ctx->T;
+    q.T_out = ctx->T2;
+    q.Cb = ctx->Cb;
+    q.theta = ctx->theta;
+    q.cw = ctx->cw_diag;
+    q.W = ctx->W;
+    q.rtol = ctx->opt.newton_rtol;
+    q.maxit = ctx->opt.newton_max_iter;
+    q.iter_max = ctx->d_iter_max;
+    q.fail = ctx->d_fail;
+    q.single = rule == 2;
+    if (ctx->td) {
+        q.td = 1;
+        q.tr_step = 0;
+        q.r2 = rule == 0;
+        q.ra = ctx->d_ra;
+        q.rb = ctx->d_rb;
+        q.rth = ctx->d_rth;
+        q.inv_v = ctx->d_inv_v;
+        q.Tr = ctx->Tr;
+    }
+    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
+    CUDA_TRY(ctx, cudaGetLastError());
+    STATUS_TRY(check_newton(ctx));
+    return rows_to_host(ctx, ctx->T2, ctx->nc, 1, T);
 }
 
 bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {

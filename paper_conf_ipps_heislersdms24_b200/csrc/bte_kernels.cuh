@@ -1093,6 +1093,8 @@ struct NewtonParams {
     const double *ra, *rb, *rth, *inv_v;  // [nb] global
     double *Tr;            // [nc] rate temperature
     double *rate_out;      // [nb_loc][nc] rates of the local rows at the new T
+    int32_t single;        // R3: one linearised first-law step, no convergence test (N4)
+    double *T_out;         // diagnostic solve: write T here only (state untouched)
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1171,7 +1173,15 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     double T = T0;
     bool ok = false;
     int it = 0;
-    if (E > 0.0 && isfinite(E)) {
+    if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
+        const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+        const double Tn = T - gs.g / gs.gp;
+        it = 1;
+        if (Tn > 0.0 && isfinite(Tn)) {
+            T = Tn;
+            ok = true;
+        }
+    } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
             const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
             const double delta = gs.g / gs.gp;
@@ -1200,6 +1210,10 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         T = T0;
     }
     atomicMax(p.iter_max, it);
+    if (p.T_out) {
+        p.T_out[c] = T;
+        return;
+    }
     p.T[c] = T;
     const double iT = 1.0 / T;
     for (int k = 0; k < p.nb_loc; ++k) {

@@ -98,3 +98,35 @@ def test_n2_fig10_corner_source_stays_bounded(oracle_mod, name):
     cen = cfg.mesh["cell_centre"]
     hot = cen[np.argmax(T)]
     assert hot[0] < 0.25 * cen[:, 0].max() and hot[1] > 0.75 * cen[:, 1].max()
+
+
+# ----------------------------------------------------------------- N4 (R3 first-law step)
+def _rule_run(oracle_mod, rule, eps, steps=1, t_hot=350.0):
+    mesh = gen.gen_mesh((6, 5), (1e-6, 1e-6))
+    bands, dirs = gen.gen_bands_si(4), gen.gen_dirs_product(4, 8)
+    bcs = gen.gen_bcs_fig1(mesh, t_hot=t_hot, radius=2e-6)
+    p = oracle_mod.Problem(mesh, bands, dirs, bcs, temp_rule=rule)
+    T0 = np.full(mesh["n_cells"], 300.0)
+    I0 = p.equilibrium(T0)
+    from paper_conf_ipps_heislersdms24_b200.inputs import ic_multiplier
+    for b in range(bands["n_bands"]):
+        I0[b] *= ic_multiplier(dirs["n_dirs"], mesh["n_cells"], b, eps)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+    return p.run(I0, T0, dt, steps)
+
+
+def test_n4_r3_is_second_order_close_to_r1(oracle_mod):
+    """R3 is one Newton step of the R1 equation from T^n: its error against the
+    converged R1 temperature is quadratic in the temperature change, so halving
+    the perturbation divides the gap by ~4 (and equilibrium gives no change)."""
+    gaps, moves = [], []
+    for eps in (0.08, 0.04, 0.02):
+        _, T1 = _rule_run(oracle_mod, 1, eps)
+        _, T3 = _rule_run(oracle_mod, 2, eps)
+        gaps.append(np.max(np.abs(T3 - T1)))
+        moves.append(np.max(np.abs(T1 - 300.0)))
+    assert gaps[0] > 0 and all(g < 1e-2 * m for g, m in zip(gaps, moves))
+    r1, r2 = gaps[0] / gaps[1], gaps[1] / gaps[2]
+    assert 3.0 < r1 < 5.0 and 3.0 < r2 < 5.0, (gaps, moves)
+    _, Te = _rule_run(oracle_mod, 2, 0.0, steps=5, t_hot=300.0)  # equilibrium: nothing moves
+    assert np.max(np.abs(Te / 300.0 - 1)) < 1e-14
