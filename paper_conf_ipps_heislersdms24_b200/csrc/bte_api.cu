@@ -86,6 +86,11 @@ struct bte_ctx {
     bool td = false;  // temperature-dependent relaxation times (rate tables)
     std::vector<double> h_ra, h_rb, h_rth, h_vg_all, h_inv_tau_all;  // rate law, constants (global rows)
     double *E2 = nullptr, *T2 = nullptr, *cw_diag = nullptr;  // bte_get_temperature_rule scratch
+    // band-sharded step (world > 1 with a communicator): reduce-scatter of E,
+    // temperature solve on this rank's chunk of cells, all-gather of T
+    bool shard_newton = false;
+    int32_t nc_pad = 0, chunk = 0;
+    double *Echunk = nullptr, *Tg = nullptr;
     double *d_ra = nullptr, *d_rb = nullptr, *d_rth = nullptr, *d_inv_v = nullptr;
     double *rates = nullptr;  // [2][nb_loc][nc]: 1/tau at the rate temperature / at the current T
     double *Tr = nullptr;     // [nc] rate temperature
@@ -512,11 +517,29 @@ BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
     b.tiles0 = (ctx->bn[0] + bte::kBoxTX - 1) / bte::kBoxTX;
     b.tiles1 = (ctx->bn[1] + bte::kBoxTY - 1) / bte::kBoxTY;
     b.zranges = (ctx->bn[2] + ctx->box_L - 1) / ctx->box_L;
-    // band-rows per item: 5 when a slice's tiles all fit in the resident CTAs
-    // (C4), else 1 so that a slice is swept quickly and neighbouring tiles stay
-    // close in time (C5); measured on B200, DESIGN.md 10
+    // band-rows per item (measured on B200): up to 5 when a
+    // slice's tiles all fit in the resident CTAs (C4), the largest that still
+    // gives >= 8 waves of CTAs (band-sharded launches have few rows); 1 when a
+    // slice has more tiles than resident CTAs, so it is swept quickly and
+    // neighbouring tiles stay close in time (C5)
     const int tiles = b.tiles0 * b.tiles1 * b.zranges;
-    const int auto_nbb = tiles <= ctx->sm_count * ctx->box_ctas_per_sm ? ctx->box_nbb : 1;
+    const int64_t slots = (int64_t)ctx->sm_count * ctx->box_ctas_per_sm;
+    int oc_pre = 1;
+    for (int c = std::min({ctx->n_orb, kBoxMaxOrbChunk, ctx->box_oc}); c >= 1; --c)
+        if (ctx->n_orb % c == 0) {
+            oc_pre = c;
+            break;
+        }
+    if (ctx->opt.dir_chunk > 0) oc_pre = std::max(1, std::min({ctx->n_orb, kBoxMaxOrbChunk, (int)ctx->opt.dir_chunk / 4}));
+    int auto_nbb = 1;
+    if (tiles <= slots)
+        for (int n = std::min(nbl, ctx->box_nbb); n >= 1; --n) {
+            const int64_t ctas = (int64_t)tiles * ((nbl + n - 1) / n) * ((ctx->n_orb + oc_pre - 1) / oc_pre);
+            if (ctas >= 8 * slots) {
+                auto_nbb = n;
+                break;
+            }
+        }
     b.nbb = std::min(nbl, ctx->opt.band_group > 0 ? (int)ctx->opt.band_group : auto_nbb);
     if (ctx->opt.dir_chunk > 0) {
         b.oc = std::max(1, std::min({ctx->n_orb, kBoxMaxOrbChunk, (int)ctx->opt.dir_chunk / 4}));
@@ -757,7 +780,21 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
 // the new rates go to the current half, which the caller then swaps); else a
 // re-solve of the current state (weights at the kept rate temperature, the
 // new rates go to the "next" half).
+bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step);
+
 bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
+    bte::NewtonParams q = newton_params(ctx, E_or_null, step);
+    const int tb = 128;
+    ev_mark(ctx, kPhNewton, true);
+    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
+    ev_mark(ctx, kPhNewton, false);
+    ctx->st.kernel_launches++;
+    if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step) {
     bte::NewtonParams q{};
     if (ctx->td) {
         q.td = 1;
@@ -788,14 +825,7 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
     q.single = ctx->opt.temp_rule == 2;
-    const int tb = 128;
-    ev_mark(ctx, kPhNewton, true);
-    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
-    if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
-    ev_mark(ctx, kPhNewton, false);
-    ctx->st.kernel_launches++;
-    CUDA_TRY(ctx, cudaGetLastError());
-    return BTE_OK;
+    return q;
 }
 
 bte_status allreduce_E(bte_ctx *ctx, double *E = nullptr) {
@@ -816,6 +846,41 @@ bte_status reduce_slots(bte_ctx *ctx) {
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
 }
+
+// Band-sharded step exchange (SURVEY 8(e) alternative, no replicated solve):
+// E (slot sum, padded to world x chunk) -> reduce-scatter -> Newton on this
+// rank's chunk of cells -> all-gather of T -> every rank finishes its rows.
+bte_status shard_newton_step(bte_ctx *ctx) {
+    std::string e;
+    ev_mark(ctx, kPhAllreduce, true);
+    STATUS_TRY(reduce_slots(ctx));
+    if (!bte::nccl::reduce_scatter_sum_f64(ctx->comm, ctx->E, ctx->Echunk, ctx->chunk, ctx->stream, &e))
+        return set_err(&ctx->err, "NCCL reduce-scatter failed: %s", e.c_str()), BTE_ENCCL;
+    ev_mark(ctx, kPhAllreduce, false);
+    ev_mark(ctx, kPhNewton, true);
+    bte::NewtonParams q = newton_params(ctx, ctx->Echunk, /*step=*/true);
+    q.c_lo = ctx->opt.rank * ctx->chunk;
+    q.nc = std::max(0, std::min(ctx->chunk, ctx->nc - q.c_lo));
+    q.T_out = ctx->Tg;
+    q.neg_fail = 1;
+    const int tb = 128;
+    if (q.nc > 0) {
+        bte::newton_kernel<<<(q.nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
+        ctx->st.kernel_launches++;
+    }
+    double *mine = ctx->Tg + (size_t)ctx->opt.rank * ctx->chunk;
+    if (!bte::nccl::allgather_f64(ctx->comm, mine, ctx->Tg, ctx->chunk, ctx->stream, &e))
+        return set_err(&ctx->err, "NCCL all-gather failed: %s", e.c_str()), BTE_ENCCL;
+    bte::newton_finish_kernel<<<(ctx->nc + 255) / 256, 256, 0, ctx->stream>>>(
+        ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
+        ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail);
+    ctx->st.kernel_launches++;
+    ev_mark(ctx, kPhNewton, false);
+    if (ctx->td) ctx->rsel = 1 - ctx->rsel;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
 
 bte_status check_newton(bte_ctx *ctx) {
     int32_t h[2];
@@ -987,7 +1052,7 @@ void bte_destroy(bte_ctx *ctx) {
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
-                    ctx->E2, ctx->T2, ctx->cw_diag};
+                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -1391,7 +1456,17 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(dalloc(ctx, &ctx->part, (size_t)max_slots * nc));
     CREATE_TRY(dalloc(ctx, &ctx->i0, (size_t)nb_loc * nc));
     CREATE_TRY(dalloc(ctx, &ctx->T, (size_t)nc));
-    CREATE_TRY(dalloc(ctx, &ctx->E, (size_t)nc));
+    // E padded to world x chunk for the reduce-scatter of the sharded step
+    ctx->chunk = (int32_t)((nc64 + o->world - 1) / o->world);
+    ctx->nc_pad = ctx->chunk * o->world;
+    CREATE_TRY(dalloc(ctx, &ctx->E, (size_t)ctx->nc_pad));
+    CREATE_CUDA(cudaMemset(ctx->E, 0, (size_t)ctx->nc_pad * sizeof(double)));
+    if (ctx->have_comm) {
+        const char *ev = std::getenv("BTE_SHARD_NEWTON");  // "replicated": all-reduce + replicated solve
+        ctx->shard_newton = !(ev && std::strcmp(ev, "replicated") == 0);
+        CREATE_TRY(dalloc(ctx, &ctx->Echunk, (size_t)ctx->chunk));
+        CREATE_TRY(dalloc(ctx, &ctx->Tg, (size_t)ctx->nc_pad));
+    }
     ctx->staging_elems = std::min<int64_t>((int64_t)nd * nc, std::max<int64_t>(nc, (int64_t)8 << 20));
     CREATE_TRY(dalloc(ctx, &ctx->staging, (size_t)ctx->staging_elems));
     CREATE_TRY(upload(ctx, &ctx->d_cur_slot, ctx->cur_slot));
@@ -1547,7 +1622,9 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int64_t s = 0; s < n; ++s) {
         STATUS_TRY(run_flux(ctx, dt));
-        if (ctx->have_comm) {
+        if (ctx->have_comm && ctx->shard_newton) {
+            STATUS_TRY(shard_newton_step(ctx));
+        } else if (ctx->have_comm) {
             ev_mark(ctx, kPhAllreduce, true);
             STATUS_TRY(reduce_slots(ctx));
             STATUS_TRY(allreduce_E(ctx));

@@ -1094,7 +1094,9 @@ struct NewtonParams {
     double *Tr;            // [nc] rate temperature
     double *rate_out;      // [nb_loc][nc] rates of the local rows at the new T
     int32_t single;        // R3: one linearised first-law step, no convergence test (N4)
-    double *T_out;         // diagnostic solve: write T here only (state untouched)
+    double *T_out;         // diagnostic / chunk solve: write T here only (state untouched)
+    int32_t c_lo;          // chunk solve: cells [c_lo, c_lo + nc) of the mesh, E indexed from c_lo
+    int32_t neg_fail;      // chunk solve: a failed cell writes -T^n (decoded by newton_finish_kernel)
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1155,11 +1157,12 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         }
     }
     __syncthreads();
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= p.nc) return;
+    const int cl = blockIdx.x * blockDim.x + threadIdx.x;  // chunk-local index
+    if (cl >= p.nc) return;
+    const int c = p.c_lo + cl;
     double E;
     if (p.E) {
-        E = p.E[c];
+        E = p.E[cl];
     } else {
         E = 0.0;
         for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
@@ -1168,7 +1171,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     Weights wt{sW, sA, sB, sR, sV, p.td && p.r2, 0.0};
     if (p.td) {
         wt.Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
-        if (p.tr_step) p.Tr[c] = T0;
+        if (p.tr_step && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
     }
     double T = T0;
     bool ok = false;
@@ -1207,7 +1210,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     }
     if (!ok) {
         atomicExch(p.fail, 1);
-        T = T0;
+        T = p.neg_fail ? -T0 : T0;
     }
     atomicMax(p.iter_max, it);
     if (p.T_out) {
@@ -1220,6 +1223,33 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         const int b = p.b_lo + k;
         p.i0[(size_t)k * p.nc + c] = sC[b] / expm1(sTh[b] * iT);
         if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(sA[b], sB[b], sR[b], T);
+    }
+}
+
+// Band-sharded step, after the all-gather of the chunk solves:
+// T^{n+1} for every cell (a negative value marks a failed cell of some rank:
+// flag it on every rank and keep T^n), the rate temperature Tr <- T^n, and the
+// local rows of I0 and of the rate table at T^{n+1} -- the epilogue of
+// newton_kernel, bit for bit.
+__global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__restrict__ T, int nc, int b_lo,
+                                     int nb_loc, const double *__restrict__ Cb, const double *__restrict__ theta,
+                                     double *__restrict__ i0, int td, const double *__restrict__ ra,
+                                     const double *__restrict__ rb, const double *__restrict__ rth,
+                                     double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    double t = Tg[c];
+    if (!(t > 0.0)) {
+        atomicExch(fail, 1);
+        t = -t;
+    }
+    if (td) Tr[c] = T[c];
+    T[c] = t;
+    const double iT = 1.0 / t;
+    for (int k = 0; k < nb_loc; ++k) {
+        const int b = b_lo + k;
+        i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * iT);
+        if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
     }
 }
 

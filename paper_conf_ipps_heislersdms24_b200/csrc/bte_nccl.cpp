@@ -18,6 +18,9 @@ struct Api {
     ncclResult_t (*commInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
     ncclResult_t (*allReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
                               cudaStream_t) = nullptr;
+    ncclResult_t (*reduceScatter)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                                  cudaStream_t) = nullptr;
+    ncclResult_t (*allGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
     const char *(*getErrorString)(ncclResult_t) = nullptr;
     std::string why;
@@ -41,9 +44,12 @@ Api *api() {
         a.getUniqueId = (decltype(a.getUniqueId))dlsym(a.h, "ncclGetUniqueId");
         a.commInitRank = (decltype(a.commInitRank))dlsym(a.h, "ncclCommInitRank");
         a.allReduce = (decltype(a.allReduce))dlsym(a.h, "ncclAllReduce");
+        a.reduceScatter = (decltype(a.reduceScatter))dlsym(a.h, "ncclReduceScatter");
+        a.allGather = (decltype(a.allGather))dlsym(a.h, "ncclAllGather");
         a.commDestroy = (decltype(a.commDestroy))dlsym(a.h, "ncclCommDestroy");
         a.getErrorString = (decltype(a.getErrorString))dlsym(a.h, "ncclGetErrorString");
-        if (!a.getUniqueId || !a.commInitRank || !a.allReduce || !a.commDestroy || !a.getErrorString) {
+        if (!a.getUniqueId || !a.commInitRank || !a.allReduce || !a.reduceScatter || !a.allGather || !a.commDestroy ||
+            !a.getErrorString) {
             a.why = "libnccl is missing a required symbol";
             a.h = nullptr;
         }
@@ -82,6 +88,24 @@ bool allreduce_sum_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, st
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->allReduce(buf, buf, (size_t)n, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    return true;
+}
+
+bool reduce_scatter_sum_f64(const Comm &c, const double *send, double *recv, int64_t recvcount, cudaStream_t s,
+                            std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    ncclResult_t r = a->reduceScatter(send, recv, (size_t)recvcount, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    return true;
+}
+
+bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t sendcount, cudaStream_t s,
+                   std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    ncclResult_t r = a->allGather(send, recv, (size_t)sendcount, ncclFloat64, (ncclComm_t)c.comm, s);
     if (r != ncclSuccess) return *err = a->getErrorString(r), false;
     return true;
 }

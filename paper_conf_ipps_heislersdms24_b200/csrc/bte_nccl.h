@@ -1,7 +1,9 @@
 // bte_nccl.h -- NCCL, loaded at run time with dlopen so that single-GPU use
 // needs no NCCL and the library links against nothing but the CUDA runtime.
-// Used for the one per-step collective of the band-sharded step: the
-// all-reduce of the per-cell energy partials (L760-763).
+// Used for the per-step exchange of the band-sharded step (L760-763, SURVEY
+// 8(e)): reduce-scatter of the per-cell energy partials, the temperature solve
+// on this rank's cell chunk, all-gather of T (or one all-reduce of E and a
+// replicated solve).
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -19,6 +21,12 @@ bool unique_id(void *id128, std::string *err);
 bool init(Comm *c, const void *id128, int rank, int world, std::string *err);
 // in-place sum of n doubles on stream
 bool allreduce_sum_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err);
+// recv[recvcount] = this rank's chunk of the sum of every rank's send[world * recvcount]
+bool reduce_scatter_sum_f64(const Comm &c, const double *send, double *recv, int64_t recvcount, cudaStream_t s,
+                            std::string *err);
+// recv[world * sendcount] = every rank's send[sendcount] in rank order (in place: send = recv + rank * sendcount)
+bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t sendcount, cudaStream_t s,
+                   std::string *err);
 void destroy(Comm &c);
 
 }  // namespace nccl

@@ -361,3 +361,36 @@ def test_nan_energy_reports_enoconv(bte):
         with pytest.raises(bte.BTEError) as e:
             s.solve_temperature()
         assert e.value.status == bte.BTE_ENOCONV
+
+
+def test_nccl_sharded_solve_modes_one_rank(bte, monkeypatch):
+    """The band-sharded step exchange on a one-rank communicator, both modes:
+    reduce-scatter + chunk solve + all-gather (default) and all-reduce +
+    replicated solve (BTE_SHARD_NEWTON=replicated); both bitwise equal to the
+    single-GPU path, with and without the rate law, on the box kernel."""
+    cfg = gen.small_3d_config((34, 9, 5), n_spectral=3)
+    law = dataclasses.replace(cfg, bands=gen.with_rate_law(cfg.bands),
+                              dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, gen.with_rate_law(cfg.bands), cfg.dirs,
+                                                               t_max=350.0))
+    for c in (cfg, law):
+        a = gpu_run(c, 6)
+        for mode in ("shard", "replicated"):
+            monkeypatch.setenv("BTE_SHARD_NEWTON", mode)
+            b = gpu_run(c, 6, nccl_id=bte.nccl_unique_id())
+            assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1]), mode
+        monkeypatch.delenv("BTE_SHARD_NEWTON")
+
+
+def test_nccl_sharded_step_reports_enoconv(bte):
+    """A failed cell in the chunk solve is flagged on every rank (negative
+    marker through the all-gather) and keeps T^n."""
+    cfg = _cfg("C1")
+    with bte.solver_from_config(cfg, nccl_id=bte.nccl_unique_id()) as s:
+        T_before = s.temperature()
+        I = s.intensity()
+        I[:, :, 5] = -1e13  # the step's energy of cell 5 stays negative
+        s.set_intensity(I)
+        with pytest.raises(bte.BTEError) as e:
+            s.step(cfg.dt, 1)
+        assert e.value.status == bte.BTE_ENOCONV
+        assert s.temperature()[5] == T_before[5]
