@@ -213,7 +213,13 @@ def run_ours(args):
         from paper_conf_ipps_heislersdms24_b200.dist import share_nccl_id
         nccl_id = share_nccl_id(pg, rank)
     stream = torch.cuda.current_stream()
-    s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream,
+    part_kw = {}
+    if args.cell_parts > 1:  # cell partitioning, x band groups = world / cell_parts
+        from paper_conf_ipps_heislersdms24_b200.dist import partition_cells
+        assert world % args.cell_parts == 0, "--cell-parts must divide the number of GPUs"
+        part_kw = dict(cell_part=partition_cells(cfg.mesh["cell_centre"], args.cell_parts),
+                       n_cell_parts=args.cell_parts)
+    s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream, **part_kw,
                                profile=True, band_group=args.band_group, block_threads=args.block_threads,
                                max_spare_slabs=args.max_spare, dir_chunk=args.dir_chunk,
                                locality=not args.no_locality, tma=not args.no_tma, stencil=args.stencil,
@@ -221,6 +227,7 @@ def run_ours(args):
     bte.apply_ic(s, cfg)
     nb_loc = s.b_hi - s.b_lo
     nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
+    nc_loc = s.n_cells  # owned cells (all of them without --cell-parts)
     dt = cfg.dt
 
     def barrier():
@@ -257,8 +264,10 @@ def run_ours(args):
     # timed region.  A step launches it once per band-group segment; achieved =
     # algorithmic bytes of all flux launches of a step / their summed time.
     flux_launches_per_step = max(1, (st["kernel_launches"] // args.steps) - 1 - (1 if world > 1 else 0))
+    if args.cell_parts > 1:
+        flux_launches_per_step = None  # (halo pack / unpack launches too)
     t_flux = st["ms_flux_interior"] / args.steps / 1e3
-    alg_bytes = BYTES_PER_UPDATE * nc * nd * nb_loc  # per step, this rank
+    alg_bytes = BYTES_PER_UPDATE * nc_loc * nd * nb_loc  # per step, this rank
     peak, peak_src = _peaks()
     achieved = alg_bytes / t_flux / 1e9 if t_flux > 0 else None
     traffic = _traffic_from_profiles(args.config)
@@ -268,17 +277,18 @@ def run_ours(args):
             "alg_bytes_per_step": alg_bytes, "flux_launches_per_step": flux_launches_per_step,
             "kernel_ms_per_step": t_flux * 1e3,
             "share_of_step": st["ms_flux_interior"] / ms if ms > 0 else None,
-            "step_alg_GBs": BYTES_PER_UPDATE * nc * nd * nb_loc * args.steps / (ms / 1e3) / 1e9}
-    phases = {k: st[k] / args.steps for k in ("ms_flux_interior", "ms_flux_boundary", "ms_allreduce", "ms_newton")}
+            "step_alg_GBs": BYTES_PER_UPDATE * nc_loc * nd * nb_loc * args.steps / (ms / 1e3) / 1e9}
+    phases = {k: st[k] / args.steps for k in ("ms_flux_interior", "ms_flux_boundary", "ms_allreduce", "ms_newton",
+                                              "ms_halo")}
 
     # ---- end-to-end through the public API with host buffers: upload the state
     # (pinned host -> device) once, then every step bte_step + read T back.
     e2e = None
-    state_gb = nb_loc * nd * nc * 8 / 1e9
+    state_gb = nb_loc * nd * nc_loc * 8 / 1e9
     if not args.no_e2e and state_gb > E2E_MAX_GB:  # C5: the host copy would need ~156 GB of pinned RAM
         e2e = {"skipped": f"state {state_gb:.0f} GB per rank > {E2E_MAX_GB} GB of pinned host memory"}
     elif not args.no_e2e:
-        e2e = _e2e(s, pg, world, nb_loc, nb, nd, nc, dt, total_updates, args)
+        e2e = _e2e(s, pg, world, nb_loc, nb, nd, nc_loc, dt, total_updates, args)
 
     cb = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -330,7 +340,10 @@ def _emit(v):
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOADS[args.config], "name": args.config, "n_cells": nc, "n_dirs": nd,
-                       "n_band_rows": nb, "dt": dt, "parallelism": f"band-shard x{world}",
+                       "n_band_rows": nb, "dt": dt,
+                       "parallelism": (f"band-shard x{world}" if args.cell_parts == 1 else
+                                       f"band-shard x{world // args.cell_parts} x cell-part x{args.cell_parts}"),
+                       "halo_bytes_per_step_rank0": st["halo_bytes"],
                        "relaxation": "tau(T) law" if args.rate_law else "constant tau",
                        "l2": f"state {nc * nd * nb * 8 / 1e9:.1f} GB per copy >> 126 MB L2 (no flush needed)"},
             "roofline": roof, "cpu_baseline": cb, "e2e": e2e, "clocks": clocks,
@@ -365,6 +378,8 @@ def main():
     ap.add_argument("--ic-eps", type=float, default=None, help="override the IC perturbation (0: equilibrium IC)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")
+    ap.add_argument("--cell-parts", type=int, default=1,
+                    help="cell partitioning (SURVEY 8(f) N3) into K parts x world/K band groups (default 1)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

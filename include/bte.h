@@ -158,6 +158,21 @@ typedef struct {
                                  per thread block, any >= 1) */
     int32_t dir_chunk;        /* 0 auto; else directions per thread block (box kernel: rounded
                                  down to whole 4-direction orbits) */
+    /* Cell partitioning (the paper's cell-parallel split with a
+     * Metis-style partition, L728-735, L768-772, Fig. 3-4), optionally combined
+     * with band sharding.  NULL cell_part: none (band sharding only).  Else
+     * every rank passes the WHOLE mesh and the same partition; rank r owns the
+     * cells of part r % n_cell_parts and the band-rows of band group
+     * r / n_cell_parts (world / n_cell_parts groups, rows split as above).
+     * Every step first exchanges, with the ranks of the same band group, the
+     * old-level intensities its cut faces read (halo; only the directions that
+     * flow across the cut), then runs the same step on the owned cells; the
+     * energy is reduced over the ranks of the same part.  All cell-indexed
+     * arrays at the ABI (T, E, I) then hold the OWNED cells in ascending global
+     * id (bte_local_cells).  Without a communicator the caller moves the halo
+     * with bte_halo_export / bte_halo_import before bte_step_begin. */
+    const int32_t *cell_part; /* [n_cells] part id in [0, n_cell_parts) */
+    int32_t n_cell_parts;     /* >= 1; world must be a multiple of it */
 } bte_options;
 
 /* Per-context counters since creation / the last bte_reset_stats. Phase
@@ -182,6 +197,8 @@ typedef struct {
                                   uniform geometry, 3 TMA-staged, 4 TMA-staged + uniform
                                   geometry, 5 stencil-staged (structured order), 6 box
                                   (structured 3-D grid, tensor copies, z-marching) */
+    double ms_halo;            /* cell partitioning: halo pack + exchange + unpack */
+    int64_t halo_bytes;        /* halo bytes this rank sends per step (all segments) */
 } bte_stats;
 
 /* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,
@@ -249,6 +266,28 @@ BTE_API bte_status bte_step_begin(bte_ctx *ctx, double dt);
 BTE_API bte_status bte_get_energy(const bte_ctx *ctx, double *E);
 BTE_API bte_status bte_set_energy(bte_ctx *ctx, const double *E);
 BTE_API bte_status bte_step_finish(bte_ctx *ctx);
+
+/* Cell partitioning (see bte_options.cell_part).  Owned cells of this rank:
+ * *n_local, and (ids != NULL) their global ids ascending into ids[*n_local]
+ * (host).  Without partitioning: all cells, ids 0..n_cells-1. */
+BTE_API bte_status bte_local_cells(const bte_ctx *ctx, int64_t *n_local, int64_t *ids);
+
+/* Halo segment sizes with part `part` (doubles): *n_send = values this rank
+ * sends to it, *n_recv = values it receives from it (0 and 0 if the parts share
+ * no face or part is this rank's own).  Segment layout [k][j][i]: local band-row
+ * k, the segment's directions j (ascending ids d with s_d . n_f < 0 at the
+ * reading cell's cut face f), the segment's cells i (ascending global id of
+ * the writing part's cells that cut faces of the reading part point to). */
+BTE_API bte_status bte_halo_size(const bte_ctx *ctx, int32_t part, int64_t *n_send, int64_t *n_recv);
+
+/* Caller-driven halo exchange (no communicator, e.g. partitions emulated on one
+ * device): export writes the current I^n values this rank sends to `part` into
+ * buf[n_send] (host); import stores the values received from `part`
+ * (buf[n_recv], host) as this rank's halo.  Call import for every neighbour
+ * part before bte_step_begin; the halo is read by the next flux only.  EINVAL
+ * for a part out of range, ESTATE inside a split step. */
+BTE_API bte_status bte_halo_export(const bte_ctx *ctx, int32_t part, double *buf);
+BTE_API bte_status bte_halo_import(bte_ctx *ctx, int32_t part, const double *buf);
 
 /* Counters (see bte_stats). */
 BTE_API bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st);

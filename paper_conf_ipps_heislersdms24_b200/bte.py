@@ -61,7 +61,8 @@ class Options(C.Structure):
                 ("newton_max_iter", C.c_int32), ("rank", C.c_int32), ("world", C.c_int32),
                 ("device", C.c_int32), ("nccl_unique_id", C.c_void_p), ("stream", C.c_void_p),
                 ("flags", C.c_uint32), ("max_spare_slabs", C.c_int32), ("block_threads", C.c_int32),
-                ("band_group", C.c_int32), ("dir_chunk", C.c_int32)]
+                ("band_group", C.c_int32), ("dir_chunk", C.c_int32), ("cell_part", C.c_void_p),
+                ("n_cell_parts", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -70,7 +71,8 @@ class Stats(C.Structure):
                 ("ms_allreduce", C.c_double), ("ms_newton", C.c_double), ("ms_total", C.c_double),
                 ("newton_iter_max", C.c_int32), ("spare_slabs", C.c_int32),
                 ("n_interior_cells", C.c_int32), ("band_group", C.c_int32),
-                ("block_threads", C.c_int32), ("dir_chunks", C.c_int32), ("flux_variant", C.c_int32)]
+                ("block_threads", C.c_int32), ("dir_chunks", C.c_int32), ("flux_variant", C.c_int32),
+                ("ms_halo", C.c_double), ("halo_bytes", C.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -82,7 +84,8 @@ EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",
            "bte_band_range", "bte_step_begin", "bte_get_energy", "bte_set_energy", "bte_step_finish",
            "bte_get_stats", "bte_reset_stats", "bte_nccl_unique_id", "bte_last_error",
-           "bte_status_string", "bte_destroy", "bte_get_temperature_rule"]
+           "bte_status_string", "bte_destroy", "bte_get_temperature_rule", "bte_local_cells",
+           "bte_halo_size", "bte_halo_export", "bte_halo_import"]
 
 
 def _load():
@@ -122,6 +125,10 @@ def _load():
         "bte_last_error": ([vp], C.c_char_p),
         "bte_status_string": ([i32], C.c_char_p),
         "bte_destroy": ([vp], None),
+        "bte_local_cells": ([vp, P(i64), vp], i32),
+        "bte_halo_size": ([vp, i32, P(i64), P(i64)], i32),
+        "bte_halo_export": ([vp, i32, vp], i32),
+        "bte_halo_import": ([vp, i32, vp], i32),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -158,7 +165,8 @@ class Solver:
     def __init__(self, mesh, bands, dirs, bcs, *, t_init=300.0, temp_rule=0, newton_rtol=1e-12,
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
                  stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
-                 generic_faces=False, locality=True, dir_chunk=0, tma=True, stencil=False, box=True):
+                 generic_faces=False, locality=True, dir_chunk=0, tma=True, stencil=False, box=True,
+                 cell_part=None, n_cell_parts=1):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -200,12 +208,21 @@ class Solver:
                    | (0 if box else BTE_FLAG_NO_BOX))
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)
         o.dir_chunk = int(dir_chunk)
+        if cell_part is not None:  # cell partitioning (N3): this rank owns part rank % n_cell_parts
+            k["part"] = i32(cell_part)
+            assert k["part"].shape == (self.n_cells,)
+            o.cell_part, o.n_cell_parts = _p(k["part"]).value, int(n_cell_parts)
         ctx = C.c_void_p()
         _check(lib.bte_create(C.byref(m), C.byref(b), C.byref(d), C.byref(bc), C.byref(o), C.byref(ctx)))
         self.ctx = ctx
         lo, hi = C.c_int32(), C.c_int32()
         _check(lib.bte_band_range(self.ctx, C.byref(lo), C.byref(hi)), self.ctx)
         self.b_lo, self.b_hi = lo.value, hi.value
+        self.n_cell_parts = int(n_cell_parts) if cell_part is not None else 1
+        self.n_global_cells = self.n_cells
+        n = C.c_int64()
+        _check(lib.bte_local_cells(self.ctx, C.byref(n), None), self.ctx)
+        self.n_cells = n.value  # owned cells (all of them without cell partitioning)
 
     # -- lifecycle ---------------------------------------------------------------
     def close(self):
@@ -284,6 +301,31 @@ class Solver:
         T = np.ascontiguousarray(np.broadcast_to(np.asarray(T, np.float64), (self.n_cells,)))
         _check(lib.bte_set_equilibrium(self.ctx, _p(T)), self.ctx)
 
+    # -- cell partitioning (N3) ----------------------------------------------------
+    def local_cells(self):
+        """Global ids (ascending) of the owned cells; cell-indexed arrays follow this order."""
+        ids = np.empty(self.n_cells, np.int64)
+        n = C.c_int64()
+        _check(lib.bte_local_cells(self.ctx, C.byref(n), _p(ids)), self.ctx)
+        return ids
+
+    def halo_size(self, part):
+        s, r = C.c_int64(), C.c_int64()
+        _check(lib.bte_halo_size(self.ctx, int(part), C.byref(s), C.byref(r)), self.ctx)
+        return s.value, r.value
+
+    def halo_export(self, part):
+        n, _ = self.halo_size(part)
+        buf = np.empty(n)
+        if n:
+            _check(lib.bte_halo_export(self.ctx, int(part), _p(buf)), self.ctx)
+        return buf
+
+    def halo_import(self, part, buf):
+        buf = np.ascontiguousarray(buf, np.float64)
+        if buf.size:
+            _check(lib.bte_halo_import(self.ctx, int(part), _p(buf)), self.ctx)
+
     def stats(self):
         s = Stats()
         _check(lib.bte_get_stats(self.ctx, C.byref(s)), self.ctx)
@@ -317,8 +359,10 @@ def apply_ic(solver, cfg, seed=None):
     if not cfg.ic_eps:
         return
     seed = SEED if seed is None else seed
+    cells = solver.local_cells() if solver.n_cell_parts > 1 else None
     for b in range(solver.b_lo, solver.b_hi):
         I = solver.intensity(b, b + 1)
-        I[0] *= ic_multiplier(solver.n_dirs, solver.n_cells, b, cfg.ic_eps, seed)
+        mult = ic_multiplier(solver.n_dirs, solver.n_global_cells, b, cfg.ic_eps, seed)
+        I[0] *= mult if cells is None else mult[:, cells]
         solver.set_intensity(I, b, b + 1)
     solver.solve_temperature()

@@ -18,7 +18,9 @@
 #include <cstring>
 #include <cstdlib>
 #include <functional>
+#include <array>
 #include <map>
+#include <set>
 #include <string>
 #include <vector>
 
@@ -45,7 +47,18 @@ struct PhaseEvent {
     int phase;
     cudaEvent_t a, b;
 };
-enum Phase { kPhFlux = 0, kPhAllreduce = 2, kPhNewton = 3 };
+enum Phase { kPhFlux = 0, kPhAllreduce = 2, kPhNewton = 3, kPhHalo = 4 };
+
+// One halo segment of a cell-partitioned run: the values this
+// rank sends to / receives from one neighbour part, buffers [k][j][i].
+struct HaloSeg {
+    int part = 0;
+    int32_t n_send_cells = 0, n_send_dirs = 0, n_recv_cells = 0, n_recv_dirs = 0, col0 = 0;
+    int32_t *send_cells = nullptr, *send_dirs = nullptr, *recv_dirs = nullptr;  // device
+    double *sbuf = nullptr, *rbuf = nullptr;                                      // device
+    int64_t n_send() const { return (int64_t)n_send_cells * n_send_dirs; }  // per band-row
+    int64_t n_recv() const { return (int64_t)n_recv_cells * n_recv_dirs; }
+};
 
 }  // namespace
 
@@ -120,6 +133,14 @@ struct bte_ctx {
     bool own_stream = false;
     bte::nccl::Comm comm{};
     bool have_comm = false;
+    // cell partitioning (N3): part of this rank, band groups, halo segments;
+    // the energy is reduced over the ranks of the same part (bcomm, G ranks)
+    int n_parts = 1, my_part = 0, G = 1, gband = 0;
+    int32_t n_halo = 0;
+    std::vector<HaloSeg> hsegs;
+    std::vector<int64_t> gid;  // owned cells: global ids ascending (caller order of the ABI)
+    bte::nccl::Comm bcomm{};
+    bool have_bcomm = false, own_bcomm = false;
     bool begun = false;  // split step in flight
     // stats
     bte_stats st{};
@@ -297,6 +318,7 @@ void ev_collect(bte_ctx *ctx) {  // after a stream sync
         cudaEventElapsedTime(&ms, pe.a, pe.b);
         double *dst = pe.phase == kPhFlux ? &ctx->st.ms_flux_interior
                       : pe.phase == kPhAllreduce ? &ctx->st.ms_allreduce
+                      : pe.phase == kPhHalo      ? &ctx->st.ms_halo
                                                  : &ctx->st.ms_newton;
         *dst += ms;
         ctx->ev_pool.push_back(pe);
@@ -829,9 +851,9 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
 }
 
 bte_status allreduce_E(bte_ctx *ctx, double *E = nullptr) {
-    if (!ctx->have_comm) return BTE_OK;
+    if (!ctx->have_bcomm) return BTE_OK;
     std::string e;
-    if (!bte::nccl::allreduce_sum_f64(ctx->comm, E ? E : ctx->E, ctx->nc, ctx->stream, &e)) {
+    if (!bte::nccl::allreduce_sum_f64(ctx->bcomm, E ? E : ctx->E, ctx->nc, ctx->stream, &e)) {
         set_err(&ctx->err, "NCCL all-reduce failed: %s", e.c_str());
         return BTE_ENCCL;
     }
@@ -854,12 +876,12 @@ bte_status shard_newton_step(bte_ctx *ctx) {
     std::string e;
     ev_mark(ctx, kPhAllreduce, true);
     STATUS_TRY(reduce_slots(ctx));
-    if (!bte::nccl::reduce_scatter_sum_f64(ctx->comm, ctx->E, ctx->Echunk, ctx->chunk, ctx->stream, &e))
+    if (!bte::nccl::reduce_scatter_sum_f64(ctx->bcomm, ctx->E, ctx->Echunk, ctx->chunk, ctx->stream, &e))
         return set_err(&ctx->err, "NCCL reduce-scatter failed: %s", e.c_str()), BTE_ENCCL;
     ev_mark(ctx, kPhAllreduce, false);
     ev_mark(ctx, kPhNewton, true);
     bte::NewtonParams q = newton_params(ctx, ctx->Echunk, /*step=*/true);
-    q.c_lo = ctx->opt.rank * ctx->chunk;
+    q.c_lo = ctx->gband * ctx->chunk;
     q.nc = std::max(0, std::min(ctx->chunk, ctx->nc - q.c_lo));
     q.T_out = ctx->Tg;
     q.neg_fail = 1;
@@ -868,8 +890,8 @@ bte_status shard_newton_step(bte_ctx *ctx) {
         bte::newton_kernel<<<(q.nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
         ctx->st.kernel_launches++;
     }
-    double *mine = ctx->Tg + (size_t)ctx->opt.rank * ctx->chunk;
-    if (!bte::nccl::allgather_f64(ctx->comm, mine, ctx->Tg, ctx->chunk, ctx->stream, &e))
+    double *mine = ctx->Tg + (size_t)ctx->gband * ctx->chunk;
+    if (!bte::nccl::allgather_f64(ctx->bcomm, mine, ctx->Tg, ctx->chunk, ctx->stream, &e))
         return set_err(&ctx->err, "NCCL all-gather failed: %s", e.c_str()), BTE_ENCCL;
     bte::newton_finish_kernel<<<(ctx->nc + 255) / 256, 256, 0, ctx->stream>>>(
         ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
@@ -878,6 +900,66 @@ bte_status shard_newton_step(bte_ctx *ctx) {
     ev_mark(ctx, kPhNewton, false);
     if (ctx->td) ctx->rsel = 1 - ctx->rsel;
     CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+// ------------------------------------------------------------- halo (N3)
+// Pack / unpack one segment for every local band-row (current slabs).
+bte::HaloParams halo_params(const bte_ctx *ctx) {
+    bte::HaloParams hp{};
+    for (int k = 0; k < ctx->nb_loc; ++k) hp.row[k] = ctx->pool + (int64_t)ctx->cur_slot[k] * ctx->slab_elems;
+    hp.nb_loc = ctx->nb_loc;
+    hp.ps = ctx->ps;
+    return hp;
+}
+
+dim3 halo_grid(const bte_ctx *ctx, int64_t per) {
+    return dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(2048, (per + 255) / 256)), (unsigned)ctx->nb_loc);
+}
+
+bte_status halo_pack(bte_ctx *ctx, const HaloSeg &h) {
+    if (h.n_send() == 0) return BTE_OK;
+    bte::HaloParams hp = halo_params(ctx);
+    hp.cells = h.send_cells;
+    hp.dirs = h.send_dirs;
+    hp.n = h.n_send_cells;
+    hp.n_dirs = h.n_send_dirs;
+    bte::halo_pack_kernel<<<halo_grid(ctx, h.n_send()), 256, 0, ctx->stream>>>(hp, h.sbuf);
+    ctx->st.kernel_launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+bte_status halo_unpack(bte_ctx *ctx, const HaloSeg &h) {
+    if (h.n_recv() == 0) return BTE_OK;
+    bte::HaloParams hp = halo_params(ctx);
+    hp.dirs = h.recv_dirs;
+    hp.n = h.n_recv_cells;
+    hp.n_dirs = h.n_recv_dirs;
+    hp.col0 = h.col0;
+    bte::halo_unpack_kernel<<<halo_grid(ctx, h.n_recv()), 256, 0, ctx->stream>>>(hp, h.rbuf);
+    ctx->st.kernel_launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+// Cell-partitioned step, before the flux: every segment packed, one NCCL group
+// of sends / receives with the neighbour parts of this band group, unpacked
+// into the halo columns of the current slabs (I^n, the old level, Eq. 3).
+bte_status halo_exchange(bte_ctx *ctx) {
+    if (ctx->hsegs.empty()) return BTE_OK;
+    if (!ctx->have_comm) return set_err(&ctx->err, "halo exchange needs a communicator"), BTE_ESTATE;
+    ev_mark(ctx, kPhHalo, true);
+    for (const HaloSeg &h : ctx->hsegs) STATUS_TRY(halo_pack(ctx, h));
+    std::vector<bte::nccl::P2P> ops;
+    for (const HaloSeg &h : ctx->hsegs)
+        ops.push_back({ctx->gband * ctx->n_parts + h.part, h.sbuf, h.n_send() * ctx->nb_loc, h.rbuf,
+                       h.n_recv() * ctx->nb_loc});
+    std::string e;
+    if (!bte::nccl::exchange_f64(ctx->comm, ops.data(), (int)ops.size(), ctx->stream, &e))
+        return set_err(&ctx->err, "NCCL halo exchange failed: %s", e.c_str()), BTE_ENCCL;
+    for (const HaloSeg &h : ctx->hsegs) STATUS_TRY(halo_unpack(ctx, h));
+    ev_mark(ctx, kPhHalo, false);
     return BTE_OK;
 }
 
@@ -1002,6 +1084,109 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
     return BTE_OK;
 }
 
+// ------------------------------------------------------------- cell partition (N3)
+// The owned cells of part `me` as a mesh of their own: owned cells in ascending
+// global id (local ids 0..nc-1), faces copied in stored order; a face whose
+// neighbour lies in another part points to a halo column nc + slot (the slots
+// of one neighbour part contiguous, ascending global id).  Segments (one per
+// neighbour part): cells and directions follow the READING
+// side's faces (a cut face f of a reader cell needs the writer's value for the
+// directions with s_d . n_f < 0, the upwind inflow of Eq. 3), so both ends of
+// a segment derive the same lists from the replicated global mesh.
+struct SegPlan {
+    int part = 0;
+    std::vector<int32_t> send_local, send_dirs, recv_dirs;
+    int32_t n_recv_cells = 0, col0 = 0;
+};
+struct LocalPlan {
+    std::vector<int64_t> gid, off, nbr;
+    std::vector<double> area, nrm, vol, cen;
+    std::vector<SegPlan> segs;
+    int32_t n_halo = 0;
+    bte_mesh mesh{};
+};
+
+bte_status build_local(const bte_mesh *m, const bte_dirs *dr, const bte_options *o, int me, LocalPlan *L) {
+    const int64_t N = m->n_cells;
+    const int P = o->n_cell_parts;
+    const int32_t *part = o->cell_part;
+    for (int64_t c = 0; c < N; ++c)
+        if (part[c] < 0 || part[c] >= P)
+            return set_err(nullptr, "cell_part[%lld] = %d outside [0, %d)", (long long)c, part[c], P), BTE_EINVAL;
+    std::vector<int64_t> loc(N, -1);
+    for (int64_t c = 0; c < N; ++c)
+        if (part[c] == me) loc[c] = (int64_t)L->gid.size(), L->gid.push_back(c);
+    if (L->gid.empty()) return set_err(nullptr, "cell part %d has no cells", me), BTE_EINVAL;
+    std::vector<std::vector<int64_t>> rc(P), sc(P);
+    std::vector<std::set<std::array<double, 3>>> rn(P), sn(P);
+    for (int64_t g = 0; g < N; ++g) {
+        const int pg = part[g];
+        for (int64_t f = m->face_offsets[g]; f < m->face_offsets[g + 1]; ++f) {
+            const int64_t h = m->face_nbr[f];
+            if (h < 0 || part[h] == pg) continue;
+            const std::array<double, 3> n = {m->face_normal[3 * f], m->face_normal[3 * f + 1], m->face_normal[3 * f + 2]};
+            if (pg == me) rc[part[h]].push_back(h), rn[part[h]].insert(n);  // g reads h
+            if (part[h] == me) sc[pg].push_back(h), sn[pg].insert(n);       // h is read by g
+        }
+    }
+    auto dirs_of = [&](const std::set<std::array<double, 3>> &ns) {
+        std::vector<int32_t> out;
+        for (int d = 0; d < dr->n_dirs; ++d) {
+            const double *s = dr->s + 3 * d;
+            for (const auto &n : ns)
+                if (s[0] * n[0] + s[1] * n[1] + s[2] * n[2] < 0.0) {
+                    out.push_back(d);
+                    break;
+                }
+        }
+        return out;
+    };
+    std::vector<int32_t> hslot(N, -1);
+    for (int q = 0; q < P; ++q) {
+        if (q == me) continue;
+        auto uniq = [](std::vector<int64_t> &v) {
+            std::sort(v.begin(), v.end());
+            v.erase(std::unique(v.begin(), v.end()), v.end());
+        };
+        uniq(rc[q]);
+        uniq(sc[q]);
+        if (rc[q].empty() && sc[q].empty()) continue;
+        SegPlan s;
+        s.part = q;
+        s.col0 = L->n_halo;
+        for (int64_t h : rc[q]) hslot[h] = L->n_halo++;
+        s.n_recv_cells = (int32_t)rc[q].size();
+        s.recv_dirs = dirs_of(rn[q]);
+        for (int64_t h : sc[q]) s.send_local.push_back((int32_t)loc[h]);
+        s.send_dirs = dirs_of(sn[q]);
+        L->segs.push_back(std::move(s));
+    }
+    const int64_t nc = (int64_t)L->gid.size();
+    L->off.push_back(0);
+    for (int64_t i = 0; i < nc; ++i) {
+        const int64_t c = L->gid[i];
+        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f) {
+            const int64_t h = m->face_nbr[f];
+            L->nbr.push_back(h < 0 ? h : part[h] == me ? loc[h] : nc + hslot[h]);
+            L->area.push_back(m->face_area[f]);
+            for (int a = 0; a < 3; ++a) L->nrm.push_back(m->face_normal[3 * f + a]);
+        }
+        L->off.push_back((int64_t)L->nbr.size());
+        L->vol.push_back(m->cell_volume[c]);
+        if (m->cell_centre)
+            for (int a = 0; a < 3; ++a) L->cen.push_back(m->cell_centre[3 * c + a]);
+    }
+    L->mesh.dim = m->dim;
+    L->mesh.n_cells = nc;
+    L->mesh.face_offsets = L->off.data();
+    L->mesh.face_nbr = L->nbr.data();
+    L->mesh.face_area = L->area.data();
+    L->mesh.face_normal = L->nrm.data();
+    L->mesh.cell_volume = L->vol.data();
+    L->mesh.cell_centre = m->cell_centre ? L->cen.data() : nullptr;
+    return BTE_OK;
+}
+
 }  // namespace
 
 // ============================================================= public API
@@ -1046,7 +1231,13 @@ void bte_destroy(bte_ctx *ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    if (ctx->own_bcomm) bte::nccl::destroy(ctx->bcomm);
     if (ctx->have_comm) bte::nccl::destroy(ctx->comm);
+    for (HaloSeg &h : ctx->hsegs) {
+        void *hp[] = {h.send_cells, h.send_dirs, h.recv_dirs, h.sbuf, h.rbuf};
+        for (void *q : hp)
+            if (q) cudaFree(q);
+    }
     void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
@@ -1066,6 +1257,19 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     if (!out) return set_err(nullptr, "NULL out"), BTE_EINVAL;
     *out = nullptr;
     STATUS_TRY(validate(m, bd, dr, bc, o));
+    // --- cell partitioning (N3): rank r owns part r % P of the cells and band
+    // group r / P; from here on `m` is the owned cells' mesh with halo columns
+    const bool cpart = o->cell_part != nullptr;
+    const int n_parts = cpart ? o->n_cell_parts : 1;
+    if (cpart && (n_parts < 1 || o->world % n_parts != 0))
+        return set_err(nullptr, "world %d is not a multiple of n_cell_parts %d", o->world, n_parts), BTE_EINVAL;
+    const int my_part = o->rank % n_parts, G = o->world / n_parts, gband = o->rank / n_parts;
+    LocalPlan lplan;
+    if (cpart) {
+        STATUS_TRY(build_local(m, dr, o, my_part, &lplan));
+        m = &lplan.mesh;
+    }
+    const int32_t n_halo = lplan.n_halo;
     const int nd = dr->n_dirs, nb = bd->n_bands;
     const int64_t nc64 = m->n_cells;
     const int32_t nc = (int32_t)nc64;
@@ -1085,10 +1289,10 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     if (!any_w) return set_err(nullptr, "all temperature weights are zero (temp_rule 0 with every tau = inf)"), BTE_EINVAL;
 
     // --- band sharding: rank g owns [floor(g nb/P), floor((g+1) nb/P))  (L760-775)
-    const int b_lo = (int)((int64_t)o->rank * nb / o->world);
-    const int b_hi = (int)((int64_t)(o->rank + 1) * nb / o->world);
+    const int b_lo = (int)((int64_t)gband * nb / G);
+    const int b_hi = (int)((int64_t)(gband + 1) * nb / G);
     const int nb_loc = b_hi - b_lo;
-    if (nb_loc < 1) return set_err(nullptr, "rank %d owns no band-row (n_bands %d < world %d)", o->rank, nb, o->world), BTE_EINVAL;
+    if (nb_loc < 1) return set_err(nullptr, "rank %d owns no band-row (n_bands %d < band groups %d)", o->rank, nb, G), BTE_EINVAL;
     if (nb_loc > bte::kMaxBandsPerLaunch)
         return set_err(nullptr, "%d band-rows on one rank (max %d)", nb_loc, bte::kMaxBandsPerLaunch), BTE_EINVAL;
 
@@ -1118,7 +1322,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- stencil: every cell has dim pairs, and pair j of every cell neighbours
     // c + so[j] ("+") and c - so[j] ("-") in the caller's order (structured grids)
     int32_t so[3] = {0, 0, 0};
-    bool stencil_order = paired_geom && mf == 2 * m->dim && nc64 >= 2 * bte::kTile;
+    bool stencil_order = paired_geom && !cpart && mf == 2 * m->dim && nc64 >= 2 * bte::kTile;
     for (int64_t c = 0; c < nc64 && stencil_order; ++c) {
         int j = 0;
         if (m->face_offsets[c + 1] - m->face_offsets[c] != 2 * m->dim) stencil_order = false;
@@ -1141,7 +1345,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // --- structured box grid -> the box kernel (grid lexicographic order)
     BoxDetect bx;
     std::vector<bte::BoxOrbit> orbs;
-    if (paired_geom && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
+    if (paired_geom && !cpart && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
         bx = detect_box(m, bc);
     const bool use_box = bx.ok && box_orbits(dr, bx.ax, bx.zside[0] == 1 || bx.zside[1] == 1, &orbs);
 
@@ -1247,8 +1451,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         return set_err(nullptr, "%d distinct specular wall normals (max %d)", (int)cls_of.size(),
                        bte::kMaxGenericClasses), BTE_EINVAL;
 
-    // --- plane stride: cells padded to a whole 256-cell tile (2 KB)
-    const int32_t ps = (int32_t)((nc64 + bte::kTile - 1) / bte::kTile * bte::kTile);
+    // --- plane stride: cells (and halo columns) padded to a whole 256-cell tile (2 KB)
+    const int32_t ps = (int32_t)((nc64 + n_halo + bte::kTile - 1) / bte::kTile * bte::kTile);
 
     // (the paired layout's 5-bit face codes hold up to 16 specular classes)
     // (with the rate law only the box kernel and the generic-face kernel read rate tables)
@@ -1264,7 +1468,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     auto face_src = [&](int64_t f, int32_t *idx, int32_t *kind) {
         const int64_t v = m->face_nbr[f];
         if (v >= 0) {
-            *idx = pos_h[v];
+            *idx = v < nc ? pos_h[v] : (int32_t)v;  // (v >= nc: halo column of a cut face)
             *kind = -1;
         } else {
             const int64_t bf = -1 - v;
@@ -1380,6 +1584,23 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         }
         ctx->have_comm = true;
     }
+    ctx->n_parts = n_parts;
+    ctx->my_part = my_part;
+    ctx->G = G;
+    ctx->gband = gband;
+    ctx->n_halo = n_halo;
+    ctx->gid = lplan.gid;
+    if (ctx->have_comm && n_parts == 1) {  // band sharding: the energy goes over the whole communicator
+        ctx->bcomm = ctx->comm;
+        ctx->have_bcomm = true;
+    } else if (ctx->have_comm && G > 1) {  // hybrid: over the ranks of this cell part
+        std::string e;
+        if (!bte::nccl::split(ctx->comm, my_part, gband, &ctx->bcomm, &e)) {
+            set_err(&ctx->err, "NCCL communicator split failed: %s", e.c_str());
+            return fail(BTE_ENCCL);
+        }
+        ctx->have_bcomm = ctx->own_bcomm = true;
+    }
 
     // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
@@ -1457,11 +1678,32 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(dalloc(ctx, &ctx->i0, (size_t)nb_loc * nc));
     CREATE_TRY(dalloc(ctx, &ctx->T, (size_t)nc));
     // E padded to world x chunk for the reduce-scatter of the sharded step
-    ctx->chunk = (int32_t)((nc64 + o->world - 1) / o->world);
-    ctx->nc_pad = ctx->chunk * o->world;
+    ctx->chunk = (int32_t)((nc64 + G - 1) / G);
+    ctx->nc_pad = ctx->chunk * G;
     CREATE_TRY(dalloc(ctx, &ctx->E, (size_t)ctx->nc_pad));
     CREATE_CUDA(cudaMemset(ctx->E, 0, (size_t)ctx->nc_pad * sizeof(double)));
-    if (ctx->have_comm) {
+    if (n_halo > 0)  // halo columns are read (times a zero weight) before a direction's first exchange
+        CREATE_CUDA(cudaMemsetAsync(ctx->pool, 0, (size_t)(nb_loc + n_spare) * ctx->slab_elems * sizeof(double),
+                                    ctx->stream));
+    for (const SegPlan &sp : lplan.segs) {  // halo segments: internal columns, direction lists, buffers
+        ctx->hsegs.emplace_back();
+        HaloSeg &h = ctx->hsegs.back();
+        h.part = sp.part;
+        h.col0 = nc + sp.col0;
+        h.n_send_cells = (int32_t)sp.send_local.size();
+        h.n_send_dirs = (int32_t)sp.send_dirs.size();
+        h.n_recv_cells = sp.n_recv_cells;
+        h.n_recv_dirs = (int32_t)sp.recv_dirs.size();
+        std::vector<int32_t> cols(sp.send_local.size());
+        for (size_t i = 0; i < cols.size(); ++i) cols[i] = pos_h[sp.send_local[i]];
+        CREATE_TRY(upload(ctx, &h.send_cells, cols));
+        CREATE_TRY(upload(ctx, &h.send_dirs, sp.send_dirs));
+        CREATE_TRY(upload(ctx, &h.recv_dirs, sp.recv_dirs));
+        CREATE_TRY(dalloc(ctx, &h.sbuf, (size_t)h.n_send() * nb_loc));
+        CREATE_TRY(dalloc(ctx, &h.rbuf, (size_t)h.n_recv() * nb_loc));
+        ctx->st.halo_bytes += h.n_send() * nb_loc * (int64_t)sizeof(double);
+    }
+    if (ctx->have_bcomm) {
         const char *ev = std::getenv("BTE_SHARD_NEWTON");  // "replicated": all-reduce + replicated solve
         ctx->shard_newton = !(ev && std::strcmp(ev, "replicated") == 0);
         CREATE_TRY(dalloc(ctx, &ctx->Echunk, (size_t)ctx->chunk));
@@ -1517,6 +1759,13 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             bte::outflow_max_kernel<3><<<gb, tb, 0, ctx->stream>>>(nc, mf_t, paired, nd, ctx->gx, ctx->gy, ctx->gz,
                                                                   ctx->dirs, ctx->d_smax);
         CREATE_CUDA(cudaGetLastError());
+        if (ctx->have_comm && n_parts > 1) {  // the bound of the whole mesh on every rank (S_max >= 0: bits = value)
+            std::string e;
+            if (!bte::nccl::allreduce_max_f64(ctx->comm, reinterpret_cast<double *>(ctx->d_smax), 1, ctx->stream, &e)) {
+                set_err(&ctx->err, "NCCL all-reduce (max) failed: %s", e.c_str());
+                return fail(BTE_ENCCL);
+            }
+        }
         unsigned long long bits = 0;
         CREATE_CUDA(cudaMemcpyAsync(&bits, ctx->d_smax, sizeof bits, cudaMemcpyDeviceToHost, ctx->stream));
         CREATE_CUDA(cudaStreamSynchronize(ctx->stream));
@@ -1579,7 +1828,11 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         }
         CREATE_CUDA(cudaStreamSynchronize(ctx->stream));
     }
-    std::memset(&ctx->st, 0, sizeof ctx->st);
+    {
+        const int64_t hb = ctx->st.halo_bytes;
+        std::memset(&ctx->st, 0, sizeof ctx->st);
+        ctx->st.halo_bytes = hb;
+    }
     ctx->st.spare_slabs = n_spare;
     ctx->st.n_interior_cells = nc - n_bcells;
     ctx->st.band_group = ctx->box ? plan_box(ctx, std::min(ctx->n_spare, nb_loc)).nbb : ctx->bg;
@@ -1617,14 +1870,16 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
     if (n == 0) return BTE_OK;
     STATUS_TRY(check_dt(ctx, dt));
     if (ctx->opt.world > 1 && !ctx->have_comm)
-        return set_err(&ctx->err, "world > 1 without a communicator: reduce the energy with "
-                                  "bte_step_begin / bte_get_energy / bte_set_energy / bte_step_finish"), BTE_ESTATE;
+        return set_err(&ctx->err, "world > 1 without a communicator: reduce the energy (and move the halo) with "
+                                  "bte_step_begin / bte_get_energy / bte_set_energy / bte_step_finish "
+                                  "(bte_halo_export / bte_halo_import)"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int64_t s = 0; s < n; ++s) {
+        STATUS_TRY(halo_exchange(ctx));
         STATUS_TRY(run_flux(ctx, dt));
-        if (ctx->have_comm && ctx->shard_newton) {
+        if (ctx->have_bcomm && ctx->shard_newton) {
             STATUS_TRY(shard_newton_step(ctx));
-        } else if (ctx->have_comm) {
+        } else if (ctx->have_bcomm) {
             ev_mark(ctx, kPhAllreduce, true);
             STATUS_TRY(reduce_slots(ctx));
             STATUS_TRY(allreduce_E(ctx));
@@ -1645,6 +1900,7 @@ bte_status bte_step_begin(bte_ctx *ctx, double dt) {
     if (ctx->begun) return set_err(&ctx->err, "split step already begun"), BTE_ESTATE;
     STATUS_TRY(check_dt(ctx, dt));
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    if (ctx->have_comm) STATUS_TRY(halo_exchange(ctx));  // (no communicator: the caller imported the halo)
     STATUS_TRY(run_flux(ctx, dt));
     STATUS_TRY(reduce_slots(ctx));
     STATUS_TRY(upload_cur_slots(ctx));
@@ -1754,7 +2010,7 @@ bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const dou
 bte_status bte_solve_temperature(bte_ctx *ctx) {
     if (!ctx) return BTE_EINVAL;
     if (ctx->begun) return BTE_ESTATE;
-    if (ctx->opt.world > 1 && !ctx->have_comm)
+    if (ctx->G > 1 && !ctx->have_comm)
         return set_err(&ctx->err, "world > 1 without a communicator: cannot reduce the energy"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     STATUS_TRY(upload_cur_slots(ctx));
@@ -1784,7 +2040,7 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
     bte_ctx *ctx = const_cast<bte_ctx *>(cctx);
     if (rule < 0 || rule > 2) return set_err(&ctx->err, "rule must be 0, 1 or 2"), BTE_EINVAL;
     if (ctx->begun) return BTE_ESTATE;
-    if (ctx->opt.world > 1 && !ctx->have_comm)
+    if (ctx->G > 1 && !ctx->have_comm)
         return set_err(&ctx->err, "world > 1 without a communicator: cannot reduce the energy"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     if (!ctx->E2) {
@@ -1863,6 +2119,67 @@ bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
     return BTE_OK;
 }
 
+bte_status bte_local_cells(const bte_ctx *ctx, int64_t *n_local, int64_t *ids) {
+    if (!ctx || !n_local) return BTE_EINVAL;
+    *n_local = ctx->nc;
+    if (ids)
+        for (int32_t i = 0; i < ctx->nc; ++i) ids[i] = ctx->gid.empty() ? i : ctx->gid[i];
+    return BTE_OK;
+}
+
+static const HaloSeg *find_seg(const bte_ctx *ctx, int32_t part, bte_status *st) {
+    *st = BTE_OK;
+    if (part < 0 || part >= ctx->n_parts) {
+        set_err(const_cast<std::string *>(&ctx->err), "part %d outside [0, %d)", part, ctx->n_parts);
+        *st = BTE_EINVAL;
+        return nullptr;
+    }
+    for (const HaloSeg &h : ctx->hsegs)
+        if (h.part == part) return &h;
+    return nullptr;  // no shared face: empty segment
+}
+
+bte_status bte_halo_size(const bte_ctx *ctx, int32_t part, int64_t *n_send, int64_t *n_recv) {
+    if (!ctx || !n_send || !n_recv) return BTE_EINVAL;
+    bte_status st;
+    const HaloSeg *h = find_seg(ctx, part, &st);
+    STATUS_TRY(st);
+    *n_send = h ? h->n_send() * ctx->nb_loc : 0;
+    *n_recv = h ? h->n_recv() * ctx->nb_loc : 0;
+    return BTE_OK;
+}
+
+bte_status bte_halo_export(const bte_ctx *cctx, int32_t part, double *buf) {
+    if (!cctx || !buf) return BTE_EINVAL;
+    bte_ctx *ctx = const_cast<bte_ctx *>(cctx);
+    if (ctx->begun) return set_err(&ctx->err, "split step in flight"), BTE_ESTATE;
+    bte_status st;
+    const HaloSeg *h = find_seg(ctx, part, &st);
+    STATUS_TRY(st);
+    if (!h || h->n_send() == 0) return BTE_OK;
+    CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    STATUS_TRY(halo_pack(ctx, *h));
+    CUDA_TRY(ctx, cudaMemcpyAsync(buf, h->sbuf, (size_t)h->n_send() * ctx->nb_loc * sizeof(double),
+                                  cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return BTE_OK;
+}
+
+bte_status bte_halo_import(bte_ctx *ctx, int32_t part, const double *buf) {
+    if (!ctx || !buf) return BTE_EINVAL;
+    if (ctx->begun) return set_err(&ctx->err, "split step in flight"), BTE_ESTATE;
+    bte_status st;
+    const HaloSeg *h = find_seg(ctx, part, &st);
+    STATUS_TRY(st);
+    if (!h || h->n_recv() == 0) return BTE_OK;
+    CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    CUDA_TRY(ctx, cudaMemcpyAsync(h->rbuf, buf, (size_t)h->n_recv() * ctx->nb_loc * sizeof(double),
+                                  cudaMemcpyHostToDevice, ctx->stream));
+    STATUS_TRY(halo_unpack(ctx, *h));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    return BTE_OK;
+}
+
 bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st) {
     if (!ctx || !st) return BTE_EINVAL;
     *st = ctx->st;
@@ -1879,6 +2196,7 @@ bte_status bte_reset_stats(bte_ctx *ctx) {
     ctx->st.n_interior_cells = keep.n_interior_cells;
     ctx->st.band_group = keep.band_group;
     ctx->st.block_threads = keep.block_threads;
+    ctx->st.halo_bytes = keep.halo_bytes;
     return BTE_OK;
 }
 

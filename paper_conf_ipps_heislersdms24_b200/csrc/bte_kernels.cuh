@@ -1388,4 +1388,46 @@ __global__ void scatter_rows_kernel(const double *__restrict__ src, const int32_
     }
 }
 
+// ---------------------------------------------------------------------------
+// Halo exchange of a cell-partitioned run (the paper's
+// cell-parallel split, L728-735, L768-772).  The upwind values a rank reads
+// across a cut face are the neighbour part's I^n at the old level, exactly as
+// for an interior face (Eq. 3): they live in extra columns
+// [nc, nc + n_halo) of every slab, which the flux kernels read like any other
+// neighbour column and never write.  One segment per neighbour part, layout
+// buf[k][j][i] over the local band-rows k, the segment's direction list j and
+// its cell list i (only directions that flow across the cut, s_d . n < 0 at
+// the reading cell's face).
+struct HaloParams {
+    double *row[kMaxBandsPerLaunch];  // current slab of local band-row k
+    const int32_t *cells;             // pack: internal column of send cell i
+    const int32_t *dirs;              // direction list of the segment
+    int32_t n, n_dirs, nb_loc, ps;
+    int32_t col0;                     // unpack: first halo column of the segment
+};
+
+__global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf) {
+    const int64_t per = (int64_t)p.n_dirs * p.n;
+    const int k = blockIdx.y;
+    const double *s = p.row[k];
+    double *o = buf + k * per;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
+        const int j = (int)(e / p.n);
+        const int i = (int)(e - (int64_t)j * p.n);
+        o[e] = s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)];
+    }
+}
+
+__global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const double *__restrict__ buf) {
+    const int64_t per = (int64_t)p.n_dirs * p.n;
+    const int k = blockIdx.y;
+    double *s = p.row[k];
+    const double *in = buf + k * per;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
+        const int j = (int)(e / p.n);
+        const int i = (int)(e - (int64_t)j * p.n);
+        s[(int64_t)__ldg(p.dirs + j) * p.ps + p.col0 + i] = in[e];
+    }
+}
+
 }  // namespace bte

@@ -22,6 +22,11 @@ struct Api {
                                   cudaStream_t) = nullptr;
     ncclResult_t (*allGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*commSplit)(ncclComm_t, int, int, ncclComm_t *, ncclConfig_t *) = nullptr;
+    ncclResult_t (*send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*groupStart)() = nullptr;
+    ncclResult_t (*groupEnd)() = nullptr;
     const char *(*getErrorString)(ncclResult_t) = nullptr;
     std::string why;
 };
@@ -48,6 +53,12 @@ Api *api() {
         a.allGather = (decltype(a.allGather))dlsym(a.h, "ncclAllGather");
         a.commDestroy = (decltype(a.commDestroy))dlsym(a.h, "ncclCommDestroy");
         a.getErrorString = (decltype(a.getErrorString))dlsym(a.h, "ncclGetErrorString");
+        // (cell partitioning only: checked where used)
+        a.commSplit = (decltype(a.commSplit))dlsym(a.h, "ncclCommSplit");
+        a.send = (decltype(a.send))dlsym(a.h, "ncclSend");
+        a.recv = (decltype(a.recv))dlsym(a.h, "ncclRecv");
+        a.groupStart = (decltype(a.groupStart))dlsym(a.h, "ncclGroupStart");
+        a.groupEnd = (decltype(a.groupEnd))dlsym(a.h, "ncclGroupEnd");
         if (!a.getUniqueId || !a.commInitRank || !a.allReduce || !a.reduceScatter || !a.allGather || !a.commDestroy ||
             !a.getErrorString) {
             a.why = "libnccl is missing a required symbol";
@@ -106,6 +117,43 @@ bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t send
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->allGather(send, recv, (size_t)sendcount, ncclFloat64, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    return true;
+}
+
+bool allreduce_max_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    ncclResult_t r = a->allReduce(buf, buf, (size_t)n, ncclFloat64, ncclMax, (ncclComm_t)c.comm, s);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    return true;
+}
+
+bool split(const Comm &c, int color, int key, Comm *out, std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    if (!a->commSplit) return *err = "libnccl has no ncclCommSplit (NCCL >= 2.18 needed)", false;
+    ncclComm_t nc = nullptr;
+    ncclResult_t r = a->commSplit((ncclComm_t)c.comm, color, key, &nc, nullptr);
+    if (r != ncclSuccess) return *err = a->getErrorString(r), false;
+    out->comm = nc;
+    return true;
+}
+
+bool exchange_f64(const Comm &c, const P2P *ops, int n_ops, cudaStream_t s, std::string *err) {
+    Api *a = api();
+    if (!a || !c.comm) return *err = why(), false;
+    if (!a->send || !a->recv || !a->groupStart || !a->groupEnd)
+        return *err = "libnccl has no ncclSend / ncclRecv / ncclGroupStart / ncclGroupEnd", false;
+    ncclResult_t r = a->groupStart();
+    for (int i = 0; i < n_ops && r == ncclSuccess; ++i) {
+        if (ops[i].n_send > 0)
+            r = a->send(ops[i].send, (size_t)ops[i].n_send, ncclFloat64, ops[i].peer, (ncclComm_t)c.comm, s);
+        if (r == ncclSuccess && ops[i].n_recv > 0)
+            r = a->recv(ops[i].recv, (size_t)ops[i].n_recv, ncclFloat64, ops[i].peer, (ncclComm_t)c.comm, s);
+    }
+    const ncclResult_t r2 = a->groupEnd();
+    if (r == ncclSuccess) r = r2;
     if (r != ncclSuccess) return *err = a->getErrorString(r), false;
     return true;
 }

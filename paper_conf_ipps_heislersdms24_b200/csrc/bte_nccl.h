@@ -3,7 +3,7 @@
 // Used for the per-step exchange of the band-sharded step (L760-763, SURVEY
 // 8(e)): reduce-scatter of the per-cell energy partials, the temperature solve
 // on this rank's cell chunk, all-gather of T (or one all-reduce of E and a
-// replicated solve).
+// replicated solve), and the halo exchange of the cell-partitioned step.
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -27,6 +27,20 @@ bool reduce_scatter_sum_f64(const Comm &c, const double *send, double *recv, int
 // recv[world * sendcount] = every rank's send[sendcount] in rank order (in place: send = recv + rank * sendcount)
 bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t sendcount, cudaStream_t s,
                    std::string *err);
+// in-place max of n doubles (the positivity bound of a cell-partitioned run)
+bool allreduce_max_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err);
+// sub-communicator of the ranks with the same colour, ordered by key (ncclCommSplit)
+bool split(const Comm &c, int color, int key, Comm *out, std::string *err);
+// halo exchange of a cell-partitioned run: one NCCL group of
+// point-to-point sends and receives of doubles, peer[i] = world rank
+struct P2P {
+    int peer;
+    const double *send;
+    int64_t n_send;
+    double *recv;
+    int64_t n_recv;
+};
+bool exchange_f64(const Comm &c, const P2P *ops, int n_ops, cudaStream_t s, std::string *err);
 void destroy(Comm &c);
 
 }  // namespace nccl

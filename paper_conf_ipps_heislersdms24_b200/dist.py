@@ -16,6 +16,40 @@ def band_range(rank: int, world: int, n_bands: int) -> tuple[int, int]:
     return rank * n_bands // world, (rank + 1) * n_bands // world
 
 
+def rank_grid(rank: int, world: int, n_cell_parts: int = 1) -> tuple[int, int]:
+    """(cell part, band group) of a rank under cell partitioning (SURVEY 8(f)
+    N3): part = rank % P, group = rank // P; the rule bte_create applies."""
+    assert world % n_cell_parts == 0
+    return rank % n_cell_parts, rank // n_cell_parts
+
+
+def partition_cells(centres, n_parts: int):
+    """Recursive coordinate bisection of the cells (a Metis-style partition
+    without the library dependency; the paper partitions its meshes with Metis,
+    L728-735): split the cell set at the median of its longest extent, in
+    proportion to the parts on each side, until every part has its cells.
+    Deterministic (ties broken by cell id); parts are spatially compact, so a
+    part's halo is its surface.  Returns part[n_cells] (int32)."""
+    import numpy as np
+    x = np.asarray(centres, dtype=np.float64)
+    out = np.zeros(x.shape[0], np.int32)
+
+    def rec(ids, p0, n):
+        if n == 1:
+            out[ids] = p0
+            return
+        ext = x[ids].max(axis=0) - x[ids].min(axis=0)
+        ax = int(np.argmax(ext))
+        order = ids[np.lexsort((ids, x[ids, ax]))]
+        nl = n // 2
+        k = int(round(len(ids) * nl / n))
+        rec(order[:k], p0, nl)
+        rec(order[k:], p0 + nl, n - nl)
+
+    rec(np.arange(x.shape[0]), 0, int(n_parts))
+    return out
+
+
 def env_rank_world():
     return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
             int(os.environ.get("LOCAL_RANK", "0")))
@@ -33,9 +67,13 @@ def share_nccl_id(pg, rank: int, make_id=None) -> bytes:
     return bytes(nid)
 
 
-def make_solver(cfg, pg=None, **kw):
-    """Solver for this rank (world from the process group, if any)."""
+def make_solver(cfg, pg=None, n_cell_parts=1, **kw):
+    """Solver for this rank (world from the process group, if any).
+    n_cell_parts > 1: cell partitioning (N3) by partition_cells of the cell
+    centres, combined with band sharding over world / n_cell_parts groups."""
     from . import bte
+    if n_cell_parts > 1:
+        kw.update(cell_part=partition_cells(cfg.mesh["cell_centre"], n_cell_parts), n_cell_parts=n_cell_parts)
     if pg is None or pg.get_world_size() == 1:
         return bte.solver_from_config(cfg, **kw)
     rank, world = pg.get_rank(), pg.get_world_size()
