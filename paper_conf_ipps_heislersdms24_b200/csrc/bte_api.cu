@@ -94,6 +94,7 @@ struct bte_ctx {
     // box path (structured hex grid in lexicographic order, flux_box_kernel)
     bool box = false;
     int32_t bn[3] = {0, 0, 0}, bzside[2] = {0, 0};
+    bool bflat = false;  // 2-D box grid (no axis-2 faces; isothermal walls on grid axis 1)
     double bgeo[3] = {0, 0, 0};
     int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
     bool td = false;  // temperature-dependent relaxation times (rate tables)
@@ -340,10 +341,118 @@ struct BoxDetect {
     int ax[3] = {0, 1, 2};      // grid axis -> mesh axis
     int32_t n[3] = {0, 0, 0};   // extents along grid axes
     double g[3] = {0, 0, 0};    // A / V along grid axes
-    int zside[2] = {1, 1};      // grid axis-2 low / high side: 0 isothermal, 1 specular
+    int zside[2] = {1, 1};      // ghost axis (3-D: grid axis 2; 2-D: grid axis 1) low / high side:
+                                // 0 isothermal, 1 specular
+    bool flat = false;          // 2-D grid: n[2] = 1, no axis-2 faces (g[2] = 0)
     std::vector<int32_t> cell_at;
-    std::vector<int64_t> zbface[2];  // [n1][n0] boundary face id of the axis-2 side faces
+    std::vector<int64_t> zbface[2];  // boundary face ids of the ghost-axis sides: 3-D [n1][n0], 2-D [n0]
 };
+
+// 2-D structured quad grid (the paper's Fig.-1 and Fig.-10 meshes): four faces
+// per cell with normals exactly +-e_x, +-e_y, an n_0 x n_1 lattice, uniform
+// A / V per axis, each side uniformly isothermal or specular with isothermal
+// sides on at most one axis, which becomes grid axis 1 (its wall ghosts are
+// staged rows of I0_b(T_wall), Eq. 6); grid axis 0 (contiguous, specular
+// sides) must have even extent.  Grid axis 2 is a single layer with no faces.
+BoxDetect detect_box2d(const bte_mesh *m, const bte_bcs *bc) {
+    BoxDetect r;
+    if (m->dim != 2) return r;
+    const int64_t nc = m->n_cells;
+    std::vector<int64_t> fa((size_t)nc * 4, -1);  // [cell][2 axis + (normal > 0)] -> face
+    for (int64_t c = 0; c < nc; ++c) {
+        if (m->face_offsets[c + 1] - m->face_offsets[c] != 4) return r;
+        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1]; ++f) {
+            const double *nv = m->face_normal + 3 * f;
+            int a = -1;
+            for (int t = 0; t < 2; ++t)
+                if (nv[t] == 1.0 || nv[t] == -1.0) a = t;
+            if (a < 0 || nv[1 - a] != 0.0 || nv[2] != 0.0) return r;
+            int64_t &slot = fa[(size_t)c * 4 + 2 * a + (nv[a] > 0.0)];
+            if (slot >= 0) return r;
+            slot = f;
+        }
+    }
+    auto nbr = [&](int64_t c, int a, int sd) { return m->face_nbr[fa[(size_t)c * 4 + 2 * a + sd]]; };
+    int64_t corner = -1;
+    for (int64_t c = 0; c < nc && corner < 0; ++c)
+        if (nbr(c, 0, 0) < 0 && nbr(c, 1, 0) < 0) corner = c;
+    if (corner < 0) return r;
+    int64_t n[2];
+    for (int a = 0; a < 2; ++a) {
+        n[a] = 1;
+        for (int64_t c = corner; nbr(c, a, 1) >= 0; c = nbr(c, a, 1))
+            if (++n[a] > nc) return r;
+    }
+    if (n[0] * n[1] != nc) return r;
+    std::vector<int32_t> at(nc, -1);  // mesh-axis lexicographic position -> cell
+    std::vector<char> seen(nc, 0);
+    int64_t ys = corner;
+    for (int64_t y = 0; y < n[1]; ++y) {
+        if (y > 0 && (ys = nbr(ys, 1, 1)) < 0) return r;
+        int64_t c = ys;
+        for (int64_t x = 0; x < n[0]; ++x) {
+            if (x > 0 && (c = nbr(c, 0, 1)) < 0) return r;
+            if (seen[c]) return r;
+            seen[c] = 1;
+            at[y * n[0] + x] = (int32_t)c;
+        }
+    }
+    int kind[2][2] = {{-1, -1}, {-1, -1}};  // -1 none yet, 0 iso, 1 sym, 2 mixed
+    double g[2];
+    for (int a = 0; a < 2; ++a) g[a] = m->face_area[fa[(size_t)at[0] * 4 + 2 * a + 1]] / m->cell_volume[at[0]];
+    for (int64_t y = 0; y < n[1]; ++y)
+        for (int64_t x = 0; x < n[0]; ++x) {
+            const int64_t p[2] = {x, y};
+            const int64_t c = at[y * n[0] + x];
+            for (int a = 0; a < 2; ++a)
+                for (int sd = 0; sd < 2; ++sd) {
+                    const int64_t f = fa[(size_t)c * 4 + 2 * a + sd];
+                    if (m->face_area[f] / m->cell_volume[c] != g[a]) return r;
+                    int64_t q[2] = {p[0], p[1]};
+                    q[a] += sd ? 1 : -1;
+                    const int64_t v = m->face_nbr[f];
+                    if (q[a] >= 0 && q[a] < n[a]) {
+                        if (v != at[q[1] * n[0] + q[0]]) return r;
+                    } else {
+                        if (v >= 0) return r;
+                        const int k = bc->kind[-1 - v] == BTE_BC_ISOTHERMAL ? 0 : 1;
+                        int &s = kind[a][sd];
+                        s = s < 0 ? k : (s == k ? k : 2);
+                    }
+                }
+        }
+    int isoax = -1;
+    for (int a = 0; a < 2; ++a) {
+        if (kind[a][0] == 2 || kind[a][1] == 2) return r;
+        if (kind[a][0] == 0 || kind[a][1] == 0) {
+            if (isoax >= 0) return r;
+            isoax = a;
+        }
+    }
+    if (isoax >= 0) r.ax[0] = 1 - isoax, r.ax[1] = isoax;
+    else if (n[0] % 2 == 0) r.ax[0] = 0, r.ax[1] = 1;
+    else r.ax[0] = 1, r.ax[1] = 0;
+    r.ax[2] = 2;
+    if (n[r.ax[0]] % 2 != 0) return r;
+    r.flat = true;
+    for (int t = 0; t < 2; ++t) r.n[t] = (int32_t)n[r.ax[t]], r.g[t] = g[r.ax[t]];
+    r.n[2] = 1;
+    r.g[2] = 0.0;
+    for (int sd = 0; sd < 2; ++sd) r.zside[sd] = kind[r.ax[1]][sd];
+    r.cell_at.resize(nc);
+    for (int sd = 0; sd < 2; ++sd) r.zbface[sd].assign((size_t)r.n[0], -1);
+    for (int64_t i1 = 0; i1 < r.n[1]; ++i1)
+        for (int64_t i0 = 0; i0 < r.n[0]; ++i0) {
+            int64_t p[2];
+            p[r.ax[0]] = i0, p[r.ax[1]] = i1;
+            const int32_t c = at[p[1] * n[0] + p[0]];
+            r.cell_at[i1 * r.n[0] + i0] = c;
+            for (int sd = 0; sd < 2; ++sd)
+                if (i1 == (sd ? r.n[1] - 1 : 0)) r.zbface[sd][i0] = -1 - nbr(c, r.ax[1], sd);
+        }
+    r.ok = true;
+    return r;
+}
 
 BoxDetect detect_box(const bte_mesh *m, const bte_bcs *bc) {
     BoxDetect r;
@@ -578,21 +687,32 @@ BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
     return b;
 }
 
+// doubles per ring stage (2-D: + the two isothermal wall rows of grid axis 1)
+int box_stage(const bte_ctx *ctx) {
+    return (ctx->td ? bte::box_stage_elems<true>() : bte::box_stage_elems<false>()) + (ctx->bflat ? 2 * bte::kBoxTX : 0);
+}
+
 size_t box_smem(const bte_ctx *ctx) {
-    const int stage = ctx->td ? bte::box_stage_elems<true>() : bte::box_stage_elems<false>();
+    const int stage = box_stage(ctx);
     return ((size_t)ctx->box_stages * stage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
                sizeof(double) +
            (size_t)kBoxMaxOrbChunk * sizeof(bte::BoxOrbitC);
 }
 
-template <bool TD>
+// The box kernel instantiation of a context: rate tables or not, 2-D (3 CTAs
+// per SM) or 3-D (2).
+using BoxKernel = void (*)(const bte::BoxParams, const CUtensorMap, const CUtensorMap, const CUtensorMap,
+                           const CUtensorMap, const CUtensorMap);
+BoxKernel box_kernel(const bte_ctx *ctx) {
+    if (ctx->bflat) return ctx->td ? bte::flux_box_kernel<true, true> : bte::flux_box_kernel<false, true>;
+    return ctx->td ? bte::flux_box_kernel<true, false> : bte::flux_box_kernel<false, false>;
+}
+
 bte_status box_setup_kernel(bte_ctx *ctx) {
     const size_t smem = box_smem(ctx);
-    CUDA_TRY(ctx, cudaFuncSetAttribute(bte::flux_box_kernel<TD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem));
+    CUDA_TRY(ctx, cudaFuncSetAttribute(box_kernel(ctx), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int occ = 0;
-    CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, bte::flux_box_kernel<TD>, bte::kBoxThreads,
-                                                                smem));
+    CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, box_kernel(ctx), bte::kBoxThreads, smem));
     ctx->box_ctas_per_sm = std::max(1, occ);
     return BTE_OK;
 }
@@ -714,12 +834,8 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
         if (items > INT32_MAX) return set_err(&ctx->err, "box kernel: %lld work items", (long long)items), BTE_EINVAL;
         const dim3 grid((unsigned)items);
         ev_mark(ctx, kPhFlux, true);
-        if (ctx->td)
-            bte::flux_box_kernel<true><<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(
-                p, ctx->tm_in, ctx->tm_out, ctx->tm_i0, ctx->tm_side, ctx->tm_rate);
-        else
-            bte::flux_box_kernel<false><<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(
-                p, ctx->tm_in, ctx->tm_out, ctx->tm_i0, ctx->tm_side, ctx->tm_rate);
+        box_kernel(ctx)<<<grid, dim3(bte::kBoxThreads), smem, ctx->stream>>>(p, ctx->tm_in, ctx->tm_out, ctx->tm_i0,
+                                                                           ctx->tm_side, ctx->tm_rate);
         ev_mark(ctx, kPhFlux, false);
         ctx->st.kernel_launches++;
         slot += p.n_slices;
@@ -1346,8 +1462,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     BoxDetect bx;
     std::vector<bte::BoxOrbit> orbs;
     if (paired_geom && !cpart && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
-        bx = detect_box(m, bc);
-    const bool use_box = bx.ok && box_orbits(dr, bx.ax, bx.zside[0] == 1 || bx.zside[1] == 1, &orbs);
+        bx = m->dim == 3 ? detect_box(m, bc) : detect_box2d(m, bc);
+    const bool use_box = bx.ok && box_orbits(dr, bx.ax, !bx.flat && (bx.zside[0] == 1 || bx.zside[1] == 1), &orbs);
 
     // --- internal cell order from the optional centroids: cells are grouped
     // into bricks of 8 x 8 x 4 (2-D: 16 x 16) typical cell sizes, Morton order
@@ -1631,18 +1747,22 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         for (int a = 0; a < 3; ++a) ctx->bn[a] = bx.n[a], ctx->bgeo[a] = bx.g[a];
         ctx->bzside[0] = bx.zside[0];
         ctx->bzside[1] = bx.zside[1];
+        ctx->bflat = bx.flat;
         ctx->n_orb = (int)orbs.size();
         // shared memory for 2 CTAs per SM: ring stages x 12 KB + 16 KB output + L x 2 KB energy
         // (rate law: 16 KB stages; 5 stages x 4 layers fit twice per SM, measured best)
         const char *ev = std::getenv("BTE_BOX_STAGES");
-        ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : (td ? 5 : 6)));
+        // (2-D, 3 CTAs per SM: 4 stages, 3 with the rate rows; orbit chunks of 25 (a C3 slice = 4 chunks))
+        const int def_stages = bx.flat ? (td ? 3 : 4) : (td ? 5 : 6);
+        ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : def_stages));
+        if (bx.flat) ctx->box_oc = 25;
         ev = std::getenv("BTE_BOX_L");
         ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : (td ? 4 : 8)));
         ev = std::getenv("BTE_BOX_NBB");
         if (ev) ctx->box_nbb = std::max(1, std::atoi(ev));
         ev = std::getenv("BTE_BOX_OC");
         if (ev) ctx->box_oc = std::max(1, std::atoi(ev));
-        CREATE_TRY(ctx->td ? box_setup_kernel<true>(ctx) : box_setup_kernel<false>(ctx));
+        CREATE_TRY(box_setup_kernel(ctx));
     }
 
     // --- slab pool: nb_loc current slabs + n_spare workspace slabs
@@ -1799,7 +1919,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             db[d] = make_double4(sd[bx.ax[0]], sd[bx.ax[1]], sd[bx.ax[2]], dr->w[d]);
         }
         CREATE_TRY(upload(ctx, &ctx->dirs_box, db));
-        const int64_t nside = (int64_t)bx.n[0] * bx.n[1];
+        const int64_t nside = bx.flat ? (int64_t)bx.n[0] : (int64_t)bx.n[0] * bx.n[1];
         std::vector<int32_t> col(2 * nside, -1);
         for (int sd = 0; sd < 2; ++sd)
             if (bx.zside[sd] == 0)
@@ -1815,12 +1935,16 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         const uint32_t bin[5] = {bte::kBoxBX, bte::kBoxBY, 1, 1, 1}, bout[5] = {bte::kBoxTX, bte::kBoxTY, 1, 1, 1};
         const uint64_t di0[4] = {n0, n1, n2, (uint64_t)nb_loc}, si0[3] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8};
         const uint64_t dsd[4] = {n0, n1, 2, (uint64_t)nb_loc}, ssd[3] = {n0 * 8, n0 * n1 * 8, 2 * n0 * n1 * 8};
+        // 2-D: the wall rows of grid axis 1 as {n0, 2, nb_loc}, one 32-cell row per load
+        const uint64_t dsf[3] = {n0, 2, (uint64_t)nb_loc}, ssf[2] = {n0 * 8, 2 * n0 * 8};
+        const uint32_t bsf[3] = {bte::kBoxTX, 1, 1};
         const uint64_t drt[5] = {n0, n1, n2, (uint64_t)nb_loc, 2},
                        srt[4] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8, (uint64_t)nb_loc * nc * 8};
         if (!encode_map(&ctx->tm_in, ctx->pool, 5, dpool, spool, bin) ||
             !encode_map(&ctx->tm_out, ctx->pool, 5, dpool, spool, bout) ||
             !encode_map(&ctx->tm_i0, ctx->i0, 4, di0, si0, bout) ||
-            !encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin) ||
+            !(bx.flat ? encode_map(&ctx->tm_side, ctx->side_tab, 3, dsf, ssf, bsf)
+                      : encode_map(&ctx->tm_side, ctx->side_tab, 4, dsd, ssd, bin)) ||
             !encode_map(&ctx->tm_rate, ctx->td ? ctx->rates : ctx->i0, ctx->td ? 5 : 4, ctx->td ? drt : di0,
                         ctx->td ? srt : si0, bout)) {
             set_err(&ctx->err, "cuTensorMapEncodeTiled failed for the box kernel maps");

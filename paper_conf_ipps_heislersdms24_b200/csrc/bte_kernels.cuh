@@ -742,9 +742,12 @@ constexpr int kBoxPlane = 320;               // doubles per staged plane (128-by
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
 constexpr int kBoxMaxStages = 12;
-#ifndef BTE_BOX_MIN_BLOCKS
-#define BTE_BOX_MIN_BLOCKS 2
-#endif
+// Resident CTAs per SM the kernel is compiled for (register cap): 3-D grids 2
+// (96 registers, 6 stages of 12 KB plus L x 2 KB of energy rows); 2-D grids 3
+// (72 registers, no spills, 4 stages): a 2-D stage is one layer, so CTAs are
+// short and more of them per SM hide the per-stage handshake (C3 flux 0.83 ->
+// 0.96 of measured HBM, measured on B200; 3-D loses with 3).
+constexpr int kBoxMinBlocks3D = 2, kBoxMinBlocks2D = 3;
 // doubles per stage: 4 direction planes + the I0 row (+ the two rate rows with
 // temperature-dependent relaxation times)
 template <bool TD>
@@ -767,7 +770,7 @@ struct BoxParams {
     int32_t band0, slot0;      // rank-local first band-row; first energy slot
     int32_t nc;
     int32_t stages;            // shared-memory ring depth
-    int32_t zside[2];          // axis-2 low / high side: 0 isothermal, 1 specular
+    int32_t zside[2];          // ghost-axis low / high side (3-D: axis 2; 2-D: axis 1): 0 isothermal, 1 specular
     int32_t rsel_cur, rsel_next;  // temperature-dependent rates: table halves (current, next)
     int32_t rate_r2;           // ... R2 weights rate_next / v_b (else the constant cw)
     double dt;
@@ -789,6 +792,13 @@ __device__ __forceinline__ void tma_load_5d(void *dst, const void *tmap, int c0,
         "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
         " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_3d(void *dst, const void *tmap, int c0, int c1, int c2, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
         : "memory");
 }
 __device__ __forceinline__ void tma_load_4d(void *dst, const void *tmap, int c0, int c1, int c2, int c3,
@@ -827,6 +837,7 @@ __device__ __forceinline__ void bar_compute() { asm volatile("bar.sync 1, %0;" :
 //   tm_out  same tensor, box {32, 8, 1, 1, 1} (stores)
 //   tm_i0   I0 table as {n0, n1, n2, nb_loc}, box {32, 8, 1, 1}
 //   tm_side isothermal axis-2 side tables as {n0, n1, 2, nb_loc}, box {34, 9, 1, 1}
+//           (2-D: the axis-1 wall rows as {n0, 2, nb_loc}, box {32, 1, 1})
 //   tm_rate rate tables 1/tau_b(T) as {n0, n1, n2, nb_loc, 2}, box {32, 8, 1, 1, 1}
 // Box origin of slot j: axis 0 at x0 - 2 (s_0 > 0: upwind is x - 1) or x0
 // (s_0 < 0: x + 1); axis 1 at y0 - 1 (s_1 > 0) or y0.
@@ -873,12 +884,14 @@ struct BoxOrbitC {
     int32_t pad;
 };
 
-template <bool TD>
-__global__ void __launch_bounds__(kBoxThreads, BTE_BOX_MIN_BLOCKS)
+template <bool TD, bool FLAT>
+__global__ void __launch_bounds__(kBoxThreads, FLAT ? kBoxMinBlocks2D : kBoxMinBlocks3D)
 flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUtensorMap tm_in,
                 const __grid_constant__ CUtensorMap tm_out, const __grid_constant__ CUtensorMap tm_i0,
                 const __grid_constant__ CUtensorMap tm_side, const __grid_constant__ CUtensorMap tm_rate) {
-    constexpr int kStage = box_stage_elems<TD>();
+    constexpr int kGhost = box_stage_elems<TD>();  // 2-D: stage offset of the two wall rows
+    constexpr int kStage = kGhost + (FLAT ? 2 * kBoxTX : 0);
+    constexpr bool flat = FLAT;
     extern __shared__ __align__(128) double bsm[];
 #ifdef BTE_BOX_FIXED_S
     constexpr int S = BTE_BOX_FIXED_S;
@@ -928,7 +941,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                 for (int o = w.o0; o < w.o1; ++o) {
                     const BoxOrbitC &ob = sorb[o - w.o0];
                     const bool asc = ob.asc;
-                    for (int j = 0; j <= w.Lc; ++j) {
+                    for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                         if (wrapped)
                             while (!mbar_try_wait(&empty[s], ph ^ 1u)) {
                             }
@@ -948,8 +961,13 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             }
                         } else {
                             const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
-                            mbar_arrive_expect_tx(&full[s],
-                                                  (4 * kBoxBoxElems + (TD ? 3 : 1) * kBoxCells) * sizeof(double));
+                            // 2-D: the isothermal wall rows I0_b(T_wall) of the tiles on those walls (Eq. 6)
+                            const bool glo = flat && p.zside[0] == 0 && w.y0 == 0;
+                            const bool ghi = flat && p.zside[1] == 0 && w.y0 + kBoxTY >= p.n1;
+                            mbar_arrive_expect_tx(&full[s], (4 * kBoxBoxElems + (TD ? 3 : 1) * kBoxCells +
+                                                             (glo + ghi) * kBoxTX) * sizeof(double));
+                            if (glo) tma_load_3d(st + kGhost, &tm_side, w.x0, 0, bl, &full[s]);
+                            if (ghi) tma_load_3d(st + kGhost + kBoxTX, &tm_side, w.x0, 1, bl, &full[s]);
                             for (int q = 0; q < 4; ++q)
                                 tma_load_5d(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
                                             ob.d[q], slab, &full[s]);
@@ -988,6 +1006,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         const bool wall1 = (q & 2) ? gy == p.n1 - 1 : gy == 0;
         ux[q] = wall0 ? own[q ^ 1] : own[q] + ((q & 1) ? 1 : -1);
         uy[q] = wall1 ? own[q ^ 2] : own[q] + ((q & 2) ? kBoxBX : -kBoxBX);
+        if (flat && wall1 && p.zside[(q & 2) ? 1 : 0] == 0) uy[q] = kGhost + ((q & 2) ? kBoxTX : 0) + tx;
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
 
@@ -1004,7 +1023,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             const double kvout = kv * ((orb.a[0] + orb.a[1]) + orb.a[2]);
             const double coef_c = (1.0 - p.dtit[k]) - kvout;  // constant rates
             const double m0 = -orb.a[0], m1 = -orb.a[1], m2 = -orb.a[2];
-            for (int j = 0; j <= w.Lc; ++j) {
+            for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
                 if (j == 0) {
@@ -1031,7 +1050,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         const double ic = cur[own[q]];
                         double infl = m0 * cur[ux[q]];
                         infl = fma(m1, cur[uy[q]], infl);
-                        infl = fma(m2, prv[own[q]], infl);
+                        if (!flat) infl = fma(m2, prv[own[q]], infl);
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
                         out[q * kBoxCells + tid] = inew;
                         acc = fma(wq[q], inew, acc);
@@ -1040,8 +1059,12 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                     *ea = fma(cw, acc, *ea);
                     __syncwarp();
                     if (lane == 0) {  // the previous layer's stage is no longer needed
-                        mbar_arrive(&empty[sp]);
-                        if (j == w.Lc) mbar_arrive(&empty[s]);
+                        if (flat) {
+                            mbar_arrive(&empty[s]);
+                        } else {
+                            mbar_arrive(&empty[sp]);
+                            if (j == w.Lc) mbar_arrive(&empty[s]);
+                        }
                     }
                     sp = s;
                     fence_smem_to_async();

@@ -24,7 +24,7 @@ def bte_lib():
     return mod
 
 
-@pytest.mark.parametrize("name,variant", [("C6", 4), ("C6t", 0)])
+@pytest.mark.parametrize("name,variant", [("C6", 6), ("C6t", 0)])
 def test_fig10_workload(bte_lib, oracle_mod, name, variant):
     cfg = gen.make_config(name)
     Io, To = oracle_run(oracle_mod, cfg, 100)

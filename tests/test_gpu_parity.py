@@ -38,7 +38,7 @@ def test_c1_full_50_steps(bte, oracle_mod):
     Io, To = oracle_run(oracle_mod, cfg, cfg.nsteps)
     Ig, Tg, st = gpu_run(cfg, cfg.nsteps)
     assert_parity(Ig, Tg, Io, To)
-    assert st["flux_variant"] == 4  # 256 cells: too small for the stencil windows
+    assert st["flux_variant"] == 6  # a 2-D quad grid with Fig.-1 walls: the box kernel
     assert st["steps"] == cfg.nsteps
     assert To.max() > 300.5  # the hot spot moved heat in
 

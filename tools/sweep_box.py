@@ -2,6 +2,7 @@
 """Box-kernel work-split sweep (one process, the config built once).
 
     python tools/sweep_box.py C4 "5:80 5:60:6:8 1:80 ..."   (band_group:dir_chunk[:stages:L], 0 = auto)
+    python tools/sweep_box.py C3:128x120 "..."               (C3's tables on another grid)
 
 Equilibrium IC (the flux kernel's time does not depend on the values); prints
 the flux-kernel time per step from the library's CUDA events and the fraction
@@ -23,7 +24,16 @@ def main():
     name = sys.argv[1]
     combos = [tuple(int(x) for x in c.split(":")) for c in sys.argv[2].split()]
     steps = int(sys.argv[3]) if len(sys.argv) > 3 else 10
-    cfg = gen.make_config(name)
+    if ":" in name:  # e.g. "C3:128x120": the config's bands / directions / walls on another grid
+        base, shape = name.split(":")
+        cfg = gen.make_config(base)
+        shape = tuple(int(v) for v in shape.split("x"))
+        h = cfg.mesh["spacing"][0]
+        mesh = gen.gen_mesh(shape, (h,) * len(shape))
+        import dataclasses
+        cfg = dataclasses.replace(cfg, mesh=mesh, bcs=gen.gen_bcs_fig1(mesh, radius=4 * h))
+    else:
+        cfg = gen.make_config(name)
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
     nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
     for combo in combos:
