@@ -123,9 +123,10 @@ def _dist():
     return rank, world, local
 
 
-def cpu_baseline(cfg, budget_s=15.0, max_rows=16):
+def cpu_baseline(cfg, budget_s=15.0, max_rows=None):
     """The oracle as it stands, on this host's cores, on a bounded sample of the
-    workload: the full mesh and direction set, the first k band-rows, 1 step."""
+    workload (about budget_s of CPU work): the full mesh and direction set, the
+    first k band-rows, and with all rows in the sample as many steps as fit."""
     import numpy as np
     import oracle
     from paper_conf_ipps_heislersdms24_b200 import inputs as gen
@@ -144,8 +145,9 @@ def cpu_baseline(cfg, budget_s=15.0, max_rows=16):
         return time.perf_counter() - t0
 
     t1 = run(1, 1)
-    k = int(max(1, min(max_rows, cfg.bands["n_bands"], budget_s / max(t1, 1e-3))))
-    steps = 1
+    nb = cfg.bands["n_bands"]
+    k = int(max(1, min(max_rows or nb, nb, budget_s / max(t1, 1e-3))))
+    steps = int(max(1, min(50, budget_s / max(t1 * k, 1e-3)))) if k == nb else 1
     t = run(k, steps)
     upd = cfg.mesh["n_cells"] * cfg.dirs["n_dirs"] * k * steps
     return {"value": upd / t, "unit": METRIC.replace("updates/s", "updates/s"), "cores": cores,
