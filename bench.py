@@ -33,6 +33,7 @@ sys.path.insert(0, ROOT)
 METRIC = "cell*dir*band updates/s"
 WORKLOADS = {
     "C3": "2-D 120x120 quad mesh (525 um), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
+    "C3t": "2-D 120x120 quads split into 28800 triangles (525 um), 55 band-rows, 400 dirs, Fig.1 walls",
     "C4": "3-D 64x64x32 hex mesh (8.2 um cells), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
     "C5": "3-D 96x96x96 hex mesh (8.2 um cells), 55 band-rows (40 spectral), 400 dirs, Fig.1 walls",
 }

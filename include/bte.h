@@ -126,7 +126,7 @@ typedef struct {
 /* bte_options.flags */
 #define BTE_FLAG_PROFILE 1u       /* record CUDA events around every phase (see bte_stats) */
 #define BTE_FLAG_GENERIC_FACES 2u /* never use the opposite-face-pair layout (testing) */
-#define BTE_FLAG_NO_TMA 4u        /* paired meshes: register-pipelined kernel instead of the
+#define BTE_FLAG_NO_TMA 4u        /* register-pipelined flux kernel instead of the
                                      TMA-staged one (testing / comparison) */
 #define BTE_FLAG_STENCIL 8u       /* structured index order: stencil-staged kernel (near/far
                                      TMA windows; L2-bandwidth-heavy, opt-in) */
@@ -196,7 +196,8 @@ typedef struct {
     int32_t flux_variant;      /* flux kernel in use: 0 generic faces, 1 paired, 2 paired +
                                   uniform geometry, 3 TMA-staged, 4 TMA-staged + uniform
                                   geometry, 5 stencil-staged (structured order), 6 box
-                                  (structured 3-D grid, tensor copies, z-marching) */
+                                  (structured 2-D / 3-D grid, tensor copies), 7 TMA-staged
+                                  generic faces (unstructured meshes) */
     double ms_halo;            /* cell partitioning: halo pack + exchange + unpack */
     int64_t halo_bytes;        /* halo bytes this rank sends per step (all segments) */
 } bte_stats;

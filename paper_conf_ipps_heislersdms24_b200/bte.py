@@ -78,7 +78,8 @@ class Stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
-FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil", 6: "box"}
+FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil", 6: "box",
+                 7: "tma-generic"}
 
 EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte_get_temperature",
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",

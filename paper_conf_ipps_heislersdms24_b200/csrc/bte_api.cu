@@ -204,6 +204,28 @@ void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p)
     bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
 }
 
+// TMA-staged generic-face kernel (general meshes): kStages x BG x 2 KB ring.
+template <int DIM, int MF, int BG>
+void flux_tma_generic_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    const size_t smem = (size_t)bte::kStagesG * BG * bte::kTile * sizeof(double);
+    static size_t attr = 0;
+    if (attr < smem) {
+        cudaFuncSetAttribute(bte::flux_tma_generic_kernel<DIM, MF, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smem);
+        attr = smem;
+    }
+    bte::flux_tma_generic_kernel<DIM, MF, BG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+}
+
+template <int DIM, int MF>
+FluxLaunch pick_tma_generic(int bg) {
+    switch (bg) {
+        case 1: return flux_tma_generic_launch_t<DIM, MF, 1>;
+        case 2: return flux_tma_generic_launch_t<DIM, MF, 2>;
+        default: return flux_tma_generic_launch_t<DIM, MF, 4>;
+    }
+}
+
 // Stencil-staged kernel (structured meshes): near + far windows per plane.
 template <int DIM, int NP, int BG>
 void flux_stencil_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
@@ -279,8 +301,14 @@ FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, boo
     }
     if (paired && uniform_g) return dim == 2 ? pick_paired<2, 2, true>(bg) : pick_paired<3, 3, true>(bg);
     if (paired) return dim == 2 ? pick_paired<2, 2, false>(bg) : pick_paired<3, 3, false>(bg);
-    if (dim == 2) return mf_t == 4 ? pick_generic<2, 4>(bg) : pick_generic<2, 8>(bg);
-    return mf_t == 6 ? pick_generic<3, 6>(bg) : pick_generic<3, 8>(bg);
+    if (tma) {
+        if (dim == 2) return mf_t == 3 ? pick_tma_generic<2, 3>(bg) : mf_t == 4 ? pick_tma_generic<2, 4>(bg)
+                                                                               : pick_tma_generic<2, 8>(bg);
+        return mf_t == 4 ? pick_tma_generic<3, 4>(bg) : mf_t == 6 ? pick_tma_generic<3, 6>(bg)
+                                                                  : pick_tma_generic<3, 8>(bg);
+    }
+    if (dim == 2) return mf_t == 3 ? pick_generic<2, 3>(bg) : mf_t == 4 ? pick_generic<2, 4>(bg) : pick_generic<2, 8>(bg);
+    return mf_t == 4 ? pick_generic<3, 4>(bg) : mf_t == 6 ? pick_generic<3, 6>(bg) : pick_generic<3, 8>(bg);
 }
 
 int legal_bg(int bg, bool paired) {
@@ -1573,7 +1601,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // (the paired layout's 5-bit face codes hold up to 16 specular classes)
     // (with the rate law only the box kernel and the generic-face kernel read rate tables)
     const bool paired = paired_geom && (int)cls_of.size() <= bte::kMaxPairedClasses && !(td && !use_box);
-    const int mf_t = paired ? m->dim : (m->dim == 2 ? (mf <= 4 ? 4 : 8) : (mf <= 6 ? 6 : 8));
+    const int mf_t = paired ? m->dim
+                            : (m->dim == 2 ? (mf <= 3 ? 3 : mf <= 4 ? 4 : 8) : (mf <= 4 ? 4 : mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
     std::vector<int32_t> nbr_h(ell), nbm_h(paired ? ell : 1, 0);
     std::vector<uint32_t> fcode_h(paired ? nc : 1, (1u << (10 * m->dim)) - 1u);  // all interior
@@ -1720,7 +1749,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
 
     // --- launch plan knobs (band group: measured best on B200)
     ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
-    ctx->tma = paired && ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);
+    ctx->tma = ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);  // (paired or generic faces)
     if (ctx->tma && ctx->uniform_g && stencil_order && (o->flags & BTE_FLAG_STENCIL)) {  // near / far windows
         int32_t halo = 0, nfar = 0;
         for (int j = 0; j < m->dim; ++j) {
@@ -1739,7 +1768,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     // auto band group (measured on B200): the largest group that
     // compiles without spills for the chosen kernel
-    const int auto_bg = !paired ? 2 : ctx->stencil ? 4 : ctx->tma ? (ctx->uniform_g ? 5 : 3) : 8;
+    const int auto_bg = !paired ? 4 : ctx->stencil ? 4 : ctx->tma ? (ctx->uniform_g ? 5 : 3) : 8;
     ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : auto_bg, paired);
     if (use_box) {  // one band-row per stage; band_group / dir_chunk size the CTA's work instead
         ctx->box = true;
@@ -2308,7 +2337,8 @@ bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st) {
     if (!ctx || !st) return BTE_EINVAL;
     *st = ctx->st;
     st->dir_chunks = ctx->dir_chunks;
-    st->flux_variant = ctx->box ? 6 : ctx->stencil ? 5 : ctx->tma ? (ctx->uniform_g ? 4 : 3) : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
+    st->flux_variant = ctx->box ? 6 : ctx->stencil ? 5 : ctx->tma ? (!ctx->paired ? 7 : ctx->uniform_g ? 4 : 3)
+                                                 : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
     return BTE_OK;
 }
 

@@ -537,6 +537,150 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
 }
 
 // ---------------------------------------------------------------------------
+// TMA-staged kernel for general meshes (unstructured: triangles, split faces,
+// any face-based mesh).  The staging of flux_tma_kernel (one
+// 256-cell tile per block in the locality order, every (band-row, direction)
+// plane segment streamed into a kStages ring by cp.async.bulk, in-tile upwind
+// values from shared memory, halo / boundary values as global loads issued
+// before the stage wait) with the arithmetic of flux_kernel: up to MF faces per
+// cell, outflow sum_j max(alpha_j, 0), inflow sum_j min(alpha_j, 0) I_up
+// (Eq. 3/5 with the Eq. 6 ghosts), and with the rate law the cell's own rates.
+#ifndef BTE_TMA_GENERIC_STAGES
+#define BTE_TMA_GENERIC_STAGES 8
+#endif
+// Ring depth of the generic-face kernel: its per-thread state (faces x band
+// rows) keeps BG small, so the producer runs further ahead instead.
+constexpr int kStagesG = BTE_TMA_GENERIC_STAGES;
+template <int DIM, int MF, int BG>
+__global__ void __launch_bounds__(kTmaThreads, BTE_MIN_BLOCKS)
+flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
+    extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][kTile]
+    __shared__ __align__(8) uint64_t full[kStagesG];
+    __shared__ __align__(8) uint64_t empty[kStagesG];
+    const int tid = threadIdx.x;
+    const int tile0 = blockIdx.x * kTile;
+    const int grp = blockIdx.y / p.n_dchunks;
+    const int dch = blockIdx.y - grp * p.n_dchunks;
+    const int lg0 = grp * BG;
+    const int d0 = dch * p.dchunk;
+    const int nit = min(p.nd, d0 + p.dchunk) - d0;
+    const int nc = p.nc;
+    const int ps = p.ps;
+    constexpr uint32_t kBytes = BG * kTile * sizeof(double);
+
+    if (tid == 0) {
+#pragma unroll
+        for (int s = 0; s < kStagesG; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kComputeWarps);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (tid >= kTile) {  // ------------------------------------------ producer warp
+        if (tid == kTile) {
+            for (int i = 0; i < nit; ++i) {
+                const int st = i % kStagesG;
+                if (i >= kStagesG)
+                    while (!mbar_try_wait(&empty[st], ((i / kStagesG) - 1) & 1)) {
+                    }
+                mbar_arrive_expect_tx(&full[st], kBytes);
+                const int64_t off = (int64_t)(d0 + i) * ps + tile0;
+#pragma unroll
+                for (int k = 0; k < BG; ++k)
+                    bulk_g2s(ring + (st * BG + k) * kTile, p.in_ptr[lg0 + k] + off, kTile * sizeof(double), &full[st]);
+            }
+        }
+        return;
+    }
+
+    // --------------------------------------------------------------- compute warps
+    const int c = tile0 + tid;
+    const bool valid = c < nc;
+    const int lane = tid & 31;
+    int nbr[MF];
+    uint32_t code[MF];
+    double gx[MF], gy[MF], gz[MF];
+    bool has_bnd = false;
+#pragma unroll
+    for (int j = 0; j < MF; ++j) {
+        const int q = j * nc + c;
+        nbr[j] = valid ? __ldg(p.nbr + q) : c;
+        gx[j] = valid ? __ldg(p.gx + q) : 0.0;
+        gy[j] = valid ? __ldg(p.gy + q) : 0.0;
+        gz[j] = (DIM == 3 && valid) ? __ldg(p.gz + q) : 0.0;
+        code[j] = valid ? __ldg(p.fcode8 + q) : kCode8Interior;
+        has_bnd |= code[j] != kCode8Interior;
+    }
+    double src[BG], dtk[BG], cwk[BG];
+#pragma unroll
+    for (int k = 0; k < BG; ++k) {  // dt/tau I0_b(T_c); the cell's rates with the rate law
+        const int64_t row = (int64_t)(p.band0 + lg0 + k) * nc + c;
+        dtk[k] = (p.rate_cur && valid) ? p.dt * __ldg(p.rate_cur + row) : p.dtit[lg0 + k];
+        cwk[k] = (p.rate_cur && p.rate_r2 && valid) ? __ldg(p.rate_next + row) * p.inv_v[lg0 + k] : p.cw[lg0 + k];
+        src[k] = valid ? dtk[k] * __ldg(p.i0 + row) : 0.0;
+    }
+
+    double e = 0.0;
+    for (int i = 0; i < nit; ++i) {
+        const int d = d0 + i;
+        const double4 sd = load_dir(p.dirs, d);
+        double a[MF];
+        int idx[MF];
+        bool glob[MF], iso[MF];
+        double out = 0.0;
+#pragma unroll
+        for (int j = 0; j < MF; ++j) {
+            a[j] = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
+            out += fmax(a[j], 0.0);  // outflow faces carry the cell's own value
+            idx[j] = nbr[j];
+            iso[j] = false;
+            if (has_bnd) {
+                iso[j] = code[j] == kCode8Iso;
+                if (code[j] < kCode8Iso) idx[j] = (__ldg(p.refl + code[j] * p.nd + d) - d) * ps + c;
+            }
+            glob[j] = iso[j] || (unsigned)(idx[j] - tile0) >= (unsigned)kTile;
+        }
+        // halo / boundary values of the inflow faces: global loads first (overlap the stage wait)
+        const int64_t po = (int64_t)d * ps;
+        double nv[BG][MF];
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            const double *pl = p.in_ptr[lg0 + k] + po;
+            const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
+#pragma unroll
+            for (int j = 0; j < MF; ++j)
+                nv[k][j] = (valid && glob[j] && a[j] < 0.0) ? __ldg((iso[j] ? isot : pl) + idx[j]) : 0.0;
+        }
+        const int st = i % kStagesG;
+        while (!mbar_try_wait(&full[st], (i / kStagesG) & 1)) {
+        }
+        const double *stage = ring + st * BG * kTile;
+        double inew[BG];
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            const double *sk = stage + k * kTile;
+            const double ic = sk[tid];
+            double infl = 0.0;
+#pragma unroll
+            for (int j = 0; j < MF; ++j)
+                infl = fma(fmin(a[j], 0.0), glob[j] ? nv[k][j] : sk[idx[j] - tile0], infl);
+            const double kv = p.kv[lg0 + k];
+            inew[k] = fma(ic, (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done with the stage
+#pragma unroll
+        for (int k = 0; k < BG; ++k) {
+            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew[k]);
+            e = fma(cwk[k] * sd.w, inew[k], e);
+        }
+    }
+    if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
+}
+
+// ---------------------------------------------------------------------------
 // Stencil-staged kernel for structured meshes (uniform geometry, constant
 // neighbour offsets so[q] in the stored cell order: +-1, +-nx, +-nx*ny).  For
 // every (band-row, direction) plane one elected thread bulk-copies (TMA) a

@@ -499,9 +499,11 @@ def make_config(name, variant="scaled"):
         dirs = gen_dirs_product(4, 20)
         bcs = gen_bcs_fig1(mesh, radius=4e-6)
         nsteps, eps = 500, 0.10
-    elif name == "C3":
+    elif name in ("C3", "C3t"):
+        # C3t: the same domain as an unstructured triangle mesh
+        # (every quad split on a seeded diagonal: 28,800 cells) for the generic-face path
         h = 525e-6 / 120
-        mesh = gen_mesh((120, 120), (h, h))
+        mesh = gen_mesh((120, 120), (h, h)) if name == "C3" else gen_mesh_tri((120, 120), (h, h))
         bands = gen_bands_si(40)
         dirs = gen_dirs_product(20, 20)
         bcs = gen_bcs_fig1(mesh, radius=10e-6)

@@ -46,7 +46,8 @@ def _check(oracle_mod, cfg, variant, steps=None, **kw):
 
 @pytest.mark.parametrize("rule", [0, 1])
 def test_law_2d_generic_kernel(bte_lib, oracle_mod, rule):
-    _check(oracle_mod, _law_cfg((19, 13), rule=rule, steps=25), variant=0)
+    _check(oracle_mod, _law_cfg((19, 13), rule=rule, steps=25), variant=7)  # TMA-staged generic faces
+    _check(oracle_mod, _law_cfg((19, 13), rule=rule, steps=25), variant=0, tma=False)
 
 
 @pytest.mark.parametrize("rule", [0, 1])
@@ -62,7 +63,8 @@ def test_law_box_rotation_and_work_split(bte_lib, oracle_mod, spare, nbb, dc):
 
 def test_law_3d_non_box_mesh_uses_generic(bte_lib, oracle_mod):
     """Odd extents: not a box grid for the tensor copies -> generic-face kernel."""
-    _check(oracle_mod, _law_cfg((7, 5, 3)), variant=0)
+    _check(oracle_mod, _law_cfg((7, 5, 3)), variant=7)
+    _check(oracle_mod, _law_cfg((7, 5, 3)), variant=0, tma=False)
 
 
 def test_law_dt_bound_uses_hottest_wall(bte_lib):

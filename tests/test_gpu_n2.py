@@ -24,7 +24,7 @@ def bte_lib():
     return mod
 
 
-@pytest.mark.parametrize("name,variant", [("C6", 6), ("C6t", 0)])
+@pytest.mark.parametrize("name,variant", [("C6", 6), ("C6t", 7)])
 def test_fig10_workload(bte_lib, oracle_mod, name, variant):
     cfg = gen.make_config(name)
     Io, To = oracle_run(oracle_mod, cfg, 100)
@@ -49,7 +49,7 @@ def test_triangles_with_rate_law(bte_lib, oracle_mod):
     cfg = dataclasses.replace(cfg, bands=bands, dt=0.5 * gen.general_dt_bound(cfg.mesh, bands, cfg.dirs, t_max=150.0))
     Io, To = oracle_run(oracle_mod, cfg, 40)
     Ig, Tg, st = gpu_run(cfg, 40)
-    assert st["flux_variant"] == 0
+    assert st["flux_variant"] == 7
     assert_parity(Ig, Tg, Io, To)
 
 
@@ -59,3 +59,25 @@ def test_triangles_band_groups(bte_lib, oracle_mod, bg):
     Io, To = oracle_run(oracle_mod, cfg, 20)
     Ig, Tg, _ = gpu_run(cfg, 20, band_group=bg)
     assert_parity(Ig, Tg, Io, To)
+
+
+@pytest.mark.parametrize("bg", [1, 2, 4])
+@pytest.mark.parametrize("tma", [True, False])
+def test_triangles_kernels_and_groups(bte_lib, oracle_mod, bg, tma):
+    """Both generic-face kernels (TMA-staged 7, register 0) in every band group."""
+    cfg = gen.make_config("C6t")
+    Io, To = oracle_run(oracle_mod, cfg, 20)
+    Ig, Tg, st = gpu_run(cfg, 20, band_group=bg, tma=tma)
+    assert st["flux_variant"] == (7 if tma else 0)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_split_faces_3d_generic(bte_lib, oracle_mod):
+    """A 3-D mesh with split (hanging) faces: more than 6 faces per cell (MF 8)."""
+    cfg = gen.small_3d_config((7, 6, 5), n_spectral=3)
+    cfg = dataclasses.replace(cfg, mesh=gen.split_faces(cfg.mesh))
+    Io, To = oracle_run(oracle_mod, cfg, 10)
+    for tma, v in ((True, 7), (False, 0)):
+        Ig, Tg, st = gpu_run(cfg, 10, tma=tma)
+        assert st["flux_variant"] == v
+        assert_parity(Ig, Tg, Io, To)
