@@ -87,7 +87,11 @@ struct bte_ctx {
     double *gx = nullptr, *gy = nullptr, *gz = nullptr;
     bool paired = false;     // every cell's faces are exact opposite pairs
     bool uniform_g = false;  // ... and every cell has the same g per pair
-    bool tma = false;        // paired + 256-thread blocks: the TMA-staged kernel
+    bool tma = false;        // 256-thread blocks: the TMA-staged kernel (paired or generic faces)
+    int32_t *hl_off = nullptr, *hl_cell = nullptr;  // generic TMA kernel: per-tile halo lists,
+    int32_t *bl_off = nullptr, *bl_col = nullptr, *bl_cls = nullptr;  // ... boundary-face ghost lists
+    uint16_t *sidx = nullptr;                        // ... per face slot: shared-memory index of the upwind value
+    int32_t hstride = 0;
     bool stencil = false;    // ... + constant neighbour offsets: the stencil-staged kernel
     int32_t so[3] = {0, 0, 0}, halo = 0, wmain = 0, nfar = 0, farq[3] = {0, 0, 0};
     double gu[3][3] = {};
@@ -207,7 +211,7 @@ void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p)
 // TMA-staged generic-face kernel (general meshes): kStages x BG x 2 KB ring.
 template <int DIM, int MF, int BG>
 void flux_tma_generic_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    const size_t smem = (size_t)bte::kStagesG * BG * bte::kTile * sizeof(double);
+    const size_t smem = (size_t)bte::kStagesG * BG * p.hstride * sizeof(double) + (size_t)p.dchunk * sizeof(double4);
     static size_t attr = 0;
     if (attr < smem) {
         cudaFuncSetAttribute(bte::flux_tma_generic_kernel<DIM, MF, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -900,6 +904,13 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.refl = ctx->refl;
     p.dirs = ctx->dirs;
     p.dt = dt;
+    p.hl_off = ctx->hl_off;
+    p.hl_cell = ctx->hl_cell;
+    p.bl_off = ctx->bl_off;
+    p.bl_col = ctx->bl_col;
+    p.bl_cls = ctx->bl_cls;
+    p.sidx = ctx->sidx;
+    p.hstride = ctx->hstride;
     if (ctx->td) {
         p.rate_cur = rate_half(ctx, ctx->rsel);
         p.rate_next = rate_half(ctx, 1 - ctx->rsel);
@@ -1387,7 +1398,7 @@ void bte_destroy(bte_ctx *ctx) {
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
-                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg};
+                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -1860,6 +1871,63 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
     ctx->staging_elems = std::min<int64_t>((int64_t)nd * nc, std::max<int64_t>(nc, (int64_t)8 << 20));
     CREATE_TRY(dalloc(ctx, &ctx->staging, (size_t)ctx->staging_elems));
+    if (ctx->tma && !paired) {  // generic TMA kernel: per-tile staging lists and shared-memory indices
+        // per tile: own cells [0, 256), halo cells (interior faces pointing out of the
+        // tile) [256, 256 + nh), boundary-face ghosts [256 + nh, 256 + nh + ng)
+        const int32_t ntiles = (nc + bte::kTile - 1) / bte::kTile;
+        std::vector<int32_t> hoff(ntiles + 1, 0), hcell, goff(ntiles + 1, 0), gcol, gcls;
+        std::vector<uint16_t> sidx_h(ell, 0);
+        int32_t smax = 0;
+        std::map<int32_t, int32_t> slot_of;
+        std::vector<size_t> bq;
+        for (int32_t t = 0; t < ntiles; ++t) {
+            const int32_t t0 = t * bte::kTile, t1 = std::min(nc, t0 + bte::kTile);
+            slot_of.clear();
+            bq.clear();
+            for (int j = 0; j < mf_t; ++j)
+                for (int32_t i = t0; i < t1; ++i) {
+                    const size_t q = (size_t)j * nc + i;
+                    if (fcode8_h[q] != bte::kCode8Interior) {
+                        bq.push_back(q);
+                        continue;
+                    }
+                    const int32_t v = nbr_h[q];
+                    if (v >= t0 && v < t0 + bte::kTile) {
+                        sidx_h[q] = (uint16_t)(v - t0);
+                    } else {
+                        auto it = slot_of.find(v);
+                        if (it == slot_of.end()) it = slot_of.emplace(v, (int32_t)slot_of.size()).first;
+                        sidx_h[q] = (uint16_t)(bte::kTile + it->second);
+                    }
+                }
+            const int32_t nh = (int32_t)slot_of.size();
+            std::vector<int32_t> cells(nh);
+            for (const auto &kv : slot_of) cells[kv.second] = kv.first;
+            hcell.insert(hcell.end(), cells.begin(), cells.end());
+            hoff[t + 1] = (int32_t)hcell.size();
+            for (size_t g = 0; g < bq.size(); ++g) {  // Eq. 6 ghosts: isothermal table column / reflected plane
+                const size_t q = bq[g];
+                const int32_t i = (int32_t)(q % (size_t)nc);
+                const bool iso = fcode8_h[q] == bte::kCode8Iso;
+                gcol.push_back(iso ? nbr_h[q] : i);
+                gcls.push_back(iso ? -1 : (int32_t)fcode8_h[q]);
+                sidx_h[q] = (uint16_t)(bte::kTile + nh + (int32_t)g);
+            }
+            goff[t + 1] = (int32_t)gcol.size();
+            smax = std::max<int32_t>(smax, nh + (int32_t)bq.size());
+        }
+        if (smax <= bte::kMaxTileStaged) {
+            ctx->hstride = bte::kTile + (smax + 31) / 32 * 32;
+            CREATE_TRY(upload(ctx, &ctx->hl_off, hoff));
+            CREATE_TRY(upload(ctx, &ctx->hl_cell, hcell));
+            CREATE_TRY(upload(ctx, &ctx->bl_off, goff));
+            CREATE_TRY(upload(ctx, &ctx->bl_col, gcol));
+            CREATE_TRY(upload(ctx, &ctx->bl_cls, gcls));
+            CREATE_TRY(upload(ctx, &ctx->sidx, sidx_h));
+        } else {
+            ctx->tma = false;  // too much to stage per tile: the register kernel
+        }
+    }
     CREATE_TRY(upload(ctx, &ctx->d_cur_slot, ctx->cur_slot));
     CREATE_TRY(upload(ctx, &ctx->nbr, nbr_h));
     CREATE_TRY(upload(ctx, &ctx->nbm, nbm_h));

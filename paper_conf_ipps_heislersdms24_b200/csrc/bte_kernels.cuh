@@ -78,6 +78,17 @@ struct FluxParams {
     double dtit[kMaxBandsPerLaunch];           // dt / tau_b
     double kv[kMaxBandsPerLaunch];             // dt v_b
     double cw[kMaxBandsPerLaunch];             // temperature weight c_b
+    // TMA-staged generic-face kernel: per tile (256 cells) the out-of-tile
+    // upwind cells its interior faces read, then its boundary faces' ghosts,
+    // gathered into the stage behind the tile's own values; per face slot the
+    // shared-memory index of its upwind value
+    const int32_t *hl_off;   // [n_tiles + 1] halo cells of tile t: [hl_off[t], hl_off[t+1])
+    const int32_t *hl_cell;  // plane columns of the halo cells
+    const int32_t *bl_off;   // [n_tiles + 1] boundary-face ghosts of tile t
+    const int32_t *bl_col;   // specular: the cell's column; isothermal: the I0w table column
+    const int32_t *bl_cls;   // specular class (reflected direction refl[cls][d]); -1: isothermal
+    const uint16_t *sidx;    // [MF][nc] staged index: own tile < kTile <= halo < kTile + nh <= ghosts
+    int32_t hstride;         // doubles per staged band-row: kTile + halo + ghost capacity
 };
 
 // L2 eviction-priority policies (createpolicy) for the streamed intensity planes.
@@ -538,23 +549,37 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
 
 // ---------------------------------------------------------------------------
 // TMA-staged kernel for general meshes (unstructured: triangles, split faces,
-// any face-based mesh).  The staging of flux_tma_kernel (one
-// 256-cell tile per block in the locality order, every (band-row, direction)
-// plane segment streamed into a kStages ring by cp.async.bulk, in-tile upwind
-// values from shared memory, halo / boundary values as global loads issued
-// before the stage wait) with the arithmetic of flux_kernel: up to MF faces per
-// cell, outflow sum_j max(alpha_j, 0), inflow sum_j min(alpha_j, 0) I_up
-// (Eq. 3/5 with the Eq. 6 ghosts), and with the rate law the cell's own rates.
+// any face-based mesh).  One 256-cell tile of the locality
+// order per block.  For every (band-row, direction) plane the producer warp
+// stages, kStagesG iterations ahead, everything the tile's faces read: the
+// tile's own 2 KB segment (lane 0, cp.async.bulk), its halo -- the out-of-tile
+// cells its interior faces point to -- and the Eq. 6 ghosts of its boundary
+// faces (isothermal: I0_b(T_wall) from the table; specular: the same cell's
+// value in the reflected direction's plane), both gathered by the 32 lanes with
+// 8-byte cp.async whose completion the same mbarrier tracks
+// (cp.async.mbarrier.arrive.noinc).  The lists are built on the host.  The
+// compute warps then read every upwind value from shared memory at a
+// host-computed index: no global loads and no boundary branch in the update.
+// Arithmetic of flux_kernel: up to MF faces per cell, outflow
+// sum_j max(alpha_j, 0), inflow sum_j min(alpha_j, 0) I_up (Eq. 3/5), with the
+// rate law the cell's own rates.
 #ifndef BTE_TMA_GENERIC_STAGES
-#define BTE_TMA_GENERIC_STAGES 8
+#define BTE_TMA_GENERIC_STAGES 3  // measured on B200 (C3t): 3 > 6 > 12 stages
 #endif
-// Ring depth of the generic-face kernel: its per-thread state (faces x band
-// rows) keeps BG small, so the producer runs further ahead instead.
 constexpr int kStagesG = BTE_TMA_GENERIC_STAGES;
+constexpr int kMaxTileStaged = 768;  // halo + ghost values per tile (else the register kernel)
+
+__device__ __forceinline__ void cp_async_8(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
 template <int DIM, int MF, int BG>
 __global__ void __launch_bounds__(kTmaThreads, BTE_MIN_BLOCKS)
 flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
-    extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][kTile]
+    extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][hstride], then double4 dirs[dchunk]
     __shared__ __align__(8) uint64_t full[kStagesG];
     __shared__ __align__(8) uint64_t empty[kStagesG];
     const int tid = threadIdx.x;
@@ -566,31 +591,56 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     const int nit = min(p.nd, d0 + p.dchunk) - d0;
     const int nc = p.nc;
     const int ps = p.ps;
+    const int hs = p.hstride;
     constexpr uint32_t kBytes = BG * kTile * sizeof(double);
+    double4 *sdir = reinterpret_cast<double4 *>(ring + kStagesG * BG * hs);  // this chunk's {s, w}
 
     if (tid == 0) {
 #pragma unroll
         for (int s = 0; s < kStagesG; ++s) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], 1 + 32);  // lane 0's expect-tx arrive + one async arrive per producer lane
             mbar_init(&empty[s], kComputeWarps);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    for (int i = tid; i < nit; i += kTmaThreads) sdir[i] = load_dir(p.dirs, d0 + i);
     __syncthreads();
 
     if (tid >= kTile) {  // ------------------------------------------ producer warp
-        if (tid == kTile) {
-            for (int i = 0; i < nit; ++i) {
-                const int st = i % kStagesG;
-                if (i >= kStagesG)
-                    while (!mbar_try_wait(&empty[st], ((i / kStagesG) - 1) & 1)) {
-                    }
+        const int lane = tid - kTile;
+        const int h0 = __ldg(p.hl_off + blockIdx.x), nh = __ldg(p.hl_off + blockIdx.x + 1) - h0;
+        const int g0 = __ldg(p.bl_off + blockIdx.x), ng = __ldg(p.bl_off + blockIdx.x + 1) - g0;
+        int st = 0;
+        uint32_t ph = 0;
+        for (int i = 0; i < nit; ++i) {
+            const int d = d0 + i;
+            if (i >= kStagesG)
+                while (!mbar_try_wait(&empty[st], ph ^ 1u)) {
+                }
+            const int64_t po = (int64_t)d * ps;
+            double *sbase = ring + st * BG * hs;
+            if (lane == 0) {
                 mbar_arrive_expect_tx(&full[st], kBytes);
-                const int64_t off = (int64_t)(d0 + i) * ps + tile0;
 #pragma unroll
                 for (int k = 0; k < BG; ++k)
-                    bulk_g2s(ring + (st * BG + k) * kTile, p.in_ptr[lg0 + k] + off, kTile * sizeof(double), &full[st]);
+                    bulk_g2s(sbase + k * hs, p.in_ptr[lg0 + k] + po + tile0, kTile * sizeof(double), &full[st]);
             }
+            for (int h = lane; h < nh; h += 32) {  // halo: neighbour cells outside the tile
+                const int col = __ldg(p.hl_cell + h0 + h);
+#pragma unroll
+                for (int k = 0; k < BG; ++k) cp_async_8(sbase + k * hs + kTile + h, p.in_ptr[lg0 + k] + po + col);
+            }
+            for (int g = lane; g < ng; g += 32) {  // boundary-face ghosts (Eq. 6, old level)
+                const int col = __ldg(p.bl_col + g0 + g), cls = __ldg(p.bl_cls + g0 + g);
+                const int64_t off = cls < 0 ? (int64_t)col
+                                            : (int64_t)__ldg(p.refl + cls * p.nd + d) * ps + col;
+#pragma unroll
+                for (int k = 0; k < BG; ++k)
+                    cp_async_8(sbase + k * hs + kTile + nh + g,
+                               (cls < 0 ? p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso : p.in_ptr[lg0 + k]) + off);
+            }
+            cp_async_mbar_arrive(&full[st]);
+            if (++st == kStagesG) st = 0, ph ^= 1u;
         }
         return;
     }
@@ -599,19 +649,15 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     const int c = tile0 + tid;
     const bool valid = c < nc;
     const int lane = tid & 31;
-    int nbr[MF];
-    uint32_t code[MF];
+    int sx[MF];  // staged index of each face's upwind value
     double gx[MF], gy[MF], gz[MF];
-    bool has_bnd = false;
 #pragma unroll
     for (int j = 0; j < MF; ++j) {
         const int q = j * nc + c;
-        nbr[j] = valid ? __ldg(p.nbr + q) : c;
+        sx[j] = valid ? (int)__ldg(p.sidx + q) : tid;
         gx[j] = valid ? __ldg(p.gx + q) : 0.0;
         gy[j] = valid ? __ldg(p.gy + q) : 0.0;
         gz[j] = (DIM == 3 && valid) ? __ldg(p.gz + q) : 0.0;
-        code[j] = valid ? __ldg(p.fcode8 + q) : kCode8Interior;
-        has_bnd |= code[j] != kCode8Interior;
     }
     double src[BG], dtk[BG], cwk[BG];
 #pragma unroll
@@ -623,57 +669,37 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     }
 
     double e = 0.0;
+    int st = 0;
+    uint32_t ph = 0;
     for (int i = 0; i < nit; ++i) {
-        const int d = d0 + i;
-        const double4 sd = load_dir(p.dirs, d);
-        double a[MF];
-        int idx[MF];
-        bool glob[MF], iso[MF];
+        const double4 sd = sdir[i];
+        double am[MF];  // min(alpha_j, 0): the inflow weights
         double out = 0.0;
 #pragma unroll
         for (int j = 0; j < MF; ++j) {
-            a[j] = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
-            out += fmax(a[j], 0.0);  // outflow faces carry the cell's own value
-            idx[j] = nbr[j];
-            iso[j] = false;
-            if (has_bnd) {
-                iso[j] = code[j] == kCode8Iso;
-                if (code[j] < kCode8Iso) idx[j] = (__ldg(p.refl + code[j] * p.nd + d) - d) * ps + c;
-            }
-            glob[j] = iso[j] || (unsigned)(idx[j] - tile0) >= (unsigned)kTile;
+            const double a = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
+            out += fmax(a, 0.0);  // outflow faces carry the cell's own value
+            am[j] = fmin(a, 0.0);
         }
-        // halo / boundary values of the inflow faces: global loads first (overlap the stage wait)
-        const int64_t po = (int64_t)d * ps;
-        double nv[BG][MF];
-#pragma unroll
-        for (int k = 0; k < BG; ++k) {
-            const double *pl = p.in_ptr[lg0 + k] + po;
-            const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
-#pragma unroll
-            for (int j = 0; j < MF; ++j)
-                nv[k][j] = (valid && glob[j] && a[j] < 0.0) ? __ldg((iso[j] ? isot : pl) + idx[j]) : 0.0;
+        while (!mbar_try_wait(&full[st], ph)) {
         }
-        const int st = i % kStagesG;
-        while (!mbar_try_wait(&full[st], (i / kStagesG) & 1)) {
-        }
-        const double *stage = ring + st * BG * kTile;
+        const double *stage = ring + st * BG * hs;
         double inew[BG];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
-            const double *sk = stage + k * kTile;
-            const double ic = sk[tid];
+            const double *sk = stage + k * hs;
             double infl = 0.0;
 #pragma unroll
-            for (int j = 0; j < MF; ++j)
-                infl = fma(fmin(a[j], 0.0), glob[j] ? nv[k][j] : sk[idx[j] - tile0], infl);
+            for (int j = 0; j < MF; ++j) infl = fma(am[j], sk[sx[j]], infl);
             const double kv = p.kv[lg0 + k];
-            inew[k] = fma(ic, (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
+            inew[k] = fma(sk[tid], (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done with the stage
+        if (++st == kStagesG) st = 0, ph ^= 1u;
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
-            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew[k]);
+            if (valid) __stcs(p.out_ptr[lg0 + k] + (int64_t)(d0 + i) * ps + c, inew[k]);
             e = fma(cwk[k] * sd.w, inew[k], e);
         }
     }
