@@ -209,16 +209,22 @@ void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p)
 }
 
 // TMA-staged generic-face kernel (general meshes): kStages x BG x 2 KB ring.
-template <int DIM, int MF, int BG>
-void flux_tma_generic_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+template <int DIM, int MF, int BG, bool TD>
+void flux_tma_generic_launch_td(dim3 g, const bte::FluxParams &p, cudaStream_t s) {
     const size_t smem = (size_t)bte::kStagesG * BG * p.hstride * sizeof(double) + (size_t)p.dchunk * sizeof(double4);
     static size_t attr = 0;
     if (attr < smem) {
-        cudaFuncSetAttribute(bte::flux_tma_generic_kernel<DIM, MF, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem);
+        cudaFuncSetAttribute(bte::flux_tma_generic_kernel<DIM, MF, BG, TD>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
-    bte::flux_tma_generic_kernel<DIM, MF, BG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+    bte::flux_tma_generic_kernel<DIM, MF, BG, TD><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+}
+
+template <int DIM, int MF, int BG>
+void flux_tma_generic_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    if (p.rate_cur) flux_tma_generic_launch_td<DIM, MF, BG, true>(g, p, s);
+    else flux_tma_generic_launch_td<DIM, MF, BG, false>(g, p, s);
 }
 
 template <int DIM, int MF>

@@ -576,8 +576,11 @@ __device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
     asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <int DIM, int MF, int BG>
-__global__ void __launch_bounds__(kTmaThreads, BTE_MIN_BLOCKS)
+#ifndef BTE_TMA_GENERIC_MIN_BLOCKS
+#define BTE_TMA_GENERIC_MIN_BLOCKS 3
+#endif
+template <int DIM, int MF, int BG, bool TD>
+__global__ void __launch_bounds__(kTmaThreads, BTE_TMA_GENERIC_MIN_BLOCKS)
 flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][hstride], then double4 dirs[dchunk]
     __shared__ __align__(8) uint64_t full[kStagesG];
@@ -659,13 +662,16 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
         gy[j] = valid ? __ldg(p.gy + q) : 0.0;
         gz[j] = (DIM == 3 && valid) ? __ldg(p.gz + q) : 0.0;
     }
-    double src[BG], dtk[BG], cwk[BG];
+    // dt/tau I0_b(T_c); TD (rate law): the cell's own rates, else the band's constants
+    double src[BG], dtk[TD ? BG : 1], cwk[TD ? BG : 1];
 #pragma unroll
-    for (int k = 0; k < BG; ++k) {  // dt/tau I0_b(T_c); the cell's rates with the rate law
+    for (int k = 0; k < BG; ++k) {
         const int64_t row = (int64_t)(p.band0 + lg0 + k) * nc + c;
-        dtk[k] = (p.rate_cur && valid) ? p.dt * __ldg(p.rate_cur + row) : p.dtit[lg0 + k];
-        cwk[k] = (p.rate_cur && p.rate_r2 && valid) ? __ldg(p.rate_next + row) * p.inv_v[lg0 + k] : p.cw[lg0 + k];
-        src[k] = valid ? dtk[k] * __ldg(p.i0 + row) : 0.0;
+        if (TD) {
+            dtk[k] = valid ? p.dt * __ldg(p.rate_cur + row) : 0.0;
+            cwk[k] = (p.rate_r2 && valid) ? __ldg(p.rate_next + row) * p.inv_v[lg0 + k] : p.cw[lg0 + k];
+        }
+        src[k] = valid ? (TD ? dtk[k] : p.dtit[lg0 + k]) * __ldg(p.i0 + row) : 0.0;
     }
 
     double e = 0.0;
@@ -692,7 +698,8 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
             for (int j = 0; j < MF; ++j) infl = fma(am[j], sk[sx[j]], infl);
             const double kv = p.kv[lg0 + k];
-            inew[k] = fma(sk[tid], (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
+            const double dt_tau = TD ? dtk[k] : p.dtit[lg0 + k];
+            inew[k] = fma(sk[tid], (1.0 - dt_tau) - kv * out, fma(-kv, infl, src[k]));
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done with the stage
@@ -700,7 +707,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
             if (valid) __stcs(p.out_ptr[lg0 + k] + (int64_t)(d0 + i) * ps + c, inew[k]);
-            e = fma(cwk[k] * sd.w, inew[k], e);
+            e = fma((TD ? cwk[k] : p.cw[lg0 + k]) * sd.w, inew[k], e);
         }
     }
     if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
