@@ -266,9 +266,7 @@ def run_ours(args):
     # cell), from the library's CUDA events on the launching stream over the
     # timed region.  A step launches it once per band-group segment; achieved =
     # algorithmic bytes of all flux launches of a step / their summed time.
-    flux_launches_per_step = max(1, (st["kernel_launches"] // args.steps) - 1 - (1 if world > 1 else 0))
-    if args.cell_parts > 1:
-        flux_launches_per_step = None  # (halo pack / unpack launches too)
+    flux_launches_per_step = st["flux_launches"] / args.steps
     t_flux = st["ms_flux_interior"] / args.steps / 1e3
     alg_bytes = BYTES_PER_UPDATE * nc_loc * nd * nb_loc  # per step, this rank
     peak, peak_src = _peaks()

@@ -1426,6 +1426,132 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     }
 }
 
+// ---------------------------------------------------------------------------
+// The same per-cell temperature solve with one WARP per cell (the step's
+// solve; newton_kernel serves the re-solves): lane l evaluates band-rows
+// l, l + 32, ... and butterfly shuffles give every lane the same sums, so the
+// Newton iterates (and the bisection safeguard) are warp-uniform.  A cell's
+// 55 rows x ~4 iterations of expm1 are spread over 32 lanes, so small meshes
+// (C3: 14,400 cells) fill the GPU instead of a few warps per SM.  Output like
+// newton_kernel's chunk solve: T_out[c] = T^{n+1} (or -T^n on failure), the
+// epilogue (T, Tr, I0, rates) is newton_finish_kernel's.
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    return v;
+}
+
+constexpr int kNewtonRowsPerLane = kMaxBandsPerLaunch / 32;  // nb <= 128
+
+__device__ __forceinline__ Gsum g_eval_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
+                                            double E, double T, int lane) {
+    double g = 0.0, gp = 0.0;
+    const double it = 1.0 / T;
+#pragma unroll
+    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+        const int b = lane + 32 * r;
+        if (b < nb) {
+            const double x = sTh[b] * it;
+            const double em1 = expm1(x);
+            const double i0 = sC[b] / em1;
+            g = fma(wl[r], i0, g);
+            gp = fma(wl[r], i0 * (x * it) * (1.0 + 1.0 / em1), gp);
+        }
+    }
+    return {W * warp_sum(g) - E, W * warp_sum(gp)};
+}
+
+__device__ __forceinline__ double g_only_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
+                                              double E, double T, int lane) {
+    double g = 0.0;
+#pragma unroll
+    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+        const int b = lane + 32 * r;
+        if (b < nb) g = fma(wl[r], sC[b] / expm1(sTh[b] / T), g);
+    }
+    return W * warp_sum(g) - E;
+}
+
+__global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
+    extern __shared__ double sm[];
+    double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
+    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
+    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
+        sC[b] = p.Cb[b];
+        sTh[b] = p.theta[b];
+        sW[b] = p.cw[b];
+        if (p.td) {
+            sA[b] = p.ra[b];
+            sB[b] = p.rb[b];
+            sR[b] = p.rth[b];
+            sV[b] = p.inv_v[b];
+        }
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int cl = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);  // chunk-local cell
+    if (cl >= p.nc) return;
+    const int c = p.c_lo + cl;
+    double E;
+    if (p.E) {
+        E = p.E[cl];
+    } else {
+        E = 0.0;
+        for (int s = lane; s < p.n_slots; s += 32) E += p.part[(size_t)s * p.nc + c];
+        E = warp_sum(E);
+    }
+    const double T0 = p.T[c];
+    const bool law = p.td && p.r2;
+    const double Tw = p.td ? (p.tr_step ? T0 : p.Tr[c]) : 0.0;  // a step: weights at T^n
+    double wl[kNewtonRowsPerLane];
+#pragma unroll
+    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+        const int b = lane + 32 * r;
+        wl[r] = b >= p.nb ? 0.0 : law ? tau_rate(sA[b], sB[b], sR[b], Tw) * sV[b] : sW[b];
+    }
+    double T = T0;
+    bool ok = false;
+    int it = 0;
+    if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
+        const Gsum gs = g_eval_warp(sC, sTh, wl, p.nb, p.W, E, T, lane);
+        const double Tn = T - gs.g / gs.gp;
+        it = 1;
+        if (Tn > 0.0 && isfinite(Tn)) {
+            T = Tn;
+            ok = true;
+        }
+    } else if (E > 0.0 && isfinite(E)) {
+        for (it = 1; it <= p.maxit; ++it) {
+            const Gsum gs = g_eval_warp(sC, sTh, wl, p.nb, p.W, E, T, lane);
+            const double delta = gs.g / gs.gp;
+            const double Tn = T - delta;
+            if (!(Tn > 0.0) || !isfinite(Tn)) break;
+            T = Tn;
+            if (fabs(delta) <= p.rtol * T) { ok = true; break; }
+        }
+        if (!ok) {  // bisection safeguard on a bracket grown from T0
+            double lo = T0, hi = T0;
+            for (int k = 0; k < 2000 && g_only_warp(sC, sTh, wl, p.nb, p.W, E, lo, lane) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only_warp(sC, sTh, wl, p.nb, p.W, E, hi, lane) < 0.0; ++k) hi *= 2.0;
+            if (g_only_warp(sC, sTh, wl, p.nb, p.W, E, lo, lane) <= 0.0 &&
+                g_only_warp(sC, sTh, wl, p.nb, p.W, E, hi, lane) >= 0.0) {
+                for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
+                    const double mid = 0.5 * (lo + hi);
+                    if (g_only_warp(sC, sTh, wl, p.nb, p.W, E, mid, lane) < 0.0) lo = mid; else hi = mid;
+                }
+                T = 0.5 * (lo + hi);
+                ok = true;
+            }
+            it = p.maxit + 1;
+        }
+    }
+    if (lane == 0) {
+        if (!ok) atomicExch(p.fail, 1);
+        atomicMax(p.iter_max, it);
+        p.T_out[c] = ok ? T : (p.neg_fail ? -T0 : T0);
+    }
+}
+
 // Band-sharded step, after the all-gather of the chunk solves:
 // T^{n+1} for every cell (a negative value marks a failed cell of some rank:
 // flag it on every rank and keep T^n), the rate temperature Tr <- T^n, and the
