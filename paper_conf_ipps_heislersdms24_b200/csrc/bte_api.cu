@@ -147,6 +147,13 @@ struct bte_ctx {
     bte::nccl::Comm bcomm{};
     bool have_bcomm = false, own_bcomm = false;
     bool begun = false;  // split step in flight
+    // CUDA graph of two steps (double-buffered single-GPU runs: after two steps the
+    // slab pointers and rate halves are back where they were, so it replays)
+    cudaGraphExec_t gexec = nullptr;
+    double g_dt = 0.0;
+    int g_key = -1;
+    int64_t g_launches = 0, g_flux = 0;
+    bool graphs_ok = true;
     // stats
     bte_stats st{};
     std::vector<PhaseEvent> ev_live, ev_pool;
@@ -1433,6 +1440,7 @@ void bte_destroy(bte_ctx *ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
     if (ctx->own_bcomm) bte::nccl::destroy(ctx->bcomm);
     if (ctx->have_comm) bte::nccl::destroy(ctx->comm);
     for (HaloSeg &h : ctx->hsegs) {
@@ -2131,6 +2139,65 @@ static bte_status check_dt(bte_ctx *ctx, double dt) {
     return BTE_OK;
 }
 
+// One explicit step (Eq. 2-3): halo exchange (cell partitioning), flux +
+// relaxation + energy partials, the energy exchange and the temperature solve.
+static bte_status one_step(bte_ctx *ctx, double dt) {
+    STATUS_TRY(halo_exchange(ctx));
+    STATUS_TRY(run_flux(ctx, dt));
+    if (ctx->have_bcomm && ctx->shard_newton) {
+        STATUS_TRY(shard_newton_step(ctx));
+    } else if (ctx->have_bcomm) {
+        ev_mark(ctx, kPhAllreduce, true);
+        STATUS_TRY(reduce_slots(ctx));
+        STATUS_TRY(allreduce_E(ctx));
+        ev_mark(ctx, kPhAllreduce, false);
+        STATUS_TRY(run_newton(ctx, ctx->E));
+    } else {
+        STATUS_TRY(run_newton(ctx, nullptr));
+    }
+    return BTE_OK;
+}
+
+// State key of the double-buffered pointers: which slab holds row 0 and which
+// rate half is current (both flip every step).
+static int graph_key(const bte_ctx *ctx) { return ctx->cur_slot[0] * 2 + ctx->rsel; }
+
+// Capture two steps into a CUDA graph on the library stream (launch-bound
+// small problems: one replay instead of ~8 launches).  The host-side pointer
+// rotation of the two captured steps cancels out; their launch counters are
+// moved to the per-replay count.  Any failure disables graphs for the context.
+static void capture_two_steps(bte_ctx *ctx, double dt) {
+    if (ctx->gexec) {
+        cudaGraphExecDestroy(ctx->gexec);
+        ctx->gexec = nullptr;
+    }
+    const int64_t l0 = ctx->st.kernel_launches, f0 = ctx->st.flux_launches;
+    const int key = graph_key(ctx);
+    cudaGraph_t g = nullptr;
+    bool ok = cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+    bte_status s1 = BTE_OK, s2 = BTE_OK;
+    if (ok) {
+        s1 = one_step(ctx, dt);
+        if (s1 == BTE_OK) s2 = one_step(ctx, dt);
+        ok = cudaStreamEndCapture(ctx->stream, &g) == cudaSuccess && s1 == BTE_OK && s2 == BTE_OK && g;
+    }
+    if (ok) ok = cudaGraphInstantiate(&ctx->gexec, g, 0) == cudaSuccess;
+    if (g) cudaGraphDestroy(g);
+    ctx->g_launches = ctx->st.kernel_launches - l0;
+    ctx->g_flux = ctx->st.flux_launches - f0;
+    ctx->st.kernel_launches = l0;
+    ctx->st.flux_launches = f0;
+    if (!ok || graph_key(ctx) != key) {  // (the rotation did not close: never replay)
+        if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
+        ctx->gexec = nullptr;
+        ctx->graphs_ok = false;
+        cudaGetLastError();
+        return;
+    }
+    ctx->g_key = key;
+    ctx->g_dt = dt;
+}
+
 bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
     if (!ctx) return BTE_EINVAL;
     if (ctx->begun) return set_err(&ctx->err, "split step in flight"), BTE_ESTATE;
@@ -2142,23 +2209,34 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
                                   "bte_step_begin / bte_get_energy / bte_set_energy / bte_step_finish "
                                   "(bte_halo_export / bte_halo_import)"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
-    for (int64_t s = 0; s < n; ++s) {
-        STATUS_TRY(halo_exchange(ctx));
-        STATUS_TRY(run_flux(ctx, dt));
-        if (ctx->have_bcomm && ctx->shard_newton) {
-            STATUS_TRY(shard_newton_step(ctx));
-        } else if (ctx->have_bcomm) {
-            ev_mark(ctx, kPhAllreduce, true);
-            STATUS_TRY(reduce_slots(ctx));
-            STATUS_TRY(allreduce_E(ctx));
-            ev_mark(ctx, kPhAllreduce, false);
-            STATUS_TRY(run_newton(ctx, ctx->E));
-        } else {
-            STATUS_TRY(run_newton(ctx, nullptr));
-        }
+    const int64_t upd = (int64_t)ctx->nc * ctx->nd * ctx->nb_loc;
+    int64_t s = 0;
+    auto step1 = [&]() -> bte_status {
+        STATUS_TRY(one_step(ctx, dt));
         ctx->st.steps++;
-        ctx->st.updates += (int64_t)ctx->nc * ctx->nd * ctx->nb_loc;
+        ctx->st.updates += upd;
+        ++s;
+        return BTE_OK;
+    };
+    // CUDA graphs: single GPU, double buffering, no per-phase events (BTE_NO_GRAPH=1 disables)
+    const bool no_graph_env = std::getenv("BTE_NO_GRAPH") != nullptr;
+    const bool graphs = ctx->graphs_ok && !no_graph_env && n >= 4 && !(ctx->opt.flags & BTE_FLAG_PROFILE) &&
+                        !ctx->have_comm && ctx->hsegs.empty() && ctx->n_spare == ctx->nb_loc;
+    if (graphs) {
+        if (!ctx->gexec || ctx->g_dt != dt) {
+            STATUS_TRY(step1());  // (first launches set the kernels' shared-memory attributes)
+            capture_two_steps(ctx, dt);
+        }
+        if (ctx->gexec && graph_key(ctx) != ctx->g_key) STATUS_TRY(step1());
+        for (; ctx->gexec && s + 2 <= n; s += 2) {
+            CUDA_TRY(ctx, cudaGraphLaunch(ctx->gexec, ctx->stream));
+            ctx->st.steps += 2;
+            ctx->st.updates += 2 * upd;
+            ctx->st.kernel_launches += ctx->g_launches;
+            ctx->st.flux_launches += ctx->g_flux;
+        }
     }
+    while (s < n) STATUS_TRY(step1());
     STATUS_TRY(upload_cur_slots(ctx));
     return check_newton(ctx);
 }

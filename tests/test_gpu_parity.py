@@ -434,3 +434,36 @@ def test_c3_full_size_elementwise(bte, oracle_mod):
     Ig, Tg, st = gpu_run(cfg, 3)
     assert st["flux_variant"] == 6
     assert_parity(Ig, Tg, Io, To)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "box3d", "law2d"])
+def test_cuda_graph_replay_is_bitwise_equal(bte, oracle_mod, name):
+    """bte_step(n >= 4) on one GPU replays a captured 2-step CUDA graph; the
+    per-phase profiling mode launches every kernel instead.  Same bits, for odd
+    n, a dt change (re-capture) and the rate law (rate halves flip per step)."""
+    if name == "box3d":
+        cfg = gen.small_3d_config((34, 9, 5), n_spectral=3)
+    elif name == "law2d":
+        c0 = _cfg("C2")
+        law = gen.with_rate_law(c0.bands)
+        cfg = dataclasses.replace(c0, bands=law, dt=0.5 * gen.cartesian_dt_bound(c0.mesh, law, c0.dirs, t_max=350.0))
+    else:
+        cfg = _cfg(name)
+    out = []
+    for profile in (False, True):
+        with bte.solver_from_config(cfg, profile=profile) as s:
+            bte.apply_ic(s, cfg)
+            s.step(cfg.dt, 7)
+            s.step(0.5 * cfg.dt, 6)
+            s.step(cfg.dt, 5)
+            st = s.stats()
+            out.append((s.intensity(), s.temperature(), st["steps"], st["updates"]))
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+    assert out[0][2:] == out[1][2:] == (18, 18 * cfg.n_updates_per_step)
+    if name == "C1":  # and the graph path against the oracle
+        p = oracle_mod.problem_from_config(cfg)
+        I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps, with_tr=True)
+        I, T, Tr = p.run(I, T, cfg.dt, 7, Tr=Tr)
+        I, T, Tr = p.run(I, T, 0.5 * cfg.dt, 6, Tr=Tr)
+        I, T, Tr = p.run(I, T, cfg.dt, 5, Tr=Tr)
+        assert_parity(out[0][0], out[0][1], I, T)
