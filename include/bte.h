@@ -201,6 +201,8 @@ typedef struct {
     double ms_halo;            /* cell partitioning: halo pack + exchange + unpack */
     int64_t halo_bytes;        /* halo bytes this rank sends per step (all segments) */
     int64_t flux_launches;     /* flux-kernel launches (a1-a3), part of kernel_launches */
+    int64_t graph_replays;     /* 2-step CUDA-graph replays inside bte_step (their kernels are
+                                  counted in kernel_launches) */
 } bte_stats;
 
 /* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,

@@ -72,7 +72,8 @@ class Stats(C.Structure):
                 ("newton_iter_max", C.c_int32), ("spare_slabs", C.c_int32),
                 ("n_interior_cells", C.c_int32), ("band_group", C.c_int32),
                 ("block_threads", C.c_int32), ("dir_chunks", C.c_int32), ("flux_variant", C.c_int32),
-                ("ms_halo", C.c_double), ("halo_bytes", C.c_int64), ("flux_launches", C.c_int64)]
+                ("ms_halo", C.c_double), ("halo_bytes", C.c_int64), ("flux_launches", C.c_int64),
+                ("graph_replays", C.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

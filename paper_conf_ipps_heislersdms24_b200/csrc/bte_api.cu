@@ -2218,10 +2218,12 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
         ++s;
         return BTE_OK;
     };
-    // CUDA graphs: single GPU, double buffering, no per-phase events (BTE_NO_GRAPH=1 disables)
+    // CUDA graphs: double buffering, no per-phase events (BTE_NO_GRAPH=1 disables).  The
+    // NCCL exchanges of band sharding / cell partitioning are captured too (NCCL supports
+    // stream capture); every rank replays the same sequence of collectives.
     const bool no_graph_env = std::getenv("BTE_NO_GRAPH") != nullptr;
     const bool graphs = ctx->graphs_ok && !no_graph_env && n >= 4 && !(ctx->opt.flags & BTE_FLAG_PROFILE) &&
-                        !ctx->have_comm && ctx->hsegs.empty() && ctx->n_spare == ctx->nb_loc;
+                        ctx->n_spare == ctx->nb_loc;
     if (graphs) {
         if (!ctx->gexec || ctx->g_dt != dt) {
             STATUS_TRY(step1());  // (first launches set the kernels' shared-memory attributes)
@@ -2234,6 +2236,7 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
             ctx->st.updates += 2 * upd;
             ctx->st.kernel_launches += ctx->g_launches;
             ctx->st.flux_launches += ctx->g_flux;
+            ctx->st.graph_replays++;
         }
     }
     while (s < n) STATUS_TRY(step1());

@@ -457,9 +457,10 @@ def test_cuda_graph_replay_is_bitwise_equal(bte, oracle_mod, name):
             s.step(0.5 * cfg.dt, 6)
             s.step(cfg.dt, 5)
             st = s.stats()
-            out.append((s.intensity(), s.temperature(), st["steps"], st["updates"]))
+            out.append((s.intensity(), s.temperature(), st["steps"], st["updates"], st["graph_replays"]))
     assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
-    assert out[0][2:] == out[1][2:] == (18, 18 * cfg.n_updates_per_step)
+    assert out[0][2:4] == out[1][2:4] == (18, 18 * cfg.n_updates_per_step)
+    assert out[0][4] >= 6 and out[1][4] == 0  # graph replays (7 + 6 + 5 steps) / none when profiling
     if name == "C1":  # and the graph path against the oracle
         p = oracle_mod.problem_from_config(cfg)
         I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps, with_tr=True)
@@ -467,3 +468,15 @@ def test_cuda_graph_replay_is_bitwise_equal(bte, oracle_mod, name):
         I, T, Tr = p.run(I, T, 0.5 * cfg.dt, 6, Tr=Tr)
         I, T, Tr = p.run(I, T, cfg.dt, 5, Tr=Tr)
         assert_parity(out[0][0], out[0][1], I, T)
+
+
+def test_cuda_graph_with_nccl_one_rank(bte, monkeypatch):
+    """The graph path with the NCCL exchange captured (one-rank communicator,
+    both exchange modes): bitwise equal to launching every kernel."""
+    cfg = _cfg("C2")
+    ref = gpu_run(cfg, 9, profile=True)  # no graph, no communicator
+    for mode in ("shard", "replicated"):
+        monkeypatch.setenv("BTE_SHARD_NEWTON", mode)
+        g = gpu_run(cfg, 9, nccl_id=bte.nccl_unique_id())
+        assert np.array_equal(ref[0], g[0]) and np.array_equal(ref[1], g[1]), mode
+        assert g[2]["graph_replays"] >= 3 and ref[2]["graph_replays"] == 0, mode
