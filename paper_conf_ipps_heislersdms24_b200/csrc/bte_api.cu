@@ -720,12 +720,26 @@ BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
     if (ctx->opt.dir_chunk > 0) {
         b.oc = std::max(1, std::min({ctx->n_orb, kBoxMaxOrbChunk, (int)ctx->opt.dir_chunk / 4}));
     } else {
-        b.oc = 1;
-        for (int c = std::min({ctx->n_orb, kBoxMaxOrbChunk, ctx->box_oc}); c >= 1; --c)
-            if (ctx->n_orb % c == 0) {
-                b.oc = c;
-                break;
+        b.oc = oc_pre;
+        // small launches (few band-rows: band sharding over many GPUs) that give fewer
+        // than 8 waves even at one row per item: smaller orbit chunks, and then the most
+        // work per item (rows x orbits) that still gives 8 waves (measured on B200: C4
+        // 7 rows 0.994 -> 0.958 ms with 5 rows x 5 orbits instead of 1 x 20)
+        const int64_t ctas1 = (int64_t)tiles * nbl * ((ctx->n_orb + oc_pre - 1) / oc_pre);
+        if (tiles <= slots && ctas1 < 8 * slots && ctx->opt.band_group <= 0) {
+            int best_w = 0;
+            for (int c = oc_pre; c >= 1; --c) {
+                if (ctx->n_orb % c) continue;
+                for (int n = std::min(nbl, ctx->box_nbb); n >= 1; --n) {
+                    const int64_t ctas = (int64_t)tiles * ((nbl + n - 1) / n) * (ctx->n_orb / c);
+                    if (ctas >= 8 * slots && n * c > best_w) {
+                        best_w = n * c;
+                        b.oc = c;
+                        b.nbb = n;
+                    }
+                }
             }
+        }
     }
     b.n_batches = (nbl + b.nbb - 1) / b.nbb;
     b.n_chunks = (ctx->n_orb + b.oc - 1) / b.oc;
