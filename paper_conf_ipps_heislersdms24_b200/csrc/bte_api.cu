@@ -721,24 +721,22 @@ BoxPlan plan_box(const bte_ctx *ctx, int nbl) {
         b.oc = std::max(1, std::min({ctx->n_orb, kBoxMaxOrbChunk, (int)ctx->opt.dir_chunk / 4}));
     } else {
         b.oc = oc_pre;
-        // small launches (few band-rows: band sharding over many GPUs) that give fewer
-        // than 8 waves even at one row per item: smaller orbit chunks, and then the most
-        // work per item (rows x orbits) that still gives 8 waves (measured on B200: C4
-        // 7 rows 0.994 -> 0.958 ms with 5 rows x 5 orbits instead of 1 x 20)
-        const int64_t ctas1 = (int64_t)tiles * nbl * ((ctx->n_orb + oc_pre - 1) / oc_pre);
-        if (tiles <= slots && ctas1 < 8 * slots && ctx->opt.band_group <= 0) {
-            int best_w = 0;
-            for (int c = oc_pre; c >= 1; --c) {
-                if (ctx->n_orb % c) continue;
-                for (int n = std::min(nbl, ctx->box_nbb); n >= 1; --n) {
-                    const int64_t ctas = (int64_t)tiles * ((nbl + n - 1) / n) * (ctx->n_orb / c);
-                    if (ctas >= 8 * slots && n * c > best_w) {
-                        best_w = n * c;
+        // 3-D launches whose items got one row each (few band-rows per launch: band
+        // sharding over 4-8 GPUs): the most rows per item, then the largest orbit
+        // chunk, that still give 8 waves (measured on B200, C4 emulated ranks: 7 rows
+        // 0.994 -> 0.958 ms with 5 rows x 5 orbits instead of 1 x 20; 14 rows 1.942 ->
+        // 1.879 ms)
+        if (!ctx->bflat && tiles <= slots && auto_nbb == 1 && ctx->opt.band_group <= 0) {
+            bool done = false;
+            for (int n = std::min(nbl, ctx->box_nbb); n >= 1 && !done; --n)
+                for (int c = oc_pre; c >= 1 && !done; --c) {
+                    if (ctx->n_orb % c) continue;
+                    if ((int64_t)tiles * ((nbl + n - 1) / n) * (ctx->n_orb / c) >= 8 * slots) {
                         b.oc = c;
                         b.nbb = n;
+                        done = true;
                     }
                 }
-            }
         }
     }
     b.n_batches = (nbl + b.nbb - 1) / b.nbb;
