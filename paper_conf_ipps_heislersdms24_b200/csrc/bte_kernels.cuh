@@ -91,18 +91,6 @@ struct FluxParams {
     int32_t hstride;         // doubles per staged band-row: kTile + halo + ghost capacity
 };
 
-// L2 eviction-priority policies (createpolicy) for the streamed intensity planes.
-__device__ __forceinline__ uint64_t l2_policy_evict_last() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-    return pol;
-}
-__device__ __forceinline__ double ldg_hint(const double *ptr, uint64_t pol) {
-    double v;
-    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(ptr), "l"(pol));
-    return v;
-}
-
 __device__ __forceinline__ double4 load_dir(const double4 *dirs, int d) {
     const double2 a = __ldg(reinterpret_cast<const double2 *>(dirs + d));
     const double2 b = __ldg(reinterpret_cast<const double2 *>(dirs + d) + 1);
@@ -250,9 +238,6 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
         }
     }
     const uint32_t codes = __ldg(p.fcode + c);
-#ifdef BTE_EXP_KEEP
-    const uint64_t pol = l2_policy_evict_last();
-#endif
     constexpr uint32_t kAllInterior = (1u << (10 * NP)) - 1u;
     const bool has_bnd = codes != kAllInterior;
     double src[BG];  // dt/tau I0_b(T_c) per band-row of the group
@@ -285,18 +270,10 @@ flux_paired_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
         for (int k = 0; k < BG; ++k) {  // every load of the iteration first
             const double *pl = p.in_ptr[lg0 + k] + po;  // slab bases come from the constant bank
-#ifdef BTE_EXP_KEEP
-            ic[k] = ldg_hint(pl + c, pol);
-#else
             ic[k] = __ldg(pl + c);
-#endif
             if (!has_bnd) {
 #pragma unroll
-#ifdef BTE_EXP_NO_NBR
-                for (int q = 0; q < NP; ++q) nv[k][q] = ic[k];
-#else
                 for (int q = 0; q < NP; ++q) nv[k][q] = __ldg(pl + idx[q]);
-#endif
             } else {
                 const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
 #pragma unroll
