@@ -218,10 +218,11 @@ def run_ours(args):
     stream = torch.cuda.current_stream()
     part_kw = {}
     if args.cell_parts > 1:  # cell partitioning, x band groups = world / cell_parts
-        from paper_conf_ipps_heislersdms24_b200.dist import partition_cells
+        from paper_conf_ipps_heislersdms24_b200.dist import partition_cells, slab_partition
         assert world % args.cell_parts == 0, "--cell-parts must divide the number of GPUs"
-        part_kw = dict(cell_part=partition_cells(cfg.mesh["cell_centre"], args.cell_parts),
-                       n_cell_parts=args.cell_parts)
+        cen = cfg.mesh["cell_centre"]  # 3-D grids: z slabs (the box kernel keeps running); else bisection
+        parts = slab_partition(cen, args.cell_parts) if cfg.mesh["dim"] == 3 else partition_cells(cen, args.cell_parts)
+        part_kw = dict(cell_part=parts, n_cell_parts=args.cell_parts)
     s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream, **part_kw,
                                profile=True, band_group=args.band_group, block_threads=args.block_threads,
                                max_spare_slabs=args.max_spare, dir_chunk=args.dir_chunk,

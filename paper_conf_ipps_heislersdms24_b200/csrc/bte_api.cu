@@ -55,6 +55,7 @@ struct HaloSeg {
     int part = 0;
     int32_t n_send_cells = 0, n_send_dirs = 0, n_recv_cells = 0, n_recv_dirs = 0, col0 = 0;
     int32_t *send_cells = nullptr, *send_dirs = nullptr, *recv_dirs = nullptr;  // device
+    int32_t *recv_cols = nullptr;  // device: halo column of each received cell (relative to pool_cells)
     double *sbuf = nullptr, *rbuf = nullptr;                                      // device
     int64_t n_send() const { return (int64_t)n_send_cells * n_send_dirs; }  // per band-row
     int64_t n_recv() const { return (int64_t)n_recv_cells * n_recv_dirs; }
@@ -72,6 +73,8 @@ struct bte_ctx {
     double W = 0.0, s_max = 0.0, dt_bound = 0.0;
     // slab pool: nb_loc current slabs + n_spare workspace slabs of nd x ps doubles
     double *pool = nullptr;
+    double *pool_cells = nullptr;  // pool + the column of the first owned cell (cell index 0); halo
+                                   // layers of a z-slab cell partition sit before / after the owned cells
     int64_t slab_elems = 0;
     int n_spare = 0;
     std::vector<int32_t> cur_slot, spare_slot;
@@ -99,6 +102,7 @@ struct bte_ctx {
     bool box = false;
     int32_t bn[3] = {0, 0, 0}, bzside[2] = {0, 0};
     bool bflat = false;  // 2-D box grid (no axis-2 faces; isothermal walls on grid axis 1)
+    int32_t bz_t = 0, bz_lo = 0;  // z-slab partition: tensor layers (owned + halo), first owned layer
     double bgeo[3] = {0, 0, 0};
     int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
     bool td = false;  // temperature-dependent relaxation times (rate tables)
@@ -767,7 +771,14 @@ BoxKernel box_kernel(const bte_ctx *ctx) {
 
 bte_status box_setup_kernel(bte_ctx *ctx) {
     const size_t smem = box_smem(ctx);
-    CUDA_TRY(ctx, cudaFuncSetAttribute(box_kernel(ctx), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    // the attribute is per function, shared by every context of the process: only ever raise it
+    // (contexts with different layer ranges need different amounts)
+    static std::map<const void *, size_t> granted;
+    size_t &g = granted[(const void *)box_kernel(ctx)];
+    if (smem > g) {
+        CUDA_TRY(ctx, cudaFuncSetAttribute(box_kernel(ctx), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        g = smem;
+    }
     int occ = 0;
     CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, box_kernel(ctx), bte::kBoxThreads, smem));
     ctx->box_ctas_per_sm = std::max(1, occ);
@@ -846,7 +857,9 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     bte::BoxParams p{};
     p.n0 = ctx->bn[0];
     p.n1 = ctx->bn[1];
-    p.n2 = ctx->bn[2];
+    p.n2 = ctx->bz_t;  // tensor layers (z-slab partition: + halo layers)
+    p.zlo = ctx->bz_lo;
+    p.nown = ctx->bn[2];
     p.L = ctx->box_L;
     p.n_orb = ctx->n_orb;
     p.nc = ctx->nc;
@@ -957,8 +970,8 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
             p.slot0 = slot;
             for (int k = 0; k < sg.nbl; ++k) {
                 const int b = l0 + sg.off + k;  // rank-local band-row
-                p.in_ptr[k] = ctx->pool + (int64_t)ctx->cur_slot[b] * ctx->slab_elems;
-                p.out_ptr[k] = ctx->pool + (int64_t)ctx->spare_slot[sg.off + k] * ctx->slab_elems;
+                p.in_ptr[k] = ctx->pool_cells + (int64_t)ctx->cur_slot[b] * ctx->slab_elems;
+                p.out_ptr[k] = ctx->pool_cells + (int64_t)ctx->spare_slot[sg.off + k] * ctx->slab_elems;
                 p.dtit[k] = dt * ctx->h_inv_tau[b];
                 p.kv[k] = dt * ctx->h_vg[b];
                 p.cw[k] = ctx->h_cw[b];
@@ -1117,7 +1130,7 @@ bte_status shard_newton_step(bte_ctx *ctx) {
 // Pack / unpack one segment for every local band-row (current slabs).
 bte::HaloParams halo_params(const bte_ctx *ctx) {
     bte::HaloParams hp{};
-    for (int k = 0; k < ctx->nb_loc; ++k) hp.row[k] = ctx->pool + (int64_t)ctx->cur_slot[k] * ctx->slab_elems;
+    for (int k = 0; k < ctx->nb_loc; ++k) hp.row[k] = ctx->pool_cells + (int64_t)ctx->cur_slot[k] * ctx->slab_elems;
     hp.nb_loc = ctx->nb_loc;
     hp.ps = ctx->ps;
     return hp;
@@ -1146,7 +1159,7 @@ bte_status halo_unpack(bte_ctx *ctx, const HaloSeg &h) {
     hp.dirs = h.recv_dirs;
     hp.n = h.n_recv_cells;
     hp.n_dirs = h.n_recv_dirs;
-    hp.col0 = h.col0;
+    hp.cells = h.recv_cols;
     bte::halo_unpack_kernel<<<halo_grid(ctx, h.n_recv()), 256, 0, ctx->stream>>>(hp, h.rbuf);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
@@ -1305,6 +1318,57 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
     return BTE_OK;
 }
 
+// ------------------------------------------------------------- z-slab partitions of box grids
+// A cell partition of a structured 3-D box grid into slabs of whole grid
+// axis-2 layers (each part a contiguous layer range) keeps the box kernel: the
+// rank's slab tensor holds its owned layers plus the neighbour parts' adjacent
+// layer (halo) below / above, the kernel updates the owned layers only and
+// takes the upwind layer of a range from the halo layer exactly as from a
+// neighbouring range (Eq. 3); the global walls stay wall ghosts (Eq. 6).
+struct ZSlab {
+    bool on = false;
+    int32_t za = 0, zb = 0, h_lo = 0, h_hi = 0;
+    int64_t off = 0;                // columns before the first owned cell (the lower halo layer)
+    BoxDetect gbx;                  // the global box
+    std::vector<bte::BoxOrbit> orbs;
+    std::vector<int64_t> grid_of;   // global cell -> grid lexicographic position
+};
+
+ZSlab detect_zslab(const bte_mesh *m, const bte_dirs *dr, const bte_bcs *bc, const bte_options *o, int me) {
+    ZSlab z;
+    if (m->dim != 3 || (o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA | BTE_FLAG_GENERIC_FACES)))
+        return z;
+    z.gbx = detect_box(m, bc);
+    const BoxDetect &g = z.gbx;
+    if (!g.ok || !box_orbits(dr, g.ax, g.zside[0] == 1 || g.zside[1] == 1, &z.orbs)) return z;
+    const int64_t plane = (int64_t)g.n[0] * g.n[1];
+    std::vector<int32_t> layer_part(g.n[2], -1);
+    for (int32_t l = 0; l < g.n[2]; ++l)
+        for (int64_t i = 0; i < plane; ++i) {
+            const int32_t pp = o->cell_part[g.cell_at[l * plane + i]];
+            if (pp < 0 || pp >= o->n_cell_parts) return z;
+            if (layer_part[l] < 0) layer_part[l] = pp;
+            else if (layer_part[l] != pp) return z;  // a layer split between parts
+        }
+    int32_t za = -1, zb = -1;
+    for (int32_t l = 0; l < g.n[2]; ++l)
+        if (layer_part[l] == me) {
+            if (za < 0) za = l;
+            else if (zb != l) return z;  // not contiguous
+            zb = l + 1;
+        }
+    if (za < 0) return z;
+    z.za = za;
+    z.zb = zb;
+    z.h_lo = za > 0;
+    z.h_hi = zb < g.n[2];
+    z.off = z.h_lo * plane;
+    z.grid_of.assign(m->n_cells, -1);
+    for (int64_t i = 0; i < (int64_t)g.cell_at.size(); ++i) z.grid_of[g.cell_at[i]] = i;
+    z.on = true;
+    return z;
+}
+
 // ------------------------------------------------------------- cell partition (N3)
 // The owned cells of part `me` as a mesh of their own: owned cells in ascending
 // global id (local ids 0..nc-1), faces copied in stored order; a face whose
@@ -1317,6 +1381,7 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
 struct SegPlan {
     int part = 0;
     std::vector<int32_t> send_local, send_dirs, recv_dirs;
+    std::vector<int64_t> recv_global;  // the halo cells (global ids, ascending)
     int32_t n_recv_cells = 0, col0 = 0;
 };
 struct LocalPlan {
@@ -1377,6 +1442,7 @@ bte_status build_local(const bte_mesh *m, const bte_dirs *dr, const bte_options 
         s.col0 = L->n_halo;
         for (int64_t h : rc[q]) hslot[h] = L->n_halo++;
         s.n_recv_cells = (int32_t)rc[q].size();
+        s.recv_global = rc[q];
         s.recv_dirs = dirs_of(rn[q]);
         for (int64_t h : sc[q]) s.send_local.push_back((int32_t)loc[h]);
         s.send_dirs = dirs_of(sn[q]);
@@ -1456,7 +1522,7 @@ void bte_destroy(bte_ctx *ctx) {
     if (ctx->own_bcomm) bte::nccl::destroy(ctx->bcomm);
     if (ctx->have_comm) bte::nccl::destroy(ctx->comm);
     for (HaloSeg &h : ctx->hsegs) {
-        void *hp[] = {h.send_cells, h.send_dirs, h.recv_dirs, h.sbuf, h.rbuf};
+        void *hp[] = {h.send_cells, h.send_dirs, h.recv_dirs, h.recv_cols, h.sbuf, h.rbuf};
         for (void *q : hp)
             if (q) cudaFree(q);
     }
@@ -1487,7 +1553,9 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         return set_err(nullptr, "world %d is not a multiple of n_cell_parts %d", o->world, n_parts), BTE_EINVAL;
     const int my_part = o->rank % n_parts, G = o->world / n_parts, gband = o->rank / n_parts;
     LocalPlan lplan;
+    ZSlab zs;
     if (cpart) {
+        zs = detect_zslab(m, dr, bc, o, my_part);
         STATUS_TRY(build_local(m, dr, o, my_part, &lplan));
         m = &lplan.mesh;
     }
@@ -1569,7 +1637,21 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     std::vector<bte::BoxOrbit> orbs;
     if (paired_geom && !cpart && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
         bx = m->dim == 3 ? detect_box(m, bc) : detect_box2d(m, bc);
-    const bool use_box = bx.ok && box_orbits(dr, bx.ax, !bx.flat && (bx.zside[0] == 1 || bx.zside[1] == 1), &orbs);
+    if (zs.on) {  // z-slab partition: the owned layers of the global box, in grid order (local ids)
+        const BoxDetect &g = zs.gbx;
+        const int64_t plane = (int64_t)g.n[0] * g.n[1];
+        bx = g;
+        bx.n[2] = zs.zb - zs.za;
+        for (int sd = 0; sd < 2; ++sd)  // a side facing a neighbour part reads its halo layer, never a wall
+            if (sd ? zs.h_hi : zs.h_lo) bx.zside[sd] = 1;
+        bx.cell_at.resize((size_t)plane * bx.n[2]);
+        for (int64_t i = 0; i < (int64_t)bx.cell_at.size(); ++i) {
+            const int64_t gcell = g.cell_at[(int64_t)zs.za * plane + i];
+            bx.cell_at[i] = (int32_t)(std::lower_bound(lplan.gid.begin(), lplan.gid.end(), gcell) - lplan.gid.begin());
+        }
+        orbs = zs.orbs;
+    }
+    const bool use_box = bx.ok && (zs.on || box_orbits(dr, bx.ax, !bx.flat && (bx.zside[0] == 1 || bx.zside[1] == 1), &orbs));
 
     // --- internal cell order from the optional centroids: cells are grouped
     // into bricks of 8 x 8 x 4 (2-D: 16 x 16) typical cell sizes, Morton order
@@ -1852,6 +1934,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->box = true;
         ctx->bg = 1;
         for (int a = 0; a < 3; ++a) ctx->bn[a] = bx.n[a], ctx->bgeo[a] = bx.g[a];
+        ctx->bz_lo = zs.on ? zs.h_lo : 0;
+        ctx->bz_t = bx.n[2] + (zs.on ? zs.h_lo + zs.h_hi : 0);
         ctx->bzside[0] = bx.zside[0];
         ctx->bzside[1] = bx.zside[1];
         ctx->bflat = bx.flat;
@@ -1899,6 +1983,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     for (int k = 0; k < nb_loc; ++k) ctx->cur_slot[k] = k;
     for (int k = 0; k < n_spare; ++k) ctx->spare_slot[k] = nb_loc + k;
     CREATE_TRY(dalloc(ctx, &ctx->pool, (size_t)(nb_loc + n_spare) * ctx->slab_elems));
+    ctx->pool_cells = ctx->pool + zs.off;
 
     const int max_slots = count_slots(ctx);
     CREATE_TRY(dalloc(ctx, &ctx->part, (size_t)max_slots * nc));
@@ -1917,6 +2002,20 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         HaloSeg &h = ctx->hsegs.back();
         h.part = sp.part;
         h.col0 = nc + sp.col0;
+        {  // halo columns relative to pool_cells: after the owned cells, or (z-slab box) the halo layers
+            std::vector<int32_t> rc(sp.n_recv_cells);
+            const int64_t plane = zs.on ? (int64_t)zs.gbx.n[0] * zs.gbx.n[1] : 0;
+            for (int32_t i = 0; i < sp.n_recv_cells; ++i) {
+                if (!zs.on) {
+                    rc[i] = nc + sp.col0 + i;
+                } else {
+                    const int64_t gp = zs.grid_of[sp.recv_global[i]];
+                    const int64_t layer = gp / plane;
+                    rc[i] = (int32_t)((layer - zs.za + zs.h_lo) * plane + gp % plane - zs.off);
+                }
+            }
+            CREATE_TRY(upload(ctx, &h.recv_cols, rc));
+        }
         h.n_send_cells = (int32_t)sp.send_local.size();
         h.n_send_dirs = (int32_t)sp.send_dirs.size();
         h.n_recv_cells = sp.n_recv_cells;
@@ -2032,7 +2131,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         const int gb = (nc + tb - 1) / tb;
         bte::i0_table_kernel<<<gb, tb, 0, ctx->stream>>>(ctx->T, nc, b_lo, nb_loc, ctx->Cb, ctx->theta, ctx->i0);
         bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)nd * nc + tb - 1) / tb), nb_loc), tb, 0,
-                                  ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ps, nd, nc, ctx->i0);
+                                  ctx->stream>>>(ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ps, nd, nc, ctx->i0);
         if (ctx->n_iso > 0)
             bte::i0w_kernel<<<(ctx->n_iso + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->twall, ctx->n_iso, b_lo, nb_loc,
                                                                                ctx->Cb, ctx->theta, ctx->i0w);
@@ -2094,7 +2193,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                                                             nb_loc, ctx->side_tab);
         CREATE_CUDA(cudaGetLastError());
         const uint64_t n0 = bx.n[0], n1 = bx.n[1], n2 = bx.n[2];
-        const uint64_t dpool[5] = {n0, n1, n2, (uint64_t)nd, (uint64_t)(nb_loc + n_spare)};
+        const uint64_t dpool[5] = {n0, n1, (uint64_t)ctx->bz_t, (uint64_t)nd, (uint64_t)(nb_loc + n_spare)};
         const uint64_t spool[4] = {n0 * 8, n0 * n1 * 8, (uint64_t)ps * 8, (uint64_t)ctx->slab_elems * 8};
         const uint32_t bin[5] = {bte::kBoxBX, bte::kBoxBY, 1, 1, 1}, bout[5] = {bte::kBoxTX, bte::kBoxTY, 1, 1, 1};
         const uint64_t di0[4] = {n0, n1, n2, (uint64_t)nb_loc}, si0[3] = {n0 * 8, n0 * n1 * 8, (uint64_t)nc * 8};
@@ -2350,7 +2449,7 @@ bte_status bte_get_intensity(const bte_ctx *ctx, int32_t b_lo, int32_t b_hi, dou
     STATUS_TRY(check_rows(ctx, b_lo, b_hi));
     CUDA_TRY(const_cast<bte_ctx *>(ctx), cudaSetDevice(ctx->device));
     for (int32_t b = b_lo; b < b_hi; ++b) {
-        const double *slab = ctx->pool + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
+        const double *slab = ctx->pool_cells + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
         STATUS_TRY(rows_to_host(ctx, slab, ctx->ps, ctx->nd, I + (int64_t)(b - b_lo) * ctx->nd * ctx->nc));
     }
     return BTE_OK;
@@ -2361,7 +2460,7 @@ bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const dou
     STATUS_TRY(check_rows(ctx, b_lo, b_hi));
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     for (int32_t b = b_lo; b < b_hi; ++b) {
-        double *slab = ctx->pool + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
+        double *slab = ctx->pool_cells + (int64_t)ctx->cur_slot[b - ctx->b_lo] * ctx->slab_elems;
         STATUS_TRY(rows_from_host(ctx, I + (int64_t)(b - b_lo) * ctx->nd * ctx->nc, ctx->ps, ctx->nd, slab));
     }
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
@@ -2378,7 +2477,7 @@ bte_status bte_solve_temperature(bte_ctx *ctx) {
     const int tb = 128;
     const bool law_r2 = ctx->td && ctx->opt.temp_rule == 0;  // weights at the kept rate temperature
     bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
-        ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc,
+        ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc,
         law_r2 ? rate_half(ctx, ctx->rsel) : nullptr, ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E);
     CUDA_TRY(ctx, cudaGetLastError());
     STATUS_TRY(allreduce_E(ctx));
@@ -2422,7 +2521,7 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
     const bool law_r2 = ctx->td && rule == 0;
     const int tb = 128;
     bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
-        ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs,
+        ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs,
         ctx->cw_diag + ctx->b_lo, law_r2 ? rate_half(ctx, ctx->rsel) : nullptr,
         ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E2);
     CUDA_TRY(ctx, cudaGetLastError());
@@ -2473,7 +2572,7 @@ bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T) {
     STATUS_TRY(upload_cur_slots(ctx));
     const int tb = 256;
     bte::equilibrium_kernel<<<dim3(std::min<int64_t>(4096, ((int64_t)ctx->nd * ctx->nc + tb - 1) / tb), ctx->nb_loc),
-                              tb, 0, ctx->stream>>>(ctx->pool, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nd,
+                              tb, 0, ctx->stream>>>(ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nd,
                                                     ctx->nc, ctx->i0);
     CUDA_TRY(ctx, cudaGetLastError());
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));

@@ -916,7 +916,9 @@ struct BoxOrbit {
 };
 
 struct BoxParams {
-    int32_t n0, n1, n2;        // grid extents, axis 0 contiguous
+    int32_t n0, n1, n2;        // grid extents, axis 0 contiguous (n2: layers of the slab tensor)
+    int32_t zlo, nown;         // computed layers [zlo, zlo + nown) of the tensor (a z-slab cell
+                               // partition keeps halo layers around them; else 0, n2)
     int32_t tiles0, tiles1;    // 32-cell tiles along axis 0, 8-cell tiles along axis 1
     int32_t L, zranges;        // layers per work item, ranges along axis 2
     int32_t n_orb, orb_chunk, n_chunks;  // orbits, orbits per item, chunks
@@ -1017,8 +1019,8 @@ __device__ __forceinline__ BoxItem box_item(const BoxParams &p, int item) {
     const int zr = t / p.tiles1;
     w.x0 = t0 * kBoxTX;
     w.y0 = t1 * kBoxTY;
-    w.z0 = zr * p.L;
-    w.Lc = min(p.L, p.n2 - w.z0);
+    w.z0 = p.zlo + zr * p.L;
+    w.Lc = min(p.L, p.zlo + p.nown - w.z0);
     const int chunk = w.slice % p.n_chunks, batch = w.slice / p.n_chunks;
     w.k0 = batch * p.nbb;
     w.k1 = min(p.nbl, w.k0 + p.nbb);
@@ -1125,11 +1127,11 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             for (int q = 0; q < 4; ++q)
                                 tma_load_5d(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
                                             ob.d[q], slab, &full[s]);
-                            tma_load_4d(st + 4 * kBoxPlane, &tm_i0, w.x0, w.y0, z, bl, &full[s]);
+                            tma_load_4d(st + 4 * kBoxPlane, &tm_i0, w.x0, w.y0, z - p.zlo, bl, &full[s]);
                             if (TD) {
-                                tma_load_5d(st + 4 * kBoxPlane + kBoxCells, &tm_rate, w.x0, w.y0, z, bl,
+                                tma_load_5d(st + 4 * kBoxPlane + kBoxCells, &tm_rate, w.x0, w.y0, z - p.zlo, bl,
                                             p.rsel_cur, &full[s]);
-                                tma_load_5d(st + 4 * kBoxPlane + 2 * kBoxCells, &tm_rate, w.x0, w.y0, z, bl,
+                                tma_load_5d(st + 4 * kBoxPlane + 2 * kBoxCells, &tm_rate, w.x0, w.y0, z - p.zlo, bl,
                                             p.rsel_next, &full[s]);
                             }
                         }
@@ -1242,7 +1244,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     if (valid) {
         double *part = p.part + (int64_t)(p.slot0 + w.slice) * p.nc;
         for (int l = 0; l < w.Lc; ++l)
-            part[((int64_t)(w.z0 + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
+            part[((int64_t)(w.z0 - p.zlo + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
     if (tid == 0) bulk_wait_all();
 }
@@ -1697,16 +1699,16 @@ __global__ void scatter_rows_kernel(const double *__restrict__ src, const int32_
 // across a cut face are the neighbour part's I^n at the old level, exactly as
 // for an interior face (Eq. 3): they live in extra columns
 // [nc, nc + n_halo) of every slab, which the flux kernels read like any other
-// neighbour column and never write.  One segment per neighbour part, layout
+// neighbour column and never write (z-slab partitions of box grids: whole
+// halo layers before / after the owned ones).  One segment per neighbour part, layout
 // buf[k][j][i] over the local band-rows k, the segment's direction list j and
 // its cell list i (only directions that flow across the cut, s_d . n < 0 at
 // the reading cell's face).
 struct HaloParams {
     double *row[kMaxBandsPerLaunch];  // current slab of local band-row k
-    const int32_t *cells;             // pack: internal column of send cell i
+    const int32_t *cells;             // column of send cell i (pack) / of halo cell i (unpack)
     const int32_t *dirs;              // direction list of the segment
     int32_t n, n_dirs, nb_loc, ps;
-    int32_t col0;                     // unpack: first halo column of the segment
 };
 
 __global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf) {
@@ -1729,7 +1731,7 @@ __global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const d
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
         const int j = (int)(e / p.n);
         const int i = (int)(e - (int64_t)j * p.n);
-        s[(int64_t)__ldg(p.dirs + j) * p.ps + p.col0 + i] = in[e];
+        s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)] = in[e];
     }
 }
 

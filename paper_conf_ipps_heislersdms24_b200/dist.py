@@ -50,6 +50,20 @@ def partition_cells(centres, n_parts: int):
     return out
 
 
+def slab_partition(centres, n_parts: int, axis: int = 2):
+    """Slabs of whole cell layers along one axis (equal cell counts up to a
+    layer): on the paper's structured 3-D grids, z slabs keep the box kernel
+    (bte_options.cell_part, DESIGN.md 9 N3).  Returns part[n_cells] (int32)."""
+    import numpy as np
+    x = np.asarray(centres, dtype=np.float64)[:, axis]
+    levels = np.unique(x)
+    layer = np.searchsorted(levels, x)
+    counts = np.bincount(layer, minlength=levels.size)
+    cum = np.cumsum(counts) - counts  # cells before each layer
+    part_of_layer = np.minimum(n_parts - 1, (cum * n_parts) // x.size).astype(np.int32)
+    return part_of_layer[layer]
+
+
 def env_rank_world():
     return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
             int(os.environ.get("LOCAL_RANK", "0")))

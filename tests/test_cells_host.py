@@ -42,6 +42,18 @@ def test_partition_cells_bisects_longest_axis():
     assert x[parts == 0].max() < x[parts == 1].min()
 
 
+@pytest.mark.parametrize("n_parts", [1, 2, 3, 5, 8])
+def test_slab_partition_whole_layers(n_parts):
+    cfg = gen.small_3d_config((6, 5, 8))
+    parts = bdist.slab_partition(cfg.mesh["cell_centre"], n_parts)
+    z = cfg.mesh["cell_centre"][:, 2]
+    for p in range(n_parts):  # every part a contiguous range of whole z layers
+        zs = np.unique(z[parts == p])
+        assert zs.size >= 1
+        assert not np.isin(zs, z[parts != p]).any()
+    assert np.all(np.diff([z[parts == p].min() for p in range(n_parts)]) > 0)
+
+
 @pytest.mark.parametrize("world,P", [(8, 8), (8, 4), (8, 2), (6, 3), (4, 1)])
 def test_rank_grid(world, P):
     seen = {bdist.rank_grid(r, world, P) for r in range(world)}

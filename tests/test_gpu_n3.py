@@ -190,3 +190,47 @@ def test_partition_errors(bte):
     with bte.solver_from_config(cfg, cell_part=one, n_cell_parts=1) as s:
         assert s.n_cells == nc and s.stats()["halo_bytes"] == 0
         assert np.array_equal(s.local_cells(), np.arange(nc))
+
+
+def _zslab_parts(cfg, bounds):
+    """Part id per cell from the z layer: part k owns layers [bounds[k], bounds[k+1])."""
+    nx, ny, nz = cfg.mesh["shape"]
+    z = np.arange(cfg.mesh["n_cells"]) // (nx * ny)
+    return (np.searchsorted(np.asarray(bounds[1:-1]), z, side="right")).astype(np.int32)
+
+
+@pytest.mark.parametrize("shape,bounds", [((34, 9, 8), (0, 4, 8)), ((34, 9, 8), (0, 2, 5, 8)),
+                                          ((16, 9, 6), (0, 1, 2, 4, 6)), ((32, 16, 9), (0, 5, 9))])
+def test_zslab_partition_box_kernel(bte, oracle_mod, shape, bounds):
+    """Cell parts made of whole z layers of a structured 3-D grid keep the box
+    kernel (halo layers around the owned ones; 1-layer parts included)."""
+    cfg = gen.small_3d_config(shape, n_spectral=3)
+    parts = _zslab_parts(cfg, bounds)
+    Io, To = oracle_run(oracle_mod, cfg, 8)
+    Ig, Tg, st = run_partitioned(bte, cfg, len(bounds) - 1, 1, 8, parts=parts)
+    assert all(s["flux_variant"] == 6 for s in st)
+    assert_parity(Ig, Tg, Io, To)
+
+
+def test_zslab_partition_walls_law_hybrid(bte, oracle_mod):
+    """z-slab parts with specular z walls (the z-mirrored ghost at the global
+    walls), the rate law, and a 2 x 2 hybrid with band groups."""
+    cfg = gen.small_3d_config((34, 9, 8), n_spectral=3)
+    bcs = gen.gen_bcs_walls(cfg.mesh, {w: (gen.SYMMETRY, 0) for w in range(6)})
+    law = gen.with_rate_law(cfg.bands)
+    c_spec = dataclasses.replace(cfg, bcs=bcs)
+    c_law = dataclasses.replace(cfg, bands=law,
+                                dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, law, cfg.dirs, t_max=350.0))
+    parts = _zslab_parts(cfg, (0, 3, 8))
+    for c in (c_spec, c_law):
+        Io, To = oracle_run(oracle_mod, c, 6)
+        Ig, Tg, st = run_partitioned(bte, c, 2, 1, 6, parts=parts)
+        assert all(s["flux_variant"] == 6 for s in st)
+        assert_parity(Ig, Tg, Io, To)
+    rng = np.random.default_rng(4)
+    T0 = 300.0 + 20 * rng.random(cfg.mesh["n_cells"])
+    p = oracle_mod.problem_from_config(cfg)
+    Io, To = p.run(p.equilibrium(T0), T0, cfg.dt, 6)
+    Ig, Tg, st = run_partitioned(bte, cfg, 2, 2, 6, parts=parts, T0=T0)
+    assert all(s["flux_variant"] == 6 for s in st)
+    assert_parity(Ig, Tg, Io, To)

@@ -30,9 +30,9 @@ cstlaw = dataclasses.replace(cst, bands=law2, dt=0.5 * gen.cartesian_dt_bound(cs
 c6t = dataclasses.replace(gen.make_config("C6t"), nsteps=2)
 
 
-def run_parts(cfg, n_parts):
-    from paper_conf_ipps_heislersdms24_b200.dist import partition_cells
-    parts = partition_cells(cfg.mesh["cell_centre"], n_parts)
+def run_parts(cfg, n_parts, slabs=False):
+    from paper_conf_ipps_heislersdms24_b200.dist import partition_cells, slab_partition
+    parts = (slab_partition if slabs else partition_cells)(cfg.mesh["cell_centre"], n_parts)
     ss = [bte.solver_from_config(cfg, rank=r, world=n_parts, cell_part=parts, n_cell_parts=n_parts)
           for r in range(n_parts)]
     try:
@@ -51,6 +51,7 @@ def run_parts(cfg, n_parts):
 
 
 print("parts-3d", run_parts(c3d, 3), flush=True)
+print("parts-zslab-box", run_parts(box3, 2, slabs=True), flush=True)
 print("parts-tri", run_parts(c6t, 2), flush=True)
 for name, cfg, kw in [("C1", c1, {}), ("box3d", box3, {}), ("box3d-law", box3law, {}), ("box2d", cst, {}),
                       ("box2d-law", cstlaw, {}), ("box2d-rotation", cst, {"max_spare_slabs": 2}),
