@@ -83,11 +83,14 @@ def share_nccl_id(pg, rank: int, make_id=None) -> bytes:
 
 def make_solver(cfg, pg=None, n_cell_parts=1, **kw):
     """Solver for this rank (world from the process group, if any).
-    n_cell_parts > 1: cell partitioning (N3) by partition_cells of the cell
-    centres, combined with band sharding over world / n_cell_parts groups."""
+    n_cell_parts > 1: cell partitioning (N3) -- z slabs on 3-D meshes (the box
+    kernel keeps running on structured grids), coordinate bisection on 2-D --
+    combined with band sharding over world / n_cell_parts groups."""
     from . import bte
     if n_cell_parts > 1:
-        kw.update(cell_part=partition_cells(cfg.mesh["cell_centre"], n_cell_parts), n_cell_parts=n_cell_parts)
+        cen = cfg.mesh["cell_centre"]
+        parts = slab_partition(cen, n_cell_parts) if cfg.mesh["dim"] == 3 else partition_cells(cen, n_cell_parts)
+        kw.update(cell_part=parts, n_cell_parts=n_cell_parts)
     if pg is None or pg.get_world_size() == 1:
         return bte.solver_from_config(cfg, **kw)
     rank, world = pg.get_rank(), pg.get_world_size()
