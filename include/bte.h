@@ -23,8 +23,10 @@
  * Storage is band-major I[b][d][c] (L777-840: band-parallel loop order) with
  * the cell index fastest.  Band-rows are sharded across ranks (L760-775): rank g
  * of P owns rows [floor(g nb/P), floor((g+1) nb/P)); bands couple only through
- * the per-cell energy, which is summed across ranks with one NCCL all-reduce of
- * n_cells doubles per step.
+ * the per-cell energy, which is summed across ranks once per step (NCCL
+ * reduce-scatter of the n_cells partial energies, each rank solves its chunk of
+ * cells, all-gather of T: the bytes of one all-reduce).  Cells may be
+ * partitioned too (bte_options.cell_part, a halo exchange per step).
  *
  * Conventions for every call:
  *   - All pointers passed IN are borrowed for the duration of the call only and
@@ -130,7 +132,7 @@ typedef struct {
                                      TMA-staged one (testing / comparison) */
 #define BTE_FLAG_STENCIL 8u       /* structured index order: stencil-staged kernel (near/far
                                      TMA windows; L2-bandwidth-heavy, opt-in) */
-#define BTE_FLAG_NO_BOX 16u       /* structured 3-D box grids: do not use the box kernel
+#define BTE_FLAG_NO_BOX 16u       /* structured 2-D / 3-D box grids: do not use the box kernel
                                      (tensor-copy z-marching tiles, the default there) */
 
 typedef struct {
@@ -184,7 +186,7 @@ typedef struct {
     int64_t updates;           /* (cell, dir, band) unknowns advanced on this rank */
     double ms_flux_interior;   /* interior-cell flux + relaxation + energy partial */
     double ms_flux_boundary;   /* boundary-cell kernel */
-    double ms_allreduce;       /* slot reduce + NCCL all-reduce (world > 1) */
+    double ms_allreduce;       /* slot reduce + NCCL energy exchange (world > 1) */
     double ms_newton;          /* temperature solve + I0 refresh */
     double ms_total;           /* first to last event of the profiled steps */
     int32_t newton_iter_max;   /* max Newton iterations of any cell */
