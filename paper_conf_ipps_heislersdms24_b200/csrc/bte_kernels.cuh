@@ -1166,8 +1166,9 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
 
-    int s = 0, sp = 0;
+    int s = 0;
     uint32_t ph = 0, ob = 0;
+    double pv[4] = {0.0, 0.0, 0.0, 0.0};  // the previous layer's own values: this layer's axis-2 upwind values
     for (int k = w.k0; k < w.k1; ++k) {
         const double kv = p.kv[k];
         for (int o = w.o0; o < w.o1; ++o) {
@@ -1182,12 +1183,15 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
-                if (j == 0) {
-                    sp = s;
+                if (j == 0) {  // the range's upwind layer: its values to registers, the stage back at once
+                    const double *cur = ring + s * kStage;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) pv[q] = cur[own[q]];
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&empty[s]);
                 } else {
                     const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
                     const double *cur = ring + s * kStage;
-                    const double *prv = ring + sp * kStage;
                     double dtit, coef, cw;
                     if (TD) {  // 1/tau_b of this cell at the rate temperature; R2 weight at the next one
                         dtit = p.dt * cur[4 * kBoxPlane + kBoxCells + tid];
@@ -1206,7 +1210,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         const double ic = cur[own[q]];
                         double infl = m0 * cur[ux[q]];
                         infl = fma(m1, cur[uy[q]], infl);
-                        if (!flat) infl = fma(m2, prv[own[q]], infl);
+                        if (!flat) infl = fma(m2, pv[q], infl);
+                        pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
                         out[q * kBoxCells + tid] = inew;
                         acc = fma(wq[q], inew, acc);
@@ -1214,15 +1219,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
                     *ea = fma(cw, acc, *ea);
                     __syncwarp();
-                    if (lane == 0) {  // the previous layer's stage is no longer needed
-                        if (flat) {
-                            mbar_arrive(&empty[s]);
-                        } else {
-                            mbar_arrive(&empty[sp]);
-                            if (j == w.Lc) mbar_arrive(&empty[s]);
-                        }
-                    }
-                    sp = s;
+                    if (lane == 0) mbar_arrive(&empty[s]);  // this stage is no longer needed
                     fence_smem_to_async();
                     if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
                     bar_compute();
