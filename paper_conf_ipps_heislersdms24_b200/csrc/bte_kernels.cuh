@@ -1166,7 +1166,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
 
-    int s = 0;
+    int s = 0, sp = 0;
     uint32_t ph = 0, ob = 0;
     double pv[4] = {0.0, 0.0, 0.0, 0.0};  // the previous layer's own values: this layer's axis-2 upwind values
     for (int k = w.k0; k < w.k1; ++k) {
@@ -1183,12 +1183,11 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
-                if (j == 0) {  // the range's upwind layer: its values to registers, the stage back at once
+                if (j == 0) {  // the range's upwind layer: its values to registers
                     const double *cur = ring + s * kStage;
 #pragma unroll
                     for (int q = 0; q < 4; ++q) pv[q] = cur[own[q]];
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&empty[s]);
+                    sp = s;
                 } else {
                     const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
                     const double *cur = ring + s * kStage;
@@ -1219,7 +1218,17 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
                     *ea = fma(cw, acc, *ea);
                     __syncwarp();
-                    if (lane == 0) mbar_arrive(&empty[s]);  // this stage is no longer needed
+                    // release the previous layer's stage now (one layer late: keeps the producer
+                    // from running further ahead, which measured more DRAM re-reads of halo boxes)
+                    if (lane == 0) {
+                        if (flat) {
+                            mbar_arrive(&empty[s]);
+                        } else {
+                            mbar_arrive(&empty[sp]);
+                            if (j == w.Lc) mbar_arrive(&empty[s]);
+                        }
+                    }
+                    sp = s;
                     fence_smem_to_async();
                     if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
                     bar_compute();
