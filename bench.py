@@ -86,7 +86,15 @@ class ClockSampler:
                  "-lms", "100"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
         except Exception:
             self.proc = None
-        time.sleep(0.3)
+        # Wait until the sampler is live (its first row written), so that a
+        # short timed region is still bracketed by samples.
+        t0 = time.time()
+        self.n0 = 0
+        while self.proc is not None and time.time() - t0 < 10.0:
+            self.n0 = len(self._rows())
+            if self.n0:
+                break
+            time.sleep(0.05)
         return self
 
     def __exit__(self, *a):
@@ -97,7 +105,7 @@ class ClockSampler:
             except Exception:
                 self.proc.kill()
 
-    def summary(self):
+    def _rows(self):
         rows = []
         try:
             for line in open(self.path):
@@ -106,6 +114,13 @@ class ClockSampler:
                     rows.append(f)
         except Exception:
             pass
+        return rows
+
+    def summary(self):
+        rows = self._rows()
+        during = rows[self.n0:] if self.proc is not None else []
+        if during:
+            rows = during
         if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
@@ -113,8 +128,11 @@ class ClockSampler:
         loaded = [x for x in sm if x > 0.5 * smax] or sm
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower().startswith("active")})
-        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
-                "samples": len(rows)}
+        out = {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
+               "samples": len(rows)}
+        if not during:
+            out["note"] = "timed region shorter than the sampling interval: samples bracketing it"
+        return out
 
 
 def _dist():
