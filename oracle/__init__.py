@@ -72,6 +72,10 @@ def lib():
         _lib.oracle_equilibrium.restype = None
         _lib.oracle_run.argtypes = [P, dbl, i64, vp, vp, vp]
         _lib.oracle_step_cells_equilibrium.argtypes = [P, vp, vp, vp, i64, dbl, vp, vp]
+        _lib.oracle_energy_subset.argtypes = [P, i64, vp, vp, vp]
+        _lib.oracle_energy_subset.restype = None
+        _lib.oracle_newton_subset.argtypes = [P, i64, vp, vp, vp]
+        _lib.oracle_step_subset.argtypes = [P, vp, i64, vp, vp, vp, vp, i64, vp, dbl, vp, vp]
     return _lib
 
 
@@ -225,6 +229,51 @@ class Problem:
             raise RuntimeError(f"oracle sampled step failed rc={rc}")
         return out, T1
 
+    def run_until_failure(self, I, T, dt, nsteps, Tr=None):
+        """Up to nsteps steps, one at a time; stops after the step whose
+        temperature solve fails (ENOCONV, the state of that step: the failed
+        cells keep their previous T).  Returns (I, T, Tr, steps_taken, rc)."""
+        I = np.array(I, dtype=np.float64, order="C")
+        T = np.array(T, dtype=np.float64, order="C")
+        Tr = None if Tr is None else np.array(np.broadcast_to(np.asarray(Tr, np.float64), (self.nc,)))
+        self._need_tr(Tr)
+        self.reflection_map()
+        rc, k = OK, 0
+        while k < nsteps and rc == OK:
+            rc = lib().oracle_run(self.ref, float(dt), 1, _ptr(I), _ptr(T), _optr(Tr))
+            k += 1
+        return I, T, Tr, k, rc
+
+    # -- subsets of cells (sampled checks of full fields) ------------------------
+    def subset_initial(self, sub, I_sub, T_guess, Tr_sub=None):
+        """T of the subset cells' intensities I_sub[b][d][k] (Newton from T_guess)."""
+        sub = np.ascontiguousarray(sub, np.int64)
+        I_sub = np.ascontiguousarray(I_sub, np.float64)
+        Tr = None if Tr_sub is None else np.ascontiguousarray(np.broadcast_to(np.asarray(Tr_sub, np.float64), sub.shape))
+        E = np.empty(sub.size)
+        lib().oracle_energy_subset(self.ref, int(sub.size), _ptr(I_sub), _optr(Tr), _ptr(E))
+        T = np.array(np.broadcast_to(np.asarray(T_guess, np.float64), sub.shape))
+        rc = lib().oracle_newton_subset(self.ref, int(sub.size), _ptr(E), _optr(Tr), _ptr(T))
+        if rc != OK:
+            raise RuntimeError(f"oracle subset newton failed rc={rc}")
+        return T
+
+    def step_subset(self, sub, I_sub, T_sub, sel, dt, Tr_sub=None):
+        """One step of cells sub[sel] from a subset state (neighbours in sub)."""
+        sub = np.ascontiguousarray(sub, np.int64)
+        sel = np.ascontiguousarray(sel, np.int64)
+        I_sub = np.ascontiguousarray(I_sub, np.float64)
+        T_sub = np.ascontiguousarray(T_sub, np.float64)
+        Tr = None if Tr_sub is None else np.ascontiguousarray(Tr_sub, np.float64)
+        out = np.empty((sel.size, self.nb, self.nd))
+        T1 = np.empty(sel.size)
+        rc = lib().oracle_step_subset(self.ref, _ptr(self.reflection_map()), int(sub.size), _ptr(sub), _ptr(I_sub),
+                                      _ptr(T_sub), _optr(Tr), int(sel.size), _ptr(sel), float(dt), _ptr(out),
+                                      _ptr(T1))
+        if rc != OK:
+            raise RuntimeError(f"oracle subset step failed rc={rc}")
+        return out, T1
+
     # -- initial state ----------------------------------------------------------
     def initial_state(self, t_init, ic_eps=0.0, seed=None, mult_fn=None, with_tr=False):
         """IC of the synthetic configs: I = I0_b(t_init) * multiplier, then
@@ -233,10 +282,11 @@ class Problem:
         T = np.full(self.nc, float(t_init))
         Tr = np.full(self.nc, float(t_init)) if (with_tr or self.has_rates) else None
         I = self.equilibrium(T)
-        if ic_eps:
+        if ic_eps or mult_fn is not None:
             from paper_conf_ipps_heislersdms24_b200.inputs import ic_multiplier, SEED
             for b in range(self.nb):
-                I[b] *= ic_multiplier(self.nd, self.nc, b, ic_eps, SEED if seed is None else seed)
+                I[b] *= (mult_fn(self.nd, self.nc, b) if mult_fn is not None else
+                         ic_multiplier(self.nd, self.nc, b, ic_eps, SEED if seed is None else seed))
             T, _ = self.newton(self.energy(I, Tr=Tr), T, Tr=Tr)
         return (I, T, Tr) if with_tr else (I, T)
 

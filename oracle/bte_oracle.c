@@ -340,3 +340,107 @@ int oracle_step_cells_equilibrium(const oracle_problem *p, const int32_t *r, con
     }
     return status;
 }
+
+/* ------------------------------------------------------------------ subsets */
+
+typedef struct {
+    const double *I; /* [nb][nd][n_sub] */
+    const int64_t *sub;
+    int64_t n_sub;
+    int32_t nd;
+    int missing;     /* set when a requested cell is not in sub */
+} subset_ctx;
+
+static int64_t subset_index(const int64_t *sub, int64_t n, int64_t c) {
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+        int64_t mid = lo + (hi - lo) / 2;
+        if (sub[mid] < c) lo = mid + 1; else hi = mid;
+    }
+    return (lo < n && sub[lo] == c) ? lo : -1;
+}
+
+static double subset_in(const void *vctx, int32_t b, int32_t d, int64_t c) {
+    subset_ctx *x = (subset_ctx *)vctx;
+    int64_t k = subset_index(x->sub, x->n_sub, c);
+    if (k < 0) {
+        x->missing = 1;
+        return NAN;
+    }
+    return x->I[((int64_t)b * x->nd + d) * x->n_sub + k];
+}
+
+void oracle_energy_subset(const oracle_problem *p, int64_t n_sub, const double *I_sub, const double *Tr_sub,
+                          double *E_sub) {
+    const int32_t nd = p->n_dirs;
+    for (int64_t k = 0; k < n_sub; ++k) {
+        double e = 0.0;
+        for (int32_t b = 0; b < p->n_bands; ++b) {
+            double sb = 0.0;
+            for (int32_t d = 0; d < nd; ++d) sb += p->w[d] * I_sub[((int64_t)b * nd + d) * n_sub + k];
+            e += oracle_weight_at(p, b, Tr_sub ? Tr_sub[k] : NAN) * sb;
+        }
+        E_sub[k] = e;
+    }
+}
+
+int oracle_newton_subset(const oracle_problem *p, int64_t n_sub, const double *E_sub, const double *Tr_sub,
+                         double *T_sub) {
+    double W = 0.0;
+    for (int32_t d = 0; d < p->n_dirs; ++d) W += p->w[d];
+    int status = ORACLE_OK;
+    for (int64_t k = 0; k < n_sub; ++k) {
+        int rc = solve_cell(p, W, E_sub[k], Tr_sub ? Tr_sub[k] : NAN, &T_sub[k], NULL);
+        if (rc != ORACLE_OK) status = rc;
+    }
+    return status;
+}
+
+int oracle_step_subset(const oracle_problem *p, const int32_t *r, int64_t n_sub, const int64_t *sub,
+                       const double *I_sub, const double *T_sub, const double *Tr_sub, int64_t n_sel,
+                       const int64_t *sel, double dt, double *Inew_sel, double *T1_sel) {
+    const int32_t nb = p->n_bands, nd = p->n_dirs;
+    double W = 0.0;
+    for (int32_t d = 0; d < nd; ++d) W += p->w[d];
+    /* update_one reads T[c] / Tr[c] by global cell id: full-length copies with
+     * the subset's values (other entries never read for the selected cells) */
+    double *T = (double *)malloc(sizeof(double) * (size_t)p->n_cells);
+    double *Tr = (double *)malloc(sizeof(double) * (size_t)p->n_cells);
+    if (!T || !Tr) {
+        free(T);
+        free(Tr);
+        return ORACLE_EINVAL;
+    }
+    for (int64_t k = 0; k < n_sub; ++k) {
+        T[sub[k]] = T_sub[k];
+        Tr[sub[k]] = Tr_sub ? Tr_sub[k] : NAN;
+    }
+    int status = ORACLE_OK;
+    for (int64_t j = 0; j < n_sel; ++j) {
+        subset_ctx ctx = {I_sub, sub, n_sub, nd, 0};
+        const int64_t k = sel[j];
+        const int64_t c = sub[k];
+        double *out = &Inew_sel[j * nb * nd];
+        for (int32_t b = 0; b < nb; ++b)
+            for (int32_t d = 0; d < nd; ++d)
+                out[b * nd + d] = update_one(p, r, T, Tr_sub ? Tr : NULL, subset_in, &ctx, dt, b, d, c);
+        if (ctx.missing) {
+            status = ORACLE_EINVAL;
+            break;
+        }
+        /* Tr <- T^n, then E and the solve from T^n (oracle_run's order) */
+        double e = 0.0;
+        for (int32_t b = 0; b < nb; ++b) {
+            double sb = 0.0;
+            for (int32_t d = 0; d < nd; ++d) sb += p->w[d] * out[b * nd + d];
+            e += oracle_weight_at(p, b, T_sub[k]) * sb;
+        }
+        double Tc = T_sub[k];
+        int rc = solve_cell(p, W, e, T_sub[k], &Tc, NULL);
+        T1_sel[j] = Tc;
+        if (rc != ORACLE_OK) status = rc;
+    }
+    free(T);
+    free(Tr);
+    return status;
+}

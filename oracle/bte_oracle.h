@@ -122,6 +122,24 @@ int oracle_step_cells_equilibrium(const oracle_problem *p, const int32_t *r, con
                                   const int64_t *cells, int64_t n_sel, double dt,
                                   double *Inew_sel, double *T1_sel);
 
+/* The same on a SUBSET of cells whose intensities are given explicitly (full
+ * fields that do not fit on the host, with a direction-dependent state).
+ * sub[n_sub]: ascending cell ids; I_sub[b][d][k] the intensity of cell sub[k].
+ *   oracle_energy_subset: E_sub[k] = E of cell sub[k] (weights at Tr_sub[k]).
+ *   oracle_newton_subset: T_sub in/out, the per-cell solve of oracle_newton.
+ *   oracle_step_subset:   one explicit step of the cells sub[sel[j]] (their
+ *     face neighbours must be in sub): Inew_sel[j][b][d] from (I_sub, T_sub,
+ *     Tr_sub), then E and the solve with the weights at T_sub (Tr <- T^n, as
+ *     in oracle_run) from T_sub: T1_sel[j].
+ * ORACLE_EINVAL if a neighbour is missing from sub; ORACLE_ENOCONV as above. */
+void oracle_energy_subset(const oracle_problem *p, int64_t n_sub, const double *I_sub, const double *Tr_sub,
+                          double *E_sub);
+int oracle_newton_subset(const oracle_problem *p, int64_t n_sub, const double *E_sub, const double *Tr_sub,
+                         double *T_sub);
+int oracle_step_subset(const oracle_problem *p, const int32_t *r, int64_t n_sub, const int64_t *sub,
+                       const double *I_sub, const double *T_sub, const double *Tr_sub, int64_t n_sel,
+                       const int64_t *sel, double dt, double *Inew_sel, double *T1_sel);
+
 #ifdef __cplusplus
 }
 #endif

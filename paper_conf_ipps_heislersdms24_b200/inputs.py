@@ -475,6 +475,7 @@ class Config:
     temp_rule: int = 0
     note: str = ""
     extra: dict = field(default_factory=dict)
+    ic_mult: object = None  # callable (nd, nc, band) -> [nd][nc] IC multiplier (instead of ic_eps)
 
     @property
     def n_updates_per_step(self):
@@ -553,3 +554,35 @@ def small_3d_config(shape=(6, 5, 4), n_spectral=2, ntheta=4, nphi=8, eps=0.1, h=
     bound = cartesian_dt_bound(mesh, bands, dirs)
     return Config(name=f"3d{shape}", mesh=mesh, bands=bands, dirs=dirs, bcs=bcs,
                   t_init=300.0, dt=0.5 * bound, nsteps=10, ic_eps=eps, extra={"dt_bound": bound})
+
+
+# --------------------------------------------------------------------------- ENOCONV case
+def failing_strip_config(amp=11.0, comp=9.5, nx=12, x0=1):
+    """A state whose temperature solve fails in step 4 (BTE_ENOCONV semantics,
+    SURVEY 8(b)): a 2-D nx x 2 strip (1 um cells), isothermal 300 K ends,
+    specular top / bottom, the 4 diagonal in-plane directions, two gray-like
+    rows without scattering (tau = inf, temperature rule R1) whose group
+    velocities differ by 2x.  At cells x = 1, 2 the +x directions of row 0 are
+    set to -amp x equilibrium and those of row 1 to (1 + comp) x equilibrium
+    (cells x0, x0 + 1 in general):
+    the energy starts positive, but the fast negative row-0 pulse outruns the
+    slow compensating row-1 pulse and a cell's energy turns negative after a
+    few steps (step 4 for the defaults, found with the oracle).  dt = the
+    positivity bound.  Multipliers only; each side evaluates its own I0."""
+    h = 1e-6
+    mesh = gen_mesh((nx, 2), (h, h))
+    bands = gen_bands_custom(omega=[2e13, 3e13], vg=[6000.0, 3000.0], tau=np.inf, C=[1e9, 1e9])
+    dirs = gen_dirs_inplane(4)
+    bcs = gen_bcs_walls(mesh, {WALL_XM: (ISOTHERMAL, 300.0), WALL_XP: (ISOTHERMAL, 300.0),
+                               WALL_YM: (SYMMETRY, 0.0), WALL_YP: (SYMMETRY, 0.0)})
+    dp = np.where(dirs["s"][:, 0] > 0)[0]
+    cells = np.array([y * nx + x for y in range(2) for x in (x0, x0 + 1)])
+
+    def mult(nd, nc, band):
+        m = np.ones((nd, nc))
+        m[np.ix_(dp, cells)] = -amp if band == 0 else 1.0 + comp
+        return m
+
+    return Config(name="fail-strip", mesh=mesh, bands=bands, dirs=dirs, bcs=bcs, t_init=300.0,
+                  dt=cartesian_dt_bound(mesh, bands, dirs), nsteps=10, temp_rule=1, ic_mult=mult,
+                  note="temperature solve fails in step 4")

@@ -9,9 +9,10 @@ RTOL_I = 1e-10  # north star: relative 1e-10 on I after 100 FP64 steps
 RTOL_T = 1e-9   # north star: relative 1e-9 on T
 
 
-def oracle_run(oracle_mod, cfg, nsteps, ic_eps=None):
-    p = oracle_mod.problem_from_config(cfg)
-    I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps if ic_eps is None else ic_eps, with_tr=True)
+def oracle_run(oracle_mod, cfg, nsteps, ic_eps=None, **pkw):
+    p = oracle_mod.problem_from_config(cfg, **pkw)
+    I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps if ic_eps is None else ic_eps, with_tr=True,
+                               mult_fn=getattr(cfg, "ic_mult", None))
     if nsteps:
         I, T, Tr = p.run(I, T, cfg.dt, nsteps, Tr=Tr)
     return I, T
