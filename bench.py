@@ -244,7 +244,7 @@ def run_ours(args):
     s = bte.solver_from_config(cfg, rank=rank, world=world, device=local, nccl_id=nccl_id, stream=stream, **part_kw,
                                profile=True, band_group=args.band_group, block_threads=args.block_threads,
                                max_spare_slabs=args.max_spare, dir_chunk=args.dir_chunk,
-                               locality=not args.no_locality, tma=not args.no_tma, stencil=args.stencil,
+                               locality=not args.no_locality, tma=not args.no_tma,
                                box=not args.no_box)
     bte.apply_ic(s, cfg)
     nb_loc = s.b_hi - s.b_lo
@@ -391,7 +391,6 @@ def main():
     ap.add_argument("--dir-chunk", type=int, default=0)
     ap.add_argument("--no-locality", action="store_true", help="keep row-major cell order (no Morton hint)")
     ap.add_argument("--no-tma", action="store_true", help="register-pipelined flux kernel instead of TMA-staged")
-    ap.add_argument("--stencil", action="store_true", help="stencil-staged kernel (structured order, opt-in)")
     ap.add_argument("--no-box", action="store_true", help="structured grids: TMA-staged kernel instead of the box kernel")
     ap.add_argument("--rate-law", action="store_true",
                     help="temperature-dependent relaxation times (SURVEY 8(f) N1) instead of constant tau")

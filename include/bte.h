@@ -54,7 +54,8 @@
 extern "C" {
 #endif
 
-typedef struct bte_ctx bte_ctx; /* opaque; owned by the caller until bte_destroy */
+typedef struct bte_ctx bte_ctx;     /* opaque; owned by the caller until bte_destroy */
+typedef struct bte_group bte_group; /* opaque in-process communicator (bte_group_create) */
 
 typedef enum {
     BTE_OK = 0,
@@ -90,12 +91,18 @@ typedef struct {
 typedef struct {
     int32_t n_bands;
     const double *omega;         /* [n_bands] centre angular frequency, rad/s, > 0 */
-    const double *d_omega;       /* [n_bands] width, rad/s (metadata; may be NULL) */
+    const double *d_omega;       /* [n_bands] width, rad/s (only read when i0_prefactor is NULL) */
     const double *vg;            /* [n_bands] group velocity |v_g|_b, m/s, > 0 */
     const double *tau;           /* [n_bands] relaxation time, s, in (0, +inf]; ignored (may be
                                     NULL) with the rate law below */
-    const int32_t *polarization; /* [n_bands] 0 = LA, 1 = TA (metadata; may be NULL) */
-    const double *i0_prefactor;  /* [n_bands] C_b > 0; required */
+    const int32_t *polarization; /* [n_bands] 0 = LA, 1 = TA (only read when i0_prefactor is NULL) */
+    const double *i0_prefactor;  /* [n_bands] C_b > 0 of I0_b(T) = C_b / expm1(hbar omega_b / (kB T))
+                                    (SURVEY 8(c) #4).  NULL: derived from (omega, d_omega,
+                                    polarization) with the built-in quadratic Si dispersion
+                                    omega = v_s k + c k^2 (LA 9.01e3 m/s, -2.0e-7 m^2/s; TA 5.23e3,
+                                    -2.26e-7) as C_b = hbar omega k^2 d_omega / (8 pi^3);
+                                    d_omega and polarization are then required (EINVAL otherwise,
+                                    or if omega lies above the branch maximum) */
     /* Optional temperature-dependent relaxation times (the paper
      * keeps tau as a per-cell variable that depends on T, L666-669, `beta` per
      * cell L1352-1353).  NULL rate_a: constant tau.  Else, per band-row and cell,
@@ -128,10 +135,9 @@ typedef struct {
 /* bte_options.flags */
 #define BTE_FLAG_PROFILE 1u       /* record CUDA events around every phase (see bte_stats) */
 #define BTE_FLAG_GENERIC_FACES 2u /* never use the opposite-face-pair layout (testing) */
-#define BTE_FLAG_NO_TMA 4u        /* register-pipelined flux kernel instead of the
-                                     TMA-staged one (testing / comparison) */
-#define BTE_FLAG_STENCIL 8u       /* structured index order: stencil-staged kernel (near/far
-                                     TMA windows; L2-bandwidth-heavy, opt-in) */
+#define BTE_FLAG_NO_TMA 4u        /* register-pipelined generic-face flux kernel instead of the
+                                     TMA-staged ones (testing / comparison) */
+/* (8u was an opt-in stencil-window kernel, removed: L2-bound) */
 #define BTE_FLAG_NO_BOX 16u       /* structured 2-D / 3-D box grids: do not use the box kernel
                                      (tensor-copy z-marching tiles, the default there) */
 
@@ -175,6 +181,16 @@ typedef struct {
      * with bte_halo_export / bte_halo_import before bte_step_begin. */
     const int32_t *cell_part; /* [n_cells] part id in [0, n_cell_parts) */
     int32_t n_cell_parts;     /* >= 1; world must be a multiple of it */
+    /* In-process communicator instead of NCCL (bte_group_create): the `world`
+     * ranks are host threads of this process, rank r calling every collective
+     * entry point from its own thread, each context on any device (several may
+     * share one).  The per-step exchanges (reduce-scatter / all-gather of the
+     * energy and T, the all-reduce variants, the halo send / receive group, the
+     * band-group split) then run as stream-ordered device copies between the
+     * ranks' buffers with the same semantics as the NCCL calls; no CUDA graphs.
+     * NULL: NCCL (nccl_unique_id) or no communicator.  EINVAL if the group's
+     * size differs from world or an NCCL id is passed too. */
+    bte_group *group;
 } bte_options;
 
 /* Per-context counters since creation / the last bte_reset_stats. Phase
@@ -195,11 +211,10 @@ typedef struct {
     int32_t band_group;
     int32_t block_threads;
     int32_t dir_chunks;        /* direction chunks per launch (grid.y factor) */
-    int32_t flux_variant;      /* flux kernel in use: 0 generic faces, 1 paired, 2 paired +
-                                  uniform geometry, 3 TMA-staged, 4 TMA-staged + uniform
-                                  geometry, 5 stencil-staged (structured order), 6 box
-                                  (structured 2-D / 3-D grid, tensor copies), 7 TMA-staged
-                                  generic faces (unstructured meshes) */
+    int32_t flux_variant;      /* flux kernel in use: 0 register-pipelined generic faces,
+                                  3 TMA-staged opposite-face pairs, 4 ... + uniform geometry,
+                                  6 box (structured 2-D / 3-D grid, tensor copies), 7
+                                  TMA-staged generic faces (unstructured meshes) */
     double ms_halo;            /* cell partitioning: halo pack + exchange + unpack */
     int64_t halo_bytes;        /* halo bytes this rank sends per step (all segments) */
     int64_t flux_launches;     /* flux-kernel launches (a1-a3), part of kernel_launches */
@@ -208,32 +223,59 @@ typedef struct {
 } bte_stats;
 
 /* Fill *o with the defaults (t_init 300, temp_rule 0, rtol 1e-12, 50 iters,
- * rank 0 / world 1 / device 0, everything else 0/NULL). */
+ * rank 0 / world 1 / device 0, everything else 0/NULL).  Newton controls:
+ * SURVEY 8(c) #6 (the paper gives none).  EINVAL if o is NULL. */
 BTE_API bte_status bte_options_default(bte_options *o);
 
-/* Validate and deep-copy the problem, build the device layout (interior cells
- * first, padded per-cell face slots, reflection maps, isothermal ghost tables)
- * and initialise I = I0_b(t_init), T = t_init.  Collective when world > 1.
+/* In-process communicator of `world` ranks (see bte_options.group).  *out is
+ * owned by the caller; destroy it after every context that uses it.  EINVAL
+ * if world < 1 or out is NULL. */
+BTE_API bte_status bte_group_create(int32_t world, bte_group **out);
+BTE_API void bte_group_destroy(bte_group *g);
+
+/* The problem statement of the paper (mesh + FVM, L286-292, L719-722; band
+ * table with omega, v_g, tau, polarization, L507-514, L1339-1359; direction
+ * set, L514-518, L654-664; isothermal / symmetric BCs, L563-607): validate and
+ * deep-copy it, build the device layout (face slots, reflection maps,
+ * isothermal ghost tables, slab pool) and initialise the state to the
+ * equilibrium IC I = I0_b(t_init), T = t_init (L585-588, L678-684).
+ * All pointers are host pointers borrowed for the call; *out is owned by the
+ * caller (bte_destroy).  Collective when world > 1 with a communicator.
  * EINVAL on: dim not 2/3; non-positive V, A, w, C, omega, v or tau; non-unit
  * normals or directions; n_z != 0 in 2-D; a face id out of range; > 8 faces in
  * a cell; a symmetric wall whose reflected direction is not in the set (1e-10);
- * all temperature weights zero; more than 128 band-rows on one rank. */
+ * all temperature weights zero; more than 128 band-rows on one rank or 1024 in
+ * all.  ENOMEM if the state does not fit the device; ECUDA / ENCCL on runtime
+ * or communicator failures.  On error *out is NULL and bte_last_error(NULL)
+ * says why. */
 BTE_API bte_status bte_create(const bte_mesh *mesh, const bte_bands *bands, const bte_dirs *dirs,
                       const bte_bcs *bcs, const bte_options *opts, bte_ctx **out);
 
-/* n explicit steps of size dt (Eq. 2-3).  Collective when world > 1; returns
- * after the steps completed.  EINVAL if dt <= 0 or dt exceeds the positivity
- * bound 1 / max_{c,b,d} (1/tau_b + v_b sum_f (A_f/V_c) max(s_d.n_f, 0))
- * (see bte_dt_bound).  ENOCONV if a cell's temperature solve failed. */
+/* n explicit steps of size dt: forward Euler on the finite-volume form (Eq.
+ * 2-3, L269-292) of the phonon BTE (Eq. 4-5) with first-order upwind
+ * face values (L264-267, L644-647), the Eq. 6 ghosts (L563-607), the per-cell
+ * energy (L412-418) summed across ranks (L760-766) and the temperature solve
+ * that refreshes I0 (L407-418, L555-561, L707-716).  Collective when world > 1;
+ * returns after the steps completed (host-synchronous).
+ * EINVAL if dt <= 0 or dt exceeds the positivity bound
+ * 1 / max_{c,b,d} (1/tau_b + v_b sum_f (A_f/V_c) max(s_d.n_f, 0)) (see
+ * bte_dt_bound); ESTATE inside a split step or with world > 1
+ * and no communicator.  ENOCONV if a cell's temperature solve failed
+ * (E <= 0 or non-finite): stepping stops at that step, the state is the one at
+ * its end (the failed cells keep their previous T), the remaining steps are not
+ * taken, and bte_get_stats().steps counts the steps taken.  With cell
+ * partitioning the failure is reported by the ranks owning the failed cells. */
 BTE_API bte_status bte_step(bte_ctx *ctx, double dt, int64_t n);
 
 /* Largest admissible dt (the positivity bound above, over all bands; with the
  * rate law, rates at the highest temperature the state can reach: the max of
- * t_init, the wall temperatures and the last set / solved T, P10). */
+ * t_init, the wall temperatures and the last set / solved T, P10).  Host
+ * pointer out.  EINVAL on NULL. */
 BTE_API bte_status bte_dt_bound(const bte_ctx *ctx, double *dt_max);
 
 /* Temperature of the CURRENT state under `rule` (0 R2, 1 R1 energy-equivalent,
- * 2 R3 one linearised step from the current T), without changing the state:
+ * 2 R3 one linearised "first law" step from the current T, L413-415), without
+ * changing the state:
  * energy reduction with that rule's weights, all-reduce (collective when
  * world > 1), Newton from the current T.  T[n_cells] host, caller order.
  * the paper's temperature relation is under-specified
@@ -241,41 +283,61 @@ BTE_API bte_status bte_dt_bound(const bte_ctx *ctx, double *dt_max);
  * cell's solve fails; ESTATE with world > 1 and no communicator. */
 BTE_API bte_status bte_get_temperature_rule(const bte_ctx *ctx, int32_t rule, double *T);
 
-/* T[n_cells] (host, caller order).  T is replicated on every rank. */
+/* The lattice temperature T_c of the current state, the output of the
+ * per-cell solve (L407-418, L555-561; Fig. 6 "temperature"), into the
+ * caller's host buffer T[n_cells] in caller cell order (owned cells under cell
+ * partitioning).  Replicated on every rank.  Synchronises the library stream.
+ * EINVAL on NULL; ECUDA on a runtime failure. */
 BTE_API bte_status bte_get_temperature(const bte_ctx *ctx, double *T);
 
-/* I[b_hi-b_lo][n_dirs][n_cells] (host, caller order) for global band-rows
- * [b_lo, b_hi), which must lie inside this rank's bte_band_range. */
+/* The intensity field I[b][d][c] of the current state (the unknowns of Eq. 5,
+ * L546-553; band-major storage, L777-840) for global band-rows [b_lo, b_hi),
+ * which must lie inside this rank's bte_band_range, into the caller's host
+ * buffer I[b_hi-b_lo][n_dirs][n_cells] (caller cell order).  Synchronises the
+ * library stream.  EINVAL for rows outside the range or NULL; ESTATE inside a
+ * split step. */
 BTE_API bte_status bte_get_intensity(const bte_ctx *ctx, int32_t b_lo, int32_t b_hi, double *I);
 
-/* Overwrite rows [b_lo, b_hi) of I (same layout as bte_get_intensity).  T is
- * NOT changed; call bte_solve_temperature after the last row is set. */
+/* Overwrite rows [b_lo, b_hi) of I from the caller's host buffer (layout of
+ * bte_get_intensity; restart / checkpoint of the explicit state, L398-404
+ * "u = u_new").  T is NOT changed; call bte_solve_temperature after the last
+ * row is set.  Errors as bte_get_intensity. */
 BTE_API bte_status bte_set_intensity(bte_ctx *ctx, int32_t b_lo, int32_t b_hi, const double *I);
 
-/* T <- temperature of the current I (energy reduction, all-reduce, Newton from
- * the current T), and I0 refreshed.  Collective when world > 1. */
+/* T <- temperature of the current I: the energy integral over all directions
+ * and bands (L412-418), summed across ranks (L760-766), the per-cell Newton
+ * solve from the current T (L555-561), and I0 refreshed
+ * (L707-716).  Collective when world > 1.  ENOCONV if a cell's solve fails
+ * (its T is kept); ESTATE inside a split step or world > 1 without a
+ * communicator. */
 BTE_API bte_status bte_solve_temperature(bte_ctx *ctx);
 
-/* Set T (host, caller order) and I = I0_b(T_c) for every local row (local
- * thermal equilibrium).  Not collective. */
+/* Set T (host buffer, caller order) and I = I0_b(T_c) for every local row
+ * (local thermal equilibrium, the IC of L585-588, L678-684).  Not collective.
+ * EINVAL if some T_c <= 0 or non-finite; ESTATE inside a split step. */
 BTE_API bte_status bte_set_equilibrium(bte_ctx *ctx, const double *T);
 
-/* This rank's band-rows [b_lo, b_hi). */
+/* This rank's band-rows [b_lo, b_hi) (band-parallel split, L773-775:
+ * [floor(g nb / G), floor((g+1) nb / G)) for band group g of G).  EINVAL on NULL. */
 BTE_API bte_status bte_band_range(const bte_ctx *ctx, int32_t *b_lo, int32_t *b_hi);
 
-/* Split step, for callers that reduce the energy themselves (e.g. tests of
- * band sharding on one device): begin = flux/relaxation of the local rows and
- * the local energy partial; get/set energy move E[n_cells] (host, caller
- * order); finish = temperature solve from the set energy, I0 refresh and state
- * advance.  bte_step(ctx, dt, 1) == begin; (reduce E); finish. */
+/* Split step, for callers that reduce the energy themselves (the band
+ * coupling of L760-766 done outside the library): begin = flux / relaxation
+ * of the local rows (Eq. 3, 5, 6) and the local energy partial (L412-418);
+ * get / set energy move E[n_cells] (host buffer, caller order); finish =
+ * temperature solve from the set energy, I0 refresh and state advance.
+ * bte_step(ctx, dt, 1) == begin; (reduce E); finish.  ESTATE for begin twice
+ * or finish without begin; EINVAL for dt as bte_step; ENOCONV from finish as
+ * bte_step. */
 BTE_API bte_status bte_step_begin(bte_ctx *ctx, double dt);
 BTE_API bte_status bte_get_energy(const bte_ctx *ctx, double *E);
 BTE_API bte_status bte_set_energy(bte_ctx *ctx, const double *E);
 BTE_API bte_status bte_step_finish(bte_ctx *ctx);
 
-/* Cell partitioning (see bte_options.cell_part).  Owned cells of this rank:
- * *n_local, and (ids != NULL) their global ids ascending into ids[*n_local]
- * (host).  Without partitioning: all cells, ids 0..n_cells-1. */
+/* Cell partitioning (see bte_options.cell_part; the paper's cell-parallel
+ * split, L728-735, L768-772).  Owned cells of this rank: *n_local, and (ids !=
+ * NULL) their global ids ascending into the caller's host buffer ids[*n_local].
+ * Without partitioning: all cells, ids 0..n_cells-1.  EINVAL on NULL ctx / n_local. */
 BTE_API bte_status bte_local_cells(const bte_ctx *ctx, int64_t *n_local, int64_t *ids);
 
 /* Halo segment sizes with part `part` (doubles): *n_send = values this rank
@@ -295,20 +357,25 @@ BTE_API bte_status bte_halo_size(const bte_ctx *ctx, int32_t part, int64_t *n_se
 BTE_API bte_status bte_halo_export(const bte_ctx *ctx, int32_t part, double *buf);
 BTE_API bte_status bte_halo_import(bte_ctx *ctx, int32_t part, const double *buf);
 
-/* Counters (see bte_stats). */
+/* Counters (see bte_stats) into the caller's struct / reset them (the
+ * paper's per-phase timing of Figs. 5 and 8, L854-857, L871-873).  EINVAL on NULL. */
 BTE_API bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st);
 BTE_API bte_status bte_reset_stats(bte_ctx *ctx);
 
-/* 128-byte NCCL unique id (call on rank 0 only, then broadcast). ENCCL if the
- * NCCL library cannot be loaded (BTE_NCCL_LIB overrides the search). */
+/* 128-byte NCCL unique id into the caller's buffer (call on rank 0 only, then
+ * broadcast; the multi-GPU band sharding of L760-775).  ENCCL if the NCCL
+ * library cannot be loaded (BTE_NCCL_LIB overrides the search); EINVAL on NULL. */
 BTE_API bte_status bte_nccl_unique_id(void *id128);
 
 /* Message of the last failure on ctx (ctx may be NULL: last bte_create /
- * global failure of this thread).  Never NULL. */
+ * global failure of this thread).  Never NULL; owned by the library, valid
+ * until the next call on ctx. */
 BTE_API const char *bte_last_error(const bte_ctx *ctx);
 BTE_API const char *bte_status_string(bte_status s);
 
-/* Release device memory, streams and the NCCL communicator.  NULL is a no-op. */
+/* Release the context: device memory, the library-owned stream, the NCCL
+ * communicator / group endpoint (synchronises first).  Not collective.  NULL
+ * is a no-op.  Every pointer obtained from ctx is invalid afterwards. */
 BTE_API void bte_destroy(bte_ctx *ctx);
 
 #ifdef __cplusplus

@@ -20,7 +20,6 @@ BTE_OK, BTE_EINVAL, BTE_ENOMEM, BTE_ECUDA, BTE_ENCCL, BTE_ENOCONV, BTE_ESTATE = 
 BTE_FLAG_PROFILE = 1
 BTE_FLAG_GENERIC_FACES = 2
 BTE_FLAG_NO_TMA = 4
-BTE_FLAG_STENCIL = 8
 BTE_FLAG_NO_BOX = 16
 ISOTHERMAL, SYMMETRY = 0, 1
 
@@ -62,7 +61,7 @@ class Options(C.Structure):
                 ("device", C.c_int32), ("nccl_unique_id", C.c_void_p), ("stream", C.c_void_p),
                 ("flags", C.c_uint32), ("max_spare_slabs", C.c_int32), ("block_threads", C.c_int32),
                 ("band_group", C.c_int32), ("dir_chunk", C.c_int32), ("cell_part", C.c_void_p),
-                ("n_cell_parts", C.c_int32)]
+                ("n_cell_parts", C.c_int32), ("group", C.c_void_p)]
 
 
 class Stats(C.Structure):
@@ -79,15 +78,14 @@ class Stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
-FLUX_VARIANTS = {0: "generic", 1: "paired", 2: "paired-uniform", 3: "tma", 4: "tma-uniform", 5: "stencil", 6: "box",
-                 7: "tma-generic"}
+FLUX_VARIANTS = {0: "generic", 3: "tma", 4: "tma-uniform", 6: "box", 7: "tma-generic"}
 
 EXPORTS = ["bte_options_default", "bte_create", "bte_step", "bte_dt_bound", "bte_get_temperature",
            "bte_get_intensity", "bte_set_intensity", "bte_solve_temperature", "bte_set_equilibrium",
            "bte_band_range", "bte_step_begin", "bte_get_energy", "bte_set_energy", "bte_step_finish",
            "bte_get_stats", "bte_reset_stats", "bte_nccl_unique_id", "bte_last_error",
            "bte_status_string", "bte_destroy", "bte_get_temperature_rule", "bte_local_cells",
-           "bte_halo_size", "bte_halo_export", "bte_halo_import"]
+           "bte_halo_size", "bte_halo_export", "bte_halo_import", "bte_group_create", "bte_group_destroy"]
 
 
 def _load():
@@ -131,6 +129,8 @@ def _load():
         "bte_halo_size": ([vp, i32, P(i64), P(i64)], i32),
         "bte_halo_export": ([vp, i32, vp], i32),
         "bte_halo_import": ([vp, i32, vp], i32),
+        "bte_group_create": ([i32, P(vp)], i32),
+        "bte_group_destroy": ([vp], None),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -158,6 +158,36 @@ def nccl_unique_id() -> bytes:
     return buf.raw
 
 
+class Group:
+    """In-process communicator of `world` ranks (bte_group_create): every rank
+    is a host thread of this process with its own Solver(group=...), calling
+    the collective methods (step, solve_temperature, ...) from that thread.
+    The library's per-step exchanges then run as device copies between the
+    ranks (any device, several may share one).  Close it after the solvers."""
+
+    def __init__(self, world):
+        h = C.c_void_p()
+        _check(lib.bte_group_create(int(world), C.byref(h)))
+        self.handle, self.world = h, int(world)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            lib.bte_group_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
 class Solver:
     """One bte_ctx.  Arrays in caller cell order; I is [bands][dirs][cells].
 
@@ -167,8 +197,8 @@ class Solver:
     def __init__(self, mesh, bands, dirs, bcs, *, t_init=300.0, temp_rule=0, newton_rtol=1e-12,
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
                  stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
-                 generic_faces=False, locality=True, dir_chunk=0, tma=True, stencil=False, box=True,
-                 cell_part=None, n_cell_parts=1):
+                 generic_faces=False, locality=True, dir_chunk=0, tma=True, box=True,
+                 cell_part=None, n_cell_parts=1, group: Group | None = None, i0_prefactor=True):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -187,8 +217,9 @@ class Solver:
         self.n_cells, self.n_bands, self.n_dirs = int(mesh["n_cells"]), int(bands["n_bands"]), int(dirs["n_dirs"])
         m = Mesh(int(mesh["dim"]), self.n_cells, _p(k["off"]).value, _p(k["nbr"]).value, _p(k["area"]).value,
                  _p(k["nrm"]).value, _p(k["vol"]).value, _p(k["cen"]).value if k["cen"] is not None else None)
+        # i0_prefactor=False: pass NULL, the library derives C_b from its built-in dispersion
         b = Bands(self.n_bands, _p(k["omega"]).value, _p(k["dw"]).value, _p(k["vg"]).value, _p(k["tau"]).value,
-                  _p(k["pol"]).value, _p(k["C"]).value,
+                  _p(k["pol"]).value, _p(k["C"]).value if i0_prefactor else None,
                   _p(k["ra"]).value if law else None, _p(k["rb"]).value if law else None,
                   _p(k["rth"]).value if law else None)
         d = Dirs(self.n_dirs, _p(k["s"]).value, _p(k["w"]).value)
@@ -205,9 +236,11 @@ class Solver:
             o.nccl_unique_id = C.cast(self._nccl_buf, C.c_void_p).value
         if stream is not None:
             o.stream = int(getattr(stream, "cuda_stream", stream))
+        if group is not None:
+            self._group = group  # (kept alive while the context uses it)
+            o.group = group.handle.value
         o.flags = ((BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
-                   | (0 if tma else BTE_FLAG_NO_TMA) | (BTE_FLAG_STENCIL if stencil else 0)
-                   | (0 if box else BTE_FLAG_NO_BOX))
+                   | (0 if tma else BTE_FLAG_NO_TMA) | (0 if box else BTE_FLAG_NO_BOX))
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)
         o.dir_chunk = int(dir_chunk)
         if cell_part is not None:  # cell partitioning (N3): this rank owns part rank % n_cell_parts
@@ -358,13 +391,15 @@ def apply_ic(solver, cfg, seed=None):
     """Seeded IC of the synthetic configs through the public API: equilibrium
     at t_init times the generator's multiplier, then T of that field."""
     from .inputs import SEED, ic_multiplier
-    if not cfg.ic_eps:
+    fn = getattr(cfg, "ic_mult", None)
+    if not cfg.ic_eps and fn is None:
         return
     seed = SEED if seed is None else seed
     cells = solver.local_cells() if solver.n_cell_parts > 1 else None
     for b in range(solver.b_lo, solver.b_hi):
         I = solver.intensity(b, b + 1)
-        mult = ic_multiplier(solver.n_dirs, solver.n_global_cells, b, cfg.ic_eps, seed)
+        mult = (fn(solver.n_dirs, solver.n_global_cells, b) if fn is not None else
+                ic_multiplier(solver.n_dirs, solver.n_global_cells, b, cfg.ic_eps, seed))
         I[0] *= mult if cells is None else mult[:, cells]
         solver.set_intensity(I, b, b + 1)
     solver.solve_temperature()

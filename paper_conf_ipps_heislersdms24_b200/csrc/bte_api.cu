@@ -20,6 +20,7 @@
 #include <functional>
 #include <array>
 #include <map>
+#include <mutex>
 #include <set>
 #include <string>
 #include <vector>
@@ -63,6 +64,10 @@ struct HaloSeg {
 
 }  // namespace
 
+struct bte_group {
+    bte::group::Group *g = nullptr;
+};
+
 struct bte_ctx {
     std::string err = "no error";
     bte_options opt{};
@@ -95,8 +100,6 @@ struct bte_ctx {
     int32_t *bl_off = nullptr, *bl_col = nullptr, *bl_cls = nullptr;  // ... boundary-face ghost lists
     uint16_t *sidx = nullptr;                        // ... per face slot: shared-memory index of the upwind value
     int32_t hstride = 0;
-    bool stencil = false;    // ... + constant neighbour offsets: the stencil-staged kernel
-    int32_t so[3] = {0, 0, 0}, halo = 0, wmain = 0, nfar = 0, farq[3] = {0, 0, 0};
     double gu[3][3] = {};
     // box path (structured hex grid in lexicographic order, flux_box_kernel)
     bool box = false;
@@ -132,7 +135,14 @@ struct bte_ctx {
     double *cw_loc = nullptr;
     std::vector<double> h_inv_tau, h_vg, h_cw;  // local band-rows
     double *Cb = nullptr, *theta = nullptr, *cw_all = nullptr;
-    int32_t *d_iter_max = nullptr, *d_fail = nullptr;
+    int32_t *d_iter_max = nullptr;
+    // d_flags[0] fail (a temperature solve failed), [1] halt (the fail flag as the
+    // step's flux launch saw it: the rest of the step is a no-op), [2] steps done
+    // (counted by each step's last kernel; the host undoes the slab rotation of
+    // the steps skipped after a failure, so the state is that of the failing step)
+    int32_t *d_flags = nullptr, *d_fail = nullptr, *d_halt = nullptr, *d_done = nullptr;
+    int32_t done_seen = 0;
+    int newton_mode = 0;  // the step's solve: 0 by mesh size, 1 warp per cell, 2 thread per cell
     unsigned long long *d_smax = nullptr;
     // launch plan
     int bg = 4, block = 256;
@@ -195,47 +205,59 @@ bte_status upload(bte_ctx *ctx, T **p, const std::vector<T> &h) {
 }
 
 // ------------------------------------------------------------- template dispatch
-using FluxLaunch = void (*)(dim3, dim3, cudaStream_t, const bte::FluxParams &);
+// Dynamic shared memory above 48 KB needs a per-function opt-in, and the
+// attribute belongs to the device's context: remembered per (device, function),
+// raised only (contexts with different layouts need different amounts).
+cudaError_t ensure_smem(const void *fn, size_t smem) {
+    if (smem <= 48 * 1024) return cudaSuccess;
+    static std::mutex mu;
+    static std::map<std::pair<int, const void *>, size_t> granted;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lk(mu);
+    size_t &g = granted[{dev, fn}];
+    if (smem <= g) return cudaSuccess;
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess) g = smem;
+    return e;
+}
 
-template <int DIM, int MF, int BG, bool PAIRED, bool UG = false>
-void flux_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    if constexpr (PAIRED)
-        bte::flux_paired_kernel<DIM, MF, BG, UG><<<g, b, 0, s>>>(p);
-    else
-        bte::flux_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
+using FluxLaunch = cudaError_t (*)(dim3, dim3, cudaStream_t, const bte::FluxParams &);
+
+// Register-pipelined generic-face kernel (block sizes other than 256, or meshes
+// whose tiles stage too many halo / ghost values for the TMA kernel).
+template <int DIM, int MF, int BG>
+cudaError_t flux_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+    bte::flux_kernel<DIM, MF, BG><<<g, b, 0, s>>>(p);
+    return cudaGetLastError();
 }
 
 // TMA-staged paired kernel: one 256-cell tile per block, kStages x BG x 2 KB ring.
 template <int DIM, int NP, int BG, bool UG>
-void flux_tma_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
+cudaError_t flux_tma_launch_t(dim3 g, dim3, cudaStream_t s, const bte::FluxParams &p) {
     const size_t smem = (size_t)bte::kStages * BG * bte::kTile * sizeof(double) +
                         (UG ? (size_t)p.dchunk * sizeof(bte::DirEntry<NP>) : 0);
-    static size_t attr = 0;  // > 48 KB of dynamic shared memory needs an opt-in
-    if (attr < smem) {
-        cudaFuncSetAttribute(bte::flux_tma_kernel<DIM, NP, BG, UG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem);
-        attr = smem;
-    }
+    cudaError_t e = ensure_smem((const void *)bte::flux_tma_kernel<DIM, NP, BG, UG>, smem);
+    if (e != cudaSuccess) return e;
     bte::flux_tma_kernel<DIM, NP, BG, UG><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+    return cudaGetLastError();
 }
 
 // TMA-staged generic-face kernel (general meshes): kStages x BG x 2 KB ring.
 template <int DIM, int MF, int BG, bool TD>
-void flux_tma_generic_launch_td(dim3 g, const bte::FluxParams &p, cudaStream_t s) {
+cudaError_t flux_tma_generic_launch_td(dim3 g, const bte::FluxParams &p, cudaStream_t s) {
     const size_t smem = (size_t)bte::kStagesG * BG * p.hstride * sizeof(double) + (size_t)p.dchunk * sizeof(double4);
-    static size_t attr = 0;
-    if (attr < smem) {
-        cudaFuncSetAttribute(bte::flux_tma_generic_kernel<DIM, MF, BG, TD>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = smem;
-    }
+    cudaError_t e = ensure_smem((const void *)bte::flux_tma_generic_kernel<DIM, MF, BG, TD>, smem);
+    if (e != cudaSuccess) return e;
     bte::flux_tma_generic_kernel<DIM, MF, BG, TD><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+    return cudaGetLastError();
 }
 
 template <int DIM, int MF, int BG>
-void flux_tma_generic_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    if (p.rate_cur) flux_tma_generic_launch_td<DIM, MF, BG, true>(g, p, s);
-    else flux_tma_generic_launch_td<DIM, MF, BG, false>(g, p, s);
+cudaError_t flux_tma_generic_launch_t(dim3 g, dim3, cudaStream_t s, const bte::FluxParams &p) {
+    if (p.rate_cur) return flux_tma_generic_launch_td<DIM, MF, BG, true>(g, p, s);
+    return flux_tma_generic_launch_td<DIM, MF, BG, false>(g, p, s);
 }
 
 template <int DIM, int MF>
@@ -244,33 +266,6 @@ FluxLaunch pick_tma_generic(int bg) {
         case 1: return flux_tma_generic_launch_t<DIM, MF, 1>;
         case 2: return flux_tma_generic_launch_t<DIM, MF, 2>;
         default: return flux_tma_generic_launch_t<DIM, MF, 4>;
-    }
-}
-
-// Stencil-staged kernel (structured meshes): near + far windows per plane.
-template <int DIM, int NP, int BG>
-void flux_stencil_launch_t(dim3 g, dim3 b, cudaStream_t s, const bte::FluxParams &p) {
-    const size_t smem = (size_t)bte::kStages * BG * (p.wmain + p.nfar * bte::kFarWin) * sizeof(double);
-    static size_t attr = 0;
-    if (attr < smem) {
-        cudaFuncSetAttribute(bte::flux_stencil_kernel<DIM, NP, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem);
-        attr = smem;
-    }
-    bte::flux_stencil_kernel<DIM, NP, BG><<<g, dim3(bte::kTile), smem, s>>>(p);
-}
-
-template <int DIM, int NP>
-FluxLaunch pick_stencil(int bg) {
-    switch (bg) {
-        case 1: return flux_stencil_launch_t<DIM, NP, 1>;
-        case 2: return flux_stencil_launch_t<DIM, NP, 2>;
-        case 3: return flux_stencil_launch_t<DIM, NP, 3>;
-        case 4: return flux_stencil_launch_t<DIM, NP, 4>;
-        case 5: return flux_stencil_launch_t<DIM, NP, 5>;
-        case 6: return flux_stencil_launch_t<DIM, NP, 6>;
-        case 7: return flux_stencil_launch_t<DIM, NP, 7>;
-        default: return flux_stencil_launch_t<DIM, NP, 8>;
     }
 }
 
@@ -288,40 +283,23 @@ FluxLaunch pick_tma(int bg) {
     }
 }
 
-// Paired kernels exist for every band group 1..8 (per-cell or uniform geometry),
-// generic ones for 1, 2, 4.
-template <int DIM, int MF, bool UG>
-FluxLaunch pick_paired(int bg) {
-    switch (bg) {
-        case 1: return flux_launch_t<DIM, MF, 1, true, UG>;
-        case 2: return flux_launch_t<DIM, MF, 2, true, UG>;
-        case 3: return flux_launch_t<DIM, MF, 3, true, UG>;
-        case 4: return flux_launch_t<DIM, MF, 4, true, UG>;
-        case 5: return flux_launch_t<DIM, MF, 5, true, UG>;
-        case 6: return flux_launch_t<DIM, MF, 6, true, UG>;
-        case 7: return flux_launch_t<DIM, MF, 7, true, UG>;
-        default: return flux_launch_t<DIM, MF, 8, true, UG>;
-    }
-}
-
+// Generic register kernels exist for band groups 1, 2, 4.
 template <int DIM, int MF>
 FluxLaunch pick_generic(int bg) {
     switch (bg) {
-        case 1: return flux_launch_t<DIM, MF, 1, false>;
-        case 2: return flux_launch_t<DIM, MF, 2, false>;
-        default: return flux_launch_t<DIM, MF, 4, false>;
+        case 1: return flux_launch_t<DIM, MF, 1>;
+        case 2: return flux_launch_t<DIM, MF, 2>;
+        default: return flux_launch_t<DIM, MF, 4>;
     }
 }
 
-// mf_t: padded faces per cell (generic) or face pairs per cell (paired)
-FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, bool tma, bool stencil) {
-    if (stencil) return dim == 2 ? pick_stencil<2, 2>(bg) : pick_stencil<3, 3>(bg);
-    if (paired && tma) {
+// mf_t: padded faces per cell (generic) or face pairs per cell (paired; paired
+// layouts are only built for the TMA kernel)
+FluxLaunch pick_flux(int dim, int mf_t, int bg, bool paired, bool uniform_g, bool tma) {
+    if (paired) {
         if (uniform_g) return dim == 2 ? pick_tma<2, 2, true>(bg) : pick_tma<3, 3, true>(bg);
         return dim == 2 ? pick_tma<2, 2, false>(bg) : pick_tma<3, 3, false>(bg);
     }
-    if (paired && uniform_g) return dim == 2 ? pick_paired<2, 2, true>(bg) : pick_paired<3, 3, true>(bg);
-    if (paired) return dim == 2 ? pick_paired<2, 2, false>(bg) : pick_paired<3, 3, false>(bg);
     if (tma) {
         if (dim == 2) return mf_t == 3 ? pick_tma_generic<2, 3>(bg) : mf_t == 4 ? pick_tma_generic<2, 4>(bg)
                                                                                : pick_tma_generic<2, 8>(bg);
@@ -755,7 +733,12 @@ int box_stage(const bte_ctx *ctx) {
 
 size_t box_smem(const bte_ctx *ctx) {
     const int stage = box_stage(ctx);
-    return ((size_t)ctx->box_stages * stage + 2 * 4 * bte::kBoxCells + (size_t)ctx->box_L * bte::kBoxCells) *
+#ifdef BTE_BOX_TMA_STORE
+    constexpr size_t obuf = 2 * 4 * bte::kBoxCells;  // double-buffered output tiles of the tensor stores
+#else
+    constexpr size_t obuf = 0;  // results leave straight from registers
+#endif
+    return ((size_t)ctx->box_stages * stage + obuf + (size_t)ctx->box_L * bte::kBoxCells) *
                sizeof(double) +
            (size_t)kBoxMaxOrbChunk * sizeof(bte::BoxOrbitC);
 }
@@ -874,6 +857,11 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     p.orb = ctx->orb;
     p.dirs = ctx->dirs_box;
     p.part = ctx->part;
+    p.pool = ctx->pool;
+    p.slab_elems = ctx->slab_elems;
+    p.ps = ctx->ps;
+    p.fail = ctx->d_fail;
+    p.halt = ctx->d_halt;
     const size_t smem = box_smem(ctx);
     int slot = 0;
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
@@ -931,11 +919,6 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.gy = ctx->gy;
     p.gz = ctx->gz;
     std::memcpy(p.gu, ctx->gu, sizeof p.gu);
-    std::memcpy(p.so, ctx->so, sizeof p.so);
-    std::memcpy(p.farq, ctx->farq, sizeof p.farq);
-    p.halo = ctx->halo;
-    p.wmain = ctx->wmain;
-    p.nfar = ctx->nfar;
     p.fcode = ctx->fcode;
     p.fcode8 = ctx->fcode8;
     p.i0w = ctx->i0w;
@@ -950,6 +933,8 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.bl_cls = ctx->bl_cls;
     p.sidx = ctx->sidx;
     p.hstride = ctx->hstride;
+    p.fail = ctx->d_fail;
+    p.halt = ctx->d_halt;
     if (ctx->td) {
         p.rate_cur = rate_half(ctx, ctx->rsel);
         p.rate_next = rate_half(ctx, 1 - ctx->rsel);
@@ -961,7 +946,7 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
         const int nbl_batch = std::min(ctx->n_spare, ctx->nb_loc - l0);
         for (const Segment &sg : segments(nbl_batch, ctx->bg, ctx->paired)) {
             const FluxLaunch fn =
-                pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma, ctx->stencil);
+                pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma);
             const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
             p.nbl = sg.nbl;
             p.band0 = l0 + sg.off;
@@ -980,7 +965,7 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
             if (sg.off == 0) ctx->dir_chunks = lp.n_dch;
             const dim3 grid((ctx->nc + ctx->block - 1) / ctx->block, lp.groups * lp.n_dch);
             ev_mark(ctx, kPhFlux, true);
-            fn(grid, block, ctx->stream, p);
+            CUDA_TRY(ctx, fn(grid, block, ctx->stream, p));
             ev_mark(ctx, kPhFlux, false);
             ctx->st.kernel_launches++;
             ctx->st.flux_launches++;
@@ -1008,7 +993,45 @@ bte_status reduce_slots(bte_ctx *ctx);
 // C3 (14,400 cells) 0.066 -> 0.053 ms.  Larger meshes: one thread per cell
 // (newton_kernel, one launch; C4 0.16 ms vs 0.21 with warps).  Re-solves of the
 // current state (step = false) use newton_kernel.
-bool warp_newton(const bte_ctx *ctx, int ncells) { return ncells < 32 * 8 * ctx->sm_count; }
+bool warp_newton(const bte_ctx *ctx, int ncells) {
+    if (ctx->newton_mode) return ctx->newton_mode == 1;  // (BTE_NEWTON=warp|thread: tests of both kernels)
+    return ncells < 32 * 8 * ctx->sm_count;
+}
+
+// Band constants in shared memory: C, theta, c_b (+ the four rate-law arrays).
+size_t newton_smem(const bte_ctx *ctx) { return (size_t)(ctx->td ? 7 : 3) * ctx->nb * sizeof(double); }
+
+// Thread-per-cell solve over q.nc cells (block 0 counts the step when q.done).
+bte_status launch_newton_cells(bte_ctx *ctx, const bte::NewtonParams &q) {
+    if (q.nc <= 0) return BTE_OK;
+    const int tb = 128;
+    CUDA_TRY(ctx, ensure_smem((const void *)bte::newton_kernel, newton_smem(ctx)));
+    bte::newton_kernel<<<(q.nc + tb - 1) / tb, tb, newton_smem(ctx), ctx->stream>>>(q);
+    ctx->st.kernel_launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+// Warp-per-cell solve: R = band-rows per lane, the smallest power of two >= nb / 32.
+template <int R>
+bte_status launch_newton_warp_r(bte_ctx *ctx, const bte::NewtonParams &q) {
+    CUDA_TRY(ctx, ensure_smem((const void *)bte::newton_warp_kernel<R>, newton_smem(ctx)));
+    bte::newton_warp_kernel<R><<<(q.nc + 7) / 8, 256, newton_smem(ctx), ctx->stream>>>(q);
+    ctx->st.kernel_launches++;
+    CUDA_TRY(ctx, cudaGetLastError());
+    return BTE_OK;
+}
+
+bte_status launch_newton_warp(bte_ctx *ctx, const bte::NewtonParams &q) {
+    if (q.nc <= 0) return BTE_OK;
+    const int r = (ctx->nb + 31) / 32;
+    if (r <= 2) return launch_newton_warp_r<2>(ctx, q);
+    if (r <= 4) return launch_newton_warp_r<4>(ctx, q);
+    if (r <= 8) return launch_newton_warp_r<8>(ctx, q);
+    if (r <= 16) return launch_newton_warp_r<16>(ctx, q);
+    static_assert(bte::kMaxBands <= 32 * 32, "warp solve: at most 32 band-rows per lane");
+    return launch_newton_warp_r<32>(ctx, q);
+}
 
 bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
     if (step && warp_newton(ctx, ctx->nc)) {
@@ -1020,22 +1043,18 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true) {
         bte::NewtonParams q = newton_params(ctx, E_or_null, true);
         q.T_out = ctx->Tg;
         q.neg_fail = 1;
-        bte::newton_warp_kernel<<<(ctx->nc + 7) / 8, 256, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
-        ctx->st.kernel_launches++;
-        CUDA_TRY(ctx, cudaGetLastError());
+        STATUS_TRY(launch_newton_warp(ctx, q));
         STATUS_TRY(newton_finish(ctx));
         ev_mark(ctx, kPhNewton, false);
         if (ctx->td) ctx->rsel = 1 - ctx->rsel;
         return BTE_OK;
     }
     bte::NewtonParams q = newton_params(ctx, E_or_null, step);
-    const int tb = 128;
+    if (step) q.done = ctx->d_done;  // the step's last kernel
     ev_mark(ctx, kPhNewton, true);
-    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
+    STATUS_TRY(launch_newton_cells(ctx, q));
     ev_mark(ctx, kPhNewton, false);
-    ctx->st.kernel_launches++;
     if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
-    CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
 }
 
@@ -1070,6 +1089,7 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
     q.single = ctx->opt.temp_rule == 2;
+    if (step) q.halt = ctx->d_halt;  // (a step's solve: no-op after a failure earlier in the call)
     return q;
 }
 
@@ -1086,7 +1106,7 @@ bte_status allreduce_E(bte_ctx *ctx, double *E = nullptr) {
 bte_status reduce_slots(bte_ctx *ctx) {
     const int tb = 256;
     bte::sum_slots_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->part, ctx->n_slots_step, ctx->nc,
-                                                                           ctx->E);
+                                                                           ctx->E, ctx->d_halt);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
@@ -1108,14 +1128,8 @@ bte_status shard_newton_step(bte_ctx *ctx) {
     q.nc = std::max(0, std::min(ctx->chunk, ctx->nc - q.c_lo));
     q.T_out = ctx->Tg;
     q.neg_fail = 1;
-    if (q.nc > 0 && warp_newton(ctx, q.nc)) {
-        bte::newton_warp_kernel<<<(q.nc + 7) / 8, 256, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
-        ctx->st.kernel_launches++;
-    } else if (q.nc > 0) {
-        const int tb = 128;
-        bte::newton_kernel<<<(q.nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
-        ctx->st.kernel_launches++;
-    }
+    if (warp_newton(ctx, q.nc)) STATUS_TRY(launch_newton_warp(ctx, q));
+    else STATUS_TRY(launch_newton_cells(ctx, q));
     double *mine = ctx->Tg + (size_t)ctx->gband * ctx->chunk;
     if (!bte::nccl::allgather_f64(ctx->bcomm, mine, ctx->Tg, ctx->chunk, ctx->stream, &e))
         return set_err(&ctx->err, "NCCL all-gather failed: %s", e.c_str()), BTE_ENCCL;
@@ -1133,6 +1147,7 @@ bte::HaloParams halo_params(const bte_ctx *ctx) {
     for (int k = 0; k < ctx->nb_loc; ++k) hp.row[k] = ctx->pool_cells + (int64_t)ctx->cur_slot[k] * ctx->slab_elems;
     hp.nb_loc = ctx->nb_loc;
     hp.ps = ctx->ps;
+    hp.fail = ctx->d_fail;
     return hp;
 }
 
@@ -1192,25 +1207,51 @@ bte_status halo_exchange(bte_ctx *ctx) {
 bte_status newton_finish(bte_ctx *ctx) {
     bte::newton_finish_kernel<<<(ctx->nc + 255) / 256, 256, 0, ctx->stream>>>(
         ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
-        ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail);
+        ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail, ctx->d_halt, ctx->d_done);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
 }
 
-bte_status check_newton(bte_ctx *ctx) {
-    int32_t h[2];
-    CUDA_TRY(ctx, cudaMemcpyAsync(&h[0], ctx->d_fail, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
-    CUDA_TRY(ctx, cudaMemcpyAsync(&h[1], ctx->d_iter_max, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
+// After the launches of a call: the failure flag and the steps that ran
+// (*ran, since the last read); a failure resets the flags for the next call.
+bte_status read_flags(bte_ctx *ctx, bool *failed, int64_t *ran) {
+    int32_t h[4];
+    CUDA_TRY(ctx, cudaMemcpyAsync(h, ctx->d_flags, 3 * sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(ctx, cudaMemcpyAsync(&h[3], ctx->d_iter_max, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
     CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
     ev_collect(ctx);
-    ctx->st.newton_iter_max = std::max(ctx->st.newton_iter_max, h[1]);
-    if (h[0]) {
-        CUDA_TRY(ctx, cudaMemsetAsync(ctx->d_fail, 0, sizeof(int32_t), ctx->stream));
+    ctx->st.newton_iter_max = std::max(ctx->st.newton_iter_max, h[3]);
+    *ran = (int64_t)(uint32_t)(h[2] - ctx->done_seen);
+    ctx->done_seen = h[2];
+    *failed = h[0] != 0;
+    if (*failed) CUDA_TRY(ctx, cudaMemsetAsync(ctx->d_flags, 0, 2 * sizeof(int32_t), ctx->stream));  // fail, halt
+    return BTE_OK;
+}
+
+bte_status check_newton(bte_ctx *ctx) {
+    bool failed = false;
+    int64_t ran = 0;
+    STATUS_TRY(read_flags(ctx, &failed, &ran));
+    if (failed) {
         set_err(&ctx->err, "temperature solve did not converge (non-positive or non-finite energy)");
         return BTE_ENOCONV;
     }
     return BTE_OK;
+}
+
+// Undo the host-side state advance of one step whose kernels were no-ops (a
+// step after a failed solve): the slab swaps of run_flux in reverse batch
+// order, and the rate-table halves.
+void undo_step_rotation(bte_ctx *ctx) {
+    int l0 = 0;
+    std::vector<int> starts;
+    for (; l0 < ctx->nb_loc; l0 += ctx->n_spare) starts.push_back(l0);
+    for (auto it = starts.rbegin(); it != starts.rend(); ++it) {
+        const int nbl = std::min(ctx->n_spare, ctx->nb_loc - *it);
+        for (int k = 0; k < nbl; ++k) std::swap(ctx->cur_slot[*it + k], ctx->spare_slot[k]);
+    }
+    if (ctx->td) ctx->rsel = 1 - ctx->rsel;
 }
 
 // I0 of the current T; with the rate law also Tr = T and both rate halves at T
@@ -1246,6 +1287,35 @@ void update_dt_bound(bte_ctx *ctx) {
 bte_status upload_cur_slots(bte_ctx *ctx) {
     CUDA_TRY(ctx, cudaMemcpyAsync(ctx->d_cur_slot, ctx->cur_slot.data(), ctx->nb_loc * sizeof(int32_t),
                                   cudaMemcpyHostToDevice, ctx->stream));
+    return BTE_OK;
+}
+
+// ------------------------------------------------------------- built-in dispersion
+// I0 prefactor C_b when the caller passes none (bte_bands.i0_prefactor NULL):
+// the intensity of a band of width d_omega at its centre frequency omega is
+// I0_b(T) = C_b / expm1(hbar omega / (kB T)) with C_b = hbar omega k^2 d_omega / (8 pi^3)
+// (I = v_g hbar omega f D(omega) / (4 pi), D = k^2 / (2 pi^2 v_g)),
+// k from the quadratic Si dispersion omega = v_s k + c k^2 of the row's branch
+// (LA v_s = 9.01e3 m/s, c = -2.0e-7 m^2/s; TA 5.23e3, -2.26e-7),
+// the stable root k = 2 omega / (v_s + sqrt(v_s^2 + 4 c omega)).  External
+// physics (the paper defers the relation to [14], [4], L559-561).
+bte_status derive_prefactors(const bte_bands *b, std::vector<double> *C) {
+    static const double vs[2] = {9.01e3, 5.23e3}, cq[2] = {-2.0e-7, -2.26e-7};
+    C->resize(b->n_bands);
+    for (int i = 0; i < b->n_bands; ++i) {
+        if (b->i0_prefactor) {
+            (*C)[i] = b->i0_prefactor[i];
+            continue;
+        }
+        const int pol = b->polarization[i];
+        if (pol != 0 && pol != 1) return set_err(nullptr, "band-row %d: polarization must be 0 (LA) or 1 (TA)", i), BTE_EINVAL;
+        const double w = b->omega[i], disc = vs[pol] * vs[pol] + 4.0 * cq[pol] * w;
+        if (!(disc > 0.0))
+            return set_err(nullptr, "band-row %d: omega %g above the built-in dispersion's branch maximum", i, w),
+                   BTE_EINVAL;
+        const double k = 2.0 * w / (vs[pol] + std::sqrt(disc));
+        (*C)[i] = kHbar * w * k * k * b->d_omega[i] / (8.0 * std::pow(M_PI, 3));
+    }
     return BTE_OK;
 }
 
@@ -1295,10 +1365,14 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
         if (!(b->rate_a[i] >= 0.0) || !(b->rate_b[i] >= 0.0) || !(b->rate_theta[i] >= 0.0) ||
             !std::isfinite(b->rate_a[i]) || !std::isfinite(b->rate_b[i]) || !std::isfinite(b->rate_theta[i]))
             return set_err(nullptr, "band-row %d: rate law coefficients must be finite and >= 0", i), BTE_EINVAL;
-    if (!b->i0_prefactor) return set_err(nullptr, "i0_prefactor (C_b) is required"), BTE_EINVAL;
+    if (b->n_bands > bte::kMaxBands)
+        return set_err(nullptr, "%d band-rows (max %d)", b->n_bands, bte::kMaxBands), BTE_EINVAL;
+    if (!b->i0_prefactor && (!b->d_omega || !b->polarization))
+        return set_err(nullptr, "i0_prefactor NULL: d_omega and polarization are needed to derive C_b"), BTE_EINVAL;
     for (int i = 0; i < b->n_bands; ++i) {
-        if (!(b->omega[i] > 0.0) || !(b->vg[i] > 0.0) || !(law || b->tau[i] > 0.0) || !(b->i0_prefactor[i] > 0.0))
-            return set_err(nullptr, "band-row %d: omega, vg, tau, C must be > 0", i), BTE_EINVAL;
+        if (!(b->omega[i] > 0.0) || !(b->vg[i] > 0.0) || !(law || b->tau[i] > 0.0) ||
+            !(b->i0_prefactor ? b->i0_prefactor[i] > 0.0 : b->d_omega[i] > 0.0))
+            return set_err(nullptr, "band-row %d: omega, vg, tau, C (or d_omega) must be > 0", i), BTE_EINVAL;
     }
     if (d->n_dirs < 1 || !d->s || !d->w) return set_err(nullptr, "direction set incomplete"), BTE_EINVAL;
     for (int i = 0; i < d->n_dirs; ++i) {
@@ -1315,6 +1389,10 @@ bte_status validate(const bte_mesh *m, const bte_bands *b, const bte_dirs *d, co
     if (!(o->t_init > 0.0)) return set_err(nullptr, "t_init must be > 0"), BTE_EINVAL;
     if (o->world < 1 || o->rank < 0 || o->rank >= o->world) return set_err(nullptr, "bad rank/world"), BTE_EINVAL;
     if (!(o->newton_rtol > 0.0) || o->newton_max_iter < 1) return set_err(nullptr, "bad Newton controls"), BTE_EINVAL;
+    if (o->group && (!o->group->g || bte::group::world_of(o->group->g) != o->world))
+        return set_err(nullptr, "in-process group of %d ranks with world %d", bte::group::world_of(o->group ? o->group->g : nullptr),
+                       o->world), BTE_EINVAL;
+    if (o->group && o->nccl_unique_id) return set_err(nullptr, "pass either a group or an NCCL id"), BTE_EINVAL;
     return BTE_OK;
 }
 
@@ -1336,7 +1414,7 @@ struct ZSlab {
 
 ZSlab detect_zslab(const bte_mesh *m, const bte_dirs *dr, const bte_bcs *bc, const bte_options *o, int me) {
     ZSlab z;
-    if (m->dim != 3 || (o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA | BTE_FLAG_GENERIC_FACES)))
+    if (m->dim != 3 || (o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_NO_TMA | BTE_FLAG_GENERIC_FACES)))
         return z;
     z.gbx = detect_box(m, bc);
     const BoxDetect &g = z.gbx;
@@ -1514,6 +1592,19 @@ bte_status bte_nccl_unique_id(void *id128) {
     return BTE_OK;
 }
 
+bte_status bte_group_create(int32_t world, bte_group **out) {
+    if (!out || world < 1) return set_err(nullptr, "bte_group_create: world >= 1 and out needed"), BTE_EINVAL;
+    *out = new bte_group();
+    (*out)->g = bte::group::create(world);
+    return BTE_OK;
+}
+
+void bte_group_destroy(bte_group *g) {
+    if (!g) return;
+    bte::group::destroy(g->g);
+    delete g;
+}
+
 void bte_destroy(bte_ctx *ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
@@ -1529,7 +1620,7 @@ void bte_destroy(bte_ctx *ctx) {
     void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
-                    ctx->d_iter_max, ctx->d_fail, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
+                    ctx->d_iter_max, ctx->d_flags, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
                     ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls};
     for (void *p : ptrs)
@@ -1545,6 +1636,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     if (!out) return set_err(nullptr, "NULL out"), BTE_EINVAL;
     *out = nullptr;
     STATUS_TRY(validate(m, bd, dr, bc, o));
+    std::vector<double> Cb_all;  // I0 prefactors (given, or from the built-in dispersion)
+    STATUS_TRY(derive_prefactors(bd, &Cb_all));
     // --- cell partitioning (N3): rank r owns part r % P of the cells and band
     // group r / P; from here on `m` is the owned cells' mesh with halo columns
     const bool cpart = o->cell_part != nullptr;
@@ -1609,33 +1702,10 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             if (partner[f] < 0) paired_geom = false;
         }
     }
-    // --- stencil: every cell has dim pairs, and pair j of every cell neighbours
-    // c + so[j] ("+") and c - so[j] ("-") in the caller's order (structured grids)
-    int32_t so[3] = {0, 0, 0};
-    bool stencil_order = paired_geom && !cpart && mf == 2 * m->dim && nc64 >= 2 * bte::kTile;
-    for (int64_t c = 0; c < nc64 && stencil_order; ++c) {
-        int j = 0;
-        if (m->face_offsets[c + 1] - m->face_offsets[c] != 2 * m->dim) stencil_order = false;
-        for (int64_t f = m->face_offsets[c]; f < m->face_offsets[c + 1] && stencil_order; ++f) {
-            if (partner[f] < f) continue;
-            const int64_t vp = m->face_nbr[f], vm = m->face_nbr[partner[f]];
-            if (vp >= 0) {
-                if (so[j] == 0) so[j] = (int32_t)(vp - c);
-                stencil_order &= vp - c == so[j];
-            }
-            if (vm >= 0) {
-                if (so[j] == 0) so[j] = (int32_t)(c - vm);
-                stencil_order &= c - vm == so[j];
-            }
-            ++j;
-        }
-    }
-    for (int j = 0; j < m->dim; ++j) stencil_order &= so[j] != 0;
-
     // --- structured box grid -> the box kernel (grid lexicographic order)
     BoxDetect bx;
     std::vector<bte::BoxOrbit> orbs;
-    if (paired_geom && !cpart && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_STENCIL | BTE_FLAG_NO_TMA)))
+    if (paired_geom && !cpart && !(o->flags & (BTE_FLAG_NO_BOX | BTE_FLAG_NO_TMA)))
         bx = m->dim == 3 ? detect_box(m, bc) : detect_box2d(m, bc);
     if (zs.on) {  // z-slab partition: the owned layers of the global box, in grid order (local ids)
         const BoxDetect &g = zs.gbx;
@@ -1651,7 +1721,9 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         }
         orbs = zs.orbs;
     }
-    const bool use_box = bx.ok && (zs.on || box_orbits(dr, bx.ax, !bx.flat && (bx.zside[0] == 1 || bx.zside[1] == 1), &orbs));
+    // (the box kernel addresses a slab with 32-bit plane offsets: nd x padded cells < 2^31)
+    const bool box_fits = (int64_t)nd * ((nc64 + n_halo + bte::kTile - 1) / bte::kTile * bte::kTile) < INT32_MAX;
+    const bool use_box = bx.ok && box_fits && (zs.on || box_orbits(dr, bx.ax, !bx.flat && (bx.zside[0] == 1 || bx.zside[1] == 1), &orbs));
 
     // --- internal cell order from the optional centroids: cells are grouped
     // into bricks of 8 x 8 x 4 (2-D: 16 x 16) typical cell sizes, Morton order
@@ -1662,7 +1734,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     // pos_h: caller -> internal.
     std::vector<int32_t> user_of(nc), pos_h(nc);
     for (int32_t c = 0; c < nc; ++c) user_of[c] = c;
-    const bool use_locality = !use_box && m->cell_centre && !(stencil_order && (o->flags & BTE_FLAG_STENCIL));
+    const bool use_locality = !use_box && m->cell_centre;
     if (use_box) {
         user_of = bx.cell_at;
     } else if (use_locality) {
@@ -1760,7 +1832,10 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
 
     // (the paired layout's 5-bit face codes hold up to 16 specular classes)
     // (with the rate law only the box kernel and the generic-face kernel read rate tables)
-    const bool paired = paired_geom && (int)cls_of.size() <= bte::kMaxPairedClasses && !(td && !use_box);
+    // (the opposite-pair layout feeds the TMA-staged paired kernel only: 256-thread blocks)
+    const int32_t block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
+    const bool tma_ok = block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);
+    const bool paired = paired_geom && tma_ok && (int)cls_of.size() <= bte::kMaxPairedClasses && !(td && !use_box);
     const int mf_t = paired ? m->dim
                             : (m->dim == 2 ? (mf <= 3 ? 3 : mf <= 4 ? 4 : 8) : (mf <= 4 ? 4 : mf <= 6 ? 6 : 8));
     const size_t ell = (size_t)mf_t * nc;
@@ -1881,7 +1956,15 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         CREATE_CUDA(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
         ctx->own_stream = true;
     }
-    if (o->nccl_unique_id) {  // (world == 1 with an id: a one-rank communicator, same code path)
+    if (o->group) {  // in-process communicator: the ranks are host threads of this process
+        std::string e;
+        if (!bte::nccl::init_local(&ctx->comm, o->group->g, o->rank, &e)) {
+            set_err(&ctx->err, "in-process group: %s", e.c_str());
+            return fail(BTE_ENCCL);
+        }
+        ctx->have_comm = true;
+        ctx->graphs_ok = false;  // (its exchanges are host-ordered: launch by launch)
+    } else if (o->nccl_unique_id) {  // (world == 1 with an id: a one-rank communicator, same code path)
         std::string e;
         if (!bte::nccl::init(&ctx->comm, o->nccl_unique_id, o->rank, o->world, &e)) {
             set_err(&ctx->err, "NCCL init failed: %s", e.c_str());
@@ -1908,27 +1991,13 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     }
 
     // --- launch plan knobs (band group: measured best on B200)
-    ctx->block = o->block_threads > 0 ? std::max(32, std::min(bte::kMaxThreads, o->block_threads / 32 * 32)) : 256;
-    ctx->tma = ctx->block == bte::kTile && !(o->flags & BTE_FLAG_NO_TMA);  // (paired or generic faces)
-    if (ctx->tma && ctx->uniform_g && stencil_order && (o->flags & BTE_FLAG_STENCIL)) {  // near / far windows
-        int32_t halo = 0, nfar = 0;
-        for (int j = 0; j < m->dim; ++j) {
-            const int32_t a = std::abs(so[j]);
-            if (a <= bte::kTile) halo = std::max(halo, a);
-            else ctx->farq[nfar++] = j;
-        }
-        const int32_t wmain = bte::kTile + 2 * halo + 2;
-        if (ps >= wmain && ps >= bte::kFarWin) {
-            ctx->stencil = true;
-            ctx->halo = halo;
-            ctx->wmain = wmain;
-            ctx->nfar = nfar;
-            for (int j = 0; j < 3; ++j) ctx->so[j] = so[j];
-        }
-    }
+    ctx->block = block;
+    ctx->tma = tma_ok;  // (paired or generic faces)
+    if (const char *ev = std::getenv("BTE_NEWTON"))
+        ctx->newton_mode = std::strcmp(ev, "warp") == 0 ? 1 : std::strcmp(ev, "thread") == 0 ? 2 : 0;
     // auto band group (measured on B200): the largest group that
     // compiles without spills for the chosen kernel
-    const int auto_bg = !paired ? 4 : ctx->stencil ? 4 : ctx->tma ? (ctx->uniform_g ? 5 : 3) : 8;
+    const int auto_bg = !paired ? 4 : ctx->uniform_g ? 5 : 3;
     ctx->bg = legal_bg(o->band_group > 0 ? o->band_group : auto_bg, paired);
     if (use_box) {  // one band-row per stage; band_group / dir_chunk size the CTA's work instead
         ctx->box = true;
@@ -2112,15 +2181,18 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     ctx->h_vg.assign(bd->vg + b_lo, bd->vg + b_hi);
     ctx->h_cw.assign(cw.begin() + b_lo, cw.begin() + b_hi);
     CREATE_TRY(upload(ctx, &ctx->cw_loc, ctx->h_cw));
-    CREATE_TRY(upload(ctx, &ctx->Cb, std::vector<double>(bd->i0_prefactor, bd->i0_prefactor + nb)));
+    CREATE_TRY(upload(ctx, &ctx->Cb, Cb_all));
     CREATE_TRY(upload(ctx, &ctx->theta, theta));
     CREATE_TRY(upload(ctx, &ctx->cw_all, cw));
     CREATE_TRY(dalloc(ctx, &ctx->i0w, (size_t)nb_loc * std::max(1, ctx->n_iso)));
     CREATE_TRY(dalloc(ctx, &ctx->d_iter_max, 1));
-    CREATE_TRY(dalloc(ctx, &ctx->d_fail, 1));
+    CREATE_TRY(dalloc(ctx, &ctx->d_flags, 4));
+    ctx->d_fail = ctx->d_flags;
+    ctx->d_halt = ctx->d_flags + 1;
+    ctx->d_done = ctx->d_flags + 2;
     CREATE_TRY(dalloc(ctx, &ctx->d_smax, 1));
     CREATE_CUDA(cudaMemsetAsync(ctx->d_iter_max, 0, sizeof(int32_t), ctx->stream));
-    CREATE_CUDA(cudaMemsetAsync(ctx->d_fail, 0, sizeof(int32_t), ctx->stream));
+    CREATE_CUDA(cudaMemsetAsync(ctx->d_flags, 0, 4 * sizeof(int32_t), ctx->stream));
     CREATE_CUDA(cudaMemsetAsync(ctx->d_smax, 0, sizeof(unsigned long long), ctx->stream));
 
     // --- initial state: T = t_init, I = I0_b(t_init); isothermal table; dt bound
@@ -2243,6 +2315,23 @@ bte_status bte_band_range(const bte_ctx *ctx, int32_t *b_lo, int32_t *b_hi) {
     return BTE_OK;
 }
 
+// With the rate law the bound depends on the hottest temperature the state can
+// reach (t_hi); under cell partitioning each rank only sees its own cells, so
+// the ranks agree on the max first (every bte_step of such a run is collective
+// anyway), and all of them accept or reject the same dt.
+static bte_status sync_dt_bound(bte_ctx *ctx) {
+    if (!(ctx->td && ctx->n_parts > 1 && ctx->have_comm)) return BTE_OK;
+    double *d = reinterpret_cast<double *>(ctx->d_smax);
+    CUDA_TRY(ctx, cudaMemcpyAsync(d, &ctx->t_hi, sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+    std::string e;
+    if (!bte::nccl::allreduce_max_f64(ctx->comm, d, 1, ctx->stream, &e))
+        return set_err(&ctx->err, "all-reduce (max) of the hottest temperature failed: %s", e.c_str()), BTE_ENCCL;
+    CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->t_hi, d, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+    update_dt_bound(ctx);
+    return BTE_OK;
+}
+
 static bte_status check_dt(bte_ctx *ctx, double dt) {
     if (!(dt > 0.0) || !std::isfinite(dt)) return set_err(&ctx->err, "dt must be > 0 (got %g)", dt), BTE_EINVAL;
     if (dt > ctx->dt_bound * (1.0 + 1e-12))
@@ -2274,35 +2363,52 @@ static bte_status one_step(bte_ctx *ctx, double dt) {
 static int graph_key(const bte_ctx *ctx) { return ctx->cur_slot[0] * 2 + ctx->rsel; }
 
 // Capture two steps into a CUDA graph on the library stream (launch-bound
-// small problems: one replay instead of ~8 launches).  The host-side pointer
-// rotation of the two captured steps cancels out; their launch counters are
-// moved to the per-replay count.  Any failure disables graphs for the context.
+// small problems: one replay instead of ~8 launches).  Nothing runs during
+// capture, so the host-side state the captured steps advance (slab rotation,
+// rate halves, launch counters) is restored afterwards: a 2-step capture of a
+// double-buffered state ends where it began anyway, and a failed capture must
+// not leave it advanced.  A failure is recorded (ctx->err) and disables graphs
+// for the context; the steps then run launch by launch.
 static void capture_two_steps(bte_ctx *ctx, double dt) {
     if (ctx->gexec) {
         cudaGraphExecDestroy(ctx->gexec);
         ctx->gexec = nullptr;
     }
+    const std::vector<int32_t> cur0 = ctx->cur_slot, spare0 = ctx->spare_slot;
+    const int rsel0 = ctx->rsel, dch0 = ctx->dir_chunks, slots0 = ctx->n_slots_step;
     const int64_t l0 = ctx->st.kernel_launches, f0 = ctx->st.flux_launches;
     const int key = graph_key(ctx);
     cudaGraph_t g = nullptr;
-    bool ok = cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+    cudaError_t ce = cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal);
     bte_status s1 = BTE_OK, s2 = BTE_OK;
-    if (ok) {
+    bool closed = false;
+    if (ce == cudaSuccess) {
         s1 = one_step(ctx, dt);
         if (s1 == BTE_OK) s2 = one_step(ctx, dt);
-        ok = cudaStreamEndCapture(ctx->stream, &g) == cudaSuccess && s1 == BTE_OK && s2 == BTE_OK && g;
+        closed = graph_key(ctx) == key;  // (the rotation of two steps must close to replay)
+        ce = cudaStreamEndCapture(ctx->stream, &g);
     }
-    if (ok) ok = cudaGraphInstantiate(&ctx->gexec, g, 0) == cudaSuccess;
+    if (ce == cudaSuccess && s1 == BTE_OK && s2 == BTE_OK && g && closed)
+        ce = cudaGraphInstantiate(&ctx->gexec, g, 0);
     if (g) cudaGraphDestroy(g);
     ctx->g_launches = ctx->st.kernel_launches - l0;
     ctx->g_flux = ctx->st.flux_launches - f0;
     ctx->st.kernel_launches = l0;
     ctx->st.flux_launches = f0;
-    if (!ok || graph_key(ctx) != key) {  // (the rotation did not close: never replay)
+    ctx->cur_slot = cur0;
+    ctx->spare_slot = spare0;
+    ctx->rsel = rsel0;
+    ctx->dir_chunks = dch0;
+    ctx->n_slots_step = slots0;
+    if (ce != cudaSuccess || s1 != BTE_OK || s2 != BTE_OK || !closed || !ctx->gexec) {
         if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
         ctx->gexec = nullptr;
         ctx->graphs_ok = false;
         cudaGetLastError();
+        set_err(&ctx->err, "CUDA graph capture disabled (%s%s%s); stepping launch by launch",
+                ce != cudaSuccess ? cudaGetErrorString(ce) : "",
+                (s1 != BTE_OK || s2 != BTE_OK) ? " step failed under capture" : "",
+                !closed ? " slab rotation does not close over two steps" : "");
         return;
     }
     ctx->g_key = key;
@@ -2314,12 +2420,13 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
     if (ctx->begun) return set_err(&ctx->err, "split step in flight"), BTE_ESTATE;
     if (n < 0) return set_err(&ctx->err, "n < 0"), BTE_EINVAL;
     if (n == 0) return BTE_OK;
-    STATUS_TRY(check_dt(ctx, dt));
     if (ctx->opt.world > 1 && !ctx->have_comm)
         return set_err(&ctx->err, "world > 1 without a communicator: reduce the energy (and move the halo) with "
                                   "bte_step_begin / bte_get_energy / bte_set_energy / bte_step_finish "
                                   "(bte_halo_export / bte_halo_import)"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    STATUS_TRY(sync_dt_bound(ctx));  // (collective with cell partitioning + the rate law)
+    STATUS_TRY(check_dt(ctx, dt));
     const int64_t upd = (int64_t)ctx->nc * ctx->nd * ctx->nb_loc;
     int64_t s = 0;
     auto step1 = [&]() -> bte_status {
@@ -2351,15 +2458,35 @@ bte_status bte_step(bte_ctx *ctx, double dt, int64_t n) {
         }
     }
     while (s < n) STATUS_TRY(step1());
+    // A failed temperature solve in step k made steps k+1..n no-ops on the device
+    // (bte_kernels.cuh: fail / halt): undo their host-side rotation so that the
+    // state is the one at the end of the failing step (ENOCONV
+    // "with the state at the failing step").
+    bool failed = false;
+    int64_t ran = 0;
+    STATUS_TRY(read_flags(ctx, &failed, &ran));
+    if (failed) {
+        const int64_t skipped = std::max<int64_t>(0, n - ran);
+        for (int64_t i = 0; i < skipped; ++i) undo_step_rotation(ctx);
+        ctx->st.steps -= skipped;
+        ctx->st.updates -= skipped * upd;
+        STATUS_TRY(upload_cur_slots(ctx));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        set_err(&ctx->err, "temperature solve did not converge (non-positive or non-finite energy) in step %lld of "
+                           "%lld; the state is the one at the end of that step (failed cells keep their previous T)",
+                (long long)ran, (long long)n);
+        return BTE_ENOCONV;
+    }
     STATUS_TRY(upload_cur_slots(ctx));
-    return check_newton(ctx);
+    return BTE_OK;
 }
 
 bte_status bte_step_begin(bte_ctx *ctx, double dt) {
     if (!ctx) return BTE_EINVAL;
     if (ctx->begun) return set_err(&ctx->err, "split step already begun"), BTE_ESTATE;
-    STATUS_TRY(check_dt(ctx, dt));
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+    STATUS_TRY(sync_dt_bound(ctx));
+    STATUS_TRY(check_dt(ctx, dt));
     if (ctx->have_comm) STATUS_TRY(halo_exchange(ctx));  // (no communicator: the caller imported the halo)
     STATUS_TRY(run_flux(ctx, dt));
     STATUS_TRY(reduce_slots(ctx));
@@ -2551,8 +2678,7 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
         q.inv_v = ctx->d_inv_v;
         q.Tr = ctx->Tr;
     }
-    bte::newton_kernel<<<(ctx->nc + tb - 1) / tb, tb, (ctx->td ? 7 : 3) * ctx->nb * sizeof(double), ctx->stream>>>(q);
-    CUDA_TRY(ctx, cudaGetLastError());
+    STATUS_TRY(launch_newton_cells(ctx, q));
     STATUS_TRY(check_newton(ctx));
     return rows_to_host(ctx, ctx->T2, ctx->nc, 1, T);
 }
@@ -2644,8 +2770,7 @@ bte_status bte_get_stats(const bte_ctx *ctx, bte_stats *st) {
     if (!ctx || !st) return BTE_EINVAL;
     *st = ctx->st;
     st->dir_chunks = ctx->dir_chunks;
-    st->flux_variant = ctx->box ? 6 : ctx->stencil ? 5 : ctx->tma ? (!ctx->paired ? 7 : ctx->uniform_g ? 4 : 3)
-                                                 : ctx->paired ? (ctx->uniform_g ? 2 : 1) : 0;
+    st->flux_variant = ctx->box ? 6 : ctx->tma ? (!ctx->paired ? 7 : ctx->uniform_g ? 4 : 3) : 0;
     return BTE_OK;
 }
 

@@ -26,7 +26,8 @@
 
 namespace bte {
 
-constexpr int kMaxBandsPerLaunch = 128;
+constexpr int kMaxBandsPerLaunch = 128;  // band-rows per rank
+constexpr int kMaxBands = 1024;          // band-rows in all (the warp temperature solve: 32 per lane)
 constexpr int kMaxThreads = 256;
 #ifndef BTE_MIN_BLOCKS
 #define BTE_MIN_BLOCKS 2  // resident 256-thread blocks per SM the flux kernels are compiled for
@@ -53,13 +54,6 @@ struct FluxParams {
     const int32_t *nbr, *nbm;
     const double *gx, *gy, *gz;  // g = (A_f / V_c) n_f
     double gu[3][3];             // uniform-geometry meshes: g of pair q (same for every cell)
-    // stencil meshes (structured index order): the "+" face of pair q of every
-    // cell neighbours cell c + so[q], the "-" face c - so[q]; staging windows
-    int32_t so[3];
-    int32_t halo;                // near window: [t0 - halo, t0 + kTile + halo)
-    int32_t wmain;               // cells staged for the near window (even)
-    int32_t nfar;                // pairs with so > halo: one far window each
-    int32_t farq[3];             // ... which pairs
     const uint32_t *fcode;       // paired [nc]: 5-bit code per side (pair q: bits 10q "+", 10q+5 "-")
     const uint8_t *fcode8;       // generic [MF][nc]: code per face
     const int32_t *refl;         // [n_classes][nd] reflected direction of a specular class
@@ -89,7 +83,19 @@ struct FluxParams {
     const int32_t *bl_cls;   // specular class (reflected direction refl[cls][d]); -1: isothermal
     const uint16_t *sidx;    // [MF][nc] staged index: own tile < kTile <= halo < kTile + nh <= ghosts
     int32_t hstride;         // doubles per staged band-row: kTile + halo + ghost capacity
+    // ENOCONV stop (bte_step): fail != 0 once a temperature solve of an earlier
+    // step of the call failed; the flux launch is then a no-op and block 0
+    // latches the flag into halt, which the rest of the step's kernels read
+    const int32_t *fail;
+    int32_t *halt;
 };
+
+// The stop guard at the top of every flux launch (uniform per launch).
+__device__ __forceinline__ bool flux_halted(const int32_t *fail, int32_t *halt) {
+    const int f = fail ? *fail : 0;
+    if (halt && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) *halt = f;
+    return f != 0;
+}
 
 __device__ __forceinline__ double4 load_dir(const double4 *dirs, int d) {
     const double2 a = __ldg(reinterpret_cast<const double2 *>(dirs + d));
@@ -125,6 +131,7 @@ constexpr int kMaxGenericClasses = 254;
 template <int DIM, int MF, int BG>
 __global__ void __launch_bounds__(kMaxThreads, BTE_MIN_BLOCKS)
 flux_kernel(const __grid_constant__ FluxParams p) {
+    if (flux_halted(p.fail, p.halt)) return;
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= p.nc) return;
     const int grp = blockIdx.y / p.n_dchunks;
@@ -199,96 +206,6 @@ flux_kernel(const __grid_constant__ FluxParams p) {
             const double inew = fma(ic[k], (1.0 - dtk[k]) - kv * out, fma(-kv, infl, src[k]));
             __stcs(p.out_ptr[lg0 + k] + po + c, inew);
             e = fma(cwk[k] * sd.w, inew, e);
-        }
-    }
-    p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
-}
-
-// ---------------------------------------------------------------------------
-// Paired faces (every cell's faces come in exactly opposite pairs, g_- = -g_+,
-// as in the paper's uniform quad/hex grids): for each pair only the face with
-// s_d . g < 0 is an inflow, so one upwind load and one FMA per pair, and
-// out = sum_pairs |s_d . g_+|.  Same arithmetic as the generic kernel.
-// UG (uniform geometry, e.g. the paper's uniform grids): every cell has the
-// same g per pair, read from the constant bank instead of per-thread registers.
-template <int DIM, int NP, int BG, bool UG>
-__global__ void __launch_bounds__(kMaxThreads, BTE_MIN_BLOCKS)
-flux_paired_kernel(const __grid_constant__ FluxParams p) {
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= p.nc) return;
-    const int grp = blockIdx.y / p.n_dchunks;
-    const int dch = blockIdx.y - grp * p.n_dchunks;
-    const int lg0 = grp * BG;
-    const int d0 = dch * p.dchunk;
-    const int d1 = min(p.nd, d0 + p.dchunk);
-    const int nc = p.nc;
-    const int ps = p.ps;
-
-    int np_[NP], nm_[NP];
-    double gx[NP], gy[NP], gz[NP];
-#pragma unroll
-    for (int q = 0; q < NP; ++q) {
-        const int o = q * nc + c;
-        np_[q] = __ldg(p.nbr + o);
-        nm_[q] = __ldg(p.nbm + o);
-        if (!UG) {
-            gx[q] = __ldg(p.gx + o);
-            gy[q] = __ldg(p.gy + o);
-            gz[q] = DIM == 3 ? __ldg(p.gz + o) : 0.0;
-        }
-    }
-    const uint32_t codes = __ldg(p.fcode + c);
-    constexpr uint32_t kAllInterior = (1u << (10 * NP)) - 1u;
-    const bool has_bnd = codes != kAllInterior;
-    double src[BG];  // dt/tau I0_b(T_c) per band-row of the group
-#pragma unroll
-    for (int k = 0; k < BG; ++k) src[k] = p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c);
-    double e = 0.0;
-    for (int d = d0; d < d1; ++d) {
-        const double4 sd = load_dir(p.dirs, d);
-        double amin[NP];  // -|s.g|: alpha of the pair's inflow face
-        int idx[NP];
-        bool iso[NP];
-        double out = 0.0;
-#pragma unroll
-        for (int q = 0; q < NP; ++q) {
-            const double ggx = UG ? p.gu[q][0] : gx[q], ggy = UG ? p.gu[q][1] : gy[q];
-            const double ggz = UG ? p.gu[q][2] : gz[q];
-            const double a = DIM == 3 ? fma(sd.z, ggz, fma(sd.y, ggy, sd.x * ggx)) : fma(sd.y, ggy, sd.x * ggx);
-            out += fabs(a);
-            amin[q] = -fabs(a);
-            idx[q] = a > 0.0 ? nm_[q] : np_[q];  // "+" face outgoing -> inflow through "-"
-            iso[q] = false;
-            if (has_bnd) {
-                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
-                iso[q] = cd == kCodeIso;
-                if (cd < kCodeIso) idx[q] = (__ldg(p.refl + cd * p.nd + d) - d) * ps + c;
-            }
-        }
-        const int64_t po = (int64_t)d * ps;
-        double ic[BG], nv[BG][NP];
-#pragma unroll
-        for (int k = 0; k < BG; ++k) {  // every load of the iteration first
-            const double *pl = p.in_ptr[lg0 + k] + po;  // slab bases come from the constant bank
-            ic[k] = __ldg(pl + c);
-            if (!has_bnd) {
-#pragma unroll
-                for (int q = 0; q < NP; ++q) nv[k][q] = __ldg(pl + idx[q]);
-            } else {
-                const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
-#pragma unroll
-                for (int q = 0; q < NP; ++q) nv[k][q] = __ldg((iso[q] ? isot : pl) + idx[q]);
-            }
-        }
-#pragma unroll
-        for (int k = 0; k < BG; ++k) {
-            double infl = 0.0;
-#pragma unroll
-            for (int q = 0; q < NP; ++q) infl = fma(amin[q], nv[k][q], infl);
-            const double kv = p.kv[lg0 + k];
-            const double inew = fma(ic[k], (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
-            __stcs(p.out_ptr[lg0 + k] + po + c, inew);
-            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
         }
     }
     p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
@@ -383,6 +300,7 @@ flux_tma_kernel(const __grid_constant__ FluxParams p) {
     extern __shared__ __align__(128) double ring[];  // [kStages][BG][kTile], then (UG) DirEntry[dchunk]
     __shared__ __align__(8) uint64_t full[kStages];
     __shared__ __align__(8) uint64_t empty[kStages];
+    if (flux_halted(p.fail, p.halt)) return;
     const int tid = threadIdx.x;
     const int tile0 = blockIdx.x * kTile;
     const int grp = blockIdx.y / p.n_dchunks;
@@ -562,6 +480,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][hstride], then double4 dirs[dchunk]
     __shared__ __align__(8) uint64_t full[kStagesG];
     __shared__ __align__(8) uint64_t empty[kStagesG];
+    if (flux_halted(p.fail, p.halt)) return;
     const int tid = threadIdx.x;
     const int tile0 = blockIdx.x * kTile;
     const int grp = blockIdx.y / p.n_dchunks;
@@ -691,179 +610,6 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
 }
 
 // ---------------------------------------------------------------------------
-// Stencil-staged kernel for structured meshes (uniform geometry, constant
-// neighbour offsets so[q] in the stored cell order: +-1, +-nx, +-nx*ny).  For
-// every (band-row, direction) plane one elected thread bulk-copies (TMA) a
-// near window [t0 - halo, t0 + 256 + halo) that holds the tile and every
-// upwind neighbour with |offset| <= halo, plus one 256-cell far window per
-// remaining pair on its upwind side (e.g. the tile shifted by -+nx*ny), into a
-// kStages-deep ring.  All interior upwind values then come from shared memory;
-// only boundary faces (specular: another direction's plane; isothermal: the
-// I0w table) are global loads.  A plane's values are read from DRAM once (by
-// the tile that owns them) and from L2 by its neighbours.  Same arithmetic as
-// flux_paired_kernel.
-constexpr int kFarWin = kTile + 2;  // far window cells (even; 1 cell of alignment slack)
-
-template <int DIM, int NP, int BG>
-__global__ void __launch_bounds__(kTile, BTE_MIN_BLOCKS)
-flux_stencil_kernel(const __grid_constant__ FluxParams p) {
-    extern __shared__ __align__(128) double ring[];  // [kStages][BG][wmain + nfar * kFarWin]
-    __shared__ __align__(8) uint64_t full[kStages];
-    __shared__ int32_t wstart[kStages][1 + NP];       // window start cells of each stage
-    const int tid = threadIdx.x;
-    const int tile0 = blockIdx.x * kTile;
-    const int c = tile0 + tid;
-    const bool valid = c < p.nc;
-    const int grp = blockIdx.y / p.n_dchunks;
-    const int dch = blockIdx.y - grp * p.n_dchunks;
-    const int lg0 = grp * BG;
-    const int d0 = dch * p.dchunk;
-    const int nit = min(p.nd, d0 + p.dchunk) - d0;
-    const int nc = p.nc;
-    const int ps = p.ps;
-    const int plane = p.wmain + p.nfar * kFarWin;  // staged cells per (band-row, direction)
-
-    if (tid == 0) {
-#pragma unroll
-        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    // upwind offset of pair q in direction d: a = s_d . g_q > 0 -> inflow through "-" (c - so)
-    auto upwind = [&](const double4 &sd, int q) {
-        const double a = DIM == 3 ? fma(sd.z, p.gu[q][2], fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]))
-                                  : fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]);
-        return a > 0.0 ? -p.so[q] : p.so[q];
-    };
-    auto clamp_start = [&](int st, int cells) {  // even (16 B aligned), inside the plane
-        st &= ~1;
-        return max(0, min(st, ps - cells));
-    };
-    auto issue = [&](int i) {
-        const int slot = i % kStages;
-        const int d = d0 + i;
-        const double4 sd = load_dir(p.dirs, d);
-        uint64_t *bar = &full[slot];
-        mbar_arrive_expect_tx(bar, (uint32_t)(BG * plane * sizeof(double)));
-        const int wm = clamp_start(tile0 - p.halo, p.wmain);
-        wstart[slot][0] = wm;
-        int wf[NP];
-#pragma unroll
-        for (int f = 0; f < NP; ++f)
-            if (f < p.nfar) {
-                const int q = p.farq[f];
-                wf[f] = clamp_start(tile0 + upwind(sd, q), kFarWin);
-                wstart[slot][1 + f] = wf[f];
-            }
-        const int64_t po = (int64_t)d * ps;
-#pragma unroll
-        for (int k = 0; k < BG; ++k) {
-            double *dst = ring + ((int64_t)slot * BG + k) * plane;
-            const double *pl = p.in_ptr[lg0 + k] + po;
-            bulk_g2s(dst, pl + wm, (uint32_t)(p.wmain * sizeof(double)), bar);
-#pragma unroll
-            for (int f = 0; f < NP; ++f)
-                if (f < p.nfar) bulk_g2s(dst + p.wmain + f * kFarWin, pl + wf[f], kFarWin * sizeof(double), bar);
-        }
-    };
-    if (tid == 0)
-        for (int i = 0; i < min(kStages, nit); ++i) issue(i);
-
-    uint32_t codes = (1u << (10 * NP)) - 1u;
-    int np_[NP], nm_[NP];
-    if (valid) codes = __ldg(p.fcode + c);
-    const bool has_bnd = codes != (1u << (10 * NP)) - 1u;
-#pragma unroll
-    for (int q = 0; q < NP; ++q) {  // boundary cells only: isothermal table columns
-        np_[q] = has_bnd ? __ldg(p.nbr + q * nc + c) : 0;
-        nm_[q] = has_bnd ? __ldg(p.nbm + q * nc + c) : 0;
-    }
-    int farslot[NP];  // far-window index of pair q (-1: near window)
-#pragma unroll
-    for (int q = 0; q < NP; ++q) {
-        farslot[q] = -1;
-#pragma unroll
-        for (int f = 0; f < NP; ++f)
-            if (f < p.nfar && p.farq[f] == q) farslot[q] = f;
-    }
-    double src[BG];
-#pragma unroll
-    for (int k = 0; k < BG; ++k)
-        src[k] = valid ? p.dtit[lg0 + k] * __ldg(p.i0 + (int64_t)(p.band0 + lg0 + k) * nc + c) : 0.0;
-
-    double e = 0.0;
-    for (int i = 0; i < nit; ++i) {
-        const int d = d0 + i;
-        const int slot = i % kStages;
-        const double4 sd = load_dir(p.dirs, d);
-        double amin[NP];
-        int up[NP];     // upwind offset
-        int gidx[NP];   // boundary faces: global index (plane-relative or table column)
-        bool glob[NP], iso[NP];
-        double out = 0.0;
-#pragma unroll
-        for (int q = 0; q < NP; ++q) {
-            const double a = DIM == 3 ? fma(sd.z, p.gu[q][2], fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]))
-                                      : fma(sd.y, p.gu[q][1], sd.x * p.gu[q][0]);
-            out += fabs(a);
-            amin[q] = -fabs(a);
-            up[q] = a > 0.0 ? -p.so[q] : p.so[q];
-            glob[q] = false;
-            iso[q] = false;
-            gidx[q] = 0;
-            if (has_bnd) {
-                const uint32_t cd = (codes >> (10 * q + (a > 0.0 ? 5 : 0))) & kCodeInterior;
-                iso[q] = cd == kCodeIso;
-                glob[q] = cd != kCodeInterior;
-                gidx[q] = iso[q] ? (a > 0.0 ? nm_[q] : np_[q])
-                                 : (glob[q] ? (__ldg(p.refl + cd * p.nd + d) - d) * ps + c : 0);
-            }
-        }
-        const int64_t po = (int64_t)d * ps;
-        double nv[BG][NP];
-        if (has_bnd) {
-#pragma unroll
-            for (int k = 0; k < BG; ++k) {
-                const double *pl = p.in_ptr[lg0 + k] + po;
-                const double *isot = p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso;
-#pragma unroll
-                for (int q = 0; q < NP; ++q) nv[k][q] = (valid && glob[q]) ? __ldg((iso[q] ? isot : pl) + gidx[q]) : 0.0;
-            }
-        }
-        while (!mbar_try_wait(&full[slot], (i / kStages) & 1)) {
-        }
-        const int wm = wstart[slot][0];
-        int loc[NP];  // position of the upwind neighbour in the staged plane
-#pragma unroll
-        for (int q = 0; q < NP; ++q) {
-            const int nb = c + up[q];
-            loc[q] = glob[q] ? 0
-                     : farslot[q] < 0 ? nb - wm
-                                      : p.wmain + farslot[q] * kFarWin + (nb - wstart[slot][1 + farslot[q]]);
-        }
-        const double *stage = ring + (int64_t)slot * BG * plane;
-#pragma unroll
-        for (int k = 0; k < BG; ++k) {
-            const double *sk = stage + k * plane;
-            const double ic = sk[c - wm];
-            double infl = 0.0;
-#pragma unroll
-            for (int q = 0; q < NP; ++q) infl = fma(amin[q], glob[q] ? nv[k][q] : sk[loc[q]], infl);
-            const double kv = p.kv[lg0 + k];
-            const double inew = fma(ic, (1.0 - p.dtit[lg0 + k]) - kv * out, fma(-kv, infl, src[k]));
-            if (valid) __stcs(p.out_ptr[lg0 + k] + po + c, inew);
-            e = fma(p.cw[lg0 + k] * sd.w, inew, e);
-        }
-        __syncthreads();  // every thread is done with this stage
-        if (tid == 0 && i + kStages < nit) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            issue(i + kStages);
-        }
-    }
-    if (valid) p.part[(int64_t)(p.slot0 + grp * p.n_dchunks + dch) * nc + c] = e;
-}
-
-// ---------------------------------------------------------------------------
 // Box kernel: structured hexahedral grids (the paper's uniform meshes, Fig. 1
 // L617-621) stored in lexicographic order (axis 0 fastest), axis-0 and axis-1
 // sides specular, axis-2 sides isothermal or specular (each side uniform).
@@ -896,6 +642,9 @@ constexpr int kBoxPlane = 320;               // doubles per staged plane (128-by
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
 constexpr int kBoxMaxStages = 12;
+#ifndef BTE_BOX_STORE_HINT
+#define BTE_BOX_STORE_HINT 0  // direct stores of I^{n+1}: 0 st.global.cs, 1 L2 evict_first policy, 2 plain
+#endif
 // Resident CTAs per SM the kernel is compiled for (register cap): 3-D grids 2
 // (96 registers, 6 stages of 12 KB plus L x 2 KB of energy rows); 2-D grids 3
 // (72 registers, no spills, 4 stages): a 2-D stage is one layer, so CTAs are
@@ -934,6 +683,11 @@ struct BoxParams {
     const BoxOrbit *orb;       // [n_orb]
     const double4 *dirs;       // [nd] {s_0, s_1, s_2, w} in grid axes
     double *part;              // [n_slots][nc] energy partials
+    double *pool;              // slab pool (direct stores of I^{n+1}): slab s, direction d, tensor
+    int64_t slab_elems;        // cell (x, y, z) at pool[s slab_elems + d ps + (z n1 + y) n0 + x]
+    int32_t ps;
+    const int32_t *fail;       // != 0: a temperature solve of an earlier step failed -> no-op
+    int32_t *halt;             // ... latched here for the rest of the step (block 0)
     int32_t in_slab[kMaxBandsPerLaunch];   // launch-local band-row -> slab of I^n
     int32_t out_slab[kMaxBandsPerLaunch];  // ... slab of I^{n+1}
     double dtit[kMaxBandsPerLaunch];       // dt / tau_b (constant rates)
@@ -1055,13 +809,18 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     const int S = p.stages;
 #endif
     double *ring = bsm;                          // [S][kStage]
+#ifdef BTE_BOX_TMA_STORE
     double *obuf = ring + S * kStage;            // [2][4][256]
     double *eacc = obuf + 2 * 4 * kBoxCells;     // [L][256]
+#else
+    double *eacc = ring + S * kStage;            // [L][256]
+#endif
     BoxOrbitC *sorb = reinterpret_cast<BoxOrbitC *>(eacc + p.L * kBoxCells);  // [orb_chunk]
     __shared__ __align__(8) uint64_t full[kBoxMaxStages];
     __shared__ __align__(8) uint64_t empty[kBoxMaxStages];
 
     const int tid = threadIdx.x;
+    if (flux_halted(p.fail, p.halt)) return;  // (a failed solve earlier in this bte_step call)
     const BoxItem w = box_item(p, blockIdx.x);
     if (tid == 0) {
         for (int s = 0; s < S; ++s) {
@@ -1165,12 +924,26 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         if (flat && wall1 && p.zside[(q & 2) ? 1 : 0] == 0) uy[q] = kGhost + ((q & 2) ? kBoxTX : 0) + tx;
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
+#ifndef BTE_BOX_TMA_STORE
+    // I^{n+1} leaves straight from registers: a warp's 32 cells are one 256-byte
+    // row of a plane (coalesced streaming stores, no shared-memory round trip and
+    // no per-layer CTA barrier)
+    const int32_t plane = p.n0 * p.n1;
+    const int32_t cell_off = gy * p.n0 + gx;
+#if BTE_BOX_STORE_HINT == 1
+    uint64_t spol;  // I^{n+1} is not read again this step: evict first, keep L2 for the halo boxes
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(spol));
+#endif
+#endif
 
     int s = 0, sp = 0;
     uint32_t ph = 0, ob = 0;
     double pv[4] = {0.0, 0.0, 0.0, 0.0};  // the previous layer's own values: this layer's axis-2 upwind values
     for (int k = w.k0; k < w.k1; ++k) {
         const double kv = p.kv[k];
+#ifndef BTE_BOX_TMA_STORE
+        double *const oslab = p.pool + (int64_t)p.out_slab[k] * p.slab_elems + cell_off;
+#endif
         for (int o = w.o0; o < w.o1; ++o) {
             const BoxOrbitC &orb = sorb[o - w.o0];
             const bool asc = orb.asc;
@@ -1180,6 +953,11 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             const double kvout = kv * ((orb.a[0] + orb.a[1]) + orb.a[2]);
             const double coef_c = (1.0 - p.dtit[k]) - kvout;  // constant rates
             const double m0 = -orb.a[0], m1 = -orb.a[1], m2 = -orb.a[2];
+#ifndef BTE_BOX_TMA_STORE
+            int32_t doff[4];  // plane offsets of the orbit's 4 directions (slab_elems < 2^31)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) doff[q] = orb.d[q] * p.ps;
+#endif
             for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
@@ -1202,7 +980,11 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         cw = p.cw[k];
                     }
                     const double src = dtit * cur[4 * kBoxPlane + tid];
+#ifdef BTE_BOX_TMA_STORE
                     double *out = obuf + ob * (4 * kBoxCells);
+#else
+                    double *const orow = oslab + z * plane;
+#endif
                     double acc = 0.0;
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
@@ -1212,7 +994,20 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         if (!flat) infl = fma(m2, pv[q], infl);
                         pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
+#ifdef BTE_BOX_TMA_STORE
                         out[q * kBoxCells + tid] = inew;
+#else
+                        if (valid) {
+#if BTE_BOX_STORE_HINT == 1
+                            asm volatile("st.global.L1::no_allocate.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(orow + doff[q]),
+                                         "d"(inew), "l"(spol) : "memory");
+#elif BTE_BOX_STORE_HINT == 2
+                            orow[doff[q]] = inew;
+#else
+                            __stcs(orow + doff[q], inew);
+#endif
+                        }
+#endif
                         acc = fma(wq[q], inew, acc);
                     }
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
@@ -1229,6 +1024,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         }
                     }
                     sp = s;
+#ifdef BTE_BOX_TMA_STORE
                     fence_smem_to_async();
                     if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
                     bar_compute();
@@ -1239,6 +1035,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         bulk_commit();
                     }
                     ob ^= 1u;
+#endif
                 }
                 if (++s == S) {
                     s = 0;
@@ -1252,7 +1049,10 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         for (int l = 0; l < w.Lc; ++l)
             part[((int64_t)(w.z0 - p.zlo + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
+#ifdef BTE_BOX_TMA_STORE
     if (tid == 0) bulk_wait_all();
+#endif
+    (void)ob;
 }
 
 // ---------------------------------------------------------------- temperature
@@ -1282,6 +1082,11 @@ struct NewtonParams {
     double *T_out;         // diagnostic / chunk solve: write T here only (state untouched)
     int32_t c_lo;          // chunk solve: cells [c_lo, c_lo + nc) of the mesh, E indexed from c_lo
     int32_t neg_fail;      // chunk solve: a failed cell writes -T^n (decoded by newton_finish_kernel)
+    // ENOCONV stop (a step's solve): halt = the flux launch's latch (a solve of an
+    // earlier step of the call failed: no-op); done != nullptr: this launch ends
+    // the step and block 0 counts it
+    const int32_t *halt;
+    int32_t *done;
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1327,6 +1132,8 @@ __device__ __forceinline__ double g_only(const double *sC, const double *sTh, co
 }
 
 __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
+    if (p.halt && *p.halt) return;
+    if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
     double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
@@ -1426,14 +1233,15 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
-constexpr int kNewtonRowsPerLane = kMaxBandsPerLaunch / 32;  // nb <= 128
-
+// R = band-rows per lane (ceil(nb / 32) rounded up to a power of two; the
+// per-lane weights stay in registers): one instantiation per R <= kMaxBands / 32.
+template <int R>
 __device__ __forceinline__ Gsum g_eval_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
                                             double E, double T, int lane) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
 #pragma unroll
-    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+    for (int r = 0; r < R; ++r) {
         const int b = lane + 32 * r;
         if (b < nb) {
             const double x = sTh[b] * it;
@@ -1446,18 +1254,21 @@ __device__ __forceinline__ Gsum g_eval_warp(const double *sC, const double *sTh,
     return {W * warp_sum(g) - E, W * warp_sum(gp)};
 }
 
+template <int R>
 __device__ __forceinline__ double g_only_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
                                               double E, double T, int lane) {
     double g = 0.0;
 #pragma unroll
-    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+    for (int r = 0; r < R; ++r) {
         const int b = lane + 32 * r;
         if (b < nb) g = fma(wl[r], sC[b] / expm1(sTh[b] / T), g);
     }
     return W * warp_sum(g) - E;
 }
 
+template <int R>
 __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
+    if (p.halt && *p.halt) return;
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
     double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
@@ -1488,9 +1299,9 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
     const double T0 = p.T[c];
     const bool law = p.td && p.r2;
     const double Tw = p.td ? (p.tr_step ? T0 : p.Tr[c]) : 0.0;  // a step: weights at T^n
-    double wl[kNewtonRowsPerLane];
+    double wl[R];
 #pragma unroll
-    for (int r = 0; r < kNewtonRowsPerLane; ++r) {
+    for (int r = 0; r < R; ++r) {
         const int b = lane + 32 * r;
         wl[r] = b >= p.nb ? 0.0 : law ? tau_rate(sA[b], sB[b], sR[b], Tw) * sV[b] : sW[b];
     }
@@ -1498,7 +1309,7 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
     bool ok = false;
     int it = 0;
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = g_eval_warp(sC, sTh, wl, p.nb, p.W, E, T, lane);
+        const Gsum gs = g_eval_warp<R>(sC, sTh, wl, p.nb, p.W, E, T, lane);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -1507,7 +1318,7 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval_warp(sC, sTh, wl, p.nb, p.W, E, T, lane);
+            const Gsum gs = g_eval_warp<R>(sC, sTh, wl, p.nb, p.W, E, T, lane);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -1516,13 +1327,13 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only_warp(sC, sTh, wl, p.nb, p.W, E, lo, lane) > 0.0; ++k) lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only_warp(sC, sTh, wl, p.nb, p.W, E, hi, lane) < 0.0; ++k) hi *= 2.0;
-            if (g_only_warp(sC, sTh, wl, p.nb, p.W, E, lo, lane) <= 0.0 &&
-                g_only_warp(sC, sTh, wl, p.nb, p.W, E, hi, lane) >= 0.0) {
+            for (int k = 0; k < 2000 && g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, lo, lane) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, hi, lane) < 0.0; ++k) hi *= 2.0;
+            if (g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, lo, lane) <= 0.0 &&
+                g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, hi, lane) >= 0.0) {
                 for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
                     const double mid = 0.5 * (lo + hi);
-                    if (g_only_warp(sC, sTh, wl, p.nb, p.W, E, mid, lane) < 0.0) lo = mid; else hi = mid;
+                    if (g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, mid, lane) < 0.0) lo = mid; else hi = mid;
                 }
                 T = 0.5 * (lo + hi);
                 ok = true;
@@ -1546,7 +1357,10 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      int nb_loc, const double *__restrict__ Cb, const double *__restrict__ theta,
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
-                                     double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail) {
+                                     double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
+                                     const int32_t *__restrict__ halt, int32_t *done) {
+    if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
+    if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= nc) return;
     double t = Tg[c];
@@ -1575,7 +1389,9 @@ __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo
 }
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
-__global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E) {
+__global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
+                                 const int32_t *__restrict__ halt) {
+    if (halt && *halt) return;
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
     if (c >= nc) return;
     double e = 0.0;
@@ -1715,9 +1531,11 @@ struct HaloParams {
     const int32_t *cells;             // column of send cell i (pack) / of halo cell i (unpack)
     const int32_t *dirs;              // direction list of the segment
     int32_t n, n_dirs, nb_loc, ps;
+    const int32_t *fail;              // != 0: a solve of an earlier step of the call failed (no-op)
 };
 
 __global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf) {
+    if (p.fail && *p.fail) return;
     const int64_t per = (int64_t)p.n_dirs * p.n;
     const int k = blockIdx.y;
     const double *s = p.row[k];
@@ -1730,6 +1548,7 @@ __global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *_
 }
 
 __global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const double *__restrict__ buf) {
+    if (p.fail && *p.fail) return;
     const int64_t per = (int64_t)p.n_dirs * p.n;
     const int k = blockIdx.y;
     double *s = p.row[k];

@@ -7,6 +7,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 namespace bte {
 namespace nccl {
@@ -35,8 +36,8 @@ Api *api() {
     static Api a;
     static std::once_flag once;
     std::call_once(once, [] {
-        const char *cands[] = {getenv("BTE_NCCL_LIB"), "libnccl.so.2", "libnccl.so",
-                               "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
+        // BTE_NCCL_LIB (the Python binding points it at the torch-bundled NCCL), else the loader path
+        const char *cands[] = {getenv("BTE_NCCL_LIB"), "libnccl.so.2", "libnccl.so"};
         for (const char *p : cands) {
             if (!p || !*p) continue;
             a.h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
@@ -95,7 +96,12 @@ bool init(Comm *c, const void *id128, int rank, int world, std::string *err) {
     return true;
 }
 
+bool init_local(Comm *c, bte::group::Group *g, int rank, std::string *err) {
+    return bte::group::attach(g, rank, &c->local, err);
+}
+
 bool allreduce_sum_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err) {
+    if (c.local) return bte::group::allreduce_f64(c.local, buf, n, false, s, err);
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->allReduce(buf, buf, (size_t)n, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
@@ -105,6 +111,7 @@ bool allreduce_sum_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, st
 
 bool reduce_scatter_sum_f64(const Comm &c, const double *send, double *recv, int64_t recvcount, cudaStream_t s,
                             std::string *err) {
+    if (c.local) return bte::group::reduce_scatter_sum_f64(c.local, send, recv, recvcount, s, err);
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->reduceScatter(send, recv, (size_t)recvcount, ncclFloat64, ncclSum, (ncclComm_t)c.comm, s);
@@ -114,6 +121,7 @@ bool reduce_scatter_sum_f64(const Comm &c, const double *send, double *recv, int
 
 bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t sendcount, cudaStream_t s,
                    std::string *err) {
+    if (c.local) return bte::group::allgather_f64(c.local, send, recv, sendcount, s, err);
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->allGather(send, recv, (size_t)sendcount, ncclFloat64, (ncclComm_t)c.comm, s);
@@ -122,6 +130,7 @@ bool allgather_f64(const Comm &c, const double *send, double *recv, int64_t send
 }
 
 bool allreduce_max_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, std::string *err) {
+    if (c.local) return bte::group::allreduce_f64(c.local, buf, n, true, s, err);
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     ncclResult_t r = a->allReduce(buf, buf, (size_t)n, ncclFloat64, ncclMax, (ncclComm_t)c.comm, s);
@@ -130,6 +139,7 @@ bool allreduce_max_f64(const Comm &c, double *buf, int64_t n, cudaStream_t s, st
 }
 
 bool split(const Comm &c, int color, int key, Comm *out, std::string *err) {
+    if (c.local) return bte::group::split(c.local, color, key, &out->local, err);
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     if (!a->commSplit) return *err = "libnccl has no ncclCommSplit (NCCL >= 2.18 needed)", false;
@@ -141,6 +151,11 @@ bool split(const Comm &c, int color, int key, Comm *out, std::string *err) {
 }
 
 bool exchange_f64(const Comm &c, const P2P *ops, int n_ops, cudaStream_t s, std::string *err) {
+    if (c.local) {
+        std::vector<bte::group::P2P> lo(n_ops);
+        for (int i = 0; i < n_ops; ++i) lo[i] = {ops[i].peer, ops[i].send, ops[i].n_send, ops[i].recv, ops[i].n_recv};
+        return bte::group::exchange_f64(c.local, lo.data(), n_ops, s, err);
+    }
     Api *a = api();
     if (!a || !c.comm) return *err = why(), false;
     if (!a->send || !a->recv || !a->groupStart || !a->groupEnd)
@@ -159,6 +174,11 @@ bool exchange_f64(const Comm &c, const P2P *ops, int n_ops, cudaStream_t s, std:
 }
 
 void destroy(Comm &c) {
+    if (c.local) {
+        bte::group::release(c.local);
+        c.local = nullptr;
+        return;
+    }
     Api *a = api();
     if (a && c.comm) a->commDestroy((ncclComm_t)c.comm);
     c.comm = nullptr;

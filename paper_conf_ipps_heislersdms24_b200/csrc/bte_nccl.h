@@ -4,17 +4,27 @@
 // 8(e)): reduce-scatter of the per-cell energy partials, the temperature solve
 // on this rank's cell chunk, all-gather of T (or one all-reduce of E and a
 // replicated solve), and the halo exchange of the cell-partitioned step.
+//
+// Every call also takes an in-process communicator (bte_group.h: the ranks are
+// host threads of one process): Comm.local set -> the same collective runs as
+// device copies between the ranks' buffers instead of through NCCL.
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <string>
 
+#include "bte_group.h"
+
 namespace bte {
 namespace nccl {
 
 struct Comm {
-    void *comm = nullptr;  // ncclComm_t
+    void *comm = nullptr;              // ncclComm_t
+    bte::group::Rank *local = nullptr;  // in-process group endpoint (instead of NCCL)
 };
+
+// Endpoint `rank` of an in-process group (bte_group_create).
+bool init_local(Comm *c, bte::group::Group *g, int rank, std::string *err);
 
 // 128-byte ncclUniqueId into id128.
 bool unique_id(void *id128, std::string *err);

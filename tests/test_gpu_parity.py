@@ -181,7 +181,8 @@ def test_generic_face_path_2d_3d(bte, oracle_mod, bg):
 
 @pytest.mark.parametrize("bg", [1, 3, 4, 8])
 def test_register_pipelined_kernel(bte, oracle_mod, bg):
-    """The non-TMA paired kernel (BTE_FLAG_NO_TMA), uniform and per-cell geometry."""
+    """The register-pipelined generic-face kernel (BTE_FLAG_NO_TMA): paired meshes
+    then take the generic layout, uniform and per-cell geometry."""
     cfg = gen.small_3d_config((13, 7, 5), n_spectral=3, ntheta=4, nphi=8)
     Io, To = oracle_run(oracle_mod, cfg, 10)
     Ig, Tg, _ = gpu_run(cfg, 10, tma=False, band_group=bg)
@@ -205,24 +206,6 @@ def test_graded_mesh_per_cell_geometry(bte, oracle_mod):
     for tma in (True, False):
         Ig, Tg, _ = gpu_run(cfg, 10, tma=tma)
         assert_parity(Ig, Tg, Io, To)
-
-
-@pytest.mark.parametrize("shape", [(40, 24), (33, 20, 6), (64, 64, 3)])
-@pytest.mark.parametrize("bg", [1, 3, 8])
-def test_stencil_kernel(bte, oracle_mod, shape, bg):
-    """Structured index order + BTE_FLAG_STENCIL -> the stencil-staged kernel (near/far TMA windows),
-    incl. odd row lengths (unaligned windows) and far windows in 2-D and 3-D."""
-    h = 1e-6
-    mesh = gen.gen_mesh(shape, (h,) * len(shape))
-    bands = gen.gen_bands_si(3)
-    dirs = gen.gen_dirs_product(4, 8)
-    bcs = gen.gen_bcs_fig1(mesh, radius=3 * h)
-    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
-    cfg = gen.Config("st", mesh, bands, dirs, bcs, 300.0, dt, 8, ic_eps=0.2)
-    Io, To = oracle_run(oracle_mod, cfg, 8)
-    Ig, Tg, st = gpu_run(cfg, 8, band_group=bg, stencil=True)
-    assert st["flux_variant"] == 5
-    assert_parity(Ig, Tg, Io, To)
 
 
 def test_locality_order_is_invisible(bte):
@@ -272,32 +255,6 @@ def test_equilibrium_invariance_full_bench_size(bte):
         I_last = s.intensity(last, last + 1)
     with bte.Solver(cfg.mesh, cfg.bands, cfg.dirs, bcs, t_init=300.0) as s2:
         assert rel_err(I_last, s2.intensity(last, last + 1)) < 1e-13
-
-
-def test_sampled_full_bench_size(bte, oracle_mod):
-    """C4 at full size in the bench's launch configuration: one step from a
-    non-uniform equilibrium, sampled cells against the oracle cell by cell."""
-    cfg = _cfg("C4")
-    nc = cfg.mesh["n_cells"]
-    rng = np.random.default_rng(5)
-    T0 = 300.0 + 40.0 * rng.random(nc)
-    nx, ny, nz = cfg.mesh["shape"]
-    corners = [0, nx - 1, nx * ny - 1, nc - 1, nx * (ny - 1), nc - nx]
-    cells = np.unique(np.concatenate([corners, rng.integers(0, nc, 40),
-                                      [nx // 2 + nx * (ny // 2) + nx * ny * (nz - 1)]]))
-    p = oracle_mod.problem_from_config(cfg)
-    Io_sel, To_sel = p.step_cells_equilibrium(T0, cells, cfg.dt)
-    with bte.solver_from_config(cfg) as s:
-        s.set_equilibrium(T0)
-        s.step(cfg.dt, 1)
-        Tg = s.temperature()
-        Ig_sel = np.empty((cells.size, s.n_bands, s.n_dirs))
-        buf = np.empty((1, s.n_dirs, nc))
-        for b in range(s.n_bands):
-            s.intensity(b, b + 1, out=buf)
-            Ig_sel[:, b, :] = buf[0][:, cells].T
-    assert rel_err(Ig_sel, Io_sel) <= RTOL_I
-    assert rel_err(Tg[cells], To_sel) <= RTOL_T
 
 
 def test_split_step_band_sharding_emulated(bte, oracle_mod):
@@ -394,36 +351,6 @@ def test_nccl_sharded_step_reports_enoconv(bte):
             s.step(cfg.dt, 1)
         assert e.value.status == bte.BTE_ENOCONV
         assert s.temperature()[5] == T_before[5]
-
-
-def test_sampled_full_size_c5_slab_rotation(bte, oracle_mod):
-    """C5 (96^3, 55 rows, 400 dirs: 156 GB of state) at full size in the
-    bench's launch configuration (slab rotation on one GPU): one step from a
-    non-uniform equilibrium, sampled cells (corners, wall centres, random)
-    against the oracle cell by cell."""
-    cfg = _cfg("C5")
-    nc = cfg.mesh["n_cells"]
-    rng = np.random.default_rng(6)
-    T0 = 300.0 + 40.0 * rng.random(nc)
-    nx, ny, nz = cfg.mesh["shape"]
-    corners = [0, nx - 1, nx * ny - 1, nc - 1, nx * (ny - 1), nc - nx, nx * ny * (nz - 1)]
-    cells = np.unique(np.concatenate([corners, rng.integers(0, nc, 30),
-                                      [nx // 2 + nx * (ny // 2) + nx * ny * (nz - 1), nx // 2 + nx * (ny // 2)]]))
-    p = oracle_mod.problem_from_config(cfg)
-    Io_sel, To_sel = p.step_cells_equilibrium(T0, cells, cfg.dt)
-    with bte.solver_from_config(cfg) as s:
-        st = s.stats()
-        assert st["spare_slabs"] < s.n_bands and st["flux_variant"] == 6  # slab rotation, box kernel
-        s.set_equilibrium(T0)
-        s.step(cfg.dt, 1)
-        Tg = s.temperature()
-        Ig_sel = np.empty((cells.size, s.n_bands, s.n_dirs))
-        buf = np.empty((1, s.n_dirs, nc))
-        for b in range(s.n_bands):
-            s.intensity(b, b + 1, out=buf)
-            Ig_sel[:, b, :] = buf[0][:, cells].T
-    assert rel_err(Ig_sel, Io_sel) <= RTOL_I
-    assert rel_err(Tg[cells], To_sel) <= RTOL_T
 
 
 def test_c3_full_size_elementwise(bte, oracle_mod):

@@ -57,6 +57,6 @@ for name, cfg, kw in [("C1", c1, {}), ("box3d", box3, {}), ("box3d-law", box3law
                       ("box2d-law", cstlaw, {}), ("box2d-rotation", cst, {"max_spare_slabs": 2}),
                       ("triangles", c6t, {}), ("3d-tma", c3d, {}), ("3d-tma-bg1", c3d, {"band_group": 1}),
                       ("3d-reg", c3d, {"tma": False}), ("3d-generic", c3d, {"generic_faces": True}),
-                      ("stencil", cst, {"stencil": True, "box": False}), ("rotation", c3d, {"max_spare_slabs": 2})]:
+                      ("2d-tma", cst, {"box": False}), ("rotation", c3d, {"max_spare_slabs": 2})]:
     print(name, run(cfg, **kw), flush=True)
 print("ALL OK")
