@@ -51,18 +51,21 @@ def _peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def _traffic_from_profiles(config):
-    """Per-launch DRAM bytes of the interior flux kernel from the committed
-    `ncu --set full` summary, if one exists for this workload."""
+def _traffic_from_profiles(config, launches_per_step):
+    """DRAM bytes (read + write) of the dominant flux kernel per step, like
+    `achieved`: the committed `ncu --set full` capture of one launch of this
+    workload (profiles/ncu_flux_summary.json, one entry per config) times the
+    launches of a step.  None if no capture exists for the workload."""
     path = os.path.join(ROOT, "profiles", "ncu_flux_summary.json")
     try:
         with open(path) as f:
             d = json.load(f)
-        if d.get("config") == config:  # per step, like `achieved` (see tools/ncu_summary.py)
-            return d.get("dram_bytes_per_step")
+        e = d.get(config)
+        if e and e.get("dram_bytes_per_launch"):
+            return float(e["dram_bytes_per_launch"]) * launches_per_step, e.get("source")
     except Exception:
         pass
-    return None
+    return None, None
 
 
 class ClockSampler:
@@ -142,37 +145,82 @@ def _dist():
     return rank, world, local
 
 
-def cpu_baseline(cfg, budget_s=15.0, max_rows=None):
-    """The oracle as it stands, on this host's cores, on a bounded sample of the
-    workload (about budget_s of CPU work): the full mesh and direction set, the
-    first k band-rows, and with all rows in the sample as many steps as fit."""
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.lower().startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def _oracle_sample(cfg, rows):
+    """The oracle's problem on a bounded sample of the workload -- the full
+    mesh and direction set, the first `rows` band-rows -- in the state the GPU
+    arm starts from: the seeded IC (equilibrium at t_init x the generator's
+    multiplier), T from the sample's energy (oracle Newton).  Untimed."""
     import numpy as np
     import oracle
     from paper_conf_ipps_heislersdms24_b200 import inputs as gen
+    bands = gen.select_bands(cfg.bands, np.arange(rows))
+    p = oracle.Problem(cfg.mesh, bands, cfg.dirs, cfg.bcs, temp_rule=cfg.temp_rule)
+    I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps, with_tr=True)
+    p.reflection_map()
+    return p, I, T, Tr
 
+
+def _time_oracle_steps(p, I, T, Tr, dt, steps):
+    """Per-step wall times of the oracle's explicit step (oracle_run, one step each)."""
+    out = []
+    for _ in range(steps):
+        t0 = time.perf_counter()
+        I, T, Tr = p.run(I, T, dt, 1, Tr=Tr)
+        out.append(time.perf_counter() - t0)
+    return out, (I, T, Tr)
+
+
+def cpu_baseline(cfg, budget_s=12.0):
+    """The oracle as it stands, on this host's cores (OpenMP over cells, all
+    cores), on a bounded sample of the workload (about budget_s of CPU work):
+    the full mesh and direction set, the first k band-rows, from the seeded IC
+    the GPU arm runs, 3 timed steps (Newton takes its steady-state iteration
+    count after the first).  Plus the same oracle on ONE core (a subprocess with
+    OMP_NUM_THREADS=1, one row, one step)."""
     cores = os.cpu_count() or 1
     os.environ.setdefault("OMP_NUM_THREADS", str(cores))
+    nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
+    p, I, T, Tr = _oracle_sample(cfg, 1)
+    t1 = _time_oracle_steps(p, I, T, Tr, cfg.dt, 1)[0][0]
+    k = int(max(1, min(nb, budget_s / 3.0 / max(t1, 1e-3))))
+    p, I, T, Tr = _oracle_sample(cfg, k)
+    ts, _ = _time_oracle_steps(p, I, T, Tr, cfg.dt, 3)
+    t = sum(ts)
+    upd = nc * nd * k * len(ts)
+    out = {"value": upd / t, "unit": "updates/s", "cores": int(os.environ["OMP_NUM_THREADS"]), "kind": "oracle",
+           "cpu_model": _cpu_model(), "host_cores": cores,
+           "sample": f"{cfg.name}: full mesh ({nc} cells) x {nd} dirs x first {k} of {nb} band-rows, seeded IC, "
+                     f"3 steps, {t:.2f} s, OMP_NUM_THREADS={os.environ['OMP_NUM_THREADS']}"}
+    try:  # one core
+        env = dict(os.environ, OMP_NUM_THREADS="1")
+        r = subprocess.run([sys.executable, os.path.abspath(__file__), "--_oracle-1core", "--config", cfg.name],
+                           env=env, capture_output=True, text=True, timeout=600)
+        one = json.loads(r.stdout.strip().splitlines()[-1])
+        out["one_core"] = one
+    except Exception as e:  # noqa: BLE001 - reported, never fatal
+        out["one_core"] = {"error": str(e)[:200]}
+    return out
 
-    def run(k, steps):
-        bands = gen.select_bands(cfg.bands, np.arange(k))
-        p = oracle.Problem(cfg.mesh, bands, cfg.dirs, cfg.bcs, temp_rule=cfg.temp_rule)
-        T = np.full(cfg.mesh["n_cells"], cfg.t_init)
-        I = p.equilibrium(T)
-        p.reflection_map()
-        t0 = time.perf_counter()
-        p.run(I, T, cfg.dt, steps, Tr=T.copy() if p.has_rates else None)
-        return time.perf_counter() - t0
 
-    t1 = run(1, 1)
-    nb = cfg.bands["n_bands"]
-    k = int(max(1, min(max_rows or nb, nb, budget_s / max(t1, 1e-3))))
-    steps = int(max(1, min(50, budget_s / max(t1 * k, 1e-3)))) if k == nb else 1
-    t = run(k, steps)
-    upd = cfg.mesh["n_cells"] * cfg.dirs["n_dirs"] * k * steps
-    return {"value": upd / t, "unit": METRIC.replace("updates/s", "updates/s"), "cores": cores,
-            "kind": "oracle",
-            "sample": f"{cfg.name}: full mesh ({cfg.mesh['n_cells']} cells) x {cfg.dirs['n_dirs']} dirs x first {k} "
-                      f"of {cfg.bands['n_bands']} band-rows, {steps} step(s), {t:.2f} s, OMP_NUM_THREADS={os.environ['OMP_NUM_THREADS']}"}
+def _oracle_one_core(args):
+    cfg = _bench_config(args)
+    nc, nd = cfg.mesh["n_cells"], cfg.dirs["n_dirs"]
+    p, I, T, Tr = _oracle_sample(cfg, 1)
+    ts, _ = _time_oracle_steps(p, I, T, Tr, cfg.dt, 2)
+    t = ts[-1]  # (the second step: Newton at its steady-state iteration count)
+    print(json.dumps({"value": nc * nd / t, "unit": "updates/s", "cores": 1,
+                      "sample": f"{cfg.name}: full mesh x {nd} dirs x band-row 0, 1 step after 1 untimed, {t:.2f} s"}))
 
 
 def _bench_config(args):
@@ -189,20 +237,29 @@ def _bench_config(args):
 
 
 def run_reference(args):
-    """--impl reference: the CPU oracle on the same workload/metric (rank 0 only)."""
+    """--impl reference: the CPU oracle as it stands, on this host's cores, on
+    the same workload / metric (rank 0 only; other ranks exit 0).  One bounded
+    sample of the workload (full mesh and directions, the first k band-rows,
+    the seeded IC; built untimed), then W untimed and K timed oracle steps;
+    value = sample updates / median step time."""
     rank, world, _ = _dist()
     if rank != 0:
         return
     cfg = _bench_config(args)
-    vals = []
-    cb = None
-    for i in range(args.warmup + args.steps):
-        r = cpu_baseline(cfg, budget_s=5.0)
-        if i >= args.warmup:
-            vals.append(r["value"])
-            cb = r
-    v = statistics.median(vals)
-    cb = dict(cb, value=v)
+    cores = os.cpu_count() or 1
+    os.environ.setdefault("OMP_NUM_THREADS", str(cores))
+    nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
+    p, I, T, Tr = _oracle_sample(cfg, 1)
+    t1 = _time_oracle_steps(p, I, T, Tr, cfg.dt, 1)[0][0]
+    k = int(max(1, min(nb, 4.0 / max(t1, 1e-3))))  # ~4 s per step
+    p, I, T, Tr = _oracle_sample(cfg, k)
+    _, (I, T, Tr) = _time_oracle_steps(p, I, T, Tr, cfg.dt, args.warmup)
+    ts, _ = _time_oracle_steps(p, I, T, Tr, cfg.dt, args.steps)
+    v = nc * nd * k / statistics.median(ts)
+    cb = {"value": v, "unit": "updates/s", "cores": int(os.environ["OMP_NUM_THREADS"]), "kind": "oracle",
+          "cpu_model": _cpu_model(),
+          "sample": f"{cfg.name}: full mesh ({nc} cells) x {nd} dirs x first {k} of {nb} band-rows, seeded IC, "
+                    f"{args.warmup} untimed + {args.steps} timed steps (median {statistics.median(ts):.2f} s)"}
     line = {"metric": METRIC, "value": v, "unit": "updates/s", "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "higher_is_better": True, "impl": "reference", "dtype": "f64",
             "data": "synthetic", "scaling": "strong",
@@ -290,10 +347,11 @@ def run_ours(args):
     alg_bytes = BYTES_PER_UPDATE * nc_loc * nd * nb_loc  # per step, this rank
     peak, peak_src = _peaks()
     achieved = alg_bytes / t_flux / 1e9 if t_flux > 0 else None
-    traffic = _traffic_from_profiles(args.config)
+    traffic, traffic_src = (_traffic_from_profiles(args.config, flux_launches_per_step) if world == 1 and
+                            not args.rate_law else (None, None))
     roof = {"bound": "hbm", "kernel": "bte::flux_*_kernel (all cells; a1+a2+a3)", "achieved": achieved, "peak": peak,
             "unit": "GB/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-            "peak_source": peak_src,
+            "peak_source": peak_src, "traffic_source": traffic_src,
             "alg_bytes_per_step": alg_bytes, "flux_launches_per_step": flux_launches_per_step,
             "kernel_ms_per_step": t_flux * 1e3,
             "share_of_step": st["ms_flux_interior"] / ms if ms > 0 else None,
@@ -308,7 +366,7 @@ def run_ours(args):
     if not args.no_e2e and state_gb > E2E_MAX_GB:  # C5: the host copy would need ~156 GB of pinned RAM
         e2e = {"skipped": f"state {state_gb:.0f} GB per rank > {E2E_MAX_GB} GB of pinned host memory"}
     elif not args.no_e2e:
-        e2e = _e2e(s, pg, world, nb_loc, nb, nd, nc_loc, dt, total_updates, args)
+        e2e = _e2e(s, pg, world, nb_loc, nd, nc_loc, dt, total_updates, args)
 
     cb = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -316,7 +374,7 @@ def run_ours(args):
     _emit(locals())
 
 
-def _e2e(s, pg, world, nb_loc, nb, nd, nc, dt, total_updates, args):
+def _e2e(s, pg, world, nb_loc, nd, nc, dt, total_updates, args):
     import torch
     def barrier():
         if pg is not None:
@@ -338,8 +396,8 @@ def _e2e(s, pg, world, nb_loc, nb, nd, nc, dt, total_updates, args):
         pg.all_reduce(t, op=pg.ReduceOp.MAX)
         e2e_s = float(t.item())
     e2e = {"value": total_updates / e2e_s, "unit": "updates/s",
-           "h2d_bytes_per_step": int(nb * nd * nc * 8 / args.steps),
-           "d2h_bytes_per_step": int(nc * 8 * world),
+           "h2d_bytes_per_step": int(nb_loc * nd * nc * 8 / args.steps),  # (this rank's state, once per K steps)
+           "d2h_bytes_per_step": int(nc * 8),
            "how": "timed: bte_set_intensity(state from pinned host) once + K x (bte_step(dt,1) + "
                   "bte_get_temperature(pinned host)); wall clock, max over ranks"}
     return e2e
@@ -378,6 +436,20 @@ def _emit(v):
         pg.destroy_process_group()
 
 
+def _spawn_ranks(args):
+    """`python bench.py --gpus N` without a launcher: re-run this command under
+    torch.distributed.run, one rank per GPU on this node (127.0.0.1 rendezvous);
+    rank 0 prints the JSON line."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    sys.stdout.flush()
+    os.execv(sys.executable, cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -399,9 +471,14 @@ def main():
     ap.add_argument("--no-e2e", action="store_true", help="skip the end-to-end leg (profiling runs)")
     ap.add_argument("--cell-parts", type=int, default=1,
                     help="cell partitioning (SURVEY 8(f) N3) into K parts x world/K band groups (default 1)")
+    ap.add_argument("--_oracle-1core", dest="oracle_1core", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
+    if args.oracle_1core:
+        return _oracle_one_core(args)
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return _spawn_ranks(args)
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -1,0 +1,248 @@
+// bte_kernels.cu -- the non-template kernels of the step (temperature solve,
+// energy, I0 / rate tables, equilibrium, ghost tables, gathers / scatters,
+// halo pack / unpack); declared, with their documentation, in bte_kernels.cuh.
+#include "bte_kernels.cuh"
+
+namespace bte {
+
+__global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
+    if (p.halt && *p.halt) return;
+    if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);
+    extern __shared__ double sm[];
+    double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
+    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
+    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
+        sC[b] = p.Cb[b];
+        sTh[b] = p.theta[b];
+        sW[b] = p.cw[b];
+        if (p.td) {
+            sA[b] = p.ra[b];
+            sB[b] = p.rb[b];
+            sR[b] = p.rth[b];
+            sV[b] = p.inv_v[b];
+        }
+    }
+    __syncthreads();
+    const int cl = blockIdx.x * blockDim.x + threadIdx.x;  // chunk-local index
+    if (cl >= p.nc) return;
+    const int c = p.c_lo + cl;
+    double E;
+    if (p.E) {
+        E = p.E[cl];
+    } else {
+        E = 0.0;
+        for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
+    }
+    const double T0 = p.T[c];
+    Weights wt{sW, sA, sB, sR, sV, p.td && p.r2, 0.0};
+    if (p.td) {
+        wt.Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
+        if (p.tr_step && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
+    }
+    double T = T0;
+    bool ok = false;
+    int it = 0;
+    if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
+        const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+        const double Tn = T - gs.g / gs.gp;
+        it = 1;
+        if (Tn > 0.0 && isfinite(Tn)) {
+            T = Tn;
+            ok = true;
+        }
+    } else if (E > 0.0 && isfinite(E)) {
+        for (it = 1; it <= p.maxit; ++it) {
+            const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+            const double delta = gs.g / gs.gp;
+            const double Tn = T - delta;
+            if (!(Tn > 0.0) || !isfinite(Tn)) break;
+            T = Tn;
+            if (fabs(delta) <= p.rtol * T) { ok = true; break; }
+        }
+        if (!ok) {  // bisection safeguard on a bracket grown from T0
+            double lo = T0, hi = T0;
+            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
+            if (g_only(sC, sTh, wt, p.nb, p.W, E, lo) <= 0.0 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) >= 0.0) {
+                for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
+                    const double mid = 0.5 * (lo + hi);
+                    if (g_only(sC, sTh, wt, p.nb, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
+                }
+                T = 0.5 * (lo + hi);
+                ok = true;
+            }
+            it = p.maxit + 1;
+        }
+    }
+    if (!ok) {
+        atomicExch(p.fail, 1);
+        T = p.neg_fail ? -T0 : T0;
+    }
+    atomicMax(p.iter_max, it);
+    if (p.T_out) {
+        p.T_out[c] = T;
+        return;
+    }
+    p.T[c] = T;
+    const double iT = 1.0 / T;
+    for (int k = 0; k < p.nb_loc; ++k) {
+        const int b = p.b_lo + k;
+        p.i0[(size_t)k * p.nc + c] = sC[b] / expm1(sTh[b] * iT);
+        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(sA[b], sB[b], sR[b], T);
+    }
+}
+
+__global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__restrict__ T, int nc, int b_lo,
+                                     int nb_loc, const double *__restrict__ Cb, const double *__restrict__ theta,
+                                     double *__restrict__ i0, int td, const double *__restrict__ ra,
+                                     const double *__restrict__ rb, const double *__restrict__ rth,
+                                     double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
+                                     const int32_t *__restrict__ halt, int32_t *done) {
+    if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
+    if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    double t = Tg[c];
+    if (!(t > 0.0)) {
+        atomicExch(fail, 1);
+        t = -t;
+    }
+    if (td) Tr[c] = T[c];
+    T[c] = t;
+    const double iT = 1.0 / t;
+    for (int k = 0; k < nb_loc; ++k) {
+        const int b = b_lo + k;
+        i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * iT);
+        if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
+    }
+}
+
+__global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
+                                  const double *__restrict__ ra, const double *__restrict__ rb,
+                                  const double *__restrict__ rth, double *__restrict__ out) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    const double t = T[c];
+    for (int k = 0; k < nb_loc; ++k) out[(size_t)k * nc + c] = tau_rate(ra[b_lo + k], rb[b_lo + k], rth[b_lo + k], t);
+}
+
+__global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
+                                 const int32_t *__restrict__ halt) {
+    if (halt && *halt) return;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    double e = 0.0;
+    for (int s = 0; s < n_slots; ++s) e += part[(size_t)s * nc + c];
+    E[c] = e;
+}
+
+__global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__restrict__ slot,
+                              int64_t slab_elems, int ps, int nb_loc, int nd, int nc,
+                              const double4 *__restrict__ dirs, const double *__restrict__ cw,
+                              const double *__restrict__ rate, const double *__restrict__ inv_v,
+                              double *__restrict__ E) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    double e = 0.0;
+    for (int k = 0; k < nb_loc; ++k) {
+        const double *s = pool + (int64_t)slot[k] * slab_elems;
+        double sb = 0.0;
+        for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * ps + c], sb);
+        e = fma(rate ? rate[(size_t)k * nc + c] * inv_v[k] : cw[k], sb, e);
+    }
+    E[c] = e;
+}
+
+__global__ void i0_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
+                                const double *__restrict__ Cb, const double *__restrict__ theta,
+                                double *__restrict__ i0) {
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nc) return;
+    const double iT = 1.0 / T[c];
+    for (int k = 0; k < nb_loc; ++k)
+        i0[(size_t)k * nc + c] = Cb[b_lo + k] / expm1(theta[b_lo + k] * iT);
+}
+
+__global__ void equilibrium_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,
+                                   int64_t slab_elems, int ps, int nd, int nc,
+                                   const double *__restrict__ i0) {
+    const int64_t n = (int64_t)nd * nc;
+    const int k = blockIdx.y;
+    double *s = pool + (int64_t)slot[k] * slab_elems;
+    const double *t = i0 + (size_t)k * nc;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t d = e / nc;
+        const int c = (int)(e - d * nc);
+        s[d * ps + c] = t[c];
+    }
+}
+
+__global__ void i0w_kernel(const double *__restrict__ twall, int n_iso, int b_lo, int nb_loc,
+                           const double *__restrict__ Cb, const double *__restrict__ theta,
+                           double *__restrict__ i0w) {
+    const int f = blockIdx.x * blockDim.x + threadIdx.x;
+    if (f >= n_iso) return;
+    for (int k = 0; k < nb_loc; ++k)
+        i0w[(size_t)k * n_iso + f] = Cb[b_lo + k] / expm1(theta[b_lo + k] / twall[f]);
+}
+
+__global__ void side_table_kernel(const double *__restrict__ i0w, int n_iso, const int32_t *__restrict__ col,
+                                  int n_side, int nb_loc, double *__restrict__ out) {
+    const int64_t n = (int64_t)n_side * nb_loc;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t k = e / n_side;
+        const int c = col[e - k * n_side];
+        out[e] = c >= 0 ? i0w[k * n_iso + c] : 0.0;
+    }
+}
+
+__global__ void gather_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
+                                   int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
+    const int64_t n = rows * nc;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = e / nc;
+        const int u = (int)(e - r * nc);
+        dst[e] = src[r * stride + pos[u]];
+    }
+}
+
+__global__ void scatter_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
+                                    int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
+    const int64_t n = rows * nc;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = e / nc;
+        const int u = (int)(e - r * nc);
+        dst[r * stride + pos[u]] = src[e];
+    }
+}
+
+__global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf) {
+    if (p.fail && *p.fail) return;
+    const int64_t per = (int64_t)p.n_dirs * p.n;
+    const int k = blockIdx.y;
+    const double *s = p.row[k];
+    double *o = buf + k * per;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
+        const int j = (int)(e / p.n);
+        const int i = (int)(e - (int64_t)j * p.n);
+        o[e] = s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)];
+    }
+}
+
+__global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const double *__restrict__ buf) {
+    if (p.fail && *p.fail) return;
+    const int64_t per = (int64_t)p.n_dirs * p.n;
+    const int k = blockIdx.y;
+    double *s = p.row[k];
+    const double *in = buf + k * per;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
+        const int j = (int)(e / p.n);
+        const int i = (int)(e - (int64_t)j * p.n);
+        s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)] = in[e];
+    }
+}
+
+}  // namespace bte

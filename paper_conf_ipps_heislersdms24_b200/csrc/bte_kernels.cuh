@@ -1024,6 +1024,9 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         }
                     }
                     sp = s;
+#if defined(BTE_BOX_LAYER_BARRIER) && !defined(BTE_BOX_TMA_STORE)
+                    bar_compute();  // (experiment: the 8 compute warps in lockstep per layer)
+#endif
 #ifdef BTE_BOX_TMA_STORE
                     fence_smem_to_async();
                     if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
@@ -1131,118 +1134,36 @@ __device__ __forceinline__ double g_only(const double *sC, const double *sTh, co
     return W * g - E;
 }
 
-__global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
-    if (p.halt && *p.halt) return;
-    if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);
-    extern __shared__ double sm[];
-    double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
-    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
-    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
-        sC[b] = p.Cb[b];
-        sTh[b] = p.theta[b];
-        sW[b] = p.cw[b];
-        if (p.td) {
-            sA[b] = p.ra[b];
-            sB[b] = p.rb[b];
-            sR[b] = p.rth[b];
-            sV[b] = p.inv_v[b];
-        }
-    }
-    __syncthreads();
-    const int cl = blockIdx.x * blockDim.x + threadIdx.x;  // chunk-local index
-    if (cl >= p.nc) return;
-    const int c = p.c_lo + cl;
-    double E;
-    if (p.E) {
-        E = p.E[cl];
-    } else {
-        E = 0.0;
-        for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
-    }
-    const double T0 = p.T[c];
-    Weights wt{sW, sA, sB, sR, sV, p.td && p.r2, 0.0};
-    if (p.td) {
-        wt.Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
-        if (p.tr_step && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
-    }
-    double T = T0;
-    bool ok = false;
-    int it = 0;
-    if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
-        const double Tn = T - gs.g / gs.gp;
-        it = 1;
-        if (Tn > 0.0 && isfinite(Tn)) {
-            T = Tn;
-            ok = true;
-        }
-    } else if (E > 0.0 && isfinite(E)) {
-        for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
-            const double delta = gs.g / gs.gp;
-            const double Tn = T - delta;
-            if (!(Tn > 0.0) || !isfinite(Tn)) break;
-            T = Tn;
-            if (fabs(delta) <= p.rtol * T) { ok = true; break; }
-        }
-        if (!ok) {  // bisection safeguard on a bracket grown from T0
-            double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
-            if (g_only(sC, sTh, wt, p.nb, p.W, E, lo) <= 0.0 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) >= 0.0) {
-                for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
-                    const double mid = 0.5 * (lo + hi);
-                    if (g_only(sC, sTh, wt, p.nb, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
-                }
-                T = 0.5 * (lo + hi);
-                ok = true;
-            }
-            it = p.maxit + 1;
-        }
-    }
-    if (!ok) {
-        atomicExch(p.fail, 1);
-        T = p.neg_fail ? -T0 : T0;
-    }
-    atomicMax(p.iter_max, it);
-    if (p.T_out) {
-        p.T_out[c] = T;
-        return;
-    }
-    p.T[c] = T;
-    const double iT = 1.0 / T;
-    for (int k = 0; k < p.nb_loc; ++k) {
-        const int b = p.b_lo + k;
-        p.i0[(size_t)k * p.nc + c] = sC[b] / expm1(sTh[b] * iT);
-        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(sA[b], sB[b], sR[b], T);
-    }
-}
+__global__ void newton_kernel(const __grid_constant__ NewtonParams p);
 
 // ---------------------------------------------------------------------------
-// The same per-cell temperature solve with one WARP per cell (the step's
-// solve; newton_kernel serves the re-solves): lane l evaluates band-rows
-// l, l + 32, ... and butterfly shuffles give every lane the same sums, so the
-// Newton iterates (and the bisection safeguard) are warp-uniform.  A cell's
-// 55 rows x ~4 iterations of expm1 are spread over 32 lanes, so small meshes
-// (C3: 14,400 cells) fill the GPU instead of a few warps per SM.  Output like
-// newton_kernel's chunk solve: T_out[c] = T^{n+1} (or -T^n on failure), the
-// epilogue (T, Tr, I0, rates) is newton_finish_kernel's.
-__device__ __forceinline__ double warp_sum(double v) {
+// The same per-cell temperature solve with a GROUP of G lanes per cell (the
+// step's solve; newton_kernel serves the re-solves): lane l of the group
+// evaluates band-rows l, l + G, ... and butterfly shuffles inside the group
+// give every lane bitwise the same sums (each level adds a commutative pair),
+// so the Newton iterates and the bisection safeguard are group-uniform.  A
+// cell's nb rows x ~4 iterations of expm1 are spread over G lanes: small
+// meshes (C3: 14,400 cells, G = 32) fill the GPU instead of a few warps per
+// SM, larger ones (C4) take G = 8.  Output like newton_kernel's chunk solve:
+// T_out[c] = T^{n+1} (or -T^n on failure); the epilogue (T, Tr, I0, rates) is
+// newton_finish_kernel's.
+template <int G>
+__device__ __forceinline__ double group_sum(double v, unsigned mask) {
 #pragma unroll
-    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    for (int off = G / 2; off > 0; off >>= 1) v += __shfl_xor_sync(mask, v, off);
     return v;
 }
 
-// R = band-rows per lane (ceil(nb / 32) rounded up to a power of two; the
-// per-lane weights stay in registers): one instantiation per R <= kMaxBands / 32.
-template <int R>
-__device__ __forceinline__ Gsum g_eval_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
-                                            double E, double T, int lane) {
+// R = band-rows per lane (ceil(nb / G) rounded up to a power of two; the
+// per-lane weights stay in registers).
+template <int G, int R>
+__device__ __forceinline__ Gsum g_eval_group(const double *sC, const double *sTh, const double *wl, int nb, double W,
+                                             double E, double T, int lane, unsigned mask) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + 32 * r;
+        const int b = lane + G * r;
         if (b < nb) {
             const double x = sTh[b] * it;
             const double em1 = expm1(x);
@@ -1251,23 +1172,23 @@ __device__ __forceinline__ Gsum g_eval_warp(const double *sC, const double *sTh,
             gp = fma(wl[r], i0 * (x * it) * (1.0 + 1.0 / em1), gp);
         }
     }
-    return {W * warp_sum(g) - E, W * warp_sum(gp)};
+    return {W * group_sum<G>(g, mask) - E, W * group_sum<G>(gp, mask)};
 }
 
-template <int R>
-__device__ __forceinline__ double g_only_warp(const double *sC, const double *sTh, const double *wl, int nb, double W,
-                                              double E, double T, int lane) {
+template <int G, int R>
+__device__ __forceinline__ double g_only_group(const double *sC, const double *sTh, const double *wl, int nb,
+                                               double W, double E, double T, int lane, unsigned mask) {
     double g = 0.0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + 32 * r;
+        const int b = lane + G * r;
         if (b < nb) g = fma(wl[r], sC[b] / expm1(sTh[b] / T), g);
     }
-    return W * warp_sum(g) - E;
+    return W * group_sum<G>(g, mask) - E;
 }
 
-template <int R>
-__global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
+template <int G, int R>
+__global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     if (p.halt && *p.halt) return;
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
@@ -1284,17 +1205,18 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
         }
     }
     __syncthreads();
-    const int lane = threadIdx.x & 31;
-    const int cl = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);  // chunk-local cell
-    if (cl >= p.nc) return;
+    const int lane = threadIdx.x & (G - 1);
+    const unsigned mask = G == 32 ? 0xffffffffu : ((1u << G) - 1u) << ((threadIdx.x & 31) & ~(G - 1));
+    const int cl = (blockIdx.x * blockDim.x + threadIdx.x) / G;  // chunk-local cell
+    if (cl >= p.nc) return;  // (whole groups)
     const int c = p.c_lo + cl;
     double E;
     if (p.E) {
         E = p.E[cl];
     } else {
         E = 0.0;
-        for (int s = lane; s < p.n_slots; s += 32) E += p.part[(size_t)s * p.nc + c];
-        E = warp_sum(E);
+        for (int s = lane; s < p.n_slots; s += G) E += p.part[(size_t)s * p.nc + c];
+        E = group_sum<G>(E, mask);
     }
     const double T0 = p.T[c];
     const bool law = p.td && p.r2;
@@ -1302,14 +1224,14 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
     double wl[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + 32 * r;
+        const int b = lane + G * r;
         wl[r] = b >= p.nb ? 0.0 : law ? tau_rate(sA[b], sB[b], sR[b], Tw) * sV[b] : sW[b];
     }
     double T = T0;
     bool ok = false;
     int it = 0;
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = g_eval_warp<R>(sC, sTh, wl, p.nb, p.W, E, T, lane);
+        const Gsum gs = g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -1318,7 +1240,7 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval_warp<R>(sC, sTh, wl, p.nb, p.W, E, T, lane);
+            const Gsum gs = g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -1327,13 +1249,15 @@ __global__ void newton_warp_kernel(const __grid_constant__ NewtonParams p) {
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, lo, lane) > 0.0; ++k) lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, hi, lane) < 0.0; ++k) hi *= 2.0;
-            if (g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, lo, lane) <= 0.0 &&
-                g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, hi, lane) >= 0.0) {
+            for (int k = 0; k < 2000 && g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, lo, lane, mask) > 0.0; ++k)
+                lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, hi, lane, mask) < 0.0; ++k)
+                hi *= 2.0;
+            if (g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, lo, lane, mask) <= 0.0 &&
+                g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, hi, lane, mask) >= 0.0) {
                 for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
                     const double mid = 0.5 * (lo + hi);
-                    if (g_only_warp<R>(sC, sTh, wl, p.nb, p.W, E, mid, lane) < 0.0) lo = mid; else hi = mid;
+                    if (g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, mid, lane, mask) < 0.0) lo = mid; else hi = mid;
                 }
                 T = 0.5 * (lo + hi);
                 ok = true;
@@ -1358,46 +1282,16 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
                                      double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
-                                     const int32_t *__restrict__ halt, int32_t *done) {
-    if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
-    if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
-    double t = Tg[c];
-    if (!(t > 0.0)) {
-        atomicExch(fail, 1);
-        t = -t;
-    }
-    if (td) Tr[c] = T[c];
-    T[c] = t;
-    const double iT = 1.0 / t;
-    for (int k = 0; k < nb_loc; ++k) {
-        const int b = b_lo + k;
-        i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * iT);
-        if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
-    }
-}
+                                     const int32_t *__restrict__ halt, int32_t *done);
 
 // Rate table of the local rows at temperature T: out[k][c] = 1/tau_{b_lo+k}(T_c).
 __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
                                   const double *__restrict__ ra, const double *__restrict__ rb,
-                                  const double *__restrict__ rth, double *__restrict__ out) {
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
-    const double t = T[c];
-    for (int k = 0; k < nb_loc; ++k) out[(size_t)k * nc + c] = tau_rate(ra[b_lo + k], rb[b_lo + k], rth[b_lo + k], t);
-}
+                                  const double *__restrict__ rth, double *__restrict__ out);
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
 __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
-                                 const int32_t *__restrict__ halt) {
-    if (halt && *halt) return;
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
-    double e = 0.0;
-    for (int s = 0; s < n_slots; ++s) e += part[(size_t)s * nc + c];
-    E[c] = e;
-}
+                                 const int32_t *__restrict__ halt);
 
 // E_loc[c] = sum_{local b} c_b sum_d w_d I[b][d][c] of the current state.
 // (rate: R2 with the rate law: c_b = rate[k][c] inv_v[k] at the rate temperature)
@@ -1405,55 +1299,22 @@ __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__
                               int64_t slab_elems, int ps, int nb_loc, int nd, int nc,
                               const double4 *__restrict__ dirs, const double *__restrict__ cw,
                               const double *__restrict__ rate, const double *__restrict__ inv_v,
-                              double *__restrict__ E) {
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
-    double e = 0.0;
-    for (int k = 0; k < nb_loc; ++k) {
-        const double *s = pool + (int64_t)slot[k] * slab_elems;
-        double sb = 0.0;
-        for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * ps + c], sb);
-        e = fma(rate ? rate[(size_t)k * nc + c] * inv_v[k] : cw[k], sb, e);
-    }
-    E[c] = e;
-}
+                              double *__restrict__ E);
 
 // I0 table of the local rows: i0[k][c] = C_{b_lo+k} / expm1(theta / T_c)
 __global__ void i0_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
                                 const double *__restrict__ Cb, const double *__restrict__ theta,
-                                double *__restrict__ i0) {
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
-    const double iT = 1.0 / T[c];
-    for (int k = 0; k < nb_loc; ++k)
-        i0[(size_t)k * nc + c] = Cb[b_lo + k] / expm1(theta[b_lo + k] * iT);
-}
+                                double *__restrict__ i0);
 
 // Equilibrium field I[k][d][c] = i0[k][c] into the current slabs (blockIdx.y = k).
 __global__ void equilibrium_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,
                                    int64_t slab_elems, int ps, int nd, int nc,
-                                   const double *__restrict__ i0) {
-    const int64_t n = (int64_t)nd * nc;
-    const int k = blockIdx.y;
-    double *s = pool + (int64_t)slot[k] * slab_elems;
-    const double *t = i0 + (size_t)k * nc;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t d = e / nc;
-        const int c = (int)(e - d * nc);
-        s[d * ps + c] = t[c];
-    }
-}
+                                   const double *__restrict__ i0);
 
 // Isothermal ghost table i0w[k][f] = I0_{b_lo+k}(T_wall(f)) (Eq. 6, constant in time).
 __global__ void i0w_kernel(const double *__restrict__ twall, int n_iso, int b_lo, int nb_loc,
                            const double *__restrict__ Cb, const double *__restrict__ theta,
-                           double *__restrict__ i0w) {
-    const int f = blockIdx.x * blockDim.x + threadIdx.x;
-    if (f >= n_iso) return;
-    for (int k = 0; k < nb_loc; ++k)
-        i0w[(size_t)k * n_iso + f] = Cb[b_lo + k] / expm1(theta[b_lo + k] / twall[f]);
-}
+                           double *__restrict__ i0w);
 
 // S_max = max_{c,d} sum_faces max(s_d . g, 0) (positivity bound of the step).
 // Paired layout: g holds the "+" face of each pair and the sum is sum |s.g|.
@@ -1482,38 +1343,15 @@ __global__ void outflow_max_kernel(int nc, int mf, int paired, int nd, const dou
 // Isothermal axis-2 side tables of the box kernel: out[k][i] = I0w[k][col[i]]
 // (Eq. 6 ghost I0_b(T_wall), already evaluated by i0w_kernel); 0 where no column.
 __global__ void side_table_kernel(const double *__restrict__ i0w, int n_iso, const int32_t *__restrict__ col,
-                                  int n_side, int nb_loc, double *__restrict__ out) {
-    const int64_t n = (int64_t)n_side * nb_loc;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t k = e / n_side;
-        const int c = col[e - k * n_side];
-        out[e] = c >= 0 ? i0w[k * n_iso + c] : 0.0;
-    }
-}
+                                  int n_side, int nb_loc, double *__restrict__ out);
 
 // dst[r][u] = src[r * stride + pos[u]]  (internal -> caller cell order).
 __global__ void gather_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
-                                   int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
-    const int64_t n = rows * nc;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = e / nc;
-        const int u = (int)(e - r * nc);
-        dst[e] = src[r * stride + pos[u]];
-    }
-}
+                                   int nc, int64_t stride, int64_t rows, double *__restrict__ dst);
 
 // dst[r * stride + pos[u]] = src[r][u]  (caller -> internal order)
 __global__ void scatter_rows_kernel(const double *__restrict__ src, const int32_t *__restrict__ pos,
-                                    int nc, int64_t stride, int64_t rows, double *__restrict__ dst) {
-    const int64_t n = rows * nc;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = e / nc;
-        const int u = (int)(e - r * nc);
-        dst[r * stride + pos[u]] = src[e];
-    }
-}
+                                    int nc, int64_t stride, int64_t rows, double *__restrict__ dst);
 
 // ---------------------------------------------------------------------------
 // Halo exchange of a cell-partitioned run (the paper's
@@ -1534,30 +1372,8 @@ struct HaloParams {
     const int32_t *fail;              // != 0: a solve of an earlier step of the call failed (no-op)
 };
 
-__global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf) {
-    if (p.fail && *p.fail) return;
-    const int64_t per = (int64_t)p.n_dirs * p.n;
-    const int k = blockIdx.y;
-    const double *s = p.row[k];
-    double *o = buf + k * per;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
-        const int j = (int)(e / p.n);
-        const int i = (int)(e - (int64_t)j * p.n);
-        o[e] = s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)];
-    }
-}
+__global__ void halo_pack_kernel(const __grid_constant__ HaloParams p, double *__restrict__ buf);
 
-__global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const double *__restrict__ buf) {
-    if (p.fail && *p.fail) return;
-    const int64_t per = (int64_t)p.n_dirs * p.n;
-    const int k = blockIdx.y;
-    double *s = p.row[k];
-    const double *in = buf + k * per;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < per; e += (int64_t)gridDim.x * blockDim.x) {
-        const int j = (int)(e / p.n);
-        const int i = (int)(e - (int64_t)j * p.n);
-        s[(int64_t)__ldg(p.dirs + j) * p.ps + __ldg(p.cells + i)] = in[e];
-    }
-}
+__global__ void halo_unpack_kernel(const __grid_constant__ HaloParams p, const double *__restrict__ buf);
 
 }  // namespace bte
