@@ -717,9 +717,23 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                         sidx_h[q] = (uint16_t)(bte::kTile + it->second);
                     }
                 }
+            // halo slots in ascending cell order, so that the producer lanes' gathers
+            // of neighbouring columns fall into shared 32-byte sectors
             const int32_t nh = (int32_t)slot_of.size();
-            std::vector<int32_t> cells(nh);
-            for (const auto &kv : slot_of) cells[kv.second] = kv.first;
+            std::vector<int32_t> cells(nh), newpos(nh);
+            {
+                int32_t r = 0;
+                for (const auto &kv : slot_of) {
+                    newpos[kv.second] = r;
+                    cells[r++] = kv.first;
+                }
+            }
+            for (int j = 0; j < mf_t; ++j)
+                for (int32_t i = t0; i < t1; ++i) {
+                    const size_t q = (size_t)j * nc + i;
+                    if (fcode8_h[q] == bte::kCode8Interior && sidx_h[q] >= bte::kTile)
+                        sidx_h[q] = (uint16_t)(bte::kTile + newpos[sidx_h[q] - bte::kTile]);
+                }
             hcell.insert(hcell.end(), cells.begin(), cells.end());
             hoff[t + 1] = (int32_t)hcell.size();
             for (size_t g = 0; g < bq.size(); ++g) {  // Eq. 6 ghosts: isothermal table column / reflected plane

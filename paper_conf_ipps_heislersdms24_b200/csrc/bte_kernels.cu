@@ -11,7 +11,9 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
     double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
+    double *sIC = sm + 7 * p.nb;  // 1 / C_b
     for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
+        sIC[b] = 1.0 / p.Cb[b];
         sC[b] = p.Cb[b];
         sTh[b] = p.theta[b];
         sW[b] = p.cw[b];
@@ -42,8 +44,10 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     double T = T0;
     bool ok = false;
     int it = 0;
+    const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+        const Gsum gs = tab ? g_eval_table(sIC, sTh, wt, p.nb, p.W, E, T, tab, p.nc_tab)
+                            : g_eval(sC, sTh, wt, p.nb, p.W, E, T);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -52,7 +56,8 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+            const Gsum gs = (it == 1 && tab) ? g_eval_table(sIC, sTh, wt, p.nb, p.W, E, T, tab, p.nc_tab)
+                                             : g_eval(sC, sTh, wt, p.nb, p.W, E, T);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -100,21 +105,21 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      const int32_t *__restrict__ halt, int32_t *done) {
     if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
     if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
+    const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= (int64_t)nc * nb_loc) return;
+    const int k = (int)(e / nc), c = (int)(e - (int64_t)k * nc);
     double t = Tg[c];
     if (!(t > 0.0)) {
-        atomicExch(fail, 1);
+        if (k == 0) atomicExch(fail, 1);
         t = -t;
     }
-    if (td) Tr[c] = T[c];
-    T[c] = t;
-    const double iT = 1.0 / t;
-    for (int k = 0; k < nb_loc; ++k) {
-        const int b = b_lo + k;
-        i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * iT);
-        if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
+    if (k == 0) {
+        if (td) Tr[c] = T[c];
+        T[c] = t;
     }
+    const int b = b_lo + k;
+    i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * (1.0 / t));
+    if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
 }
 
 __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,

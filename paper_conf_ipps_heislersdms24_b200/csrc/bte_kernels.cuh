@@ -642,9 +642,19 @@ constexpr int kBoxPlane = 320;               // doubles per staged plane (128-by
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
 constexpr int kBoxMaxStages = 12;
-#ifndef BTE_BOX_STORE_HINT
-#define BTE_BOX_STORE_HINT 0  // direct stores of I^{n+1}: 0 st.global.cs, 1 L2 evict_first policy, 2 plain
+// How I^{n+1} leaves the box kernel (measured on B200): 3-D grids
+// store straight from registers (coalesced st.global.cs, no per-layer CTA
+// barrier: C4 sustained flux 7.80 -> 7.53 ms); 2-D grids keep the
+// shared-memory tile + tensor store (C3 0.84 -> 0.83 ms).  -DBTE_BOX_TMA_STORE:
+// tensor stores everywhere.
+template <bool FLAT>
+constexpr bool box_tma_store() {
+#ifdef BTE_BOX_TMA_STORE
+    return true;
+#else
+    return FLAT;
 #endif
+}
 // Resident CTAs per SM the kernel is compiled for (register cap): 3-D grids 2
 // (96 registers, 6 stages of 12 KB plus L x 2 KB of energy rows); 2-D grids 3
 // (72 registers, no spills, 4 stages): a 2-D stage is one layer, so CTAs are
@@ -809,12 +819,9 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     const int S = p.stages;
 #endif
     double *ring = bsm;                          // [S][kStage]
-#ifdef BTE_BOX_TMA_STORE
-    double *obuf = ring + S * kStage;            // [2][4][256]
-    double *eacc = obuf + 2 * 4 * kBoxCells;     // [L][256]
-#else
-    double *eacc = ring + S * kStage;            // [L][256]
-#endif
+    constexpr bool kTmaStore = box_tma_store<FLAT>();
+    double *obuf = ring + S * kStage;                           // [2][4][256] (tensor stores)
+    double *eacc = obuf + (kTmaStore ? 2 * 4 * kBoxCells : 0);  // [L][256]
     BoxOrbitC *sorb = reinterpret_cast<BoxOrbitC *>(eacc + p.L * kBoxCells);  // [orb_chunk]
     __shared__ __align__(8) uint64_t full[kBoxMaxStages];
     __shared__ __align__(8) uint64_t empty[kBoxMaxStages];
@@ -924,26 +931,16 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         if (flat && wall1 && p.zside[(q & 2) ? 1 : 0] == 0) uy[q] = kGhost + ((q & 2) ? kBoxTX : 0) + tx;
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
-#ifndef BTE_BOX_TMA_STORE
-    // I^{n+1} leaves straight from registers: a warp's 32 cells are one 256-byte
-    // row of a plane (coalesced streaming stores, no shared-memory round trip and
-    // no per-layer CTA barrier)
+    // direct stores: a warp's 32 cells are one 256-byte row of a plane
     const int32_t plane = p.n0 * p.n1;
     const int32_t cell_off = gy * p.n0 + gx;
-#if BTE_BOX_STORE_HINT == 1
-    uint64_t spol;  // I^{n+1} is not read again this step: evict first, keep L2 for the halo boxes
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(spol));
-#endif
-#endif
 
     int s = 0, sp = 0;
     uint32_t ph = 0, ob = 0;
     double pv[4] = {0.0, 0.0, 0.0, 0.0};  // the previous layer's own values: this layer's axis-2 upwind values
     for (int k = w.k0; k < w.k1; ++k) {
         const double kv = p.kv[k];
-#ifndef BTE_BOX_TMA_STORE
         double *const oslab = p.pool + (int64_t)p.out_slab[k] * p.slab_elems + cell_off;
-#endif
         for (int o = w.o0; o < w.o1; ++o) {
             const BoxOrbitC &orb = sorb[o - w.o0];
             const bool asc = orb.asc;
@@ -953,11 +950,9 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             const double kvout = kv * ((orb.a[0] + orb.a[1]) + orb.a[2]);
             const double coef_c = (1.0 - p.dtit[k]) - kvout;  // constant rates
             const double m0 = -orb.a[0], m1 = -orb.a[1], m2 = -orb.a[2];
-#ifndef BTE_BOX_TMA_STORE
             int32_t doff[4];  // plane offsets of the orbit's 4 directions (slab_elems < 2^31)
 #pragma unroll
             for (int q = 0; q < 4; ++q) doff[q] = orb.d[q] * p.ps;
-#endif
             for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
@@ -980,11 +975,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         cw = p.cw[k];
                     }
                     const double src = dtit * cur[4 * kBoxPlane + tid];
-#ifdef BTE_BOX_TMA_STORE
-                    double *out = obuf + ob * (4 * kBoxCells);
-#else
-                    double *const orow = oslab + z * plane;
-#endif
+                    double *out = obuf + ob * (4 * kBoxCells);  // (tensor stores)
+                    double *const orow = oslab + z * plane;     // (direct stores)
                     double acc = 0.0;
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
@@ -994,20 +986,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         if (!flat) infl = fma(m2, pv[q], infl);
                         pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
-#ifdef BTE_BOX_TMA_STORE
-                        out[q * kBoxCells + tid] = inew;
-#else
-                        if (valid) {
-#if BTE_BOX_STORE_HINT == 1
-                            asm volatile("st.global.L1::no_allocate.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(orow + doff[q]),
-                                         "d"(inew), "l"(spol) : "memory");
-#elif BTE_BOX_STORE_HINT == 2
-                            orow[doff[q]] = inew;
-#else
-                            __stcs(orow + doff[q], inew);
-#endif
-                        }
-#endif
+                        if constexpr (kTmaStore) out[q * kBoxCells + tid] = inew;
+                        else if (valid) __stcs(orow + doff[q], inew);
                         acc = fma(wq[q], inew, acc);
                     }
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
@@ -1024,21 +1004,18 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         }
                     }
                     sp = s;
-#if defined(BTE_BOX_LAYER_BARRIER) && !defined(BTE_BOX_TMA_STORE)
-                    bar_compute();  // (experiment: the 8 compute warps in lockstep per layer)
-#endif
-#ifdef BTE_BOX_TMA_STORE
-                    fence_smem_to_async();
-                    if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
-                    bar_compute();
-                    if (tid == 0) {
+                    if constexpr (kTmaStore) {
+                        fence_smem_to_async();
+                        if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
+                        bar_compute();
+                        if (tid == 0) {
 #pragma unroll
-                        for (int q = 0; q < 4; ++q)
-                            tma_store_5d(&tm_out, out + q * kBoxCells, w.x0, w.y0, z, orb.d[q], p.out_slab[k]);
-                        bulk_commit();
+                            for (int q = 0; q < 4; ++q)
+                                tma_store_5d(&tm_out, out + q * kBoxCells, w.x0, w.y0, z, orb.d[q], p.out_slab[k]);
+                            bulk_commit();
+                        }
+                        ob ^= 1u;
                     }
-                    ob ^= 1u;
-#endif
                 }
                 if (++s == S) {
                     s = 0;
@@ -1052,10 +1029,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         for (int l = 0; l < w.Lc; ++l)
             part[((int64_t)(w.z0 - p.zlo + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
-#ifdef BTE_BOX_TMA_STORE
-    if (tid == 0) bulk_wait_all();
-#endif
-    (void)ob;
+    if (kTmaStore && tid == 0) bulk_wait_all();
 }
 
 // ---------------------------------------------------------------- temperature
@@ -1090,6 +1064,12 @@ struct NewtonParams {
     // the step and block 0 counts it
     const int32_t *halt;
     int32_t *done;
+    // the I0 table of ALL band-rows at the starting temperature T0 = T[c]
+    // ([nb][nc_tab], the previous step's refresh; nullptr when this rank holds
+    // only some rows): the first g / g' evaluation of a solve reads it instead
+    // of nb expm1 (I0 = C / expm1(x), 1 / expm1(x) = I0 / C)
+    const double *i0_t0;
+    int32_t nc_tab;
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1116,13 +1096,28 @@ __device__ __forceinline__ Gsum g_eval(const double *sC, const double *sTh, cons
                                        int nb, double W, double E, double T) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
-    for (int b = 0; b < nb; ++b) {
+    for (int b = 0; b < nb; ++b) {  // (one reciprocal per row: I0 = C r, I0' = I0 (x/T)(1 + r))
         const double x = sTh[b] * it;
-        const double em1 = expm1(x);
-        const double i0 = sC[b] / em1;
+        const double r = 1.0 / expm1(x);
+        const double i0 = sC[b] * r;
         const double wb = wt(b);
         g = fma(wb, i0, g);
-        gp = fma(wb, i0 * (x * it) * (1.0 + 1.0 / em1), gp);
+        gp = fma(wb, i0 * (x * it) * (1.0 + r), gp);
+    }
+    return {W * g - E, W * gp};
+}
+
+// g, g' at T0 from the stored table i0_t0[b][c] = I0_b(T0).
+__device__ __forceinline__ Gsum g_eval_table(const double *sIC, const double *sTh, const Weights &wt, int nb,
+                                             double W, double E, double T0, const double *i0_t0, int64_t stride) {
+    double g = 0.0, gp = 0.0;
+    const double it = 1.0 / T0;
+    for (int b = 0; b < nb; ++b) {
+        const double x = sTh[b] * it;
+        const double i0 = __ldg(i0_t0 + b * stride);
+        const double wb = wt(b);
+        g = fma(wb, i0, g);
+        gp = fma(wb, i0 * (x * it) * (1.0 + i0 * sIC[b]), gp);
     }
     return {W * g - E, W * gp};
 }
@@ -1166,10 +1161,29 @@ __device__ __forceinline__ Gsum g_eval_group(const double *sC, const double *sTh
         const int b = lane + G * r;
         if (b < nb) {
             const double x = sTh[b] * it;
-            const double em1 = expm1(x);
-            const double i0 = sC[b] / em1;
+            const double q = 1.0 / expm1(x);
+            const double i0 = sC[b] * q;
             g = fma(wl[r], i0, g);
-            gp = fma(wl[r], i0 * (x * it) * (1.0 + 1.0 / em1), gp);
+            gp = fma(wl[r], i0 * (x * it) * (1.0 + q), gp);
+        }
+    }
+    return {W * group_sum<G>(g, mask) - E, W * group_sum<G>(gp, mask)};
+}
+
+template <int G, int R>
+__device__ __forceinline__ Gsum g_eval_group_table(const double *sIC, const double *sTh, const double *wl, int nb,
+                                                   double W, double E, double T0, int lane, unsigned mask,
+                                                   const double *i0_t0, int64_t stride) {
+    double g = 0.0, gp = 0.0;
+    const double it = 1.0 / T0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int b = lane + G * r;
+        if (b < nb) {
+            const double x = sTh[b] * it;
+            const double i0 = __ldg(i0_t0 + b * stride);
+            g = fma(wl[r], i0, g);
+            gp = fma(wl[r], i0 * (x * it) * (1.0 + i0 * sIC[b]), gp);
         }
     }
     return {W * group_sum<G>(g, mask) - E, W * group_sum<G>(gp, mask)};
@@ -1193,7 +1207,9 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     extern __shared__ double sm[];
     double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
     double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
+    double *sIC = sm + 7 * p.nb;  // 1 / C_b
     for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
+        sIC[b] = 1.0 / p.Cb[b];
         sC[b] = p.Cb[b];
         sTh[b] = p.theta[b];
         sW[b] = p.cw[b];
@@ -1230,8 +1246,10 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     double T = T0;
     bool ok = false;
     int it = 0;
+    const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
+        const Gsum gs = tab ? g_eval_group_table<G, R>(sIC, sTh, wl, p.nb, p.W, E, T, lane, mask, tab, p.nc_tab)
+                            : g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -1240,7 +1258,9 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
+            const Gsum gs = (it == 1 && tab)
+                                ? g_eval_group_table<G, R>(sIC, sTh, wl, p.nb, p.W, E, T, lane, mask, tab, p.nc_tab)
+                                : g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -1277,6 +1297,7 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
 // flag it on every rank and keep T^n), the rate temperature Tr <- T^n, and the
 // local rows of I0 and of the rate table at T^{n+1} -- the epilogue of
 // newton_kernel, bit for bit.
+// One thread per (local row, cell): T, Tr from the k = 0 threads.
 __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__restrict__ T, int nc, int b_lo,
                                      int nb_loc, const double *__restrict__ Cb, const double *__restrict__ theta,
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,

@@ -184,11 +184,9 @@ int box_stage(const bte_ctx *ctx) {
 
 size_t box_smem(const bte_ctx *ctx) {
     const int stage = box_stage(ctx);
-#ifdef BTE_BOX_TMA_STORE
-    constexpr size_t obuf = 2 * 4 * bte::kBoxCells;  // double-buffered output tiles of the tensor stores
-#else
-    constexpr size_t obuf = 0;  // results leave straight from registers
-#endif
+    const size_t obuf = (ctx->bflat ? bte::box_tma_store<true>() : bte::box_tma_store<false>())
+                            ? 2 * 4 * bte::kBoxCells  // double-buffered output tiles of the tensor stores
+                            : 0;                      // results leave straight from registers
     return ((size_t)ctx->box_stages * stage + obuf + (size_t)ctx->box_L * bte::kBoxCells) *
                sizeof(double) +
            (size_t)kBoxMaxOrbChunk * sizeof(bte::BoxOrbitC);

@@ -208,7 +208,7 @@ int newton_lanes(const bte_ctx *ctx, int ncells) {
 bool warp_newton(const bte_ctx *ctx, int ncells) { return newton_lanes(ctx, ncells) > 0; }
 
 // Band constants in shared memory: C, theta, c_b (+ the four rate-law arrays).
-size_t newton_smem(const bte_ctx *ctx) { return (size_t)(ctx->td ? 7 : 3) * ctx->nb * sizeof(double); }
+size_t newton_smem(const bte_ctx *ctx) { return (size_t)8 * ctx->nb * sizeof(double); }
 
 // Thread-per-cell solve over q.nc cells (block 0 counts the step when q.done).
 bte_status launch_newton_cells(bte_ctx *ctx, const bte::NewtonParams &q) {
@@ -312,6 +312,10 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     q.fail = ctx->d_fail;
     q.single = ctx->opt.temp_rule == 2;
     if (step) q.halt = ctx->d_halt;  // (a step's solve: no-op after a failure earlier in the call)
+    if (ctx->nb_loc == ctx->nb) {  // this rank's I0 table holds every row at the current T
+        q.i0_t0 = ctx->i0;
+        q.nc_tab = ctx->nc;
+    }
     return q;
 }
 
@@ -328,7 +332,8 @@ bte_status reduce_slots(bte_ctx *ctx) {
 // T <- Tg (a negative entry marks a failed cell: flag, keep T^n), Tr <- T^n,
 // I0 and the rate table of the local rows at the new T.
 bte_status newton_finish(bte_ctx *ctx) {
-    bte::newton_finish_kernel<<<(ctx->nc + 255) / 256, 256, 0, ctx->stream>>>(
+    const int64_t n = (int64_t)ctx->nc * ctx->nb_loc;
+    bte::newton_finish_kernel<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(
         ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
         ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail, ctx->d_halt, ctx->d_done);
     ctx->st.kernel_launches++;

@@ -44,7 +44,10 @@ def _num(v, unit):
 
 
 def full(rep, out, config=None, bands_in_launch=None, bands=None):
-    raw = subprocess.check_output(["ncu", "-i", rep, "--page", "raw", "--csv"], text=True)
+    if rep.endswith(".csv"):  # a raw-page export (ncu -i REP --page raw --csv) made on the GPU box
+        raw = open(rep).read()
+    else:
+        raw = subprocess.check_output(["ncu", "-i", rep, "--page", "raw", "--csv"], text=True)
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
     kernels = []

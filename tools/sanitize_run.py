@@ -50,6 +50,48 @@ def run_parts(cfg, n_parts, slabs=False):
             s.close()
 
 
+def run_group(cfg, world, n_parts=1):
+    """world ranks as threads on one in-process group (bte_group_create):
+    the band-sharded / cell-partitioned step through bte_step."""
+    import threading
+    from paper_conf_ipps_heislersdms24_b200.dist import partition_cells
+    kw = {}
+    if n_parts > 1:
+        kw = dict(cell_part=partition_cells(cfg.mesh["cell_centre"], n_parts), n_cell_parts=n_parts)
+    err = []
+    with bte.Group(world) as g:
+        def rank(r):
+            try:
+                with bte.solver_from_config(cfg, rank=r, world=world, group=g, **kw) as s:
+                    bte.apply_ic(s, cfg)
+                    s.step(cfg.dt, 2)
+                    s.temperature()
+            except Exception as e:  # noqa: BLE001
+                err.append(e)
+        ts = [threading.Thread(target=rank, args=(r,)) for r in range(world)]
+        [t.start() for t in ts]
+        [t.join() for t in ts]
+    if err:
+        raise err[0]
+    return "ok"
+
+
+def run_enoconv(**kw):
+    cfg = gen.failing_strip_config()
+    with bte.solver_from_config(cfg, **kw) as s:
+        bte.apply_ic(s, cfg)
+        try:
+            s.step(cfg.dt, cfg.nsteps)
+        except bte.BTEError as e:
+            assert e.status == bte.BTE_ENOCONV and s.stats()["steps"] == 4
+            return "enoconv at step 4"
+    raise AssertionError("no ENOCONV")
+
+
+print("group-band-3", run_group(c3d, 3), flush=True)
+print("group-hybrid-2x2", run_group(dataclasses.replace(gen.make_config("C2"), nsteps=2), 4, n_parts=2), flush=True)
+print("enoconv-graph", run_enoconv(), flush=True)
+print("enoconv-profile", run_enoconv(profile=True), flush=True)
 print("parts-3d", run_parts(c3d, 3), flush=True)
 print("parts-zslab-box", run_parts(box3, 2, slabs=True), flush=True)
 print("parts-tri", run_parts(c6t, 2), flush=True)
