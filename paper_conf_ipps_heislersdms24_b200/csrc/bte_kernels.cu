@@ -131,14 +131,26 @@ __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo
     for (int k = 0; k < nb_loc; ++k) out[(size_t)k * nc + c] = tau_rate(ra[b_lo + k], rb[b_lo + k], rth[b_lo + k], t);
 }
 
+// E[c] = sum_s part[s][c]: a block of 8 warps takes 32 cells (lane = cell, so a
+// warp's loads are one coalesced 256-byte row of a slot), warp w sums slots
+// w, w + 8, ...; the 8 partial sums are added in warp order (deterministic).
 __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
                                  const int32_t *__restrict__ halt) {
     if (halt && *halt) return;
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
+    __shared__ double red[kSumSlotWarps][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int c = blockIdx.x * 32 + lane;
     double e = 0.0;
-    for (int s = 0; s < n_slots; ++s) e += part[(size_t)s * nc + c];
-    E[c] = e;
+    if (c < nc)
+        for (int s = w; s < n_slots; s += kSumSlotWarps) e += part[(size_t)s * nc + c];
+    red[w][lane] = e;
+    __syncthreads();
+    if (w == 0 && c < nc) {
+        double t = red[0][lane];
+#pragma unroll
+        for (int k = 1; k < kSumSlotWarps; ++k) t += red[k][lane];
+        E[c] = t;
+    }
 }
 
 __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__restrict__ slot,

@@ -642,6 +642,12 @@ constexpr int kBoxPlane = 320;               // doubles per staged plane (128-by
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
 constexpr int kBoxMaxStages = 12;
+#ifndef BTE_BOX_LOAD_POLICY
+#define BTE_BOX_LOAD_POLICY 0  // (experiment) L2 policy on the I^n box loads (0: none)
+#endif
+#ifndef BTE_BOX_STORE_HINT
+#define BTE_BOX_STORE_HINT 0  // (experiment) 1: direct stores with an explicit L2 evict-first policy
+#endif
 // How I^{n+1} leaves the box kernel (measured on B200): 3-D grids
 // store straight from registers (coalesced st.global.cs, no per-layer CTA
 // barrier: C4 sustained flux 7.80 -> 7.53 ms); 2-D grids keep the
@@ -655,6 +661,12 @@ constexpr bool box_tma_store() {
     return FLAT;
 #endif
 }
+// (experiment, BTE_BOX_STORE_HINT == 2) direct path through a per-warp shared
+// row + one bulk copy per direction row (no CTA barrier)
+template <bool FLAT>
+constexpr bool box_warp_bulk() { return !box_tma_store<FLAT>() && BTE_BOX_STORE_HINT == 2; }
+template <bool FLAT>
+constexpr bool box_obuf() { return box_tma_store<FLAT>() || box_warp_bulk<FLAT>(); }
 // Resident CTAs per SM the kernel is compiled for (register cap): 3-D grids 2
 // (96 registers, 6 stages of 12 KB plus L x 2 KB of energy rows); 2-D grids 3
 // (72 registers, no spills, 4 stages): a 2-D stage is one layer, so CTAs are
@@ -712,6 +724,16 @@ __device__ __forceinline__ void tma_load_5d(void *dst, const void *tmap, int c0,
         "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
         " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
+        : "memory");
+}
+// The same with an L2 cache policy (createpolicy) on the loaded lines.
+__device__ __forceinline__ void tma_load_5d_hint(void *dst, const void *tmap, int c0, int c1, int c2, int c3, int c4,
+                                                 uint64_t *bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar)),
+        "l"(pol)
         : "memory");
 }
 __device__ __forceinline__ void tma_load_3d(void *dst, const void *tmap, int c0, int c1, int c2, uint64_t *bar) {
@@ -821,7 +843,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     double *ring = bsm;                          // [S][kStage]
     constexpr bool kTmaStore = box_tma_store<FLAT>();
     double *obuf = ring + S * kStage;                           // [2][4][256] (tensor stores)
-    double *eacc = obuf + (kTmaStore ? 2 * 4 * kBoxCells : 0);  // [L][256]
+    constexpr bool kWarpBulk = box_warp_bulk<FLAT>();
+    double *eacc = obuf + (box_obuf<FLAT>() ? 2 * 4 * kBoxCells : 0);  // [L][256]
     BoxOrbitC *sorb = reinterpret_cast<BoxOrbitC *>(eacc + p.L * kBoxCells);  // [orb_chunk]
     __shared__ __align__(8) uint64_t full[kBoxMaxStages];
     __shared__ __align__(8) uint64_t empty[kBoxMaxStages];
@@ -856,6 +879,20 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
 
     if (tid >= kBoxCells) {  // ------------------------------------------- producer warp
         if (tid == kBoxCells) {
+#if BTE_BOX_LOAD_POLICY
+            // (experiment) L2 policy of the I^n boxes: 1 evict_last, 2 evict_normal, 3 evict_first
+            uint64_t lpol;
+#if BTE_BOX_LOAD_POLICY == 1
+            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(lpol));
+#elif BTE_BOX_LOAD_POLICY == 2
+            asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(lpol));
+#else
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(lpol));
+#endif
+#define BOX_LOAD_IN(dst, map, a, b, c, d, e, bar) tma_load_5d_hint(dst, map, a, b, c, d, e, bar, lpol)
+#else
+#define BOX_LOAD_IN(dst, map, a, b, c, d, e, bar) tma_load_5d(dst, map, a, b, c, d, e, bar)
+#endif
             int s = 0;
             uint32_t ph = 0, wrapped = 0;  // ring slot, its use parity, ring wrapped once
             for (int k = w.k0; k < w.k1; ++k) {
@@ -874,7 +911,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             for (int q = 0; q < 4; ++q) {
                                 const int xs = w.x0 - box_xs(q), ys = w.y0 - box_hy(q);
                                 if (zh >= 0 && zh < p.n2)
-                                    tma_load_5d(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
+                                    BOX_LOAD_IN(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
                                 else if (p.zside[asc ? 0 : 1] == 0)  // isothermal: I0_b(T_wall) side table
                                     tma_load_4d(st + q * kBoxPlane, &tm_side, xs, ys, asc ? 0 : 1, bl, &full[s]);
                                 else  // specular: the wall layer of the z-mirrored direction (old level)
@@ -891,7 +928,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             if (glo) tma_load_3d(st + kGhost, &tm_side, w.x0, 0, bl, &full[s]);
                             if (ghi) tma_load_3d(st + kGhost + kBoxTX, &tm_side, w.x0, 1, bl, &full[s]);
                             for (int q = 0; q < 4; ++q)
-                                tma_load_5d(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
+                                BOX_LOAD_IN(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
                                             ob.d[q], slab, &full[s]);
                             tma_load_4d(st + 4 * kBoxPlane, &tm_i0, w.x0, w.y0, z - p.zlo, bl, &full[s]);
                             if (TD) {
@@ -934,6 +971,10 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     // direct stores: a warp's 32 cells are one 256-byte row of a plane
     const int32_t plane = p.n0 * p.n1;
     const int32_t cell_off = gy * p.n0 + gx;
+#if BTE_BOX_STORE_HINT
+    uint64_t spol;  // (experiment) L2 evict-first policy for the direct stores
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(spol));
+#endif
 
     int s = 0, sp = 0;
     uint32_t ph = 0, ob = 0;
@@ -986,8 +1027,14 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         if (!flat) infl = fma(m2, pv[q], infl);
                         pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
-                        if constexpr (kTmaStore) out[q * kBoxCells + tid] = inew;
+                        if constexpr (kTmaStore || kWarpBulk) out[q * kBoxCells + tid] = inew;
+#if BTE_BOX_STORE_HINT == 1
+                        else if (valid)
+                            asm volatile("st.global.L1::no_allocate.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(orow + doff[q]),
+                                         "d"(inew), "l"(spol) : "memory");
+#else
                         else if (valid) __stcs(orow + doff[q], inew);
+#endif
                         acc = fma(wq[q], inew, acc);
                     }
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
@@ -1004,6 +1051,30 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         }
                     }
                     sp = s;
+#if BTE_BOX_STORE_HINT == 2
+                    if constexpr (kWarpBulk) {  // this warp's 4 rows leave by bulk copies
+                        fence_smem_to_async();
+                        __syncwarp();
+                        const bool full_row = w.x0 + kBoxTX <= p.n0 && gy < p.n1;
+                        if (lane == 0 && full_row) {
+#pragma unroll
+                            for (int q = 0; q < 4; ++q)
+                                asm volatile(
+                                    "cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], 256, %2;" ::"l"(
+                                        orow + doff[q] - tx),
+                                    "r"(smem_u32(out + q * kBoxCells + ty * 32)), "l"(spol)
+                                    : "memory");
+                            bulk_commit();
+                        }
+                        if (!full_row && valid)  // ragged rows: plain stores
+#pragma unroll
+                            for (int q = 0; q < 4; ++q) __stcs(orow + doff[q], out[q * kBoxCells + tid]);
+                        ob ^= 1u;
+                        // before this warp rewrites the other buffer: its copies have read it
+                        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                        __syncwarp();
+                    }
+#endif
                     if constexpr (kTmaStore) {
                         fence_smem_to_async();
                         if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
@@ -1030,6 +1101,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             part[((int64_t)(w.z0 - p.zlo + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
     if (kTmaStore && tid == 0) bulk_wait_all();
+    if (kWarpBulk && lane == 0) bulk_wait_all();
 }
 
 // ---------------------------------------------------------------- temperature
@@ -1311,6 +1383,7 @@ __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo
                                   const double *__restrict__ rth, double *__restrict__ out);
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
+constexpr int kSumSlotWarps = 8;  // sum_slots_kernel: warps per 32 cells
 __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
                                  const int32_t *__restrict__ halt);
 

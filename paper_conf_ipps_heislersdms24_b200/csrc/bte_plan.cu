@@ -184,7 +184,7 @@ int box_stage(const bte_ctx *ctx) {
 
 size_t box_smem(const bte_ctx *ctx) {
     const int stage = box_stage(ctx);
-    const size_t obuf = (ctx->bflat ? bte::box_tma_store<true>() : bte::box_tma_store<false>())
+    const size_t obuf = (ctx->bflat ? bte::box_obuf<true>() : bte::box_obuf<false>())
                             ? 2 * 4 * bte::kBoxCells  // double-buffered output tiles of the tensor stores
                             : 0;                      // results leave straight from registers
     return ((size_t)ctx->box_stages * stage + obuf + (size_t)ctx->box_L * bte::kBoxCells) *

@@ -271,9 +271,13 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
         if (ctx->td) ctx->rsel = 1 - ctx->rsel;
         return BTE_OK;
     }
+    ev_mark(ctx, kPhNewton, true);
+    if (step && !E_or_null) {  // the slot sum in parallel first (one thread per cell sums them serially)
+        STATUS_TRY(reduce_slots(ctx));
+        E_or_null = ctx->E;
+    }
     bte::NewtonParams q = newton_params(ctx, E_or_null, step);
     if (step) q.done = ctx->d_done;  // the step's last kernel
-    ev_mark(ctx, kPhNewton, true);
     STATUS_TRY(launch_newton_cells(ctx, q));
     ev_mark(ctx, kPhNewton, false);
     if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
@@ -320,9 +324,8 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
 }
 
 bte_status reduce_slots(bte_ctx *ctx) {
-    const int tb = 256;
-    bte::sum_slots_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(ctx->part, ctx->n_slots_step, ctx->nc,
-                                                                           ctx->E, ctx->d_halt);
+    bte::sum_slots_kernel<<<(ctx->nc + 31) / 32, 32 * bte::kSumSlotWarps, 0, ctx->stream>>>(
+        ctx->part, ctx->n_slots_step, ctx->nc, ctx->E, ctx->d_halt);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;

@@ -37,3 +37,35 @@ def test_short_region_uses_bracketing_samples_and_says_so():
 def test_no_sampler():
     out = _sampler([], n0=0, live=False).summary()
     assert out["sm_mhz"] is None and out["reasons"] == ["nvidia-smi unavailable"]
+
+
+def test_traffic_per_step_from_profiles(tmp_path, monkeypatch):
+    """roofline.traffic = the committed ncu capture of one flux launch of THIS
+    workload x the flux launches of a step; absent workloads give None."""
+    import json
+    prof = tmp_path / "profiles"
+    prof.mkdir()
+    (prof / "ncu_flux_summary.json").write_text(json.dumps(
+        {"C4": {"dram_bytes_per_launch": 4.9e10, "source": "x"}, "C5": {"dram_bytes_per_launch": 6.6e10}}))
+    monkeypatch.setattr(bench, "ROOT", str(tmp_path))
+    assert bench._traffic_from_profiles("C4", 1.0) == (4.9e10, "x")
+    assert bench._traffic_from_profiles("C5", 5.0)[0] == 5 * 6.6e10
+    assert bench._traffic_from_profiles("C3", 1.0) == (None, None)
+
+
+def test_gpus_n_spawns_torchrun(monkeypatch):
+    """`python bench.py --gpus 4` without WORLD_SIZE re-executes itself under
+    torch.distributed.run with 4 ranks on 127.0.0.1."""
+    calls = []
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setattr(sys, "argv", ["bench.py", "--gpus", "4", "--steps", "2"])
+    monkeypatch.setattr(bench.os, "execv", lambda exe, cmd: calls.append(cmd))
+    bench.main()
+    (cmd,) = calls
+    assert cmd[1:3] == ["-m", "torch.distributed.run"] and "--nproc-per-node=4" in cmd
+    assert cmd[cmd.index("--master-addr") + 1] == "127.0.0.1"
+    assert cmd[-4:] == ["--gpus", "4", "--steps", "2"] and cmd[-5].endswith("bench.py")
+
+
+def test_cpu_model_string():
+    assert isinstance(bench._cpu_model(), str) and bench._cpu_model()
