@@ -193,12 +193,15 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     return BTE_OK;
 }
 
-// The step's temperature solve.  Small meshes (fewer cells than ~8 warps of
-// threads per SM): E (the slot sum unless reduced already) -> one warp per cell
-// (newton_warp_kernel) -> the epilogue (T, Tr, I0, rates); measured on B200,
-// C3 (14,400 cells) 0.066 -> 0.053 ms.  Larger meshes: one thread per cell
-// (newton_kernel, one launch; C4 0.16 ms vs 0.21 with warps).  Re-solves of the
-// current state (step = false) use newton_kernel.
+// The step's temperature solve: E (the slot sum, sum_slots_kernel, unless
+// reduced already) -> the per-cell solve into Tg -> newton_finish_kernel (T,
+// Tr, I0, rates; one thread per row x cell).  Small meshes (fewer cells than ~8
+// warps of threads per SM) solve with one warp per cell (newton_lanes_kernel<32>:
+// C3, 14,400 cells, 0.066 -> 0.039 ms per step on B200 with the steps below),
+// larger ones with one thread per cell (newton_kernel; C4: 8 lanes per cell
+// 0.16 ms, 4 lanes 0.18, a warp 0.22, a thread 0.14).  The first evaluation of
+// g reads the stored I0 table, the slot sum runs 8 warps per 32 cells.  Re-solves
+// of the current state (step = false) use newton_kernel with its own epilogue.
 // Lanes per cell of the step's solve: 0 = thread per cell (newton_kernel), else
 // a group of G lanes per cell (newton_lanes_kernel).
 int newton_lanes(const bte_ctx *ctx, int ncells) {
@@ -256,8 +259,8 @@ bte_status launch_newton_warp(bte_ctx *ctx, const bte::NewtonParams &q) {
 }
 
 bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
-    if (step && warp_newton(ctx, ctx->nc)) {
-        ev_mark(ctx, kPhNewton, true);
+    ev_mark(ctx, kPhNewton, true);
+    if (step) {  // E (the slot sum) -> the solve into Tg -> the epilogue (T, Tr, I0, rates) in parallel
         if (!E_or_null) {
             STATUS_TRY(reduce_slots(ctx));
             E_or_null = ctx->E;
@@ -265,22 +268,17 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
         bte::NewtonParams q = newton_params(ctx, E_or_null, true);
         q.T_out = ctx->Tg;
         q.neg_fail = 1;
-        STATUS_TRY(launch_newton_warp(ctx, q));
-        STATUS_TRY(newton_finish(ctx));
+        if (warp_newton(ctx, ctx->nc)) STATUS_TRY(launch_newton_warp(ctx, q));
+        else STATUS_TRY(launch_newton_cells(ctx, q));
+        STATUS_TRY(newton_finish(ctx));  // (counts the step)
         ev_mark(ctx, kPhNewton, false);
         if (ctx->td) ctx->rsel = 1 - ctx->rsel;
         return BTE_OK;
     }
-    ev_mark(ctx, kPhNewton, true);
-    if (step && !E_or_null) {  // the slot sum in parallel first (one thread per cell sums them serially)
-        STATUS_TRY(reduce_slots(ctx));
-        E_or_null = ctx->E;
-    }
-    bte::NewtonParams q = newton_params(ctx, E_or_null, step);
-    if (step) q.done = ctx->d_done;  // the step's last kernel
+    // a re-solve of the current state: one thread per cell, epilogue in place
+    bte::NewtonParams q = newton_params(ctx, E_or_null, false);
     STATUS_TRY(launch_newton_cells(ctx, q));
     ev_mark(ctx, kPhNewton, false);
-    if (ctx->td && step) ctx->rsel = 1 - ctx->rsel;
     return BTE_OK;
 }
 

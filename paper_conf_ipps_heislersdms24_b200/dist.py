@@ -1,9 +1,10 @@
 """Band sharding across ranks: process-group plumbing around the C ABI.
 
 One process per GPU (torch.distributed, launched by torch.distributed.run).
-The library owns the data-path collective (one NCCL all-reduce of the per-cell
-energy per step, L760-763); this module only bootstraps it: rank 0 asks the
-library for an NCCL unique id and the process group broadcasts it.
+The library owns the data-path collectives (reduce-scatter of the per-cell
+energy and all-gather of T per step, L760-763); this module only bootstraps
+them: rank 0 asks the library for an NCCL unique id and the process group
+broadcasts it.  (Ranks that are threads of one process use bte.Group instead.)
 """
 from __future__ import annotations
 
@@ -91,6 +92,7 @@ def make_solver(cfg, pg=None, n_cell_parts=1, **kw):
         cen = cfg.mesh["cell_centre"]
         parts = slab_partition(cen, n_cell_parts) if cfg.mesh["dim"] == 3 else partition_cells(cen, n_cell_parts)
         kw.update(cell_part=parts, n_cell_parts=n_cell_parts)
+    kw.setdefault("device", env_rank_world()[2])  # (one process per GPU: this rank's LOCAL_RANK)
     if pg is None or pg.get_world_size() == 1:
         return bte.solver_from_config(cfg, **kw)
     rank, world = pg.get_rank(), pg.get_world_size()
