@@ -198,7 +198,7 @@ void bte_destroy(bte_ctx *ctx) {
     void *ptrs[] = {ctx->pool, ctx->d_cur_slot, ctx->i0, ctx->T, ctx->E,
                     ctx->part, ctx->staging, ctx->nbr, ctx->nbm, ctx->fcode, ctx->fcode8, ctx->pos, ctx->gx,
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
-                    ctx->d_iter_max, ctx->d_flags, ctx->d_smax, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
+                    ctx->d_iter_max, ctx->d_flags, ctx->d_smax, ctx->t_th, ctx->t_k, ctx->t_ic, ctx->t_rep, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
                     ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls};
     for (void *p : ptrs)
@@ -779,6 +779,30 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(upload(ctx, &ctx->cw_loc, ctx->h_cw));
     CREATE_TRY(upload(ctx, &ctx->Cb, Cb_all));
     CREATE_TRY(upload(ctx, &ctx->theta, theta));
+    {  // temperature-equation terms (constant weights only: not R2 with the rate law)
+        std::vector<double> th_t, k_t, ic_t;
+        std::vector<int32_t> rep_t;
+        if (!(td && o->temp_rule == 0)) {
+            std::vector<int> term_of(nb, -1);
+            for (int b = 0; b < nb; ++b) {
+                for (size_t j = 0; j < th_t.size() && term_of[b] < 0; ++j)
+                    if (th_t[j] == theta[b]) term_of[b] = (int)j;
+                if (term_of[b] < 0) {
+                    term_of[b] = (int)th_t.size();
+                    th_t.push_back(theta[b]);
+                    rep_t.push_back(b);
+                    ic_t.push_back(1.0 / Cb_all[b]);
+                    k_t.push_back(0.0);
+                }
+            }
+            for (int b = 0; b < nb; ++b) k_t[term_of[b]] += cw[b] * Cb_all[b];
+        }
+        ctx->n_terms = (int)th_t.size();
+        CREATE_TRY(upload(ctx, &ctx->t_th, th_t));
+        CREATE_TRY(upload(ctx, &ctx->t_k, k_t));
+        CREATE_TRY(upload(ctx, &ctx->t_ic, ic_t));
+        CREATE_TRY(upload(ctx, &ctx->t_rep, rep_t));
+    }
     CREATE_TRY(upload(ctx, &ctx->cw_all, cw));
     CREATE_TRY(dalloc(ctx, &ctx->i0w, (size_t)nb_loc * std::max(1, ctx->n_iso)));
     CREATE_TRY(dalloc(ctx, &ctx->d_iter_max, 1));

@@ -132,6 +132,11 @@ struct bte_ctx {
     double *cw_loc = nullptr;
     std::vector<double> h_inv_tau, h_vg, h_cw;  // local band-rows
     double *Cb = nullptr, *theta = nullptr, *cw_all = nullptr;
+    // terms of the temperature equation with constant weights: rows with the same
+    // theta (the LA and TA rows of a band) share one expm1; K_j = sum c_b C_b
+    int n_terms = 0;
+    double *t_th = nullptr, *t_k = nullptr, *t_ic = nullptr;  // theta_j, K_j, 1 / C of the representative row
+    int32_t *t_rep = nullptr;                                  // representative row (the I0 table of T^n)
     int32_t *d_iter_max = nullptr;
     // d_flags[0] fail (a temperature solve failed), [1] halt (the fail flag as the
     // step's flux launch saw it: the rest of the step is a no-op), [2] steps done

@@ -9,21 +9,8 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     if (p.halt && *p.halt) return;
     if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);
     extern __shared__ double sm[];
-    double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
-    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
-    double *sIC = sm + 7 * p.nb;  // 1 / C_b
-    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
-        sIC[b] = 1.0 / p.Cb[b];
-        sC[b] = p.Cb[b];
-        sTh[b] = p.theta[b];
-        sW[b] = p.cw[b];
-        if (p.td) {
-            sA[b] = p.ra[b];
-            sB[b] = p.rb[b];
-            sR[b] = p.rth[b];
-            sV[b] = p.inv_v[b];
-        }
-    }
+    const SolveTables tb = solve_tables(sm, p.nb, p.n_terms);
+    load_solve_tables(tb, p);
     __syncthreads();
     const int cl = blockIdx.x * blockDim.x + threadIdx.x;  // chunk-local index
     if (cl >= p.nc) return;
@@ -36,18 +23,18 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
     }
     const double T0 = p.T[c];
-    Weights wt{sW, sA, sB, sR, sV, p.td && p.r2, 0.0};
+    double Tw = 0.0;
     if (p.td) {
-        wt.Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
+        Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
         if (p.tr_step && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
     }
+    const Terms t = solve_terms(tb, p, Tw);
     double T = T0;
     bool ok = false;
     int it = 0;
     const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = tab ? g_eval_table(sIC, sTh, wt, p.nb, p.W, E, T, tab, p.nc_tab)
-                            : g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+        const Gsum gs = tab ? g_eval_table(t, p.W, E, T, tab, p.nc_tab) : g_eval(t, p.W, E, T);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -56,8 +43,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = (it == 1 && tab) ? g_eval_table(sIC, sTh, wt, p.nb, p.W, E, T, tab, p.nc_tab)
-                                             : g_eval(sC, sTh, wt, p.nb, p.W, E, T);
+            const Gsum gs = (it == 1 && tab) ? g_eval_table(t, p.W, E, T, tab, p.nc_tab) : g_eval(t, p.W, E, T);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -66,12 +52,12 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
-            if (g_only(sC, sTh, wt, p.nb, p.W, E, lo) <= 0.0 && g_only(sC, sTh, wt, p.nb, p.W, E, hi) >= 0.0) {
+            for (int k = 0; k < 2000 && g_only(t, p.W, E, lo) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only(t, p.W, E, hi) < 0.0; ++k) hi *= 2.0;
+            if (g_only(t, p.W, E, lo) <= 0.0 && g_only(t, p.W, E, hi) >= 0.0) {
                 for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
                     const double mid = 0.5 * (lo + hi);
-                    if (g_only(sC, sTh, wt, p.nb, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
+                    if (g_only(t, p.W, E, mid) < 0.0) lo = mid; else hi = mid;
                 }
                 T = 0.5 * (lo + hi);
                 ok = true;
@@ -92,10 +78,11 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     const double iT = 1.0 / T;
     for (int k = 0; k < p.nb_loc; ++k) {
         const int b = p.b_lo + k;
-        p.i0[(size_t)k * p.nc + c] = sC[b] / expm1(sTh[b] * iT);
-        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(sA[b], sB[b], sR[b], T);
+        p.i0[(size_t)k * p.nc + c] = tb.C[b] / expm1(tb.th[b] * iT);
+        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(tb.a[b], tb.b[b], tb.r[b], T);
     }
 }
+
 
 __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__restrict__ T, int nc, int b_lo,
                                      int nb_loc, const double *__restrict__ Cb, const double *__restrict__ theta,

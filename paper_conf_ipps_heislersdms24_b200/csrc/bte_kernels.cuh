@@ -1142,6 +1142,10 @@ struct NewtonParams {
     // of nb expm1 (I0 = C / expm1(x), 1 / expm1(x) = I0 / C)
     const double *i0_t0;
     int32_t nc_tab;
+    // terms of the temperature equation with constant weights (see Terms; 0: per row)
+    int32_t n_terms;
+    const double *t_th, *t_k, *t_ic;
+    const int32_t *t_rep;
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1151,53 +1155,108 @@ __device__ __forceinline__ double tau_rate(double a, double b, double th, double
 
 struct Gsum { double g, gp; };
 
-// g(T) = W sum_b c_b I0_b(T) - E and g'(T), I0 = C / expm1(theta/T),
-// I0' = I0 (x/T) (1 + 1/expm1(x)), x = theta/T.
-// Band weights of the temperature equation: the constant c_b (sW), or with the
-// rate law under R2, rate_b(Tw) / v_b at the cell's rate temperature Tw.
-struct Weights {
-    const double *sW, *ra, *rb, *rth, *iv;
-    bool law;
+// The temperature equation g(T) = W sum_j K_j I0(theta_j; T) / C_j - E as a sum
+// of TERMS j: with constant weights the rows that share theta (the LA and TA
+// rows of a band: 55 rows, 40 terms for the paper's 40 bands) are one term,
+// K_j = sum_{b in j} c_b C_b, so one expm1 serves them (bte_create builds the
+// terms); with the rate law under R2 the weights depend on the cell, and the
+// terms are the rows, K_b = rate_b(Tw) / v_b C_b.  With q = 1 / expm1(x),
+// x = theta / T: I0 = C q, dI0/dT = I0 (x / T) (1 + q).
+struct Terms {
+    const double *th, *k, *ic;  // per term: theta_j, K_j (nullptr: per row, c_b C_b), 1 / C of its representative
+    const int32_t *rep;          // representative row (nullptr: the row itself)
+    int n;
+    bool law;                    // per-cell weights: K_b = tau_rate(a, b, th, Tw) iv_b C_b
+    const double *C, *w, *ra, *rb, *rth, *iv;
     double Tw;
-    __device__ __forceinline__ double operator()(int b) const {
-        return law ? tau_rate(ra[b], rb[b], rth[b], Tw) * iv[b] : sW[b];
+    __device__ __forceinline__ double K(int j) const {
+        return law ? tau_rate(ra[j], rb[j], rth[j], Tw) * iv[j] * C[j] : k ? k[j] : w[j] * C[j];
     }
+    __device__ __forceinline__ int row(int j) const { return rep ? rep[j] : j; }
 };
 
-__device__ __forceinline__ Gsum g_eval(const double *sC, const double *sTh, const Weights &wt,
-                                       int nb, double W, double E, double T) {
+// Shared-memory band / term tables of the solve kernels (newton_smem on the host):
+// 8 row arrays [nb] (C, theta, c, rate a / b / theta, 1 / v, 1 / C), then 3 term
+// arrays [n_terms] (theta, K, 1 / C of the representative) and the int32 term
+// representatives.
+struct SolveTables {
+    double *C, *th, *w, *a, *b, *r, *v, *ic, *tth, *tk, *tic;
+    int32_t *trep;
+};
+__device__ __forceinline__ SolveTables solve_tables(double *sm, int nb, int nt) {
+    SolveTables t;
+    t.C = sm; t.th = sm + nb; t.w = sm + 2 * nb; t.a = sm + 3 * nb; t.b = sm + 4 * nb;
+    t.r = sm + 5 * nb; t.v = sm + 6 * nb; t.ic = sm + 7 * nb;
+    t.tth = sm + 8 * nb; t.tk = t.tth + nt; t.tic = t.tk + nt;
+    t.trep = reinterpret_cast<int32_t *>(t.tic + nt);
+    return t;
+}
+__device__ __forceinline__ void load_solve_tables(const SolveTables &t, const NewtonParams &p) {
+    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
+        t.ic[b] = 1.0 / p.Cb[b];
+        t.C[b] = p.Cb[b];
+        t.th[b] = p.theta[b];
+        t.w[b] = p.cw[b];
+        if (p.td) {
+            t.a[b] = p.ra[b];
+            t.b[b] = p.rb[b];
+            t.r[b] = p.rth[b];
+            t.v[b] = p.inv_v[b];
+        }
+    }
+    for (int j = threadIdx.x; j < p.n_terms; j += blockDim.x) {
+        t.tth[j] = p.t_th[j];
+        t.tk[j] = p.t_k[j];
+        t.tic[j] = p.t_ic[j];
+        t.trep[j] = p.t_rep[j];
+    }
+}
+// The terms of a cell's solve (Tw: the rate temperature of its weights).
+__device__ __forceinline__ Terms solve_terms(const SolveTables &t, const NewtonParams &p, double Tw) {
+    Terms q;
+    q.law = p.td && p.r2;
+    const bool terms = !q.law && p.n_terms > 0;  // (else one term per row: the rate law, or other weights)
+    q.th = terms ? t.tth : t.th;
+    q.k = terms ? t.tk : nullptr;
+    q.ic = terms ? t.tic : t.ic;
+    q.rep = terms ? t.trep : nullptr;
+    q.n = terms ? p.n_terms : p.nb;
+    q.C = t.C; q.w = t.w; q.ra = t.a; q.rb = t.b; q.rth = t.r; q.iv = t.v;
+    q.Tw = Tw;
+    return q;
+}
+
+__device__ __forceinline__ Gsum g_eval(const Terms &t, double W, double E, double T) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
-    for (int b = 0; b < nb; ++b) {  // (one reciprocal per row: I0 = C r, I0' = I0 (x/T)(1 + r))
-        const double x = sTh[b] * it;
-        const double r = 1.0 / expm1(x);
-        const double i0 = sC[b] * r;
-        const double wb = wt(b);
-        g = fma(wb, i0, g);
-        gp = fma(wb, i0 * (x * it) * (1.0 + r), gp);
+    for (int j = 0; j < t.n; ++j) {
+        const double x = t.th[j] * it;
+        const double q = 1.0 / expm1(x);
+        const double kq = t.K(j) * q;
+        g += kq;
+        gp = fma(kq, (x * it) * (1.0 + q), gp);
     }
     return {W * g - E, W * gp};
 }
 
-// g, g' at T0 from the stored table i0_t0[b][c] = I0_b(T0).
-__device__ __forceinline__ Gsum g_eval_table(const double *sIC, const double *sTh, const Weights &wt, int nb,
-                                             double W, double E, double T0, const double *i0_t0, int64_t stride) {
+// g, g' at T0 from the stored table i0_t0[b][c] = I0_b(T0) (q = I0 / C).
+__device__ __forceinline__ Gsum g_eval_table(const Terms &t, double W, double E, double T0, const double *i0_t0,
+                                             int64_t stride) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T0;
-    for (int b = 0; b < nb; ++b) {
-        const double x = sTh[b] * it;
-        const double i0 = __ldg(i0_t0 + b * stride);
-        const double wb = wt(b);
-        g = fma(wb, i0, g);
-        gp = fma(wb, i0 * (x * it) * (1.0 + i0 * sIC[b]), gp);
+    for (int j = 0; j < t.n; ++j) {
+        const double x = t.th[j] * it;
+        const double q = __ldg(i0_t0 + t.row(j) * stride) * t.ic[j];
+        const double kq = t.K(j) * q;
+        g += kq;
+        gp = fma(kq, (x * it) * (1.0 + q), gp);
     }
     return {W * g - E, W * gp};
 }
 
-__device__ __forceinline__ double g_only(const double *sC, const double *sTh, const Weights &wt,
-                                         int nb, double W, double E, double T) {
+__device__ __forceinline__ double g_only(const Terms &t, double W, double E, double T) {
     double g = 0.0;
-    for (int b = 0; b < nb; ++b) g = fma(wt(b), sC[b] / expm1(sTh[b] / T), g);
+    for (int j = 0; j < t.n; ++j) g += t.K(j) / expm1(t.th[j] / T);
     return W * g - E;
 }
 
@@ -1205,15 +1264,13 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p);
 
 // ---------------------------------------------------------------------------
 // The same per-cell temperature solve with a GROUP of G lanes per cell (the
-// step's solve; newton_kernel serves the re-solves): lane l of the group
-// evaluates band-rows l, l + G, ... and butterfly shuffles inside the group
-// give every lane bitwise the same sums (each level adds a commutative pair),
-// so the Newton iterates and the bisection safeguard are group-uniform.  A
-// cell's nb rows x ~4 iterations of expm1 are spread over G lanes: small
-// meshes (C3: 14,400 cells, G = 32) fill the GPU instead of a few warps per
-// SM, larger ones (C4) take G = 8.  Output like newton_kernel's chunk solve:
-// T_out[c] = T^{n+1} (or -T^n on failure); the epilogue (T, Tr, I0, rates) is
-// newton_finish_kernel's.
+// step's solve on small meshes): lane l of the group evaluates terms l, l + G,
+// ... and butterfly shuffles inside the group give every lane bitwise the same
+// sums (each level adds a commutative pair), so the Newton iterates and the
+// bisection safeguard are group-uniform.  A cell's terms x ~3 iterations of
+// expm1 are spread over G lanes: small meshes (C3: 14,400 cells, G = 32) fill
+// the GPU instead of a few warps per SM.  Output: T_out[c] = T^{n+1} (or -T^n
+// on failure); the epilogue (T, Tr, I0, rates) is newton_finish_kernel's.
 template <int G>
 __device__ __forceinline__ double group_sum(double v, unsigned mask) {
 #pragma unroll
@@ -1221,54 +1278,35 @@ __device__ __forceinline__ double group_sum(double v, unsigned mask) {
     return v;
 }
 
-// R = band-rows per lane (ceil(nb / G) rounded up to a power of two; the
-// per-lane weights stay in registers).
+// R = terms per lane (ceil(n / G) rounded up to a power of two; the per-lane
+// coefficients K stay in registers).
 template <int G, int R>
-__device__ __forceinline__ Gsum g_eval_group(const double *sC, const double *sTh, const double *wl, int nb, double W,
-                                             double E, double T, int lane, unsigned mask) {
+__device__ __forceinline__ Gsum g_eval_group(const Terms &t, const double *kl, double W, double E, double T, int lane,
+                                             unsigned mask, const double *tab, int64_t stride) {
     double g = 0.0, gp = 0.0;
     const double it = 1.0 / T;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + G * r;
-        if (b < nb) {
-            const double x = sTh[b] * it;
-            const double q = 1.0 / expm1(x);
-            const double i0 = sC[b] * q;
-            g = fma(wl[r], i0, g);
-            gp = fma(wl[r], i0 * (x * it) * (1.0 + q), gp);
+        const int j = lane + G * r;
+        if (j < t.n) {
+            const double x = t.th[j] * it;
+            const double q = tab ? __ldg(tab + t.row(j) * stride) * t.ic[j] : 1.0 / expm1(x);
+            const double kq = kl[r] * q;
+            g += kq;
+            gp = fma(kq, (x * it) * (1.0 + q), gp);
         }
     }
     return {W * group_sum<G>(g, mask) - E, W * group_sum<G>(gp, mask)};
 }
 
 template <int G, int R>
-__device__ __forceinline__ Gsum g_eval_group_table(const double *sIC, const double *sTh, const double *wl, int nb,
-                                                   double W, double E, double T0, int lane, unsigned mask,
-                                                   const double *i0_t0, int64_t stride) {
-    double g = 0.0, gp = 0.0;
-    const double it = 1.0 / T0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const int b = lane + G * r;
-        if (b < nb) {
-            const double x = sTh[b] * it;
-            const double i0 = __ldg(i0_t0 + b * stride);
-            g = fma(wl[r], i0, g);
-            gp = fma(wl[r], i0 * (x * it) * (1.0 + i0 * sIC[b]), gp);
-        }
-    }
-    return {W * group_sum<G>(g, mask) - E, W * group_sum<G>(gp, mask)};
-}
-
-template <int G, int R>
-__device__ __forceinline__ double g_only_group(const double *sC, const double *sTh, const double *wl, int nb,
-                                               double W, double E, double T, int lane, unsigned mask) {
+__device__ __forceinline__ double g_only_group(const Terms &t, const double *kl, double W, double E, double T,
+                                               int lane, unsigned mask) {
     double g = 0.0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + G * r;
-        if (b < nb) g = fma(wl[r], sC[b] / expm1(sTh[b] / T), g);
+        const int j = lane + G * r;
+        if (j < t.n) g += kl[r] / expm1(t.th[j] / T);
     }
     return W * group_sum<G>(g, mask) - E;
 }
@@ -1277,21 +1315,8 @@ template <int G, int R>
 __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     if (p.halt && *p.halt) return;
     extern __shared__ double sm[];
-    double *sC = sm, *sTh = sm + p.nb, *sW = sm + 2 * p.nb;
-    double *sA = sm + 3 * p.nb, *sB = sm + 4 * p.nb, *sR = sm + 5 * p.nb, *sV = sm + 6 * p.nb;
-    double *sIC = sm + 7 * p.nb;  // 1 / C_b
-    for (int b = threadIdx.x; b < p.nb; b += blockDim.x) {
-        sIC[b] = 1.0 / p.Cb[b];
-        sC[b] = p.Cb[b];
-        sTh[b] = p.theta[b];
-        sW[b] = p.cw[b];
-        if (p.td) {
-            sA[b] = p.ra[b];
-            sB[b] = p.rb[b];
-            sR[b] = p.rth[b];
-            sV[b] = p.inv_v[b];
-        }
-    }
+    const SolveTables tb = solve_tables(sm, p.nb, p.n_terms);
+    load_solve_tables(tb, p);
     __syncthreads();
     const int lane = threadIdx.x & (G - 1);
     const unsigned mask = G == 32 ? 0xffffffffu : ((1u << G) - 1u) << ((threadIdx.x & 31) & ~(G - 1));
@@ -1307,21 +1332,19 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
         E = group_sum<G>(E, mask);
     }
     const double T0 = p.T[c];
-    const bool law = p.td && p.r2;
-    const double Tw = p.td ? (p.tr_step ? T0 : p.Tr[c]) : 0.0;  // a step: weights at T^n
-    double wl[R];
+    const Terms t = solve_terms(tb, p, p.td ? (p.tr_step ? T0 : p.Tr[c]) : 0.0);  // a step: weights at T^n
+    double kl[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const int b = lane + G * r;
-        wl[r] = b >= p.nb ? 0.0 : law ? tau_rate(sA[b], sB[b], sR[b], Tw) * sV[b] : sW[b];
+        const int j = lane + G * r;
+        kl[r] = j < t.n ? t.K(j) : 0.0;
     }
+    const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     double T = T0;
     bool ok = false;
     int it = 0;
-    const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
-        const Gsum gs = tab ? g_eval_group_table<G, R>(sIC, sTh, wl, p.nb, p.W, E, T, lane, mask, tab, p.nc_tab)
-                            : g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
+        const Gsum gs = g_eval_group<G, R>(t, kl, p.W, E, T, lane, mask, tab, p.nc_tab);
         const double Tn = T - gs.g / gs.gp;
         it = 1;
         if (Tn > 0.0 && isfinite(Tn)) {
@@ -1330,9 +1353,7 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
         }
     } else if (E > 0.0 && isfinite(E)) {
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = (it == 1 && tab)
-                                ? g_eval_group_table<G, R>(sIC, sTh, wl, p.nb, p.W, E, T, lane, mask, tab, p.nc_tab)
-                                : g_eval_group<G, R>(sC, sTh, wl, p.nb, p.W, E, T, lane, mask);
+            const Gsum gs = g_eval_group<G, R>(t, kl, p.W, E, T, lane, mask, it == 1 ? tab : nullptr, p.nc_tab);
             const double delta = gs.g / gs.gp;
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
@@ -1341,15 +1362,13 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
-            for (int k = 0; k < 2000 && g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, lo, lane, mask) > 0.0; ++k)
-                lo *= 0.5;
-            for (int k = 0; k < 2000 && g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, hi, lane, mask) < 0.0; ++k)
-                hi *= 2.0;
-            if (g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, lo, lane, mask) <= 0.0 &&
-                g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, hi, lane, mask) >= 0.0) {
+            for (int k = 0; k < 2000 && g_only_group<G, R>(t, kl, p.W, E, lo, lane, mask) > 0.0; ++k) lo *= 0.5;
+            for (int k = 0; k < 2000 && g_only_group<G, R>(t, kl, p.W, E, hi, lane, mask) < 0.0; ++k) hi *= 2.0;
+            if (g_only_group<G, R>(t, kl, p.W, E, lo, lane, mask) <= 0.0 &&
+                g_only_group<G, R>(t, kl, p.W, E, hi, lane, mask) >= 0.0) {
                 for (int k = 0; k < 400 && (hi - lo) > p.rtol * hi; ++k) {
                     const double mid = 0.5 * (lo + hi);
-                    if (g_only_group<G, R>(sC, sTh, wl, p.nb, p.W, E, mid, lane, mask) < 0.0) lo = mid; else hi = mid;
+                    if (g_only_group<G, R>(t, kl, p.W, E, mid, lane, mask) < 0.0) lo = mid; else hi = mid;
                 }
                 T = 0.5 * (lo + hi);
                 ok = true;

@@ -194,12 +194,13 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
 }
 
 // The step's temperature solve: E (the slot sum, sum_slots_kernel, unless
-// reduced already) -> the per-cell solve into Tg -> newton_finish_kernel (T,
-// Tr, I0, rates; one thread per row x cell).  Small meshes (fewer cells than ~8
-// warps of threads per SM) solve with one warp per cell (newton_lanes_kernel<32>:
-// C3, 14,400 cells, 0.066 -> 0.039 ms per step on B200 with the steps below),
-// larger ones with one thread per cell (newton_kernel; C4: 8 lanes per cell
-// 0.16 ms, 4 lanes 0.18, a warp 0.22, a thread 0.14).  The first evaluation of
+// reduced already) -> the per-cell solve.  Small meshes (fewer cells than ~8
+// warps of threads per SM) solve with one warp per cell (newton_lanes_kernel<32>)
+// into Tg, then newton_finish_kernel writes T, Tr, I0 and the rates with one
+// thread per row x cell (C3, 14,400 cells, 0.066 -> 0.039 ms per step on B200
+// with the steps below); larger ones with one thread per cell and the epilogue
+// in the same thread (newton_kernel; C4: 8 lanes per cell 0.16 ms, 4 lanes
+// 0.18, a warp 0.22, a thread 0.14).  The first evaluation of
 // g reads the stored I0 table, the slot sum runs 8 warps per 32 cells.  Re-solves
 // of the current state (step = false) use newton_kernel with its own epilogue.
 // Lanes per cell of the step's solve: 0 = thread per cell (newton_kernel), else
@@ -211,7 +212,7 @@ int newton_lanes(const bte_ctx *ctx, int ncells) {
 bool warp_newton(const bte_ctx *ctx, int ncells) { return newton_lanes(ctx, ncells) > 0; }
 
 // Band constants in shared memory: C, theta, c_b (+ the four rate-law arrays).
-size_t newton_smem(const bte_ctx *ctx) { return (size_t)8 * ctx->nb * sizeof(double); }
+size_t newton_smem(const bte_ctx *ctx) { return (size_t)(8 * ctx->nb + 4 * ctx->n_terms) * sizeof(double); }
 
 // Thread-per-cell solve over q.nc cells (block 0 counts the step when q.done).
 bte_status launch_newton_cells(bte_ctx *ctx, const bte::NewtonParams &q) {
@@ -238,7 +239,7 @@ bte_status launch_newton_lanes_gr(bte_ctx *ctx, const bte::NewtonParams &q) {
 
 template <int G>
 bte_status launch_newton_lanes_g(bte_ctx *ctx, const bte::NewtonParams &q) {
-    const int r = (ctx->nb + G - 1) / G;
+    const int r = ((q.n_terms > 0 ? q.n_terms : ctx->nb) + G - 1) / G;
     if (r <= 2) return launch_newton_lanes_gr<G, 2>(ctx, q);
     if (r <= 4) return launch_newton_lanes_gr<G, 4>(ctx, q);
     if (r <= 8) return launch_newton_lanes_gr<G, 8>(ctx, q);
@@ -249,11 +250,12 @@ bte_status launch_newton_lanes_g(bte_ctx *ctx, const bte::NewtonParams &q) {
 
 bte_status launch_newton_warp(bte_ctx *ctx, const bte::NewtonParams &q) {
     if (q.nc <= 0) return BTE_OK;
-    static_assert(bte::kMaxBands <= 32 * 32, "group solve: at most 32 band-rows per lane");
+    static_assert(bte::kMaxBands <= 32 * 32, "group solve: at most 32 terms per lane");
+    const int n = q.n_terms > 0 ? q.n_terms : ctx->nb;  // terms a cell's solve sums
     switch (newton_lanes(ctx, q.nc)) {
-        case 4: return ctx->nb <= 64 ? launch_newton_lanes_g<4>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
-        case 8: return ctx->nb <= 128 ? launch_newton_lanes_g<8>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
-        case 16: return ctx->nb <= 256 ? launch_newton_lanes_g<16>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
+        case 4: return n <= 64 ? launch_newton_lanes_g<4>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
+        case 8: return n <= 128 ? launch_newton_lanes_g<8>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
+        case 16: return n <= 256 ? launch_newton_lanes_g<16>(ctx, q) : launch_newton_lanes_g<32>(ctx, q);
         default: return launch_newton_lanes_g<32>(ctx, q);
     }
 }
@@ -266,11 +268,15 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
             E_or_null = ctx->E;
         }
         bte::NewtonParams q = newton_params(ctx, E_or_null, true);
-        q.T_out = ctx->Tg;
-        q.neg_fail = 1;
-        if (warp_newton(ctx, ctx->nc)) STATUS_TRY(launch_newton_warp(ctx, q));
-        else STATUS_TRY(launch_newton_cells(ctx, q));
-        STATUS_TRY(newton_finish(ctx));  // (counts the step)
+        if (warp_newton(ctx, ctx->nc)) {  // solve into Tg, then the epilogue over (row, cell)
+            q.T_out = ctx->Tg;
+            q.neg_fail = 1;
+            STATUS_TRY(launch_newton_warp(ctx, q));
+            STATUS_TRY(newton_finish(ctx));  // (counts the step)
+        } else {  // one thread per cell, epilogue in the same thread (C4: 0.13 vs 0.16 ms with the finish)
+            q.done = ctx->d_done;
+            STATUS_TRY(launch_newton_cells(ctx, q));
+        }
         ev_mark(ctx, kPhNewton, false);
         if (ctx->td) ctx->rsel = 1 - ctx->rsel;
         return BTE_OK;
@@ -318,6 +324,11 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
         q.i0_t0 = ctx->i0;
         q.nc_tab = ctx->nc;
     }
+    q.n_terms = ctx->n_terms;
+    q.t_th = ctx->t_th;
+    q.t_k = ctx->t_k;
+    q.t_ic = ctx->t_ic;
+    q.t_rep = ctx->t_rep;
     return q;
 }
 
