@@ -591,11 +591,15 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->bzside[1] = bx.zside[1];
         ctx->bflat = bx.flat;
         ctx->n_orb = (int)orbs.size();
-        // shared memory for 2 CTAs per SM: ring stages x 12 KB + 16 KB output + L x 2 KB energy
-        // (rate law: 16 KB stages; 5 stages x 4 layers fit twice per SM, measured best)
+        // shared memory for 2 CTAs per SM (3-D): ring stages x 12 KB + L x 2 KB energy rows
+        // (rate law: 16 KB stages x 4 layers)
         const char *ev = std::getenv("BTE_BOX_STAGES");
-        // (2-D, 3 CTAs per SM: 4 stages, 3 with the rate rows; orbit chunks of 25 (a C3 slice = 4 chunks))
-        const int def_stages = bx.flat ? (td ? 3 : 4) : (td ? 5 : 6);
+        // (2-D, 3 CTAs per SM: 3 stages; orbit chunks of 25 (a C3 slice = 4 chunks).  Measured on B200
+        // with the direct stores, round 2: C4 5 stages 7.22 ms, 6 stages 7.63, 4 stages 8.05 -- a
+        // deeper ring lets the producer run ahead and the halo rows of the boxes are re-read from
+        // DRAM, a shallower one exposes the load latency; C5 5: 52.2 ms, 6: 52.9; C3 3: 0.814 ms,
+        // 4: 0.830, 5: 0.840)
+        const int def_stages = bx.flat ? 3 : 5;
         ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : def_stages));
         if (bx.flat) ctx->box_oc = 25;
         ev = std::getenv("BTE_BOX_L");
