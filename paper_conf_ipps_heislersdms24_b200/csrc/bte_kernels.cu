@@ -48,7 +48,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
             T = Tn;
-            if (fabs(delta) <= p.rtol * T) { ok = true; break; }
+            if (fabs(delta) <= p.rtol * T || fabs(delta) <= p.rtol_q * T) { ok = true; break; }
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;

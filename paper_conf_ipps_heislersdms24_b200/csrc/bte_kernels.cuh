@@ -642,12 +642,6 @@ constexpr int kBoxPlane = 320;               // doubles per staged plane (128-by
 constexpr int kBoxCells = kBoxTX * kBoxTY;   // 256 threads compute, one cell each
 constexpr int kBoxThreads = kBoxCells + 32;  // + the producer warp
 constexpr int kBoxMaxStages = 12;
-#ifndef BTE_BOX_LOAD_POLICY
-#define BTE_BOX_LOAD_POLICY 0  // (experiment) L2 policy on the I^n box loads (0: none)
-#endif
-#ifndef BTE_BOX_STORE_HINT
-#define BTE_BOX_STORE_HINT 0  // (experiment) 1: direct stores with an explicit L2 evict-first policy
-#endif
 // How I^{n+1} leaves the box kernel (measured on B200): 3-D grids
 // store straight from registers (coalesced st.global.cs, no per-layer CTA
 // barrier: C4 sustained flux 7.80 -> 7.53 ms); 2-D grids keep the
@@ -661,12 +655,8 @@ constexpr bool box_tma_store() {
     return FLAT;
 #endif
 }
-// (experiment, BTE_BOX_STORE_HINT == 2) direct path through a per-warp shared
-// row + one bulk copy per direction row (no CTA barrier)
 template <bool FLAT>
-constexpr bool box_warp_bulk() { return !box_tma_store<FLAT>() && BTE_BOX_STORE_HINT == 2; }
-template <bool FLAT>
-constexpr bool box_obuf() { return box_tma_store<FLAT>() || box_warp_bulk<FLAT>(); }
+constexpr bool box_obuf() { return box_tma_store<FLAT>(); }  // (the shared output tile of the tensor stores)
 // Resident CTAs per SM the kernel is compiled for (register cap): 3-D grids 2
 // (96 registers, 6 stages of 12 KB plus L x 2 KB of energy rows); 2-D grids 3
 // (72 registers, no spills, 4 stages): a 2-D stage is one layer, so CTAs are
@@ -724,16 +714,6 @@ __device__ __forceinline__ void tma_load_5d(void *dst, const void *tmap, int c0,
         "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
         " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
-        : "memory");
-}
-// The same with an L2 cache policy (createpolicy) on the loaded lines.
-__device__ __forceinline__ void tma_load_5d_hint(void *dst, const void *tmap, int c0, int c1, int c2, int c3, int c4,
-                                                 uint64_t *bar, uint64_t pol) {
-    asm volatile(
-        "cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
-        " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar)),
-        "l"(pol)
         : "memory");
 }
 __device__ __forceinline__ void tma_load_3d(void *dst, const void *tmap, int c0, int c1, int c2, uint64_t *bar) {
@@ -843,7 +823,6 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     double *ring = bsm;                          // [S][kStage]
     constexpr bool kTmaStore = box_tma_store<FLAT>();
     double *obuf = ring + S * kStage;                           // [2][4][256] (tensor stores)
-    constexpr bool kWarpBulk = box_warp_bulk<FLAT>();
     double *eacc = obuf + (box_obuf<FLAT>() ? 2 * 4 * kBoxCells : 0);  // [L][256]
     BoxOrbitC *sorb = reinterpret_cast<BoxOrbitC *>(eacc + p.L * kBoxCells);  // [orb_chunk]
     __shared__ __align__(8) uint64_t full[kBoxMaxStages];
@@ -879,20 +858,6 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
 
     if (tid >= kBoxCells) {  // ------------------------------------------- producer warp
         if (tid == kBoxCells) {
-#if BTE_BOX_LOAD_POLICY
-            // (experiment) L2 policy of the I^n boxes: 1 evict_last, 2 evict_normal, 3 evict_first
-            uint64_t lpol;
-#if BTE_BOX_LOAD_POLICY == 1
-            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(lpol));
-#elif BTE_BOX_LOAD_POLICY == 2
-            asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(lpol));
-#else
-            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(lpol));
-#endif
-#define BOX_LOAD_IN(dst, map, a, b, c, d, e, bar) tma_load_5d_hint(dst, map, a, b, c, d, e, bar, lpol)
-#else
-#define BOX_LOAD_IN(dst, map, a, b, c, d, e, bar) tma_load_5d(dst, map, a, b, c, d, e, bar)
-#endif
             int s = 0;
             uint32_t ph = 0, wrapped = 0;  // ring slot, its use parity, ring wrapped once
             for (int k = w.k0; k < w.k1; ++k) {
@@ -911,7 +876,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             for (int q = 0; q < 4; ++q) {
                                 const int xs = w.x0 - box_xs(q), ys = w.y0 - box_hy(q);
                                 if (zh >= 0 && zh < p.n2)
-                                    BOX_LOAD_IN(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
+                                    tma_load_5d(st + q * kBoxPlane, &tm_in, xs, ys, zh, ob.d[q], slab, &full[s]);
                                 else if (p.zside[asc ? 0 : 1] == 0)  // isothermal: I0_b(T_wall) side table
                                     tma_load_4d(st + q * kBoxPlane, &tm_side, xs, ys, asc ? 0 : 1, bl, &full[s]);
                                 else  // specular: the wall layer of the z-mirrored direction (old level)
@@ -928,7 +893,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                             if (glo) tma_load_3d(st + kGhost, &tm_side, w.x0, 0, bl, &full[s]);
                             if (ghi) tma_load_3d(st + kGhost + kBoxTX, &tm_side, w.x0, 1, bl, &full[s]);
                             for (int q = 0; q < 4; ++q)
-                                BOX_LOAD_IN(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
+                                tma_load_5d(st + q * kBoxPlane, &tm_in, w.x0 - box_xs(q), w.y0 - box_hy(q), z,
                                             ob.d[q], slab, &full[s]);
                             tma_load_4d(st + 4 * kBoxPlane, &tm_i0, w.x0, w.y0, z - p.zlo, bl, &full[s]);
                             if (TD) {
@@ -971,10 +936,6 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     // direct stores: a warp's 32 cells are one 256-byte row of a plane
     const int32_t plane = p.n0 * p.n1;
     const int32_t cell_off = gy * p.n0 + gx;
-#if BTE_BOX_STORE_HINT
-    uint64_t spol;  // (experiment) L2 evict-first policy for the direct stores
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(spol));
-#endif
 
     int s = 0, sp = 0;
     uint32_t ph = 0, ob = 0;
@@ -1027,14 +988,8 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         if (!flat) infl = fma(m2, pv[q], infl);
                         pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
-                        if constexpr (kTmaStore || kWarpBulk) out[q * kBoxCells + tid] = inew;
-#if BTE_BOX_STORE_HINT == 1
-                        else if (valid)
-                            asm volatile("st.global.L1::no_allocate.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(orow + doff[q]),
-                                         "d"(inew), "l"(spol) : "memory");
-#else
+                        if constexpr (kTmaStore) out[q * kBoxCells + tid] = inew;
                         else if (valid) __stcs(orow + doff[q], inew);
-#endif
                         acc = fma(wq[q], inew, acc);
                     }
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
@@ -1051,30 +1006,6 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                         }
                     }
                     sp = s;
-#if BTE_BOX_STORE_HINT == 2
-                    if constexpr (kWarpBulk) {  // this warp's 4 rows leave by bulk copies
-                        fence_smem_to_async();
-                        __syncwarp();
-                        const bool full_row = w.x0 + kBoxTX <= p.n0 && gy < p.n1;
-                        if (lane == 0 && full_row) {
-#pragma unroll
-                            for (int q = 0; q < 4; ++q)
-                                asm volatile(
-                                    "cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], 256, %2;" ::"l"(
-                                        orow + doff[q] - tx),
-                                    "r"(smem_u32(out + q * kBoxCells + ty * 32)), "l"(spol)
-                                    : "memory");
-                            bulk_commit();
-                        }
-                        if (!full_row && valid)  // ragged rows: plain stores
-#pragma unroll
-                            for (int q = 0; q < 4; ++q) __stcs(orow + doff[q], out[q * kBoxCells + tid]);
-                        ob ^= 1u;
-                        // before this warp rewrites the other buffer: its copies have read it
-                        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
-                        __syncwarp();
-                    }
-#endif
                     if constexpr (kTmaStore) {
                         fence_smem_to_async();
                         if (tid == 0) bulk_wait_read_all();  // the other output buffer has been read
@@ -1101,7 +1032,6 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
             part[((int64_t)(w.z0 - p.zlo + l) * p.n1 + gy) * p.n0 + gx] = eacc[l * kBoxCells + tid];
     }
     if (kTmaStore && tid == 0) bulk_wait_all();
-    if (kWarpBulk && lane == 0) bulk_wait_all();
 }
 
 // ---------------------------------------------------------------- temperature
@@ -1117,6 +1047,12 @@ struct NewtonParams {
     int32_t b_lo, nb_loc;
     const double *Cb, *theta, *cw;  // [nb] global
     double W, rtol;
+    // Newton converges quadratically near the root: after a step of |dT| <= rtol_q T
+    // the new iterate's error is ~ kappa dT^2 / T with kappa = T |g''| / 2|g'| ~ (x - 2) / 2,
+    // x = theta / T (5 at x = 12); with rtol_q = 0.1 sqrt(rtol) that is below rtol T for
+    // kappa <= 100 (T above ~1 % of the largest theta), so it is accepted without the
+    // confirming evaluation the |dT| <= rtol T test needs (reading 25)
+    double rtol_q;
     int32_t maxit;
     int32_t *iter_max;
     int32_t *fail;
@@ -1358,7 +1294,7 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
             const double Tn = T - delta;
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
             T = Tn;
-            if (fabs(delta) <= p.rtol * T) { ok = true; break; }
+            if (fabs(delta) <= p.rtol * T || fabs(delta) <= p.rtol_q * T) { ok = true; break; }
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;

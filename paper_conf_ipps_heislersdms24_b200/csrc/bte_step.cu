@@ -315,6 +315,7 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     q.cw = ctx->cw_all;
     q.W = ctx->W;
     q.rtol = ctx->opt.newton_rtol;
+    q.rtol_q = 0.1 * std::sqrt(ctx->opt.newton_rtol);
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
