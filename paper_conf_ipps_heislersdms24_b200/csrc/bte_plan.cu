@@ -198,14 +198,7 @@ BoxKernel box_kernel(const bte_ctx *ctx) {
 
 bte_status box_setup_kernel(bte_ctx *ctx) {
     const size_t smem = box_smem(ctx);
-    // the attribute is per function, shared by every context of the process: only ever raise it
-    // (contexts with different layer ranges need different amounts)
-    static std::map<const void *, size_t> granted;
-    size_t &g = granted[(const void *)box_kernel(ctx)];
-    if (smem > g) {
-        CUDA_TRY(ctx, cudaFuncSetAttribute(box_kernel(ctx), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        g = smem;
-    }
+    CUDA_TRY(ctx, ensure_smem((const void *)box_kernel(ctx), smem));  // (per device, raised only)
     int occ = 0;
     CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, box_kernel(ctx), bte::kBoxThreads, smem));
     ctx->box_ctas_per_sm = std::max(1, occ);
