@@ -598,8 +598,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         // with the direct stores, round 2: C4 5 stages 7.22 ms, 6 stages 7.63, 4 stages 8.05 -- a
         // deeper ring lets the producer run ahead and the halo rows of the boxes are re-read from
         // DRAM, a shallower one exposes the load latency; C5 5: 52.2 ms, 6: 52.9; C3 3: 0.814 ms,
-        // 4: 0.830, 5: 0.840)
-        const int def_stages = bx.flat ? 3 : 5;
+        // 4: 0.830, 5: 0.840; the rate law's 16 KB stages: C4 6 stages 8.03 ms, 5: 8.21, 4: 8.85)
+        const int def_stages = bx.flat ? 3 : td ? 6 : 5;
         ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : def_stages));
         if (bx.flat) ctx->box_oc = 25;
         ev = std::getenv("BTE_BOX_L");

@@ -1,24 +1,31 @@
-// bte_kernels.cuh -- sm_100a kernels of the explicit phonon-BTE step.
+// bte_kernels.cuh -- sm_100a kernels of the explicit phonon-BTE step
+// (templates, device helpers, parameter blocks; the non-template kernels are
+// defined in bte_kernels.cu).
 //
 // Paper: E. Heisler et al., IPDPS 2024; "Lnnn" = line of PAPER.md.
 //
-//   flux_kernel    Eq. 3 / Eq. 5 forward-Euler update with the first-order
-//                  upwind face flux (L264-292, L529-553, L644-647), the RTA
-//                  source (I0 - I)/tau, the Eq. 6 ghosts on boundary cells
-//                  (L563-607) and the fused per-cell energy partial
-//                  sum_b c_b sum_d w_d I' (L412-418).  HBM-bound: 16 B per
-//                  (cell, dir, band) update (read I^n, write I^{n+1}).
-//   newton_kernel  per-cell temperature from the energy (L407-418, L555-561,
-//                  L707-716) and the I0 table of the next step.
-//   small kernels  reductions, gathers/scatters into caller cell order,
-//                  equilibrium initialisation, isothermal ghost table, dt bound.
+// Every flux kernel computes the Eq. 3 / Eq. 5 forward-Euler update with the
+// first-order upwind face flux (L264-292, L529-553, L644-647), the RTA source
+// (I0 - I)/tau, the Eq. 6 ghosts on boundary faces (L563-607) and the fused
+// per-cell energy partial sum_b c_b sum_d w_d I' (L412-418).  HBM-bound: 16 B
+// per (cell, dir, band) update (read I^n, write I^{n+1}).
+//   flux_box_kernel          structured 2-D / 3-D grids (the paper's meshes):
+//                            z-marching 32 x 8 tiles, tensor-copied halo boxes
+//   flux_tma_kernel          any mesh whose faces come in opposite pairs: 256-cell
+//                            tiles staged by bulk copies
+//   flux_tma_generic_kernel  any face-based mesh (triangles, split faces): tile +
+//                            halo + ghosts staged by the producer warp
+//   flux_kernel              register-pipelined fallback (generic faces)
+//   newton_kernel / newton_lanes_kernel / newton_finish_kernel
+//                            per-cell temperature from the energy (L407-418,
+//                            L555-561, L707-716) and the I0 table of the next step
+//   small kernels            slot sums, reductions, gathers / scatters into caller
+//                            cell order, equilibrium initialisation, ghost tables,
+//                            dt bound, halo pack / unpack
 //
-// Layout: I slab of band-row b = [n_dirs][n_cells] doubles in a
-// slab pool; cells reordered interior-first; per-cell face geometry stored as
-// padded face slots j < MF in struct-of-arrays form [j][cell]:
-//   nbr[j][c] (int32), g[j][c] = (A_f / V_c) n_f (FP64, DIM components),
-//   and for boundary cells kind[j][c] (0 interior, 1 isothermal, 2 symmetric)
-//   and aux[j][c] (isothermal ghost column / reflection-class row).
+// Layout: the slab of band-row b = [n_dirs][plane stride] doubles
+// in a slab pool (cell fastest); per-cell face geometry in struct-of-arrays
+// face slots [j][cell]: nbr (int32), g = (A_f / V_c) n_f (FP64), face codes.
 #pragma once
 #include <cstdint>
 #include <cuda.h>  // CUtensorMap (box kernel tensor maps)
@@ -222,7 +229,7 @@ flux_kernel(const __grid_constant__ FluxParams p) {
 // inside the tile are read from the staged segment; only halo neighbours,
 // specular faces (another direction's plane) and isothermal faces (the I0w
 // table) are global loads, issued at the top of the iteration.  Arithmetic is
-// identical to flux_paired_kernel.
+// the same as flux_kernel's with opposite-face pairs (one inflow face per pair).
 constexpr int kTile = 256;
 #ifndef BTE_TMA_STAGES
 #define BTE_TMA_STAGES 4
@@ -614,7 +621,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
 // L617-621) stored in lexicographic order (axis 0 fastest), axis-0 and axis-1
 // sides specular, axis-2 sides isothermal or specular (each side uniform).
 //
-// Same update as flux_paired_kernel (Eq. 3/5 with the Eq. 6 ghosts, L269-292,
+// Same update as flux_kernel (Eq. 3/5 with the Eq. 6 ghosts, L269-292,
 // L546-576), organised for the bulk-copy tensor engine:
 //  * a CTA owns a tile of 32 x 8 cells (axes 0, 1) and a range of L layers
 //    along axis 2, and marches through the layers in the upwind order of the
@@ -754,7 +761,7 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 __device__ __forceinline__ void fence_smem_to_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void bar_compute() { asm volatile("bar.sync 1, %0;" ::"n"(kBoxCells) : "memory"); }
 
-// Tensor maps (host-encoded, see bte_api.cu):
+// Tensor maps (host-encoded, see bte_create.cu):
 //   tm_in   the slab pool as {n0, n1, n2, nd, n_slabs}, box {34, 9, 1, 1, 1}
 //   tm_out  same tensor, box {32, 8, 1, 1, 1} (stores)
 //   tm_i0   I0 table as {n0, n1, n2, nb_loc}, box {32, 8, 1, 1}
