@@ -772,6 +772,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(upload(ctx, &ctx->gy, gy_h));
     CREATE_TRY(upload(ctx, &ctx->gz, gz_h));
     CREATE_TRY(upload(ctx, &ctx->pos, pos_h));
+    ctx->identity_order = true;
+    for (int32_t i = 0; i < nc && ctx->identity_order; ++i) ctx->identity_order = pos_h[i] == i;
     CREATE_TRY(upload(ctx, &ctx->refl, refl_h));
     CREATE_TRY(upload(ctx, &ctx->twall, twall_h));
     std::vector<double4> dirs_h(nd);

@@ -87,6 +87,7 @@ struct bte_ctx {
     int64_t staging_elems = 0;
     // face slots [mf_t][nc]
     int32_t *nbr = nullptr, *nbm = nullptr, *pos = nullptr;
+    bool identity_order = false;  // internal cell order == the caller's (pos[i] == i): no gather / scatter
     uint32_t *fcode = nullptr;  // paired: 5-bit face codes per cell
     uint8_t *fcode8 = nullptr;  // generic: 8-bit face codes per face slot
     double *gx = nullptr, *gy = nullptr, *gz = nullptr;

@@ -23,6 +23,12 @@ bte_status bte_band_range(const bte_ctx *ctx, int32_t *b_lo, int32_t *b_hi) {
 // rows of nc doubles (device rows of `stride` elements, internal order) <-> host (caller order)
 static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t stride, int64_t rows, double *host) {
     bte_ctx *ctx = const_cast<bte_ctx *>(cctx);
+    if (ctx->identity_order) {  // one strided copy, no gather (and no staging round trip)
+        CUDA_TRY(ctx, cudaMemcpy2DAsync(host, ctx->nc * sizeof(double), dsrc, stride * sizeof(double),
+                                        ctx->nc * sizeof(double), rows, cudaMemcpyDeviceToHost, ctx->stream));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        return BTE_OK;
+    }
     const int64_t per = std::max<int64_t>(1, ctx->staging_elems / ctx->nc);
     for (int64_t r0 = 0; r0 < rows; r0 += per) {
         const int64_t nr = std::min(per, rows - r0);
@@ -40,6 +46,12 @@ static bte_status rows_to_host(const bte_ctx *cctx, const double *dsrc, int64_t 
 }
 
 static bte_status rows_from_host(bte_ctx *ctx, const double *host, int64_t stride, int64_t rows, double *ddst) {
+    if (ctx->identity_order) {  // one strided copy, no scatter (and no staging round trip)
+        CUDA_TRY(ctx, cudaMemcpy2DAsync(ddst, stride * sizeof(double), host, ctx->nc * sizeof(double),
+                                        ctx->nc * sizeof(double), rows, cudaMemcpyHostToDevice, ctx->stream));
+        CUDA_TRY(ctx, cudaStreamSynchronize(ctx->stream));
+        return BTE_OK;
+    }
     const int64_t per = std::max<int64_t>(1, ctx->staging_elems / ctx->nc);
     for (int64_t r0 = 0; r0 < rows; r0 += per) {
         const int64_t nr = std::min(per, rows - r0);
