@@ -42,6 +42,7 @@ class _Problem(C.Structure):
         ("n_bfaces", C.c_int64), ("bkind", C.c_void_p), ("t_wall", C.c_void_p),
         ("temp_rule", C.c_int32), ("newton_rtol", C.c_double), ("newton_maxit", C.c_int32),
         ("rate_a", C.c_void_p), ("rate_b", C.c_void_p), ("rate_theta", C.c_void_p),
+        ("rates_now", C.c_int32),
     ]
 
 
@@ -95,7 +96,7 @@ def _cells(x, nc):
 class Problem:
     """A mesh + band table + direction set + BCs as the oracle sees them."""
 
-    def __init__(self, mesh, bands, dirs, bcs, temp_rule=0, rtol=1e-12, maxit=50):
+    def __init__(self, mesh, bands, dirs, bcs, temp_rule=0, rtol=1e-12, maxit=50, rates_now=False):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -128,6 +129,7 @@ class Problem:
             rate_a=_ptr(k["rate_a"]).value if self.has_rates else None,
             rate_b=_ptr(k["rate_b"]).value if self.has_rates else None,
             rate_theta=_ptr(k["rate_theta"]).value if self.has_rates else None,
+            rates_now=int(bool(rates_now)),
         )
         self._r = None
 

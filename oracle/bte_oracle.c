@@ -283,7 +283,9 @@ int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, do
     for (int64_t step = 0; step < nsteps && rc == ORACLE_OK; ++step) {
         /* Finch loop (L357-372): u_new from u; then the post-step temperature
          * update (L707-716), where I0 and tau become those of the new state
-         * (L666-669; tau one step behind, reading 22); then u = u_new. */
+         * (L666-669; tau one step behind, reading 22, unless rates_now: tau
+         * of the step's own temperature, reading 26); then u = u_new. */
+        if (Tr && p->rates_now) memcpy(Tr, T, sizeof(double) * (size_t)p->n_cells);
         oracle_update_intensity(p, r, T, Tr, I, Inew, dt, 0, p->n_bands);
         if (Tr) memcpy(Tr, T, sizeof(double) * (size_t)p->n_cells);
         oracle_energy(p, Inew, Tr, 0, p->n_bands, E);

@@ -66,6 +66,13 @@ typedef struct {
      * the rates of step n are those of the temperature of step n-1, so the
      * R2 temperature equation and the relaxation use the same rates). */
     const double *rate_a, *rate_b, *rate_theta;
+    /* 0 (default): the rates lag one step (reading 22: step n relaxes with
+     * tau(T^{n-1}), its temperature solve weighs with tau(T^n)).  1: the
+     * literal post-step refresh of the Finch loop (L707-716): I0 and tau are
+     * both refreshed from the new T, so step n relaxes with tau(T^n) and its
+     * solve weighs with tau(T^n) too (Tr = T at the start of every step;
+     * DESIGN.md reading 26). */
+    int32_t rates_now;
 } oracle_problem;
 
 /* return codes */
@@ -108,8 +115,9 @@ int oracle_newton(const oracle_problem *p, const double *E, const double *Tr, do
 void oracle_equilibrium(const oracle_problem *p, const double *T, int32_t b_lo, int32_t b_hi, double *I);
 
 /* Whole explicit steps: I (all bands), T and the rate temperature Tr in/out
- * (Tr may be NULL with constant rates).  Per step: Inew from (I, T, Tr);
- * Tr <- T; E and the Newton solve with the weights at the new Tr; I <- Inew.
+ * (Tr may be NULL with constant rates).  Per step: (rates_now: Tr <- T;)
+ * Inew from (I, T, Tr); Tr <- T; E and the Newton solve with the weights at
+ * the new Tr; I <- Inew.
  * Returns 0 or an error. */
 int oracle_run(const oracle_problem *p, double dt, int64_t nsteps, double *I, double *T, double *Tr);
 

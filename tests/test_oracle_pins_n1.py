@@ -163,3 +163,77 @@ def test_n1_brute_force_dense_operator_with_rate_bookkeeping(oracle_mod):
         assert np.max(np.abs(I / I_ref - 1)) < 1e-13
         assert np.max(np.abs(T / T_ref - 1)) < 1e-12
         assert np.array_equal(Tr, Tr_ref)
+
+
+# ----------------------------------------------------------------- rates_now (reading 26)
+def test_n1_rates_now_t_independent_law_equals_lagged(oracle_mod):
+    """A T-independent law (b = 0): the two rate bookkeepings are the same
+    method, bit for bit (nothing in the rates can lag)."""
+    mesh = gen.gen_mesh((6, 5), (1e-6, 1e-6))
+    dirs = gen.gen_dirs_product(4, 8)
+    bcs = gen.gen_bcs_fig1(mesh, radius=2e-6)
+    bands = dict(gen.gen_bands_custom(omega=[1e13, 3e13, 6e13], vg=[8e3, 6e3, 3e3], tau=1.0, C=[1e5, 3e6, 2e7]),
+                 rate_a=np.array([2.0 ** 40, 2.0 ** 38, 2.0 ** 41]), rate_b=np.zeros(3), rate_theta=np.full(3, 140.0))
+    out = []
+    for now in (False, True):
+        p = oracle_mod.Problem(mesh, bands, dirs, bcs, rates_now=now)
+        I, T, Tr = p.initial_state(300.0, ic_eps=0.2, with_tr=True)
+        dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs)
+        out.append(p.run(I, T, dt, 12, Tr=Tr))
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+
+
+def test_n1_rates_now_equilibrium_invariance(oracle_mod):
+    mesh = gen.gen_mesh((4, 4, 3), (1e-6,) * 3)
+    bands = gen.with_rate_law(gen.gen_bands_si(4))
+    dirs = gen.gen_dirs_product(4, 8)
+    bcs = gen.gen_bcs_fig1(mesh, t_hot=320.0, t_cold=320.0, radius=2e-6)
+    p = oracle_mod.Problem(mesh, bands, dirs, bcs, rates_now=True)
+    T0 = np.full(mesh["n_cells"], 320.0)
+    dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs, t_max=320.0)
+    I, T, _ = p.run(p.equilibrium(T0), T0, dt, 20, Tr=T0)
+    assert np.max(np.abs(I / p.equilibrium(T0) - 1)) < 2e-14 and np.max(np.abs(T / 320.0 - 1)) < 1e-14
+
+
+def test_n1_rates_now_breaks_exact_energy_balance(oracle_mod):
+    """Why the lag is the default: with the rates of the step's own
+    temperature the R2 weights of the solve that produced T^n (rates at
+    T^{n-1}) and the relaxation of step n differ, and the specular-wall energy
+    invariant drifts (while the lagged bookkeeping keeps it to 1e-13)."""
+    mesh = gen.gen_mesh((6, 5), (1e-6, 1e-6))
+    bands = gen.with_rate_law(gen.gen_bands_si(4))
+    dirs = gen.gen_dirs_product(4, 8)
+    bcs = gen.gen_bcs_uniform(mesh, gen.SYMMETRY)
+    drift = []
+    for now in (False, True):
+        p = oracle_mod.Problem(mesh, bands, dirs, bcs, rates_now=now)
+        I0, T0, Tr0 = p.initial_state(300.0, ic_eps=0.4, with_tr=True)
+        dt = 0.5 * gen.cartesian_dt_bound(mesh, bands, dirs, t_max=T0.max() * 1.2)
+        e0 = _total_energy(p, I0, mesh["cell_volume"], bands["vg"])
+        I, _, _ = p.run(I0, T0, dt, 30, Tr=Tr0)
+        drift.append(abs(_total_energy(p, I, mesh["cell_volume"], bands["vg"]) / e0 - 1))
+    assert drift[0] < 1e-13 and drift[1] > 1e-9
+
+
+def test_n1_rates_now_brute_force_dense_operator(oracle_mod):
+    """The dense affine map with the rates of the step's own T, then E and a
+    bisection T with R2 weights at that T, kept independently of the oracle."""
+    mesh = gen.gen_mesh((4, 4), (1e-6, 1e-6))
+    bands = gen.with_rate_law(gen.select_bands(gen.gen_bands_si(3), [0, 1, 3]))
+    dirs = gen.gen_dirs_inplane(8)
+    bcs = gen.gen_bcs_fig1(mesh, radius=2e-6)
+    p = oracle_mod.Problem(mesh, bands, dirs, bcs, rates_now=True)
+    I, T, Tr = p.initial_state(300.0, ic_eps=0.2, with_tr=True)
+    dt = 0.6 * gen.cartesian_dt_bound(mesh, bands, dirs, t_max=360.0)
+    W = dirs["w"].sum()
+    ra, rb, rt = bands["rate_a"], bands["rate_b"], bands["rate_theta"]
+    for _ in range(3):
+        inv_tau = _law(ra[:, None], rb[:, None], rt[:, None], T[None, :])
+        M, q = _dense_step(mesh, bands, dirs, bcs, T, inv_tau, dt)
+        I_ref = (M @ I.ravel() + q).reshape(I.shape)
+        wts = inv_tau / bands["vg"][:, None]
+        E = np.einsum("bc,d,bdc->c", wts, dirs["w"], I_ref)
+        T_ref = np.array([_bisect_T(bands, W, wts[:, c], E[c]) for c in range(mesh["n_cells"])])
+        I, T, Tr = p.run(I, T, dt, 1, Tr=Tr)
+        assert np.max(np.abs(I / I_ref - 1)) < 1e-13
+        assert np.max(np.abs(T / T_ref - 1)) < 1e-12
