@@ -191,6 +191,13 @@ typedef struct {
      * NULL: NCCL (nccl_unique_id) or no communicator.  EINVAL if the group's
      * size differs from world or an NCCL id is passed too. */
     bte_group *group;
+    /* Temperature-dependent relaxation times only: 0 (default) the rates of a
+     * step are those of the previous step's temperature (DESIGN.md reading
+     * 22: the R2 weights of the solve that produced T^n and the relaxation of
+     * step n use the same rates, so the RTA energy balance is exact); 1 the
+     * literal post-step refresh of the Finch loop (L707-716: I0 and tau both
+     * from the new T), step n relaxes with tau(T^n) (reading 26). */
+    int32_t rates_now;
 } bte_options;
 
 /* Per-context counters since creation / the last bte_reset_stats. Phase

@@ -61,7 +61,7 @@ class Options(C.Structure):
                 ("device", C.c_int32), ("nccl_unique_id", C.c_void_p), ("stream", C.c_void_p),
                 ("flags", C.c_uint32), ("max_spare_slabs", C.c_int32), ("block_threads", C.c_int32),
                 ("band_group", C.c_int32), ("dir_chunk", C.c_int32), ("cell_part", C.c_void_p),
-                ("n_cell_parts", C.c_int32), ("group", C.c_void_p)]
+                ("n_cell_parts", C.c_int32), ("group", C.c_void_p), ("rates_now", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -198,7 +198,8 @@ class Solver:
                  newton_max_iter=50, rank=0, world=1, device=0, nccl_id: bytes | None = None,
                  stream=None, profile=False, max_spare_slabs=0, block_threads=0, band_group=0,
                  generic_faces=False, locality=True, dir_chunk=0, tma=True, box=True,
-                 cell_part=None, n_cell_parts=1, group: Group | None = None, i0_prefactor=True):
+                 cell_part=None, n_cell_parts=1, group: Group | None = None, i0_prefactor=True,
+                 rates_now=False):
         f64 = lambda x: np.ascontiguousarray(x, dtype=np.float64)
         i64 = lambda x: np.ascontiguousarray(x, dtype=np.int64)
         i32 = lambda x: np.ascontiguousarray(x, dtype=np.int32)
@@ -239,6 +240,7 @@ class Solver:
         if group is not None:
             self._group = group  # (kept alive while the context uses it)
             o.group = group.handle.value
+        o.rates_now = int(bool(rates_now))  # (rate law: tau of the step's own T, reading 26)
         o.flags = ((BTE_FLAG_PROFILE if profile else 0) | (BTE_FLAG_GENERIC_FACES if generic_faces else 0)
                    | (0 if tma else BTE_FLAG_NO_TMA) | (0 if box else BTE_FLAG_NO_BOX))
         o.max_spare_slabs, o.block_threads, o.band_group = int(max_spare_slabs), int(block_threads), int(band_group)

@@ -468,6 +468,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     bte_ctx *ctx = new bte_ctx();
     ctx->opt = *o;
     ctx->td = td;
+    ctx->rate_now = td && o->rates_now;
     ctx->dim = m->dim;
     ctx->nd = nd;
     ctx->nb = nb;

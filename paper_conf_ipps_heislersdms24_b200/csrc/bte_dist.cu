@@ -41,7 +41,7 @@ bte_status shard_newton_step(bte_ctx *ctx) {
         return set_err(&ctx->err, "NCCL all-gather failed: %s", e.c_str()), BTE_ENCCL;
     STATUS_TRY(newton_finish(ctx));
     ev_mark(ctx, kPhNewton, false);
-    if (ctx->td) ctx->rsel = 1 - ctx->rsel;
+    if (ctx->td && !ctx->rate_now) ctx->rsel = 1 - ctx->rsel;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
 }

@@ -107,6 +107,7 @@ struct bte_ctx {
     double bgeo[3] = {0, 0, 0};
     int n_orb = 0, box_L = 8, box_stages = 6, box_nbb = 5, box_oc = 20, box_ctas_per_sm = 2;
     bool td = false;  // temperature-dependent relaxation times (rate tables)
+    bool rate_now = false;  // ... of the step's own T (reading 26; else lagged one step, reading 22)
     std::vector<double> h_ra, h_rb, h_rth, h_vg_all, h_inv_tau_all;  // rate law, constants (global rows)
     double *E2 = nullptr, *T2 = nullptr, *cw_diag = nullptr;  // bte_get_temperature_rule scratch
     // band-sharded step (world > 1 with a communicator): reduce-scatter of E,

@@ -26,7 +26,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     double Tw = 0.0;
     if (p.td) {
         Tw = p.tr_step ? T0 : p.Tr[c];  // a step: the rate temperature becomes T^n
-        if (p.tr_step && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
+        if (p.tr_step && !p.tr_now && !p.T_out) p.Tr[c] = T0;  // (chunk solves: newton_finish_kernel stores Tr)
     }
     const Terms t = solve_terms(tb, p, Tw);
     double T = T0;
@@ -75,6 +75,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
         return;
     }
     p.T[c] = T;
+    if (p.td && p.tr_now) p.Tr[c] = T;  // (reading 26: the rates follow T)
     const double iT = 1.0 / T;
     for (int k = 0; k < p.nb_loc; ++k) {
         const int b = p.b_lo + k;
@@ -89,7 +90,7 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
                                      double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
-                                     const int32_t *__restrict__ halt, int32_t *done) {
+                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now) {
     if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
     if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
     const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -101,7 +102,7 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
         t = -t;
     }
     if (k == 0) {
-        if (td) Tr[c] = T[c];
+        if (td) Tr[c] = tr_now ? t : T[c];  // T^n (lagged rates), or the new T (reading 26)
         T[c] = t;
     }
     const int b = b_lo + k;

@@ -1066,6 +1066,7 @@ struct NewtonParams {
     // temperature-dependent relaxation times (N1): 1/tau_b(T) = ra + rb T exp(-rth / T)
     int32_t td;            // 0: constant rates (cw); 1: rate law
     int32_t tr_step;       // 1: a step's solve (rate temperature <- T^n, weights at T^n); 0: weights at Tr
+    int32_t tr_now;        // rates of the current T (reading 26): the rate temperature follows T
     int32_t r2;            // R2 weights rate / v_b (else R1 cw = 1 / v_b)
     const double *ra, *rb, *rth, *inv_v;  // [nb] global
     double *Tr;            // [nc] rate temperature
@@ -1337,7 +1338,7 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
                                      double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
-                                     const int32_t *__restrict__ halt, int32_t *done);
+                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now);
 
 // Rate table of the local rows at temperature T: out[k][c] = 1/tau_{b_lo+k}(T_c).
 __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,

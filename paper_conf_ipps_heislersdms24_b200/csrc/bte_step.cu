@@ -65,7 +65,7 @@ bte_status run_flux_box(bte_ctx *ctx, double dt) {
     p.zside[0] = ctx->bzside[0];
     p.zside[1] = ctx->bzside[1];
     p.rsel_cur = ctx->rsel;
-    p.rsel_next = 1 - ctx->rsel;
+    p.rsel_next = ctx->rate_now ? ctx->rsel : 1 - ctx->rsel;  // (R2 weights of this step's energy)
     p.rate_r2 = ctx->opt.temp_rule == 0;
     p.dt = dt;
     for (int a = 0; a < 3; ++a) p.g[a] = ctx->bgeo[a];
@@ -152,7 +152,7 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.halt = ctx->d_halt;
     if (ctx->td) {
         p.rate_cur = rate_half(ctx, ctx->rsel);
-        p.rate_next = rate_half(ctx, 1 - ctx->rsel);
+        p.rate_next = rate_half(ctx, ctx->rate_now ? ctx->rsel : 1 - ctx->rsel);
         p.rate_r2 = ctx->opt.temp_rule == 0;
     }
     int slot = 0;
@@ -278,7 +278,7 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
             STATUS_TRY(launch_newton_cells(ctx, q));
         }
         ev_mark(ctx, kPhNewton, false);
-        if (ctx->td) ctx->rsel = 1 - ctx->rsel;
+        if (ctx->td && !ctx->rate_now) ctx->rsel = 1 - ctx->rsel;
         return BTE_OK;
     }
     // a re-solve of the current state: one thread per cell, epilogue in place
@@ -299,7 +299,8 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
         q.rth = ctx->d_rth;
         q.inv_v = ctx->d_inv_v;
         q.Tr = ctx->Tr;
-        q.rate_out = rate_half(ctx, step ? ctx->rsel : 1 - ctx->rsel);
+        q.rate_out = rate_half(ctx, (step || ctx->rate_now) ? ctx->rsel : 1 - ctx->rsel);
+        q.tr_now = ctx->rate_now;
     }
     q.nc = ctx->nc;
     q.nb = ctx->nb;
@@ -348,7 +349,8 @@ bte_status newton_finish(bte_ctx *ctx) {
     const int64_t n = (int64_t)ctx->nc * ctx->nb_loc;
     bte::newton_finish_kernel<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(
         ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
-        ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail, ctx->d_halt, ctx->d_done);
+        ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail, ctx->d_halt, ctx->d_done,
+        ctx->rate_now ? 1 : 0);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
@@ -392,7 +394,7 @@ void undo_step_rotation(bte_ctx *ctx) {
         const int nbl = std::min(ctx->n_spare, ctx->nb_loc - *it);
         for (int k = 0; k < nbl; ++k) std::swap(ctx->cur_slot[*it + k], ctx->spare_slot[k]);
     }
-    if (ctx->td) ctx->rsel = 1 - ctx->rsel;
+    if (ctx->td && !ctx->rate_now) ctx->rsel = 1 - ctx->rsel;
 }
 
 // I0 of the current T; with the rate law also Tr = T and both rate halves at T

@@ -185,3 +185,15 @@ def test_group_size_mismatch_is_einval(bte):
         with pytest.raises(bte.BTEError) as e:
             bte.solver_from_config(cfg, rank=0, world=2, group=g)
         assert e.value.status == bte.BTE_EINVAL
+
+
+def test_band_sharding_rates_now(bte, oracle_mod):
+    """Band sharding over 3 ranks with the literal rate bookkeeping (reading
+    26): the chunk solves and the finish kernel keep the rate temperature at T."""
+    cfg = gen.small_3d_config((34, 9, 7), n_spectral=5)
+    law = gen.with_rate_law(cfg.bands)
+    cfg = dataclasses.replace(cfg, bands=law, dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, law, cfg.dirs, t_max=350.0))
+    Io, To = oracle_run(oracle_mod, cfg, 10, rates_now=True)
+    out = run_ranks(bte, cfg, 3, 10, rates_now=True)
+    Ig, Tg = assemble(cfg, out)
+    assert_parity(Ig, Tg, Io, To)

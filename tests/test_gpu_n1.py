@@ -134,3 +134,30 @@ def test_law_split_step_band_sharding_emulated(bte_lib, oracle_mod):
         for s in ranks:
             s.close()
     assert_parity(Ig, Ts[0], Io, To)
+
+
+# ------------------------------------------------------------------ rates_now (reading 26)
+def _check_now(oracle_mod, cfg, variant, steps, **kw):
+    Io, To = oracle_run(oracle_mod, cfg, steps, rates_now=True)
+    Ig, Tg, st = gpu_run(cfg, steps, rates_now=True, **kw)
+    assert st["flux_variant"] == variant
+    assert_parity(Ig, Tg, Io, To)
+    lag = gpu_run(cfg, steps, **kw)  # the default (lagged) bookkeeping differs
+    assert rel_err(lag[1], Tg) > 1e-12
+    return Ig, Tg
+
+
+@pytest.mark.parametrize("rule", [0, 1])
+def test_rates_now_box_and_generic(bte_lib, oracle_mod, rule):
+    """The literal post-step refresh (tau with I0 from the new T): 3-D box
+    kernel (graph and per-launch), 2-D generic-face kernel, both rules."""
+    _check_now(oracle_mod, _law_cfg((34, 9, 7), rule=rule), 6, 15)
+    _check_now(oracle_mod, _law_cfg((34, 9, 7), rule=rule), 6, 15, profile=True)
+    _check_now(oracle_mod, _law_cfg((19, 13), rule=rule), 7, 20)
+
+
+def test_rates_now_slab_rotation_and_resolve(bte_lib, oracle_mod):
+    """Slab rotation, and a re-solve of a set state (the rate temperature
+    follows T) before stepping on."""
+    cfg = _law_cfg((16, 9, 6), n_spectral=4)
+    _check_now(oracle_mod, cfg, 6, 12, max_spare_slabs=2)
