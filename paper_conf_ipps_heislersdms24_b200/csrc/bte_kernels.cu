@@ -141,21 +141,34 @@ __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, i
     }
 }
 
+// E_loc[c] = sum_{local b} c_b sum_d w_d I[b][d][c] of the current state.  A
+// block of 8 warps takes 32 cells (lane = cell: each load is a coalesced row of
+// a plane); warp w takes directions w, w + 8, ...; the warps' sums are added in
+// warp order.  (rate: R2 with the rate law: c_b = rate[k][c] inv_v[k].)
 __global__ void energy_kernel(const double *__restrict__ pool, const int32_t *__restrict__ slot,
                               int64_t slab_elems, int ps, int nb_loc, int nd, int nc,
                               const double4 *__restrict__ dirs, const double *__restrict__ cw,
                               const double *__restrict__ rate, const double *__restrict__ inv_v,
                               double *__restrict__ E) {
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nc) return;
+    __shared__ double red[kSumSlotWarps][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int c = blockIdx.x * 32 + lane;
     double e = 0.0;
-    for (int k = 0; k < nb_loc; ++k) {
-        const double *s = pool + (int64_t)slot[k] * slab_elems;
-        double sb = 0.0;
-        for (int d = 0; d < nd; ++d) sb = fma(dirs[d].w, s[(size_t)d * ps + c], sb);
-        e = fma(rate ? rate[(size_t)k * nc + c] * inv_v[k] : cw[k], sb, e);
+    if (c < nc)
+        for (int k = 0; k < nb_loc; ++k) {
+            const double *s = pool + (int64_t)slot[k] * slab_elems + c;
+            double sb = 0.0;
+            for (int d = w; d < nd; d += kSumSlotWarps) sb = fma(dirs[d].w, s[(size_t)d * ps], sb);
+            e = fma(rate ? rate[(size_t)k * nc + c] * inv_v[k] : cw[k], sb, e);
+        }
+    red[w][lane] = e;
+    __syncthreads();
+    if (w == 0 && c < nc) {
+        double t = red[0][lane];
+#pragma unroll
+        for (int j = 1; j < kSumSlotWarps; ++j) t += red[j][lane];
+        E[c] = t;
     }
-    E[c] = e;
 }
 
 __global__ void i0_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,

@@ -126,9 +126,8 @@ bte_status bte_solve_temperature(bte_ctx *ctx) {
         return set_err(&ctx->err, "world > 1 without a communicator: cannot reduce the energy"), BTE_ESTATE;
     CUDA_TRY(ctx, cudaSetDevice(ctx->device));
     STATUS_TRY(upload_cur_slots(ctx));
-    const int tb = 128;
     const bool law_r2 = ctx->td && ctx->opt.temp_rule == 0;  // weights at the kept rate temperature
-    bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
+    bte::energy_kernel<<<(ctx->nc + 31) / 32, 32 * bte::kSumSlotWarps, 0, ctx->stream>>>(
         ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs, ctx->cw_loc,
         law_r2 ? rate_half(ctx, ctx->rsel) : nullptr, ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E);
     CUDA_TRY(ctx, cudaGetLastError());
@@ -171,8 +170,7 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
                                   ctx->stream));
     STATUS_TRY(upload_cur_slots(ctx));
     const bool law_r2 = ctx->td && rule == 0;
-    const int tb = 128;
-    bte::energy_kernel<<<(ctx->nc + tb - 1) / tb, tb, 0, ctx->stream>>>(
+    bte::energy_kernel<<<(ctx->nc + 31) / 32, 32 * bte::kSumSlotWarps, 0, ctx->stream>>>(
         ctx->pool_cells, ctx->d_cur_slot, ctx->slab_elems, ctx->ps, ctx->nb_loc, ctx->nd, ctx->nc, ctx->dirs,
         ctx->cw_diag + ctx->b_lo, law_r2 ? rate_half(ctx, ctx->rsel) : nullptr,
         ctx->td ? ctx->d_inv_v + ctx->b_lo : nullptr, ctx->E2);
