@@ -940,6 +940,16 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
         if (flat && wall1 && p.zside[(q & 2) ? 1 : 0] == 0) uy[q] = kGhost + ((q & 2) ? kBoxTX : 0) + tx;
     }
     for (int l = 0; l < w.Lc; ++l) eacc[l * kBoxCells + tid] = 0.0;
+    // byte offsets of the staged values inside a stage (one add per shared load)
+    uint32_t own_b[4], ux_b[4], uy_b[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        own_b[q] = (uint32_t)own[q] * 8u;
+        ux_b[q] = (uint32_t)ux[q] * 8u;
+        uy_b[q] = (uint32_t)uy[q] * 8u;
+        // (keep the byte offsets in registers: the loads then address [offset + stage base])
+        asm volatile("" : "+r"(own_b[q]), "+r"(ux_b[q]), "+r"(uy_b[q]));
+    }
     // direct stores: a warp's 32 cells are one 256-byte row of a plane
     const int32_t plane = p.n0 * p.n1;
     const int32_t cell_off = gy * p.n0 + gx;
@@ -948,7 +958,7 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
     uint32_t ph = 0, ob = 0;
     double pv[4] = {0.0, 0.0, 0.0, 0.0};  // the previous layer's own values: this layer's axis-2 upwind values
     for (int k = w.k0; k < w.k1; ++k) {
-        const double kv = p.kv[k];
+        const double kv = p.kv[k], dtit_k = p.dtit[k], cw_k = p.cw[k];  // (per band-row, once)
         double *const oslab = p.pool + (int64_t)p.out_slab[k] * p.slab_elems + cell_off;
         for (int o = w.o0; o < w.o1; ++o) {
             const BoxOrbitC &orb = sorb[o - w.o0];
@@ -957,18 +967,23 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
 #pragma unroll
             for (int q = 0; q < 4; ++q) wq[q] = orb.w[q];
             const double kvout = kv * ((orb.a[0] + orb.a[1]) + orb.a[2]);
-            const double coef_c = (1.0 - p.dtit[k]) - kvout;  // constant rates
+            const double coef_c = (1.0 - dtit_k) - kvout;  // constant rates
             const double m0 = -orb.a[0], m1 = -orb.a[1], m2 = -orb.a[2];
-            int32_t doff[4];  // plane offsets of the orbit's 4 directions (slab_elems < 2^31)
+            // output pointers of the orbit's 4 directions at the first computed layer; they
+            // move one plane per layer in the marching direction (slab_elems < 2^31)
+            double *op[4];
+            const int32_t zfirst = asc ? w.z0 : w.z0 + w.Lc - 1;
+            const int64_t dz = asc ? plane : -(int64_t)plane;
 #pragma unroll
-            for (int q = 0; q < 4; ++q) doff[q] = orb.d[q] * p.ps;
+            for (int q = 0; q < 4; ++q) op[q] = oslab + (orb.d[q] * p.ps + zfirst * plane);
             for (int j = flat ? 1 : 0; j <= w.Lc; ++j) {
                 while (!mbar_try_wait(&full[s], ph)) {
                 }
+                const char *const cb = reinterpret_cast<const char *>(ring + s * kStage);  // this stage
+                auto at = [cb](uint32_t b) { return *reinterpret_cast<const double *>(cb + b); };
                 if (j == 0) {  // the range's upwind layer: its values to registers
-                    const double *cur = ring + s * kStage;
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) pv[q] = cur[own[q]];
+                    for (int q = 0; q < 4; ++q) pv[q] = at(own_b[q]);
                     sp = s;
                 } else {
                     const int z = asc ? w.z0 + j - 1 : w.z0 + w.Lc - j;
@@ -977,26 +992,29 @@ flux_box_kernel(const __grid_constant__ BoxParams p, const __grid_constant__ CUt
                     if (TD) {  // 1/tau_b of this cell at the rate temperature; R2 weight at the next one
                         dtit = p.dt * cur[4 * kBoxPlane + kBoxCells + tid];
                         coef = (1.0 - dtit) - kvout;
-                        cw = p.rate_r2 ? cur[4 * kBoxPlane + 2 * kBoxCells + tid] * p.inv_v[k] : p.cw[k];
+                        cw = p.rate_r2 ? cur[4 * kBoxPlane + 2 * kBoxCells + tid] * p.inv_v[k] : cw_k;
                     } else {
-                        dtit = p.dtit[k];
+                        dtit = dtit_k;
                         coef = coef_c;
-                        cw = p.cw[k];
+                        cw = cw_k;
                     }
                     const double src = dtit * cur[4 * kBoxPlane + tid];
                     double *out = obuf + ob * (4 * kBoxCells);  // (tensor stores)
-                    double *const orow = oslab + z * plane;     // (direct stores)
                     double acc = 0.0;
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
-                        const double ic = cur[own[q]];
-                        double infl = m0 * cur[ux[q]];
-                        infl = fma(m1, cur[uy[q]], infl);
+                        const double ic = at(own_b[q]);
+                        double infl = m0 * at(ux_b[q]);
+                        infl = fma(m1, at(uy_b[q]), infl);
                         if (!flat) infl = fma(m2, pv[q], infl);
                         pv[q] = ic;  // (the next layer's axis-2 upwind value)
                         const double inew = fma(ic, coef, fma(-kv, infl, src));
-                        if constexpr (kTmaStore) out[q * kBoxCells + tid] = inew;
-                        else if (valid) __stcs(orow + doff[q], inew);
+                        if constexpr (kTmaStore) {
+                            out[q * kBoxCells + tid] = inew;
+                        } else {
+                            if (valid) __stcs(op[q], inew);
+                            op[q] += dz;
+                        }
                         acc = fma(wq[q], inew, acc);
                     }
                     double *ea = eacc + (z - w.z0) * kBoxCells + tid;
