@@ -6,8 +6,144 @@
 #include "bte_internal.h"
 #include <map>
 #include <set>
+#include <cstring>
 
 namespace bte_host {
+
+// Shared-memory bank conflicts of the generic TMA kernel.  A warp reads face
+// slot j's upwind values with one 64-bit shared load per band-row, at the staged
+// indices sidx[j][lane]; the hardware serves each half-warp (16 lanes) in as many
+// wavefronts as the most distinct values that share a bank pair (index mod 16),
+// equal values broadcast (measured on B200: C3t 4.5 wavefronts per warp load
+// before, ncu, against 2 without conflicts).
+// cnt[k] = distinct values of v[0..n) in bank class k.
+static void class_counts(const uint16_t *v, int n, int cnt[16]) {
+    for (int k = 0; k < 16; ++k) cnt[k] = 0;
+    for (int a = 0; a < n; ++a) {
+        bool first = true;
+        for (int b = 0; b < a && first; ++b) first = v[b] != v[a];
+        if (first) ++cnt[v[a] & 15];
+    }
+}
+// Wavefronts of a half-warp's loads of every slot (cost) and a smooth version
+// that also rewards evenly spread classes (the local search's objective).
+static void half_costs(const uint16_t (*col)[16], int mf, int n, int *wave, int *smooth) {
+    int w = 0, sm = 0, cnt[16];
+    for (int j = 0; j < mf; ++j) {
+        class_counts(col[j], n, cnt);
+        int mx = 0;
+        for (int k = 0; k < 16; ++k) {
+            mx = std::max(mx, cnt[k]);
+            sm += cnt[k] * cnt[k];
+        }
+        w += mx;
+        sm += 64 * mx;
+    }
+    *wave = w;
+    *smooth = sm;
+}
+
+// The faces of a cell may be summed in any order (Eq. 3's face sum), so per
+// half-warp each cell's faces are permuted among its slots by a local search
+// (best permutation per cell in turn, from the caller's order and from random
+// ones, keeping the fewest wavefronts).  perm[c * mf + j] = the face (old slot)
+// that slot j of cell c takes.  Returns {wavefronts before, after}.
+static std::pair<int64_t, int64_t> order_face_slots(std::vector<uint16_t> &sidx, int32_t nc, int mf,
+                                                    std::vector<uint8_t> &perm) {
+    perm.assign((size_t)nc * mf, 0);
+    for (int32_t c = 0; c < nc; ++c)
+        for (int j = 0; j < mf; ++j) perm[(size_t)c * mf + j] = (uint8_t)j;
+    if (mf > 8) return {0, 0};
+    std::vector<std::array<uint8_t, 8>> perms;  // candidate permutations of a cell's slots
+    {
+        std::array<uint8_t, 8> p{};
+        for (int j = 0; j < mf; ++j) p[j] = (uint8_t)j;
+        if (mf <= 4) {
+            do perms.push_back(p); while (std::next_permutation(p.begin(), p.begin() + mf));
+        } else {
+            perms.push_back(p);
+            for (int a = 0; a < mf; ++a)
+                for (int b = a + 1; b < mf; ++b) {
+                    auto q = p;
+                    std::swap(q[a], q[b]);
+                    perms.push_back(q);
+                }
+        }
+    }
+    const int restarts = nc <= (1 << 18) ? 4 : 1;
+    uint64_t rng = 0x9e3779b97f4a7c15ull;  // (deterministic)
+    auto next = [&rng]() {
+        rng ^= rng << 13;
+        rng ^= rng >> 7;
+        rng ^= rng << 17;
+        return rng;
+    };
+    int64_t before = 0, after = 0;
+    uint16_t orig[16][8], col[8][16], best_col[8][16];
+    uint8_t cur_p[16][8], best_p[16][8];
+    for (int32_t h0 = 0; h0 < nc; h0 += 16) {
+        const int n = std::min<int32_t>(16, nc - h0);
+        for (int l = 0; l < n; ++l)
+            for (int j = 0; j < mf; ++j) {
+                orig[l][j] = sidx[(size_t)j * nc + h0 + l];
+                col[j][l] = orig[l][j];
+                cur_p[l][j] = (uint8_t)j;
+            }
+        int wave, smooth;
+        half_costs(col, mf, n, &wave, &smooth);
+        before += wave;
+        int best_wave = wave;
+        std::memcpy(best_col, col, sizeof(col));
+        std::memcpy(best_p, cur_p, sizeof(cur_p));
+        for (int r = 0; r < restarts; ++r) {
+            for (int l = 0; l < n; ++l) {  // start: the caller's order, then random ones
+                const auto &p = perms[r == 0 ? 0 : next() % perms.size()];
+                for (int j = 0; j < mf; ++j) {
+                    cur_p[l][j] = p[j];
+                    col[j][l] = orig[l][p[j]];
+                }
+            }
+            half_costs(col, mf, n, &wave, &smooth);
+            for (int pass = 0; pass < 6; ++pass) {
+                bool improved = false;
+                for (int l = 0; l < n; ++l) {
+                    int bs = smooth, bw = wave, bi = -1;
+                    for (size_t pi = 0; pi < perms.size(); ++pi) {
+                        for (int j = 0; j < mf; ++j) col[j][l] = orig[l][perms[pi][j]];
+                        int w2, s2;
+                        half_costs(col, mf, n, &w2, &s2);
+                        if (s2 < bs) bs = s2, bw = w2, bi = (int)pi;
+                    }
+                    const uint8_t *p = bi >= 0 ? perms[bi].data() : cur_p[l];
+                    uint8_t keep[8];
+                    for (int j = 0; j < mf; ++j) keep[j] = p[j];
+                    for (int j = 0; j < mf; ++j) {
+                        cur_p[l][j] = keep[j];
+                        col[j][l] = orig[l][keep[j]];
+                    }
+                    if (bi >= 0) {
+                        smooth = bs;
+                        wave = bw;
+                        improved = true;
+                    }
+                }
+                if (!improved) break;
+            }
+            if (wave < best_wave) {
+                best_wave = wave;
+                std::memcpy(best_col, col, sizeof(col));
+                std::memcpy(best_p, cur_p, sizeof(cur_p));
+            }
+        }
+        after += best_wave;
+        for (int l = 0; l < n; ++l)
+            for (int j = 0; j < mf; ++j) {
+                sidx[(size_t)j * nc + h0 + l] = best_col[j][l];
+                perm[(size_t)(h0 + l) * mf + j] = best_p[l][j];
+            }
+    }
+    return {before, after};
+}
 
 thread_local std::string g_err = "no error";
 
@@ -200,7 +336,7 @@ void bte_destroy(bte_ctx *ctx) {
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_flags, ctx->d_smax, ctx->t_th, ctx->t_k, ctx->t_ic, ctx->t_rep, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
-                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls};
+                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->hl_pos, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls, ctx->bl_pos};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -694,71 +830,135 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     ctx->staging_elems = std::min<int64_t>((int64_t)nd * nc, std::max<int64_t>(nc, (int64_t)8 << 20));
     CREATE_TRY(dalloc(ctx, &ctx->staging, (size_t)ctx->staging_elems));
     if (ctx->tma && !paired) {  // generic TMA kernel: per-tile staging lists and shared-memory indices
-        // per tile: own cells [0, 256), halo cells (interior faces pointing out of the
-        // tile) [256, 256 + nh), boundary-face ghosts [256 + nh, 256 + nh + ng)
+        // per tile: own cells at [0, 256), then the halo cells (interior faces pointing
+        // out of the tile) and the boundary-face ghosts at positions of
+        // [256, 256 + cap) placed so that each half-warp's upwind loads spread over the
+        // 16 bank pairs (fewer shared-memory bank conflicts)
         const int32_t ntiles = (nc + bte::kTile - 1) / bte::kTile;
         std::vector<int32_t> hoff(ntiles + 1, 0), hcell, goff(ntiles + 1, 0), gcol, gcls;
-        std::vector<uint16_t> sidx_h(ell, 0);
+        std::vector<std::vector<size_t>> gface(ntiles);  // face slot q of each ghost
         int32_t smax = 0;
-        std::map<int32_t, int32_t> slot_of;
-        std::vector<size_t> bq;
-        for (int32_t t = 0; t < ntiles; ++t) {
-            const int32_t t0 = t * bte::kTile, t1 = std::min(nc, t0 + bte::kTile);
-            slot_of.clear();
-            bq.clear();
-            for (int j = 0; j < mf_t; ++j)
-                for (int32_t i = t0; i < t1; ++i) {
-                    const size_t q = (size_t)j * nc + i;
-                    if (fcode8_h[q] != bte::kCode8Interior) {
-                        bq.push_back(q);
-                        continue;
+        {
+            std::set<int32_t> halo;
+            for (int32_t t = 0; t < ntiles; ++t) {
+                const int32_t t0 = t * bte::kTile, t1 = std::min(nc, t0 + bte::kTile);
+                halo.clear();
+                for (int j = 0; j < mf_t; ++j)
+                    for (int32_t i = t0; i < t1; ++i) {
+                        const size_t q = (size_t)j * nc + i;
+                        if (fcode8_h[q] != bte::kCode8Interior) {
+                            gface[t].push_back(q);
+                            const bool iso = fcode8_h[q] == bte::kCode8Iso;  // Eq. 6: isothermal table column / reflected plane
+                            gcol.push_back(iso ? nbr_h[q] : i);
+                            gcls.push_back(iso ? -1 : (int32_t)fcode8_h[q]);
+                        } else if (nbr_h[q] < t0 || nbr_h[q] >= t0 + bte::kTile) {
+                            halo.insert(nbr_h[q]);
+                        }
                     }
-                    const int32_t v = nbr_h[q];
-                    if (v >= t0 && v < t0 + bte::kTile) {
-                        sidx_h[q] = (uint16_t)(v - t0);
-                    } else {
-                        auto it = slot_of.find(v);
-                        if (it == slot_of.end()) it = slot_of.emplace(v, (int32_t)slot_of.size()).first;
-                        sidx_h[q] = (uint16_t)(bte::kTile + it->second);
-                    }
-                }
-            // halo slots in ascending cell order, so that the producer lanes' gathers
-            // of neighbouring columns fall into shared 32-byte sectors
-            const int32_t nh = (int32_t)slot_of.size();
-            std::vector<int32_t> cells(nh), newpos(nh);
-            {
-                int32_t r = 0;
-                for (const auto &kv : slot_of) {
-                    newpos[kv.second] = r;
-                    cells[r++] = kv.first;
-                }
+                // (halo list in ascending cell order: the producer lanes' gathers of
+                // neighbouring columns fall into shared 32-byte sectors)
+                hcell.insert(hcell.end(), halo.begin(), halo.end());
+                hoff[t + 1] = (int32_t)hcell.size();
+                goff[t + 1] = (int32_t)gcol.size();
+                smax = std::max<int32_t>(smax, (int32_t)halo.size() + (int32_t)gface[t].size());
             }
-            for (int j = 0; j < mf_t; ++j)
-                for (int32_t i = t0; i < t1; ++i) {
-                    const size_t q = (size_t)j * nc + i;
-                    if (fcode8_h[q] == bte::kCode8Interior && sidx_h[q] >= bte::kTile)
-                        sidx_h[q] = (uint16_t)(bte::kTile + newpos[sidx_h[q] - bte::kTile]);
-                }
-            hcell.insert(hcell.end(), cells.begin(), cells.end());
-            hoff[t + 1] = (int32_t)hcell.size();
-            for (size_t g = 0; g < bq.size(); ++g) {  // Eq. 6 ghosts: isothermal table column / reflected plane
-                const size_t q = bq[g];
-                const int32_t i = (int32_t)(q % (size_t)nc);
-                const bool iso = fcode8_h[q] == bte::kCode8Iso;
-                gcol.push_back(iso ? nbr_h[q] : i);
-                gcls.push_back(iso ? -1 : (int32_t)fcode8_h[q]);
-                sidx_h[q] = (uint16_t)(bte::kTile + nh + (int32_t)g);
-            }
-            goff[t + 1] = (int32_t)gcol.size();
-            smax = std::max<int32_t>(smax, nh + (int32_t)bq.size());
         }
         if (smax <= bte::kMaxTileStaged) {
             ctx->hstride = bte::kTile + (smax + 31) / 32 * 32;
+            if (ctx->hstride <= bte::kTileStagedFixed) ctx->hstride = bte::kTileStagedFixed;  // (compile-time stride)
+            const int32_t cap = ctx->hstride - bte::kTile;
+            std::vector<uint16_t> sidx_h(ell, 0);
+            std::vector<int32_t> hpos(hcell.size()), gpos(gcol.size());
+            std::map<int32_t, int32_t> hk;  // halo cell -> its index in the tile's list
+            std::vector<std::vector<int32_t>> readers;
+            std::vector<int32_t> order, freep;
+            for (int32_t t = 0; t < ntiles; ++t) {
+                const int32_t t0 = t * bte::kTile, t1 = std::min(nc, t0 + bte::kTile);
+                const int32_t h0 = hoff[t], nh = hoff[t + 1] - h0, g0 = goff[t], ng = goff[t + 1] - g0;
+                hk.clear();
+                for (int32_t k = 0; k < nh; ++k) hk[hcell[h0 + k]] = k;
+                int deg[bte::kTile / 16][16] = {};  // upwind reads per (half-warp, bank class)
+                readers.assign(nh + ng, {});
+                for (int j = 0; j < mf_t; ++j)
+                    for (int32_t i = t0; i < t1; ++i) {
+                        const size_t q = (size_t)j * nc + i;
+                        const int32_t H = (i - t0) >> 4, v = nbr_h[q];
+                        if (fcode8_h[q] != bte::kCode8Interior) continue;
+                        if (v >= t0 && v < t0 + bte::kTile) {
+                            sidx_h[q] = (uint16_t)(v - t0);
+                            ++deg[H][(v - t0) & 15];
+                        } else {
+                            auto &r = readers[hk[v]];
+                            if (std::find(r.begin(), r.end(), H) == r.end()) r.push_back(H);
+                        }
+                    }
+                for (int32_t g = 0; g < ng; ++g) readers[nh + g].push_back((int32_t)((gface[t][g] % nc) - t0) >> 4);
+                // the most-read values first, each at the free position whose bank class
+                // adds least to the class counts of the half-warps that read it
+                order.resize(nh + ng);
+                for (int32_t k = 0; k < nh + ng; ++k) order[k] = k;
+                std::stable_sort(order.begin(), order.end(),
+                                 [&](int32_t a, int32_t b) { return readers[a].size() > readers[b].size(); });
+                freep.resize(cap);
+                for (int32_t p = 0; p < cap; ++p) freep[p] = bte::kTile + p;
+                for (const int32_t k : order) {
+                    size_t bi = 0;
+                    int bs = INT32_MAX;
+                    for (size_t fi = 0; fi < freep.size(); ++fi) {
+                        int sc = 0;
+                        for (const int32_t H : readers[k]) sc += 2 * deg[H][freep[fi] & 15] + 1;
+                        if (sc < bs) bs = sc, bi = fi;
+                    }
+                    const int32_t p = freep[bi];
+                    freep.erase(freep.begin() + (std::ptrdiff_t)bi);
+                    for (const int32_t H : readers[k]) ++deg[H][p & 15];
+                    if (k < nh) hpos[h0 + k] = p; else gpos[g0 + k - nh] = p;
+                }
+                for (int j = 0; j < mf_t; ++j)
+                    for (int32_t i = t0; i < t1; ++i) {
+                        const size_t q = (size_t)j * nc + i;
+                        const int32_t v = nbr_h[q];
+                        if (fcode8_h[q] == bte::kCode8Interior && (v < t0 || v >= t0 + bte::kTile))
+                            sidx_h[q] = (uint16_t)hpos[h0 + hk[v]];
+                    }
+                for (int32_t g = 0; g < ng; ++g) sidx_h[gface[t][g]] = (uint16_t)gpos[g0 + g];
+            }
+            // faces of each cell permuted among its slots against the remaining conflicts
+            std::vector<uint8_t> perm;
+            const auto wf = order_face_slots(sidx_h, nc, mf_t, perm);
+            if (std::getenv("BTE_DEBUG_SLOTS"))
+                std::fprintf(stderr, "bte: upwind shared-load wavefronts (all half-warps, slots) %lld -> %lld\n",
+                             (long long)wf.first, (long long)wf.second);
+            {
+                std::vector<int32_t> t_nbr(mf_t);
+                std::vector<uint8_t> t_code(mf_t);
+                std::vector<double> t_g(3 * mf_t);
+                for (int32_t i = 0; i < nc; ++i) {
+                    for (int j = 0; j < mf_t; ++j) {
+                        const size_t q = (size_t)perm[(size_t)i * mf_t + j] * nc + i;
+                        t_nbr[j] = nbr_h[q];
+                        t_code[j] = fcode8_h[q];
+                        t_g[3 * j] = gx_h[q];
+                        t_g[3 * j + 1] = gy_h[q];
+                        t_g[3 * j + 2] = gz_h[q];
+                    }
+                    for (int j = 0; j < mf_t; ++j) {
+                        const size_t q = (size_t)j * nc + i;
+                        nbr_h[q] = t_nbr[j];
+                        fcode8_h[q] = t_code[j];
+                        gx_h[q] = t_g[3 * j];
+                        gy_h[q] = t_g[3 * j + 1];
+                        gz_h[q] = t_g[3 * j + 2];
+                    }
+                }
+            }
             CREATE_TRY(upload(ctx, &ctx->hl_off, hoff));
             CREATE_TRY(upload(ctx, &ctx->hl_cell, hcell));
+            CREATE_TRY(upload(ctx, &ctx->hl_pos, hpos));
             CREATE_TRY(upload(ctx, &ctx->bl_off, goff));
             CREATE_TRY(upload(ctx, &ctx->bl_col, gcol));
             CREATE_TRY(upload(ctx, &ctx->bl_cls, gcls));
+            CREATE_TRY(upload(ctx, &ctx->bl_pos, gpos));
             CREATE_TRY(upload(ctx, &ctx->sidx, sidx_h));
         } else {
             ctx->tma = false;  // too much to stage per tile: the register kernel

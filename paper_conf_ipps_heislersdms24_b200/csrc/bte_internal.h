@@ -94,8 +94,8 @@ struct bte_ctx {
     bool paired = false;     // every cell's faces are exact opposite pairs
     bool uniform_g = false;  // ... and every cell has the same g per pair
     bool tma = false;        // 256-thread blocks: the TMA-staged kernel (paired or generic faces)
-    int32_t *hl_off = nullptr, *hl_cell = nullptr;  // generic TMA kernel: per-tile halo lists,
-    int32_t *bl_off = nullptr, *bl_col = nullptr, *bl_cls = nullptr;  // ... boundary-face ghost lists
+    int32_t *hl_off = nullptr, *hl_cell = nullptr, *hl_pos = nullptr;  // generic TMA kernel: per-tile halo lists,
+    int32_t *bl_off = nullptr, *bl_col = nullptr, *bl_cls = nullptr, *bl_pos = nullptr;  // ... ghost lists
     uint16_t *sidx = nullptr;                        // ... per face slot: shared-memory index of the upwind value
     int32_t hstride = 0;
     double gu[3][3] = {};

@@ -80,15 +80,17 @@ struct FluxParams {
     double kv[kMaxBandsPerLaunch];             // dt v_b
     double cw[kMaxBandsPerLaunch];             // temperature weight c_b
     // TMA-staged generic-face kernel: per tile (256 cells) the out-of-tile
-    // upwind cells its interior faces read, then its boundary faces' ghosts,
-    // gathered into the stage behind the tile's own values; per face slot the
-    // shared-memory index of its upwind value
+    // upwind cells its interior faces read and its boundary faces' ghosts,
+    // gathered into the stage behind the tile's own values (at host-chosen
+    // positions >= kTile); per face slot the shared-memory index of its upwind value
     const int32_t *hl_off;   // [n_tiles + 1] halo cells of tile t: [hl_off[t], hl_off[t+1])
     const int32_t *hl_cell;  // plane columns of the halo cells
+    const int32_t *hl_pos;   // their staged positions
     const int32_t *bl_off;   // [n_tiles + 1] boundary-face ghosts of tile t
     const int32_t *bl_col;   // specular: the cell's column; isothermal: the I0w table column
     const int32_t *bl_cls;   // specular class (reflected direction refl[cls][d]); -1: isothermal
-    const uint16_t *sidx;    // [MF][nc] staged index: own tile < kTile <= halo < kTile + nh <= ghosts
+    const int32_t *bl_pos;   // their staged positions
+    const uint16_t *sidx;    // [MF][nc] staged index: own tile < kTile <= halo and ghosts
     int32_t hstride;         // doubles per staged band-row: kTile + halo + ghost capacity
     // ENOCONV stop (bte_step): fail != 0 once a temperature solve of an earlier
     // step of the call failed; the flux launch is then a no-op and block 0
@@ -481,10 +483,15 @@ __device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
 #ifndef BTE_TMA_GENERIC_MIN_BLOCKS
 #define BTE_TMA_GENERIC_MIN_BLOCKS 3
 #endif
-template <int DIM, int MF, int BG, bool TD>
+// HS: the staged band-row stride in doubles when fixed at compile time (the
+// common case kTileStagedFixed: the row offsets become load immediates), 0: p.hstride.
+constexpr int kTileStagedFixed = kTile + 128;
+template <int DIM, int MF, int BG, bool TD, int HS>
 __global__ void __launch_bounds__(kTmaThreads, BTE_TMA_GENERIC_MIN_BLOCKS)
 flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
-    extern __shared__ __align__(128) double ring[];  // [kStagesG][BG][hstride], then double4 dirs[dchunk]
+    // [kStagesG][BG][hstride] ring, double4 dirs[dchunk], then the tile's staging
+    // lists: halo columns and positions [nh], ghost columns, classes, positions [ng]
+    extern __shared__ __align__(128) double ring[];
     __shared__ __align__(8) uint64_t full[kStagesG];
     __shared__ __align__(8) uint64_t empty[kStagesG];
     if (flux_halted(p.fail, p.halt)) return;
@@ -497,9 +504,13 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     const int nit = min(p.nd, d0 + p.dchunk) - d0;
     const int nc = p.nc;
     const int ps = p.ps;
-    const int hs = p.hstride;
+    const int hs = HS ? HS : p.hstride;
     constexpr uint32_t kBytes = BG * kTile * sizeof(double);
     double4 *sdir = reinterpret_cast<double4 *>(ring + kStagesG * BG * hs);  // this chunk's {s, w}
+    int32_t *shl = reinterpret_cast<int32_t *>(sdir + p.dchunk);          // halo columns
+    const int h0 = __ldg(p.hl_off + blockIdx.x), nh = __ldg(p.hl_off + blockIdx.x + 1) - h0;
+    const int g0 = __ldg(p.bl_off + blockIdx.x), ng = __ldg(p.bl_off + blockIdx.x + 1) - g0;
+    int32_t *shp = shl + nh, *sgc = shp + nh, *sgk = sgc + ng, *sgp = sgk + ng;
 
     if (tid == 0) {
 #pragma unroll
@@ -510,12 +521,20 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     for (int i = tid; i < nit; i += kTmaThreads) sdir[i] = load_dir(p.dirs, d0 + i);
+    // the tile's lists, read once per block (every plane of the block gathers the same cells)
+    for (int i = tid; i < nh; i += kTmaThreads) {
+        shl[i] = __ldg(p.hl_cell + h0 + i);
+        shp[i] = __ldg(p.hl_pos + h0 + i);
+    }
+    for (int i = tid; i < ng; i += kTmaThreads) {
+        sgc[i] = __ldg(p.bl_col + g0 + i);
+        sgk[i] = __ldg(p.bl_cls + g0 + i);
+        sgp[i] = __ldg(p.bl_pos + g0 + i);
+    }
     __syncthreads();
 
     if (tid >= kTile) {  // ------------------------------------------ producer warp
         const int lane = tid - kTile;
-        const int h0 = __ldg(p.hl_off + blockIdx.x), nh = __ldg(p.hl_off + blockIdx.x + 1) - h0;
-        const int g0 = __ldg(p.bl_off + blockIdx.x), ng = __ldg(p.bl_off + blockIdx.x + 1) - g0;
         int st = 0;
         uint32_t ph = 0;
         for (int i = 0; i < nit; ++i) {
@@ -532,17 +551,17 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
                     bulk_g2s(sbase + k * hs, p.in_ptr[lg0 + k] + po + tile0, kTile * sizeof(double), &full[st]);
             }
             for (int h = lane; h < nh; h += 32) {  // halo: neighbour cells outside the tile
-                const int col = __ldg(p.hl_cell + h0 + h);
+                const int col = shl[h], pos = shp[h];
 #pragma unroll
-                for (int k = 0; k < BG; ++k) cp_async_8(sbase + k * hs + kTile + h, p.in_ptr[lg0 + k] + po + col);
+                for (int k = 0; k < BG; ++k) cp_async_8(sbase + k * hs + pos, p.in_ptr[lg0 + k] + po + col);
             }
             for (int g = lane; g < ng; g += 32) {  // boundary-face ghosts (Eq. 6, old level)
-                const int col = __ldg(p.bl_col + g0 + g), cls = __ldg(p.bl_cls + g0 + g);
+                const int col = sgc[g], cls = sgk[g], pos = sgp[g];
                 const int64_t off = cls < 0 ? (int64_t)col
                                             : (int64_t)__ldg(p.refl + cls * p.nd + d) * ps + col;
 #pragma unroll
                 for (int k = 0; k < BG; ++k)
-                    cp_async_8(sbase + k * hs + kTile + nh + g,
+                    cp_async_8(sbase + k * hs + pos,
                                (cls < 0 ? p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso : p.in_ptr[lg0 + k]) + off);
             }
             cp_async_mbar_arrive(&full[st]);
@@ -555,16 +574,21 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     const int c = tile0 + tid;
     const bool valid = c < nc;
     const int lane = tid & 31;
-    int sx[MF];  // staged index of each face's upwind value
+    uint32_t sxb[MF];  // byte offset (in a staged band-row) of each face's upwind value
     double gx[MF], gy[MF], gz[MF];
 #pragma unroll
     for (int j = 0; j < MF; ++j) {
         const int q = j * nc + c;
-        sx[j] = valid ? (int)__ldg(p.sidx + q) : tid;
+        sxb[j] = 8u * (valid ? (uint32_t)__ldg(p.sidx + q) : (uint32_t)tid);
         gx[j] = valid ? __ldg(p.gx + q) : 0.0;
         gy[j] = valid ? __ldg(p.gy + q) : 0.0;
         gz[j] = (DIM == 3 && valid) ? __ldg(p.gz + q) : 0.0;
     }
+    uint32_t ownb = 8u * (uint32_t)tid;
+#pragma unroll
+    for (int j = 0; j < MF; ++j) asm volatile("" : "+r"(sxb[j]));  // (loads address [offset + row base])
+    asm volatile("" : "+r"(ownb));
+    const uint32_t rowb = 8u * (uint32_t)hs;  // bytes per staged band-row (HS: a constant)
     // dt/tau I0_b(T_c); TD (rate law): the cell's own rates, else the band's constants
     double src[BG], dtk[TD ? BG : 1], cwk[TD ? BG : 1];
 #pragma unroll
@@ -576,6 +600,9 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
         }
         src[k] = valid ? (TD ? dtk[k] : p.dtit[lg0 + k]) * __ldg(p.i0 + row) : 0.0;
     }
+    double *op[BG];  // this cell's output in the chunk's first plane, one plane per iteration on
+#pragma unroll
+    for (int k = 0; k < BG; ++k) op[k] = p.out_ptr[lg0 + k] + (int64_t)d0 * ps + c;
 
     double e = 0.0;
     int st = 0;
@@ -587,29 +614,35 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
 #pragma unroll
         for (int j = 0; j < MF; ++j) {
             const double a = DIM == 3 ? fma(sd.z, gz[j], fma(sd.y, gy[j], sd.x * gx[j])) : fma(sd.y, gy[j], sd.x * gx[j]);
-            out += fmax(a, 0.0);  // outflow faces carry the cell's own value
-            am[j] = fmin(a, 0.0);
+            am[j] = a > 0.0 ? 0.0 : a;  // (select)
+            out += a - am[j];           // max(alpha_j, 0), exactly: outflow faces carry the cell's own value
         }
         while (!mbar_try_wait(&full[st], ph)) {
         }
-        const double *stage = ring + st * BG * hs;
+        const char *const cb = reinterpret_cast<const char *>(ring + st * BG * hs);
+        // per face one address (stage + offset); the band-rows are k row strides on
+        const char *fa[MF];
+#pragma unroll
+        for (int j = 0; j < MF; ++j) fa[j] = cb + sxb[j];
+        const char *const oa = cb + ownb;
+        auto at = [](const char *a, uint32_t b) { return *reinterpret_cast<const double *>(a + b); };
         double inew[BG];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
-            const double *sk = stage + k * hs;
             double infl = 0.0;
 #pragma unroll
-            for (int j = 0; j < MF; ++j) infl = fma(am[j], sk[sx[j]], infl);
+            for (int j = 0; j < MF; ++j) infl = fma(am[j], at(fa[j], k * rowb), infl);
             const double kv = p.kv[lg0 + k];
             const double dt_tau = TD ? dtk[k] : p.dtit[lg0 + k];
-            inew[k] = fma(sk[tid], (1.0 - dt_tau) - kv * out, fma(-kv, infl, src[k]));
+            inew[k] = fma(at(oa, k * rowb), (1.0 - dt_tau) - kv * out, fma(-kv, infl, src[k]));
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done with the stage
         if (++st == kStagesG) st = 0, ph ^= 1u;
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
-            if (valid) __stcs(p.out_ptr[lg0 + k] + (int64_t)(d0 + i) * ps + c, inew[k]);
+            if (valid) __stcs(op[k], inew[k]);
+            op[k] += ps;
             e = fma((TD ? cwk[k] : p.cw[lg0 + k]) * sd.w, inew[k], e);
         }
     }

@@ -48,13 +48,20 @@ cudaError_t flux_tma_launch_t(dim3 g, dim3, cudaStream_t s, const bte::FluxParam
 }
 
 // TMA-staged generic-face kernel (general meshes): kStages x BG x 2 KB ring.
+template <int DIM, int MF, int BG, bool TD, int HS>
+cudaError_t flux_tma_generic_launch_hs(dim3 g, const bte::FluxParams &p, cudaStream_t s) {
+    const size_t smem = (size_t)bte::kStagesG * BG * p.hstride * sizeof(double) + (size_t)p.dchunk * sizeof(double4) +
+                        3 * (size_t)(p.hstride - bte::kTile) * sizeof(int32_t);  // (+ the tile's staging lists)
+    cudaError_t e = ensure_smem((const void *)bte::flux_tma_generic_kernel<DIM, MF, BG, TD, HS>, smem);
+    if (e != cudaSuccess) return e;
+    bte::flux_tma_generic_kernel<DIM, MF, BG, TD, HS><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
+    return cudaGetLastError();
+}
+// (the staged row stride of the common case as a compile-time constant)
 template <int DIM, int MF, int BG, bool TD>
 cudaError_t flux_tma_generic_launch_td(dim3 g, const bte::FluxParams &p, cudaStream_t s) {
-    const size_t smem = (size_t)bte::kStagesG * BG * p.hstride * sizeof(double) + (size_t)p.dchunk * sizeof(double4);
-    cudaError_t e = ensure_smem((const void *)bte::flux_tma_generic_kernel<DIM, MF, BG, TD>, smem);
-    if (e != cudaSuccess) return e;
-    bte::flux_tma_generic_kernel<DIM, MF, BG, TD><<<g, dim3(bte::kTmaThreads), smem, s>>>(p);
-    return cudaGetLastError();
+    if (p.hstride == bte::kTileStagedFixed) return flux_tma_generic_launch_hs<DIM, MF, BG, TD, bte::kTileStagedFixed>(g, p, s);
+    return flux_tma_generic_launch_hs<DIM, MF, BG, TD, 0>(g, p, s);
 }
 
 template <int DIM, int MF, int BG>

@@ -143,9 +143,11 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     p.dt = dt;
     p.hl_off = ctx->hl_off;
     p.hl_cell = ctx->hl_cell;
+    p.hl_pos = ctx->hl_pos;
     p.bl_off = ctx->bl_off;
     p.bl_col = ctx->bl_col;
     p.bl_cls = ctx->bl_cls;
+    p.bl_pos = ctx->bl_pos;
     p.sidx = ctx->sidx;
     p.hstride = ctx->hstride;
     p.fail = ctx->d_fail;
