@@ -336,7 +336,8 @@ void bte_destroy(bte_ctx *ctx) {
                     ctx->gy, ctx->gz, ctx->refl, ctx->i0w, ctx->twall, ctx->dirs, ctx->cw_loc, ctx->Cb, ctx->theta, ctx->cw_all,
                     ctx->d_iter_max, ctx->d_flags, ctx->d_smax, ctx->t_th, ctx->t_k, ctx->t_ic, ctx->t_rep, ctx->orb, ctx->dirs_box, ctx->side_tab, ctx->side_col,
                     ctx->d_ra, ctx->d_rb, ctx->d_rth, ctx->d_inv_v, ctx->rates, ctx->Tr,
-                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->hl_pos, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls, ctx->bl_pos};
+                    ctx->E2, ctx->T2, ctx->cw_diag, ctx->Echunk, ctx->Tg, ctx->hl_off, ctx->hl_cell, ctx->hl_pos, ctx->sidx, ctx->bl_off, ctx->bl_col, ctx->bl_cls, ctx->bl_pos,
+                    ctx->t_nrow, ctx->fresh};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (auto &pe : ctx->ev_pool) cudaEventDestroy(pe.a), cudaEventDestroy(pe.b);
@@ -1005,6 +1006,16 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             for (int b = 0; b < nb; ++b) k_t[term_of[b]] += cw[b] * Cb_all[b];
         }
         ctx->n_terms = (int)th_t.size();
+        if (ctx->n_terms > 0) {  // rows of a term as a list: rep[j], nrow[rep[j]], ...
+            std::vector<int32_t> nrow(nb, -1), last(ctx->n_terms, -1);
+            for (int b = 0; b < nb; ++b) {
+                int j = 0;
+                while (th_t[j] != theta[b]) ++j;
+                if (last[j] >= 0) nrow[last[j]] = b;
+                last[j] = b;
+            }
+            CREATE_TRY(upload(ctx, &ctx->t_nrow, nrow));
+        }
         CREATE_TRY(upload(ctx, &ctx->t_th, th_t));
         CREATE_TRY(upload(ctx, &ctx->t_k, k_t));
         CREATE_TRY(upload(ctx, &ctx->t_ic, ic_t));
@@ -1013,6 +1024,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(upload(ctx, &ctx->cw_all, cw));
     CREATE_TRY(dalloc(ctx, &ctx->i0w, (size_t)nb_loc * std::max(1, ctx->n_iso)));
     CREATE_TRY(dalloc(ctx, &ctx->d_iter_max, 1));
+    CREATE_TRY(dalloc(ctx, &ctx->fresh, (size_t)nc));
     CREATE_TRY(dalloc(ctx, &ctx->d_flags, 4));
     ctx->d_fail = ctx->d_flags;
     ctx->d_halt = ctx->d_flags + 1;

@@ -34,6 +34,7 @@ bte_status shard_newton_step(bte_ctx *ctx) {
     q.nc = std::max(0, std::min(ctx->chunk, ctx->nc - q.c_lo));
     q.T_out = ctx->Tg;
     q.neg_fail = 1;
+    q.spec = 0;  // (a chunk of cells: the finish kernel refreshes every row after the all-gather)
     if (warp_newton(ctx, q.nc)) STATUS_TRY(launch_newton_warp(ctx, q));
     else STATUS_TRY(launch_newton_cells(ctx, q));
     double *mine = ctx->Tg + (size_t)ctx->gband * ctx->chunk;

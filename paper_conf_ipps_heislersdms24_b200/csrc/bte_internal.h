@@ -139,6 +139,8 @@ struct bte_ctx {
     int n_terms = 0;
     double *t_th = nullptr, *t_k = nullptr, *t_ic = nullptr;  // theta_j, K_j, 1 / C of the representative row
     int32_t *t_rep = nullptr;                                  // representative row (the I0 table of T^n)
+    int32_t *t_nrow = nullptr;                                 // [nb] next row of the same term (-1: none)
+    int8_t *fresh = nullptr;                                   // [nc] I0 stored by the step's solve (lanes path)
     int32_t *d_iter_max = nullptr;
     // d_flags[0] fail (a temperature solve failed), [1] halt (the fail flag as the
     // step's flux launch saw it: the rest of the step is a no-op), [2] steps done
@@ -314,7 +316,7 @@ bte_status launch_newton_cells(bte_ctx *ctx, const bte::NewtonParams &q);
 bte_status launch_newton_warp(bte_ctx *ctx, const bte::NewtonParams &q);
 bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step);
 bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step = true);
-bte_status newton_finish(bte_ctx *ctx);
+bte_status newton_finish(bte_ctx *ctx, const int8_t *fresh = nullptr);
 bte_status reduce_slots(bte_ctx *ctx);
 bte_status read_flags(bte_ctx *ctx, bool *failed, int64_t *ran);
 bte_status check_newton(bte_ctx *ctx);

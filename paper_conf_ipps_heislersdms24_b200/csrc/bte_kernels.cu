@@ -5,7 +5,7 @@
 
 namespace bte {
 
-__global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
+__global__ void __launch_bounds__(128, 8) newton_kernel(const __grid_constant__ NewtonParams p) {
     if (p.halt && *p.halt) return;
     if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);
     extern __shared__ double sm[];
@@ -18,9 +18,23 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     double E;
     if (p.E) {
         E = p.E[cl];
-    } else {
-        E = 0.0;
-        for (int s = 0; s < p.n_slots; ++s) E += p.part[(size_t)s * p.nc + c];
+    } else {  // the slot sum in sum_slots_kernel's order, bit for bit: partial w sums
+              // slots w, w + 8, ... in turn, then the partials in order (8 loads in flight)
+        double e[kSumSlotWarps];
+#pragma unroll
+        for (int w = 0; w < kSumSlotWarps; ++w) e[w] = 0.0;
+        for (int s0 = 0; s0 < p.n_slots; s0 += kSumSlotWarps) {
+            double v[kSumSlotWarps];
+#pragma unroll
+            for (int w = 0; w < kSumSlotWarps; ++w)
+                v[w] = s0 + w < p.n_slots ? __ldcs(p.part + (size_t)(s0 + w) * p.nc + c) : 0.0;
+#pragma unroll
+            for (int w = 0; w < kSumSlotWarps; ++w)
+                if (s0 + w < p.n_slots) e[w] += v[w];
+        }
+        E = e[0];
+#pragma unroll
+        for (int w = 1; w < kSumSlotWarps; ++w) E += e[w];
     }
     const double T0 = p.T[c];
     double Tw = 0.0;
@@ -30,7 +44,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     }
     const Terms t = solve_terms(tb, p, Tw);
     double T = T0;
-    bool ok = false;
+    bool ok = false, fresh = false;  // fresh: the rows' I0 at the accepted T are stored (or unchanged)
     int it = 0;
     const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
@@ -42,13 +56,21 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
             ok = true;
         }
     } else if (E > 0.0 && isfinite(E)) {
+        // Evaluate g and its derivatives at the iterate (the first from the stored I0
+        // table of T^n); accept the iterate once its Newton correction is within
+        // rtol T -- its I0 rows were stored by that evaluation (spec) -- else take a
+        // Householder step (L555-561: a Newton-type solve of the energy equation)
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = (it == 1 && tab) ? g_eval_table(t, p.W, E, T, tab, p.nc_tab) : g_eval(t, p.W, E, T);
-            const double delta = gs.g / gs.gp;
-            const double Tn = T - delta;
+            const bool from_tab = it == 1 && tab, store = p.spec && !from_tab;
+            const Gder d = g_eval_der(t, tb, p, E, T, from_tab ? tab : nullptr, p.nc_tab, store, c);
+            if (fabs(d.g / d.g1) <= p.rtol * T) {
+                ok = true;
+                fresh = from_tab || store;
+                break;
+            }
+            const double Tn = T - householder_step(d);
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
             T = Tn;
-            if (fabs(delta) <= p.rtol * T || fabs(delta) <= p.rtol_q * T) { ok = true; break; }
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
@@ -68,6 +90,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     if (!ok) {
         atomicExch(p.fail, 1);
         T = p.neg_fail ? -T0 : T0;
+        fresh = false;
     }
     atomicMax(p.iter_max, it);
     if (p.T_out) {
@@ -79,7 +102,7 @@ __global__ void newton_kernel(const __grid_constant__ NewtonParams p) {
     const double iT = 1.0 / T;
     for (int k = 0; k < p.nb_loc; ++k) {
         const int b = p.b_lo + k;
-        p.i0[(size_t)k * p.nc + c] = tb.C[b] / expm1(tb.th[b] * iT);
+        if (!fresh) p.i0[(size_t)k * p.nc + c] = tb.C[b] * (1.0 / expm1(tb.th[b] * iT));  // (= the solve's stores, bitwise)
         if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(tb.a[b], tb.b[b], tb.r[b], T);
     }
 }
@@ -90,7 +113,8 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
                                      double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
-                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now) {
+                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now,
+                                     const int8_t *__restrict__ fresh) {
     if (halt && *halt) return;  // (a solve of an earlier step of the call failed)
     if (done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(done, 1);  // the step's last kernel
     const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -106,7 +130,7 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
         T[c] = t;
     }
     const int b = b_lo + k;
-    i0[(size_t)k * nc + c] = Cb[b] / expm1(theta[b] * (1.0 / t));
+    if (!(fresh && fresh[c])) i0[(size_t)k * nc + c] = Cb[b] * (1.0 / expm1(theta[b] * (1.0 / t)));  // (else stored by the solve)
     if (td) rate_out[(size_t)k * nc + c] = tau_rate(ra[b], rb[b], rth[b], t);
 }
 
@@ -129,8 +153,17 @@ __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, i
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int c = blockIdx.x * 32 + lane;
     double e = 0.0;
-    if (c < nc)
-        for (int s = w; s < n_slots; s += kSumSlotWarps) e += part[(size_t)s * nc + c];
+    if (c < nc) {  // (4 loads in flight per thread, summed in slot order)
+        int s = w;
+        for (; s + 3 * kSumSlotWarps < n_slots; s += 4 * kSumSlotWarps) {
+            double v[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[u] = __ldcs(part + (size_t)(s + u * kSumSlotWarps) * nc + c);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) e += v[u];
+        }
+        for (; s < n_slots; s += kSumSlotWarps) e += __ldcs(part + (size_t)s * nc + c);
+    }
     red[w][lane] = e;
     __syncthreads();
     if (w == 0 && c < nc) {
@@ -178,7 +211,7 @@ __global__ void i0_table_kernel(const double *__restrict__ T, int nc, int b_lo, 
     if (c >= nc) return;
     const double iT = 1.0 / T[c];
     for (int k = 0; k < nb_loc; ++k)
-        i0[(size_t)k * nc + c] = Cb[b_lo + k] / expm1(theta[b_lo + k] * iT);
+        i0[(size_t)k * nc + c] = Cb[b_lo + k] * (1.0 / expm1(theta[b_lo + k] * iT));
 }
 
 __global__ void equilibrium_kernel(double *__restrict__ pool, const int32_t *__restrict__ slot,

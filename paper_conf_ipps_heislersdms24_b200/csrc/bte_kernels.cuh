@@ -1104,13 +1104,9 @@ struct NewtonParams {
     double *i0;            // [nb_loc][nc] written for global rows [b_lo, b_lo + nb_loc)
     int32_t b_lo, nb_loc;
     const double *Cb, *theta, *cw;  // [nb] global
+    // an iterate T is accepted when its Newton correction |g / g'| <= rtol T
+    // (reading 25)
     double W, rtol;
-    // Newton converges quadratically near the root: after a step of |dT| <= rtol_q T
-    // the new iterate's error is ~ kappa dT^2 / T with kappa = T |g''| / 2|g'| ~ (x - 2) / 2,
-    // x = theta / T (5 at x = 12); with rtol_q = 0.1 sqrt(rtol) that is below rtol T for
-    // kappa <= 100 (T above ~1 % of the largest theta), so it is accepted without the
-    // confirming evaluation the |dT| <= rtol T test needs (reading 25)
-    double rtol_q;
     int32_t maxit;
     int32_t *iter_max;
     int32_t *fail;
@@ -1141,6 +1137,13 @@ struct NewtonParams {
     int32_t n_terms;
     const double *t_th, *t_k, *t_ic;
     const int32_t *t_rep;
+    const int32_t *t_nrow;  // [nb] the next row of the same term (-1: none)
+    // spec != 0 (this rank holds every row, whole-mesh solve): an evaluation of g at
+    // an iterate T_k also stores I0_b(T_k) = C_b q (the I0 refresh), so a solve that
+    // accepts T_k needs no refresh of its own; fresh[c] (step solves into T_out)
+    // tells newton_finish_kernel that cell c's rows are stored already
+    int32_t spec;
+    int8_t *fresh;
 };
 
 // 1/tau_b(T) of the rate law (N1, L666-669): impurity-like + Umklapp-like terms.
@@ -1160,6 +1163,7 @@ struct Gsum { double g, gp; };
 struct Terms {
     const double *th, *k, *ic;  // per term: theta_j, K_j (nullptr: per row, c_b C_b), 1 / C of its representative
     const int32_t *rep;          // representative row (nullptr: the row itself)
+    const int32_t *nrow;         // the next row of the same term (with rep)
     int n;
     bool law;                    // per-cell weights: K_b = tau_rate(a, b, th, Tw) iv_b C_b
     const double *C, *w, *ra, *rb, *rth, *iv;
@@ -1176,7 +1180,7 @@ struct Terms {
 // representatives.
 struct SolveTables {
     double *C, *th, *w, *a, *b, *r, *v, *ic, *tth, *tk, *tic;
-    int32_t *trep;
+    int32_t *trep, *nrow;
 };
 __device__ __forceinline__ SolveTables solve_tables(double *sm, int nb, int nt) {
     SolveTables t;
@@ -1184,6 +1188,7 @@ __device__ __forceinline__ SolveTables solve_tables(double *sm, int nb, int nt) 
     t.r = sm + 5 * nb; t.v = sm + 6 * nb; t.ic = sm + 7 * nb;
     t.tth = sm + 8 * nb; t.tk = t.tth + nt; t.tic = t.tk + nt;
     t.trep = reinterpret_cast<int32_t *>(t.tic + nt);
+    t.nrow = reinterpret_cast<int32_t *>(t.tic + 2 * nt);  // (after the nt doubles holding trep)
     return t;
 }
 __device__ __forceinline__ void load_solve_tables(const SolveTables &t, const NewtonParams &p) {
@@ -1205,6 +1210,8 @@ __device__ __forceinline__ void load_solve_tables(const SolveTables &t, const Ne
         t.tic[j] = p.t_ic[j];
         t.trep[j] = p.t_rep[j];
     }
+    if (p.t_nrow)
+        for (int b = threadIdx.x; b < p.nb; b += blockDim.x) t.nrow[b] = p.t_nrow[b];
 }
 // The terms of a cell's solve (Tw: the rate temperature of its weights).
 __device__ __forceinline__ Terms solve_terms(const SolveTables &t, const NewtonParams &p, double Tw) {
@@ -1215,6 +1222,7 @@ __device__ __forceinline__ Terms solve_terms(const SolveTables &t, const NewtonP
     q.k = terms ? t.tk : nullptr;
     q.ic = terms ? t.tic : t.ic;
     q.rep = terms ? t.trep : nullptr;
+    q.nrow = t.nrow;
     q.n = terms ? p.n_terms : p.nb;
     q.C = t.C; q.w = t.w; q.ra = t.a; q.rb = t.b; q.rth = t.r; q.iv = t.v;
     q.Tw = Tw;
@@ -1255,7 +1263,78 @@ __device__ __forceinline__ double g_only(const Terms &t, double W, double E, dou
     return W * g - E;
 }
 
-__global__ void newton_kernel(const __grid_constant__ NewtonParams p);
+// g and its first three T-derivatives.  Per term, with q = 1 / expm1(x), x = theta / T,
+// s = q (1 + q), m = (1 + 2 q) x:  d/dT q = s x / T,  d2 = s x (m - 2) / T^2,
+// d3 = s x (m^2 - 6 m + 6 + 2 s x^2) / T^3 (no further exponentials: the
+// Householder step below costs a few FMAs per term on top of Newton's).
+struct Gder { double g, g1, g2, g3; };
+__device__ __forceinline__ void der_term(double K, double q, double x, double &a0, double &a1, double &a2,
+                                         double &a3) {
+    const double sx = q * (1.0 + q) * x, m = fma(2.0 * q, x, x);
+    const double ks = K * sx;
+    a0 = fma(K, q, a0);
+    a1 += ks;
+    a2 = fma(ks, m - 2.0, a2);
+    a3 = fma(ks, fma(m, m - 6.0, 6.0) + 2.0 * sx * x, a3);
+}
+__device__ __forceinline__ Gder der_finish(double W, double E, double T, double a0, double a1, double a2, double a3) {
+    const double it = 1.0 / T;
+    return {W * a0 - E, W * a1 * it, W * a2 * it * it, W * a3 * it * it * it};
+}
+// The correction h (T <- T - h) of Householder's third-order method (convergence
+// order 4): one step from the previous step's I0 table reaches |h| <= rtol T at
+// the next evaluation for the per-step temperature changes of an explicit step
+// (~1e-4 T), so a solve takes that one evaluation.  Newton's correction where the
+// higher-order one is not finite or strays from it (far from the root).
+__device__ __forceinline__ double householder_step(const Gder &d) {
+    const double newton = d.g / d.g1;
+    const double num = 3.0 * d.g * (2.0 * d.g1 * d.g1 - d.g * d.g2);
+    const double den = 6.0 * d.g1 * d.g1 * d.g1 - 6.0 * d.g * d.g1 * d.g2 + d.g * d.g * d.g3;
+    const double h = num / den;
+    return (isfinite(h) && fabs(h - newton) <= 0.5 * fabs(newton)) ? h : newton;
+}
+// I0 of the rows of term j at the iterate (q = 1 / expm1(theta_j / T)): the
+// speculative refresh of an evaluation (NewtonParams::spec), local rows only.
+__device__ __forceinline__ void store_term_rows(const Terms &t, const SolveTables &tb, const NewtonParams &p, int j,
+                                                double q, int c) {
+    for (int b = t.row(j); b >= 0; b = t.rep ? t.nrow[b] : -1) {
+        const int k = b - p.b_lo;
+        if (k >= 0 && k < p.nb_loc) p.i0[(size_t)k * p.nc + c] = tb.C[b] * q;
+    }
+}
+// One evaluation of g, g', g'', g''' at T: from the stored I0 table (tab: I0 at T,
+// q = I0 / C) or with one expm1 per term, storing the rows' I0 (store).  The
+// table loads go in batches of 8 issued together (one thread per cell: 40
+// dependent loads otherwise bound the solve, ncu C4); the sums run in term order.
+constexpr int kTermBatch = 8;
+__device__ __forceinline__ Gder g_eval_der(const Terms &t, const SolveTables &tb, const NewtonParams &p, double E,
+                                           double T, const double *tab, int64_t stride, bool store, int c) {
+    double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
+    const double it = 1.0 / T;
+    if (tab) {
+        for (int j0 = 0; j0 < t.n; j0 += kTermBatch) {
+            double qv[kTermBatch];
+#pragma unroll
+            for (int u = 0; u < kTermBatch; ++u)
+                qv[u] = __ldg(tab + t.row(min(j0 + u, t.n - 1)) * stride);  // (a clamped duplicate is not summed)
+#pragma unroll
+            for (int u = 0; u < kTermBatch; ++u) {
+                const int j = j0 + u;
+                if (j < t.n) der_term(t.K(j), qv[u] * t.ic[j], t.th[j] * it, a0, a1, a2, a3);
+            }
+        }
+    } else {
+        for (int j = 0; j < t.n; ++j) {
+            const double x = t.th[j] * it;
+            const double q = 1.0 / expm1(x);
+            if (store) store_term_rows(t, tb, p, j, q, c);
+            der_term(t.K(j), q, x, a0, a1, a2, a3);
+        }
+    }
+    return der_finish(p.W, E, T, a0, a1, a2, a3);
+}
+
+__global__ void __launch_bounds__(128, 8) newton_kernel(const __grid_constant__ NewtonParams p);
 
 // ---------------------------------------------------------------------------
 // The same per-cell temperature solve with a GROUP of G lanes per cell (the
@@ -1306,9 +1385,32 @@ __device__ __forceinline__ double g_only_group(const Terms &t, const double *kl,
     return W * group_sum<G>(g, mask) - E;
 }
 
+constexpr int kSumSlotWarps = 8;  // sum_slots_kernel: warps per 32 cells
+
+template <int G, int R>
+__device__ __forceinline__ Gder g_eval_der_group(const Terms &t, const SolveTables &tb, const NewtonParams &p,
+                                                 const double *kl, double E, double T, int lane, unsigned mask,
+                                                 const double *tab, int64_t stride, bool store, int c) {
+    double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
+    const double it = 1.0 / T;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int j = lane + G * r;
+        if (j < t.n) {
+            const double x = t.th[j] * it;
+            const double q = tab ? __ldg(tab + t.row(j) * stride) * t.ic[j] : 1.0 / expm1(x);
+            if (store) store_term_rows(t, tb, p, j, q, c);
+            der_term(kl[r], q, x, a0, a1, a2, a3);
+        }
+    }
+    return der_finish(p.W, E, T, group_sum<G>(a0, mask), group_sum<G>(a1, mask), group_sum<G>(a2, mask),
+                      group_sum<G>(a3, mask));
+}
+
 template <int G, int R>
 __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     if (p.halt && *p.halt) return;
+    if (p.done && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.done, 1);  // (the step's last kernel)
     extern __shared__ double sm[];
     const SolveTables tb = solve_tables(sm, p.nb, p.n_terms);
     load_solve_tables(tb, p);
@@ -1321,10 +1423,24 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     double E;
     if (p.E) {
         E = p.E[cl];
-    } else {
-        E = 0.0;
-        for (int s = lane; s < p.n_slots; s += G) E += p.part[(size_t)s * p.nc + c];
-        E = group_sum<G>(E, mask);
+    } else {  // the slot sum in sum_slots_kernel's order, bit for bit: lane w < 8 sums slots
+              // w, w + 8, ...; the partials are then added in lane order (G >= 8)
+        double e = 0.0;
+        if (lane < kSumSlotWarps) {
+            int s = lane;
+            for (; s + 3 * kSumSlotWarps < p.n_slots; s += 4 * kSumSlotWarps) {
+                double v[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) v[u] = __ldcs(p.part + (size_t)(s + u * kSumSlotWarps) * p.nc + c);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) e += v[u];
+            }
+            for (; s < p.n_slots; s += kSumSlotWarps) e += __ldcs(p.part + (size_t)s * p.nc + c);
+        }
+        const int base = (threadIdx.x & 31) & ~(G - 1);  // the group's first lane in the warp
+        E = __shfl_sync(mask, e, base);
+#pragma unroll
+        for (int k = 1; k < kSumSlotWarps; ++k) E += __shfl_sync(mask, e, base + k);
     }
     const double T0 = p.T[c];
     const Terms t = solve_terms(tb, p, p.td ? (p.tr_step ? T0 : p.Tr[c]) : 0.0);  // a step: weights at T^n
@@ -1336,7 +1452,7 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
     }
     const double *tab = p.i0_t0 ? p.i0_t0 + c : nullptr;  // (I0 at T0 of every row)
     double T = T0;
-    bool ok = false;
+    bool ok = false, fresh = false;
     int it = 0;
     if (E > 0.0 && isfinite(E) && p.single) {  // R3: T + (E - E_eq(T)) / C(T)
         const Gsum gs = g_eval_group<G, R>(t, kl, p.W, E, T, lane, mask, tab, p.nc_tab);
@@ -1346,14 +1462,19 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
             T = Tn;
             ok = true;
         }
-    } else if (E > 0.0 && isfinite(E)) {
+    } else if (E > 0.0 && isfinite(E)) {  // (newton_kernel's iteration, the sums over the group)
         for (it = 1; it <= p.maxit; ++it) {
-            const Gsum gs = g_eval_group<G, R>(t, kl, p.W, E, T, lane, mask, it == 1 ? tab : nullptr, p.nc_tab);
-            const double delta = gs.g / gs.gp;
-            const double Tn = T - delta;
+            const bool from_tab = it == 1 && tab, store = p.spec && !from_tab;
+            const Gder d = g_eval_der_group<G, R>(t, tb, p, kl, E, T, lane, mask, from_tab ? tab : nullptr, p.nc_tab,
+                                                  store, c);
+            if (fabs(d.g / d.g1) <= p.rtol * T) {
+                ok = true;
+                fresh = from_tab || store;
+                break;
+            }
+            const double Tn = T - householder_step(d);
             if (!(Tn > 0.0) || !isfinite(Tn)) break;
             T = Tn;
-            if (fabs(delta) <= p.rtol * T || fabs(delta) <= p.rtol_q * T) { ok = true; break; }
         }
         if (!ok) {  // bisection safeguard on a bracket grown from T0
             double lo = T0, hi = T0;
@@ -1371,10 +1492,29 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
             it = p.maxit + 1;
         }
     }
+    if (p.T_out) {  // (chunk solves: newton_finish_kernel completes the step)
+        if (lane == 0) {
+            if (!ok) atomicExch(p.fail, 1);
+            atomicMax(p.iter_max, it);
+            p.T_out[c] = ok ? T : (p.neg_fail ? -T0 : T0);
+            if (p.fresh) p.fresh[c] = (int8_t)(ok && fresh);
+        }
+        return;
+    }
+    // the epilogue of newton_finish_kernel, by the group: T, Tr, and the local rows'
+    // I0 (unless stored by the accepting evaluation) and rates at the new T
+    if (!ok) T = T0;  // (a failed cell keeps T^n)
     if (lane == 0) {
         if (!ok) atomicExch(p.fail, 1);
         atomicMax(p.iter_max, it);
-        p.T_out[c] = ok ? T : (p.neg_fail ? -T0 : T0);
+        if (p.td && (p.tr_now || p.tr_step)) p.Tr[c] = p.tr_now ? T : T0;
+        p.T[c] = T;
+    }
+    const double iT = 1.0 / T;
+    for (int k = lane; k < p.nb_loc; k += G) {
+        const int b = p.b_lo + k;
+        if (!(ok && fresh)) p.i0[(size_t)k * p.nc + c] = tb.C[b] * (1.0 / expm1(tb.th[b] * iT));
+        if (p.td) p.rate_out[(size_t)k * p.nc + c] = tau_rate(tb.a[b], tb.b[b], tb.r[b], T);
     }
 }
 
@@ -1389,7 +1529,8 @@ __global__ void newton_finish_kernel(const double *__restrict__ Tg, double *__re
                                      double *__restrict__ i0, int td, const double *__restrict__ ra,
                                      const double *__restrict__ rb, const double *__restrict__ rth,
                                      double *__restrict__ Tr, double *__restrict__ rate_out, int32_t *fail,
-                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now);
+                                     const int32_t *__restrict__ halt, int32_t *done, int tr_now,
+                                     const int8_t *__restrict__ fresh);
 
 // Rate table of the local rows at temperature T: out[k][c] = 1/tau_{b_lo+k}(T_c).
 __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo, int nb_loc,
@@ -1397,7 +1538,6 @@ __global__ void rate_table_kernel(const double *__restrict__ T, int nc, int b_lo
                                   const double *__restrict__ rth, double *__restrict__ out);
 
 // E[c] = sum_s part[s][c]  (world > 1: the local partial, all-reduced afterwards)
-constexpr int kSumSlotWarps = 8;  // sum_slots_kernel: warps per 32 cells
 __global__ void sum_slots_kernel(const double *__restrict__ part, int n_slots, int nc, double *__restrict__ E,
                                  const int32_t *__restrict__ halt);
 

@@ -187,7 +187,6 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
     q.cw = ctx->cw_diag;
     q.W = ctx->W;
     q.rtol = ctx->opt.newton_rtol;
-    q.rtol_q = 0.1 * std::sqrt(ctx->opt.newton_rtol);
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;

@@ -195,26 +195,30 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     return BTE_OK;
 }
 
-// The step's temperature solve: E (the slot sum, sum_slots_kernel, unless
-// reduced already) -> the per-cell solve.  Small meshes (fewer cells than ~8
-// warps of threads per SM) solve with one warp per cell (newton_lanes_kernel<32>)
-// into Tg, then newton_finish_kernel writes T, Tr, I0 and the rates with one
-// thread per row x cell (C3, 14,400 cells, 0.066 -> 0.039 ms per step on B200
-// with the steps below); larger ones with one thread per cell and the epilogue
-// in the same thread (newton_kernel; C4: 8 lanes per cell 0.16 ms, 4 lanes
-// 0.18, a warp 0.22, a thread 0.14).  The first evaluation of
-// g reads the stored I0 table, the slot sum runs 8 warps per 32 cells.  Re-solves
-// of the current state (step = false) use newton_kernel with its own epilogue.
+// The step's temperature solve, one kernel when this rank holds every band-row:
+// the slot sum E (in sum_slots_kernel's order, bit for bit, unless E was reduced
+// already), the per-cell solve (the first evaluation of g from the stored I0
+// table, Householder steps, the accepting evaluation storing the new I0 rows)
+// and the epilogue (T, Tr, rates; I0 only where not stored).  Small meshes (fewer
+// cells than ~8 warps of threads per SM) take a group of 16 lanes per cell
+// (newton_lanes_kernel), larger ones one thread per cell (newton_kernel).
+// Measured on B200: C3 (14,400 cells) 0.066 ms per step (round 1) -> 0.031;
+// C4 (131,072 cells) 0.155 -> ~0.07.  Band-sharded ranks (a chunk of cells for
+// all rows, the I0 of local rows only) solve into Tg; newton_finish_kernel
+// completes the step after the all-gather.  Re-solves of the current state
+// (step = false) use newton_kernel with its own epilogue.
 // Lanes per cell of the step's solve: 0 = thread per cell (newton_kernel), else
 // a group of G lanes per cell (newton_lanes_kernel).
 int newton_lanes(const bte_ctx *ctx, int ncells) {
     if (ctx->newton_mode) return ctx->newton_mode == 2 ? 0 : ctx->newton_mode;  // (BTE_NEWTON: tests / sweeps)
-    return ncells < 32 * 8 * ctx->sm_count ? 32 : 0;
+    return ncells < 32 * 8 * ctx->sm_count ? 16 : 0;  // (C3: 16 lanes 0.031 ms, 32 lanes 0.042)
 }
 bool warp_newton(const bte_ctx *ctx, int ncells) { return newton_lanes(ctx, ncells) > 0; }
 
 // Band constants in shared memory: C, theta, c_b (+ the four rate-law arrays).
-size_t newton_smem(const bte_ctx *ctx) { return (size_t)(8 * ctx->nb + 4 * ctx->n_terms) * sizeof(double); }
+size_t newton_smem(const bte_ctx *ctx) {
+    return (size_t)(8 * ctx->nb + 4 * ctx->n_terms) * sizeof(double) + (size_t)ctx->nb * sizeof(int32_t);
+}
 
 // Thread-per-cell solve over q.nc cells (block 0 counts the step when q.done).
 bte_status launch_newton_cells(bte_ctx *ctx, const bte::NewtonParams &q) {
@@ -265,6 +269,24 @@ bte_status launch_newton_warp(bte_ctx *ctx, const bte::NewtonParams &q) {
 bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
     ev_mark(ctx, kPhNewton, true);
     if (step) {  // E (the slot sum) -> the solve into Tg -> the epilogue (T, Tr, I0, rates) in parallel
+        if (warp_newton(ctx, ctx->nc) && ctx->nb_loc == ctx->nb && newton_lanes(ctx, ctx->nc) >= bte::kSumSlotWarps) {
+            // one kernel: the slot sum (unless E is given), the group-of-lanes solve and
+            // its epilogue (C3: 3 launches -> 1)
+            bte::NewtonParams q = newton_params(ctx, E_or_null, true);
+            q.done = ctx->d_done;
+            STATUS_TRY(launch_newton_warp(ctx, q));
+            ev_mark(ctx, kPhNewton, false);
+            if (ctx->td && !ctx->rate_now) ctx->rsel = 1 - ctx->rsel;
+            return BTE_OK;
+        }
+        if (!warp_newton(ctx, ctx->nc)) {  // one thread per cell: slot sum, solve and epilogue in one kernel
+            bte::NewtonParams q = newton_params(ctx, E_or_null, true);
+            q.done = ctx->d_done;
+            STATUS_TRY(launch_newton_cells(ctx, q));
+            ev_mark(ctx, kPhNewton, false);
+            if (ctx->td && !ctx->rate_now) ctx->rsel = 1 - ctx->rsel;
+            return BTE_OK;
+        }
         if (!E_or_null) {
             STATUS_TRY(reduce_slots(ctx));
             E_or_null = ctx->E;
@@ -273,8 +295,9 @@ bte_status run_newton(bte_ctx *ctx, const double *E_or_null, bool step) {
         if (warp_newton(ctx, ctx->nc)) {  // solve into Tg, then the epilogue over (row, cell)
             q.T_out = ctx->Tg;
             q.neg_fail = 1;
+            if (q.spec) q.fresh = ctx->fresh;
             STATUS_TRY(launch_newton_warp(ctx, q));
-            STATUS_TRY(newton_finish(ctx));  // (counts the step)
+            STATUS_TRY(newton_finish(ctx, q.fresh));  // (counts the step)
         } else {  // one thread per cell, epilogue in the same thread (C4: 0.13 vs 0.16 ms with the finish)
             q.done = ctx->d_done;
             STATUS_TRY(launch_newton_cells(ctx, q));
@@ -318,7 +341,6 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     q.cw = ctx->cw_all;
     q.W = ctx->W;
     q.rtol = ctx->opt.newton_rtol;
-    q.rtol_q = 0.1 * std::sqrt(ctx->opt.newton_rtol);
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
@@ -327,12 +349,14 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     if (ctx->nb_loc == ctx->nb) {  // this rank's I0 table holds every row at the current T
         q.i0_t0 = ctx->i0;
         q.nc_tab = ctx->nc;
+        q.spec = 1;  // (the accepting evaluation stores the rows' I0: no separate refresh)
     }
     q.n_terms = ctx->n_terms;
     q.t_th = ctx->t_th;
     q.t_k = ctx->t_k;
     q.t_ic = ctx->t_ic;
     q.t_rep = ctx->t_rep;
+    q.t_nrow = ctx->t_nrow;
     return q;
 }
 
@@ -346,13 +370,13 @@ bte_status reduce_slots(bte_ctx *ctx) {
 
 
 // T <- Tg (a negative entry marks a failed cell: flag, keep T^n), Tr <- T^n,
-// I0 and the rate table of the local rows at the new T.
-bte_status newton_finish(bte_ctx *ctx) {
+// I0 (unless fresh[c]: stored by the solve) and the rate table of the local rows at the new T.
+bte_status newton_finish(bte_ctx *ctx, const int8_t *fresh) {
     const int64_t n = (int64_t)ctx->nc * ctx->nb_loc;
     bte::newton_finish_kernel<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(
         ctx->Tg, ctx->T, ctx->nc, ctx->b_lo, ctx->nb_loc, ctx->Cb, ctx->theta, ctx->i0, ctx->td, ctx->d_ra, ctx->d_rb,
         ctx->d_rth, ctx->Tr, ctx->td ? rate_half(ctx, ctx->rsel) : nullptr, ctx->d_fail, ctx->d_halt, ctx->d_done,
-        ctx->rate_now ? 1 : 0);
+        ctx->rate_now ? 1 : 0, fresh);
     ctx->st.kernel_launches++;
     CUDA_TRY(ctx, cudaGetLastError());
     return BTE_OK;
