@@ -303,7 +303,7 @@ struct LaunchPlan {
 struct Segment {
     int off, nbl, bg;
 };
-std::vector<Segment> segments(int nbl, int bg, bool paired);
+std::vector<Segment> segments(const bte_ctx *ctx, int nbl);
 LaunchPlan plan_launch(const bte_ctx *ctx, int nbl, int bg);
 int count_slots(const bte_ctx *ctx);
 

@@ -500,12 +500,12 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     const int grp = blockIdx.y / p.n_dchunks;
     const int dch = blockIdx.y - grp * p.n_dchunks;
     const int lg0 = grp * BG;
+    const int nrows = min(BG, p.nbl - lg0);  // (a ragged last group: rows k >= nrows idle)
     const int d0 = dch * p.dchunk;
     const int nit = min(p.nd, d0 + p.dchunk) - d0;
     const int nc = p.nc;
     const int ps = p.ps;
     const int hs = HS ? HS : p.hstride;
-    constexpr uint32_t kBytes = BG * kTile * sizeof(double);
     double4 *sdir = reinterpret_cast<double4 *>(ring + kStagesG * BG * hs);  // this chunk's {s, w}
     int32_t *shl = reinterpret_cast<int32_t *>(sdir + p.dchunk);          // halo columns
     const int h0 = __ldg(p.hl_off + blockIdx.x), nh = __ldg(p.hl_off + blockIdx.x + 1) - h0;
@@ -545,15 +545,17 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
             const int64_t po = (int64_t)d * ps;
             double *sbase = ring + st * BG * hs;
             if (lane == 0) {
-                mbar_arrive_expect_tx(&full[st], kBytes);
+                mbar_arrive_expect_tx(&full[st], (uint32_t)(nrows * kTile * sizeof(double)));
 #pragma unroll
                 for (int k = 0; k < BG; ++k)
-                    bulk_g2s(sbase + k * hs, p.in_ptr[lg0 + k] + po + tile0, kTile * sizeof(double), &full[st]);
+                    if (k < nrows)
+                        bulk_g2s(sbase + k * hs, p.in_ptr[lg0 + k] + po + tile0, kTile * sizeof(double), &full[st]);
             }
             for (int h = lane; h < nh; h += 32) {  // halo: neighbour cells outside the tile
                 const int col = shl[h], pos = shp[h];
 #pragma unroll
-                for (int k = 0; k < BG; ++k) cp_async_8(sbase + k * hs + pos, p.in_ptr[lg0 + k] + po + col);
+                for (int k = 0; k < BG; ++k)
+                    if (k < nrows) cp_async_8(sbase + k * hs + pos, p.in_ptr[lg0 + k] + po + col);
             }
             for (int g = lane; g < ng; g += 32) {  // boundary-face ghosts (Eq. 6, old level)
                 const int col = sgc[g], cls = sgk[g], pos = sgp[g];
@@ -561,6 +563,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
                                             : (int64_t)__ldg(p.refl + cls * p.nd + d) * ps + col;
 #pragma unroll
                 for (int k = 0; k < BG; ++k)
+                    if (k < nrows)
                     cp_async_8(sbase + k * hs + pos,
                                (cls < 0 ? p.i0w + (int64_t)(p.band0 + lg0 + k) * p.n_iso : p.in_ptr[lg0 + k]) + off);
             }
@@ -593,7 +596,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     double src[BG], dtk[TD ? BG : 1], cwk[TD ? BG : 1];
 #pragma unroll
     for (int k = 0; k < BG; ++k) {
-        const int64_t row = (int64_t)(p.band0 + lg0 + k) * nc + c;
+        const int64_t row = (int64_t)(p.band0 + lg0 + min(k, nrows - 1)) * nc + c;  // (idle rows: a valid row)
         if (TD) {
             dtk[k] = valid ? p.dt * __ldg(p.rate_cur + row) : 0.0;
             cwk[k] = (p.rate_r2 && valid) ? __ldg(p.rate_next + row) * p.inv_v[lg0 + k] : p.cw[lg0 + k];
@@ -602,7 +605,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
     }
     double *op[BG];  // this cell's output in the chunk's first plane, one plane per iteration on
 #pragma unroll
-    for (int k = 0; k < BG; ++k) op[k] = p.out_ptr[lg0 + k] + (int64_t)d0 * ps + c;
+    for (int k = 0; k < BG; ++k) op[k] = p.out_ptr[lg0 + min(k, nrows - 1)] + (int64_t)d0 * ps + c;
 
     double e = 0.0;
     int st = 0;
@@ -629,6 +632,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
         double inew[BG];
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
+            if (k >= nrows) { inew[k] = 0.0; continue; }  // (idle row of a ragged group)
             double infl = 0.0;
 #pragma unroll
             for (int j = 0; j < MF; ++j) infl = fma(am[j], at(fa[j], k * rowb), infl);
@@ -641,6 +645,7 @@ flux_tma_generic_kernel(const __grid_constant__ FluxParams p) {
         if (++st == kStagesG) st = 0, ph ^= 1u;
 #pragma unroll
         for (int k = 0; k < BG; ++k) {
+            if (k >= nrows) continue;
             if (valid) __stcs(op[k], inew[k]);
             op[k] += ps;
             e = fma((TD ? cwk[k] : p.cw[lg0 + k]) * sd.w, inew[k], e);

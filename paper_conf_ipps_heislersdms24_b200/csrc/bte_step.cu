@@ -161,7 +161,7 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
     const dim3 block(ctx->block);
     for (int l0 = 0; l0 < ctx->nb_loc; l0 += ctx->n_spare) {
         const int nbl_batch = std::min(ctx->n_spare, ctx->nb_loc - l0);
-        for (const Segment &sg : segments(nbl_batch, ctx->bg, ctx->paired)) {
+        for (const Segment &sg : segments(ctx, nbl_batch)) {
             const FluxLaunch fn =
                 pick_flux(ctx->dim, ctx->mf_t, sg.bg, ctx->paired, ctx->uniform_g, ctx->tma);
             const LaunchPlan lp = plan_launch(ctx, sg.nbl, sg.bg);
