@@ -759,8 +759,17 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         CREATE_CUDA(cudaMemGetInfo(&free_b, &total_b));
         const size_t other = (size_t)nc * sizeof(double) * (size_t)(3 * nb_loc + 16) + ell * 48 + (64u << 20);
         const size_t reserve = (size_t)1 << 30;
-        while (n_spare > 1 && (size_t)(nb_loc + n_spare) * slab_bytes + other + reserve > free_b) --n_spare;
-        if ((size_t)(nb_loc + n_spare) * slab_bytes + other > free_b) {
+        // + the energy partial slots, whose count follows the batches of n_spare rows
+        auto slot_bytes = [&](int ns) {
+            const int keep = ctx->n_spare;
+            ctx->n_spare = ns;
+            const size_t b = (size_t)count_slots(ctx) * (size_t)nc * sizeof(double);
+            ctx->n_spare = keep;
+            return b;
+        };
+        while (n_spare > 1 && (size_t)(nb_loc + n_spare) * slab_bytes + other + slot_bytes(n_spare) + reserve > free_b)
+            --n_spare;
+        if ((size_t)(nb_loc + n_spare) * slab_bytes + other + slot_bytes(n_spare) > free_b) {
             set_err(&ctx->err, "intensity needs %.1f GB (%d slabs of %.2f GB); %.1f GB free",
                     (nb_loc + n_spare) * slab_bytes / 1e9, nb_loc + n_spare, slab_bytes / 1e9, free_b / 1e9);
             return fail(BTE_ENOMEM);
@@ -778,8 +787,6 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
     CREATE_TRY(dalloc(ctx, &ctx->pool, (size_t)(nb_loc + n_spare) * ctx->slab_elems));
     ctx->pool_cells = ctx->pool + zs.off;
 
-    const int max_slots = count_slots(ctx);
-    CREATE_TRY(dalloc(ctx, &ctx->part, (size_t)max_slots * nc));
     CREATE_TRY(dalloc(ctx, &ctx->i0, (size_t)nb_loc * nc));
     CREATE_TRY(dalloc(ctx, &ctx->T, (size_t)nc));
     // E padded to world x chunk for the reduce-scatter of the sharded step
@@ -965,6 +972,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
             ctx->tma = false;  // too much to stage per tile: the register kernel
         }
     }
+    // energy partial slots (after the kernel choice: the launch segments depend on it)
+    CREATE_TRY(dalloc(ctx, &ctx->part, (size_t)count_slots(ctx) * nc));
     CREATE_TRY(upload(ctx, &ctx->d_cur_slot, ctx->cur_slot));
     CREATE_TRY(upload(ctx, &ctx->nbr, nbr_h));
     CREATE_TRY(upload(ctx, &ctx->nbm, nbm_h));
