@@ -730,18 +730,20 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         ctx->bflat = bx.flat;
         ctx->n_orb = (int)orbs.size();
         // shared memory for 2 CTAs per SM (3-D): ring stages x 12 KB + L x 2 KB energy rows
-        // (rate law: 16 KB stages x 4 layers)
+        // (rate law: 16 KB stages, 5 x 16 + 8 x 2 KB)
         const char *ev = std::getenv("BTE_BOX_STAGES");
         // (2-D, 3 CTAs per SM: 3 stages; orbit chunks of 25 (a C3 slice = 4 chunks).  Measured on B200
         // with the direct stores, round 2: C4 5 stages 7.22 ms, 6 stages 7.63, 4 stages 8.05 -- a
         // deeper ring lets the producer run ahead and the halo rows of the boxes are re-read from
         // DRAM, a shallower one exposes the load latency; C5 5: 52.2 ms, 6: 52.9; C3 3: 0.814 ms,
-        // 4: 0.830, 5: 0.840; the rate law's 16 KB stages: C4 6 stages 8.03 ms, 5: 8.21, 4: 8.85)
-        const int def_stages = bx.flat ? 3 : td ? 6 : 5;
+        // 4: 0.830, 5: 0.840; the rate law's 16 KB stages, C4 with an equilibrium state
+        // (tools/sweep_box.py C4+law): 5 stages x 8 layers 7.38 ms, 6 x 4 7.46, 5 x 4 7.77,
+        // 6 x 6 8.11, 6 x 8 9.69 (one CTA per SM))
+        const int def_stages = bx.flat ? 3 : 5;
         ctx->box_stages = std::max(2, std::min(bte::kBoxMaxStages, ev ? std::atoi(ev) : def_stages));
         if (bx.flat) ctx->box_oc = 25;
         ev = std::getenv("BTE_BOX_L");
-        ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : (td ? 4 : 8)));
+        ctx->box_L = std::max(1, std::min<int>(bx.n[2], ev ? std::atoi(ev) : 8));
         ev = std::getenv("BTE_BOX_NBB");
         if (ev) ctx->box_nbb = std::max(1, std::atoi(ev));
         ev = std::getenv("BTE_BOX_OC");

@@ -3,6 +3,7 @@
 
     python tools/sweep_box.py C4 "5:80 5:60:6:8 1:80 ..."   (band_group:dir_chunk[:stages:L], 0 = auto)
     python tools/sweep_box.py C3:128x120 "..."               (C3's tables on another grid)
+    python tools/sweep_box.py C4+law "..."                   (the rate law, dt as in bench.py --rate-law)
 
 Equilibrium IC (the flux kernel's time does not depend on the values); prints
 the flux-kernel time per step from the library's CUDA events and the fraction
@@ -22,6 +23,8 @@ from paper_conf_ipps_heislersdms24_b200 import bte, inputs as gen  # noqa: E402
 
 def main():
     name = sys.argv[1]
+    law = name.endswith("+law")
+    name = name[:-4] if law else name
     combos = [tuple(int(x) for x in c.split(":")) for c in sys.argv[2].split()]
     steps = int(sys.argv[3]) if len(sys.argv) > 3 else 10
     if ":" in name:  # e.g. "C3:128x120": the config's bands / directions / walls on another grid
@@ -34,6 +37,10 @@ def main():
         cfg = dataclasses.replace(cfg, mesh=mesh, bcs=gen.gen_bcs_fig1(mesh, radius=4 * h))
     else:
         cfg = gen.make_config(name)
+    if law:  # N1: temperature-dependent tau, dt = 0.5 x the bound at the hot wall (bench.py --rate-law)
+        import dataclasses
+        lb = gen.with_rate_law(cfg.bands)
+        cfg = dataclasses.replace(cfg, bands=lb, dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, lb, cfg.dirs, t_max=350.0))
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
     nc, nd, nb = cfg.mesh["n_cells"], cfg.dirs["n_dirs"], cfg.bands["n_bands"]
     for combo in combos:
