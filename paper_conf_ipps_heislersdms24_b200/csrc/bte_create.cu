@@ -760,7 +760,7 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
         size_t free_b = 0, total_b = 0;
         CREATE_CUDA(cudaMemGetInfo(&free_b, &total_b));
         const size_t other = (size_t)nc * sizeof(double) * (size_t)(3 * nb_loc + 16) + ell * 48 + (64u << 20);
-        const size_t reserve = (size_t)1 << 30;
+        const size_t reserve = (size_t)512 << 20;  // (driver / late small allocations; the partial slots are counted)
         // + the energy partial slots, whose count follows the batches of n_spare rows
         auto slot_bytes = [&](int ns) {
             const int keep = ctx->n_spare;

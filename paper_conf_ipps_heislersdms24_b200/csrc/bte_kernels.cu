@@ -63,7 +63,7 @@ __global__ void __launch_bounds__(128, 8) newton_kernel(const __grid_constant__ 
         for (it = 1; it <= p.maxit; ++it) {
             const bool from_tab = it == 1 && tab, store = p.spec && !from_tab;
             const Gder d = g_eval_der(t, tb, p, E, T, from_tab ? tab : nullptr, p.nc_tab, store, c);
-            if (fabs(d.g / d.g1) <= p.rtol * T) {
+            if (fabs(d.g / d.g1) <= p.racc * T) {
                 ok = true;
                 fresh = from_tab || store;
                 break;

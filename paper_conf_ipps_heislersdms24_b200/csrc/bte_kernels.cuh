@@ -1109,9 +1109,11 @@ struct NewtonParams {
     double *i0;            // [nb_loc][nc] written for global rows [b_lo, b_lo + nb_loc)
     int32_t b_lo, nb_loc;
     const double *Cb, *theta, *cw;  // [nb] global
-    // an iterate T is accepted when its Newton correction |g / g'| <= rtol T
-    // (reading 25)
-    double W, rtol;
+    // an iterate T is accepted when its Newton correction |g / g'| <= racc T,
+    // racc = max(rtol / 100, 16 eps): it then lies within ~rtol / 100 of the root
+    // the oracle's |dT| <= rtol T test converges to (reading 25); rtol
+    // bounds the bisection safeguard's bracket
+    double W, rtol, racc;
     int32_t maxit;
     int32_t *iter_max;
     int32_t *fail;
@@ -1472,7 +1474,7 @@ __global__ void newton_lanes_kernel(const __grid_constant__ NewtonParams p) {
             const bool from_tab = it == 1 && tab, store = p.spec && !from_tab;
             const Gder d = g_eval_der_group<G, R>(t, tb, p, kl, E, T, lane, mask, from_tab ? tab : nullptr, p.nc_tab,
                                                   store, c);
-            if (fabs(d.g / d.g1) <= p.rtol * T) {
+            if (fabs(d.g / d.g1) <= p.racc * T) {
                 ok = true;
                 fresh = from_tab || store;
                 break;

@@ -1,5 +1,6 @@
 // bte_state.cu -- getters, setters, re-solves and counters (see bte_internal.h).
 #include "bte_internal.h"
+#include <cfloat>
 
 
 using namespace bte_host;
@@ -187,6 +188,7 @@ bte_status bte_get_temperature_rule(const bte_ctx *cctx, int32_t rule, double *T
     q.cw = ctx->cw_diag;
     q.W = ctx->W;
     q.rtol = ctx->opt.newton_rtol;
+    q.racc = std::max(0.01 * ctx->opt.newton_rtol, 16.0 * DBL_EPSILON);
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;

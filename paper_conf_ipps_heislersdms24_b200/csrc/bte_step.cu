@@ -3,6 +3,7 @@
 // (L407-418, L555-561), the device-side stop after a failed solve, the
 // 2-step CUDA graph, bte_step and the split step.
 #include "bte_internal.h"
+#include <cfloat>
 
 namespace bte_host {
 
@@ -341,6 +342,7 @@ bte::NewtonParams newton_params(bte_ctx *ctx, const double *E_or_null, bool step
     q.cw = ctx->cw_all;
     q.W = ctx->W;
     q.rtol = ctx->opt.newton_rtol;
+    q.racc = std::max(0.01 * ctx->opt.newton_rtol, 16.0 * DBL_EPSILON);
     q.maxit = ctx->opt.newton_max_iter;
     q.iter_max = ctx->d_iter_max;
     q.fail = ctx->d_fail;
