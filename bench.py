@@ -51,18 +51,19 @@ def _peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def _traffic_from_profiles(config, launches_per_step):
+def _traffic_from_profiles(config, alg_bytes_per_step):
     """DRAM bytes (read + write) of the dominant flux kernel per step, like
     `achieved`: the committed `ncu --set full` capture of one launch of this
-    workload (profiles/ncu_flux_summary.json, one entry per config) times the
-    launches of a step.  None if no capture exists for the workload."""
+    workload (profiles/ncu_flux_summary.json, one entry per config) gives its
+    DRAM bytes over the algorithmic bytes of the rows it covered; times the
+    step's algorithmic bytes.  None if no capture exists for the workload."""
     path = os.path.join(ROOT, "profiles", "ncu_flux_summary.json")
     try:
         with open(path) as f:
             d = json.load(f)
         e = d.get(config)
-        if e and e.get("dram_bytes_per_launch"):
-            return float(e["dram_bytes_per_launch"]) * launches_per_step, e.get("source")
+        if e and e.get("traffic_over_alg"):
+            return float(e["traffic_over_alg"]) * alg_bytes_per_step, e.get("source")
     except Exception:
         pass
     return None, None
@@ -347,7 +348,7 @@ def run_ours(args):
     alg_bytes = BYTES_PER_UPDATE * nc_loc * nd * nb_loc  # per step, this rank
     peak, peak_src = _peaks()
     achieved = alg_bytes / t_flux / 1e9 if t_flux > 0 else None
-    traffic, traffic_src = (_traffic_from_profiles(args.config, flux_launches_per_step) if world == 1 and
+    traffic, traffic_src = (_traffic_from_profiles(args.config, alg_bytes) if world == 1 and
                             not args.rate_law else (None, None))
     roof = {"bound": "hbm", "kernel": "bte::flux_*_kernel (all cells; a1+a2+a3)", "achieved": achieved, "peak": peak,
             "unit": "GB/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,

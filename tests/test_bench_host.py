@@ -40,16 +40,18 @@ def test_no_sampler():
 
 
 def test_traffic_per_step_from_profiles(tmp_path, monkeypatch):
-    """roofline.traffic = the committed ncu capture of one flux launch of THIS
-    workload x the flux launches of a step; absent workloads give None."""
+    """roofline.traffic = the DRAM-over-algorithmic ratio of the committed ncu
+    capture of one flux launch of THIS workload x the step's algorithmic bytes
+    (a C5 capture may cover fewer rows than the bench's launches); absent
+    workloads give None."""
     import json
     prof = tmp_path / "profiles"
     prof.mkdir()
     (prof / "ncu_flux_summary.json").write_text(json.dumps(
-        {"C4": {"dram_bytes_per_launch": 4.9e10, "source": "x"}, "C5": {"dram_bytes_per_launch": 6.6e10}}))
+        {"C4": {"traffic_over_alg": 1.02, "source": "x"}, "C5": {"traffic_over_alg": 1.05}}))
     monkeypatch.setattr(bench, "ROOT", str(tmp_path))
-    assert bench._traffic_from_profiles("C4", 1.0) == (4.9e10, "x")
-    assert bench._traffic_from_profiles("C5", 5.0)[0] == 5 * 6.6e10
+    assert bench._traffic_from_profiles("C4", 4.6e10) == (1.02 * 4.6e10, "x")
+    assert bench._traffic_from_profiles("C5", 3.1e11)[0] == 1.05 * 3.1e11
     assert bench._traffic_from_profiles("C3", 1.0) == (None, None)
 
 

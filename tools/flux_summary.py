@@ -2,7 +2,11 @@
 """Build profiles/ncu_flux_summary.json (bench.py's roofline.traffic source):
 one entry per workload from the `ncu --set full` captures of its flux kernel.
 
-    python tools/flux_summary.py TAG C4=profiles/r02_ncu_box_C4.json C5=... C3=... C3t=...
+    python tools/flux_summary.py TAG C4=profiles/r02_ncu_box_C4.json C5=...:10 C3=... C3t=...
+
+(":ROWS": the band-rows the captured launch covers, if not all of the step's --
+C5 at one GPU rotates slabs: 11 rows per launch in the bench, 10 under ncu,
+whose own allocations leave one spare slab less.)
 
 Each input is a tools/ncu_summary.py `full` JSON of ONE flux launch; the entry
 keeps its DRAM bytes (read + write, cold cache), its duration and the
@@ -24,12 +28,17 @@ def main():
     tag = sys.argv[1]
     out = {"note": "ncu --set full --clock-control none of one flux launch per workload (cold cache); "
                    "bench.py: roofline.traffic = dram_bytes_per_launch x flux launches per step",
-           "round": tag}
+           "round": tag,
+           "use": "bench.py: roofline.traffic = traffic_over_alg x the step's algorithmic bytes"}
     for spec in sys.argv[2:]:
         cfg_name, path = spec.split("=", 1)
+        rows = None
+        if ":" in path:
+            path, r = path.rsplit(":", 1)
+            rows = int(r)
         d = json.load(open(path))
         cfg = gen.make_config(cfg_name)
-        rows = ROWS_IN_LAUNCH.get(cfg_name, cfg.bands["n_bands"])
+        rows = rows or ROWS_IN_LAUNCH.get(cfg_name, cfg.bands["n_bands"])
         alg = 16.0 * cfg.mesh["n_cells"] * cfg.dirs["n_dirs"] * rows
         k = [k for k in d["kernels"] if "flux" in k["name"]][0]
         out[cfg_name] = {"source": os.path.relpath(path, ROOT), "flux_kernel": k["name"],
