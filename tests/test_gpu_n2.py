@@ -81,3 +81,16 @@ def test_split_faces_3d_generic(bte_lib, oracle_mod):
         Ig, Tg, st = gpu_run(cfg, 10, tma=tma)
         assert st["flux_variant"] == v
         assert_parity(Ig, Tg, Io, To)
+
+
+def test_c3t_full_size_bench_launch(bte_lib, oracle_mod):
+    """C3t exactly as the bench runs it (28,800 triangles, 55 rows x 400
+    directions: the TMA-staged generic kernel with its bank-conflict-aware
+    staging positions and face-slot order, 13 groups of 4 rows + a ragged
+    group of 3 in one launch), seeded IC, 3 steps, every element."""
+    cfg = gen.make_config("C3t")
+    Io, To = oracle_run(oracle_mod, cfg, 3)
+    Ig, Tg, st = gpu_run(cfg, 3)
+    assert st["flux_variant"] == 7 and st["band_group"] == 4
+    assert st["flux_launches"] == 3  # (one launch per step)
+    assert_parity(Ig, Tg, Io, To)
