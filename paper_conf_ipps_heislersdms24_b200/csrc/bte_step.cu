@@ -212,7 +212,13 @@ bte_status run_flux(bte_ctx *ctx, double dt) {
 // a group of G lanes per cell (newton_lanes_kernel).
 int newton_lanes(const bte_ctx *ctx, int ncells) {
     if (ctx->newton_mode) return ctx->newton_mode == 2 ? 0 : ctx->newton_mode;  // (BTE_NEWTON: tests / sweeps)
-    return ncells < 32 * 8 * ctx->sm_count ? 16 : 0;  // (C3: 16 lanes 0.031 ms, 32 lanes 0.042)
+    if (ncells >= 32 * 8 * ctx->sm_count) return 0;
+    // the most lanes (8 .. 32) that keep ~1,600 threads per SM (measured on B200, step
+    // solve: C3's 14,400 cells 16 lanes 0.031 ms, 8: 0.034, 32: 0.043; C3t's 28,800
+    // cells 8 lanes 0.052 ms, 16: 0.058, 32: 0.073)
+    int g = 32;
+    while (g > 8 && (int64_t)ncells * g > (int64_t)1600 * ctx->sm_count) g /= 2;
+    return g;
 }
 bool warp_newton(const bte_ctx *ctx, int ncells) { return newton_lanes(ctx, ncells) > 0; }
 
