@@ -962,6 +962,43 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                     }
                 }
             }
+            // the kernel indexes shared memory with these lists: check them (after the face-slot order: every
+            // staged index inside the row, each tile's halo / ghost positions distinct and
+            // inside [kTile, hstride), a face's index = its upwind value's position)
+            {
+                std::vector<int32_t> owner(cap);
+                for (int32_t t = 0; t < ntiles; ++t) {
+                    const int32_t t0 = t * bte::kTile, t1 = std::min(nc, t0 + bte::kTile);
+                    std::fill(owner.begin(), owner.end(), -1);
+                    bool ok = true;
+                    for (int32_t k = hoff[t]; k < hoff[t + 1] && ok; ++k) {
+                        const int32_t p = hpos[k] - bte::kTile;
+                        ok = p >= 0 && p < cap && owner[p] < 0;
+                        if (ok) owner[p] = k;
+                    }
+                    for (int32_t g = goff[t]; g < goff[t + 1] && ok; ++g) {
+                        const int32_t p = gpos[g] - bte::kTile;
+                        ok = p >= 0 && p < cap && owner[p] < 0;
+                        if (ok) owner[p] = (int32_t)hcell.size() + g;
+                    }
+                    for (int j = 0; j < mf_t && ok; ++j)
+                        for (int32_t i = t0; i < t1 && ok; ++i) {
+                            const size_t q = (size_t)j * nc + i;
+                            const int32_t v = nbr_h[q], s = sidx_h[q];
+                            if (fcode8_h[q] != bte::kCode8Interior)
+                                ok = s >= bte::kTile && s < ctx->hstride && owner[s - bte::kTile] >= (int32_t)hcell.size();
+                            else if (v >= t0 && v < t0 + bte::kTile)
+                                ok = s == v - t0 && v < nc;
+                            else
+                                ok = s >= bte::kTile && s < ctx->hstride && owner[s - bte::kTile] >= 0 &&
+                                     owner[s - bte::kTile] < (int32_t)hcell.size() && hcell[owner[s - bte::kTile]] == v;
+                        }
+                    if (!ok) {
+                        set_err(&ctx->err, "internal: inconsistent shared-memory staging lists of tile %d", t);
+                        return fail(BTE_EINVAL);
+                    }
+                }
+            }
             CREATE_TRY(upload(ctx, &ctx->hl_off, hoff));
             CREATE_TRY(upload(ctx, &ctx->hl_cell, hcell));
             CREATE_TRY(upload(ctx, &ctx->hl_pos, hpos));
