@@ -289,9 +289,14 @@ def test_split_step_band_sharding_emulated(bte, oracle_mod):
     assert_parity(Ig, Ts[0], Io, To)
 
 
-def test_nccl_allreduce_path_one_rank(bte):
-    """The NCCL code path (dlopen, ncclCommInitRank, per-step ncclAllReduce of E)
-    on a one-rank communicator: bitwise equal to the fused single-GPU path."""
+@pytest.mark.parametrize("newton", ["auto", "thread", "lanes8", "warp"])
+def test_nccl_allreduce_path_one_rank(bte, monkeypatch, newton):
+    """The NCCL code path (dlopen, ncclCommInitRank, per-step ncclAllReduce of E
+    summed by sum_slots_kernel) on a one-rank communicator: bitwise equal to the
+    fused single-GPU path, whose solve kernel sums the energy slots itself (in
+    sum_slots_kernel's order) -- for the thread-per-cell and the 8 / 32-lane solves."""
+    if newton != "auto":
+        monkeypatch.setenv("BTE_NEWTON", newton)
     cfg = _cfg("C2", steps=5)
     a = gpu_run(cfg, 5)
     b = gpu_run(cfg, 5, nccl_id=bte.nccl_unique_id(), profile=True)
