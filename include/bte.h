@@ -147,8 +147,12 @@ typedef struct {
                                  energy-equivalent temperature); 2: R3, one linearised
                                  "first-law" step T + dE / C(T) with the R1 weights per step
                                  (L413-415; reading 5) */
-    double newton_rtol;       /* stop when |dT| <= rtol T (default 1e-12) */
-    int32_t newton_max_iter;  /* default 50; bisection fallback after that */
+    double newton_rtol;       /* temperature solve tolerance (default 1e-12; L555-561): an
+                                 iterate T is accepted once its Newton correction
+                                 |g/g'| <= max(rtol/100, 16 eps) T, i.e. within ~rtol/100
+                                 of the root the oracle's |dT| <= rtol T test converges to
+                                 (reading 25); the bisection bracket to rtol T */
+    int32_t newton_max_iter;  /* default 50 (evaluations); bisection fallback after that */
     int32_t rank, world;      /* band sharding; world == 1: single GPU, no NCCL */
     int32_t device;           /* CUDA device ordinal */
     const void *nccl_unique_id; /* world > 1: 128-byte ncclUniqueId from bte_nccl_unique_id()
