@@ -837,8 +837,8 @@ bte_status bte_create(const bte_mesh *m, const bte_bands *bd, const bte_dirs *dr
                             const int32_t v = nbr_h[q], s = sidx_h[q];
                             if (fcode8_h[q] != bte::kCode8Interior)
                                 ok = s >= bte::kTile && s < ctx->hstride && owner[s - bte::kTile] >= (int32_t)hcell.size();
-                            else if (v >= t0 && v < t0 + bte::kTile)
-                                ok = s == v - t0 && v < nc;
+                            else if (v >= t0 && v < t0 + bte::kTile)  // (incl. halo columns >= nc of a cell part)
+                                ok = s == v - t0 && v < ctx->ps;
                             else
                                 ok = s >= bte::kTile && s < ctx->hstride && owner[s - bte::kTile] >= 0 &&
                                      owner[s - bte::kTile] < (int32_t)hcell.size() && hcell[owner[s - bte::kTile]] == v;
