@@ -4,6 +4,7 @@ and in the CPU oracle side by side, compared element by element every CHECK
 steps (max relative error on I and T).  Test infrastructure (loads oracle/).
 
     python tools/long_parity.py C3 1000 100      (BASELINE.json configs[2]: 1000 steps)
+    python tools/long_parity.py C4 100 25        (the bench's workload at the north star's 100 steps)
 """
 import os
 import sys
@@ -37,8 +38,9 @@ def main():
             s.step(cfg.dt, k)
             Ig, Tg = s.intensity(), s.temperature()
             done += k
-            ei = float(np.max(np.abs(Ig / I - 1.0)))
-            et = float(np.max(np.abs(Tg / T - 1.0)))
+            ei = max(float(np.max(np.abs(Ig[b] / I[b] - 1.0))) for b in range(I.shape[0]))  # (row by row: C4's
+            et = float(np.max(np.abs(Tg / T - 1.0)))                                         #  state is 23 GB)
+            del Ig
             worst_i, worst_t = max(worst_i, ei), max(worst_t, et)
             print(f"step {done:5d}: max rel err I {ei:.3e}  T {et:.3e}   T in [{T.min():.4f}, {T.max():.4f}] K"
                   f"   (oracle {t1 - t0:.1f} s)", flush=True)
