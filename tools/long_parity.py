@@ -5,6 +5,7 @@ steps (max relative error on I and T).  Test infrastructure (loads oracle/).
 
     python tools/long_parity.py C3 1000 100      (BASELINE.json configs[2]: 1000 steps)
     python tools/long_parity.py C4 100 25        (the bench's workload at the north star's 100 steps)
+    python tools/long_parity.py C4+law 40 20     (with temperature-dependent relaxation times)
 """
 import os
 import sys
@@ -21,7 +22,12 @@ from paper_conf_ipps_heislersdms24_b200 import bte, inputs as gen  # noqa: E402
 
 def main():
     name, n, check = sys.argv[1], int(sys.argv[2]), int(sys.argv[3])
-    cfg = gen.make_config(name)
+    law = name.endswith("+law")  # N1: tau(T), dt as in bench.py --rate-law
+    cfg = gen.make_config(name[:-4] if law else name)
+    if law:
+        import dataclasses
+        lb = gen.with_rate_law(cfg.bands)
+        cfg = dataclasses.replace(cfg, bands=lb, dt=0.5 * gen.cartesian_dt_bound(cfg.mesh, lb, cfg.dirs, t_max=350.0))
     p = oracle.problem_from_config(cfg)
     I, T, Tr = p.initial_state(cfg.t_init, ic_eps=cfg.ic_eps, with_tr=True, mult_fn=getattr(cfg, "ic_mult", None))
     print(f"{name}: {cfg.mesh['n_cells']} cells x {cfg.dirs['n_dirs']} dirs x {cfg.bands['n_bands']} rows, "
