@@ -5,6 +5,7 @@
 # usage: bash tools/gpu_final_r2.sh TAG [quick]
 cd $GRAFT_REPO_ROOT
 OUT=gpurun_out/${1:-r02}; mkdir -p $OUT
+MODE=$2  # (the loops below reuse the positional parameters)
 nvidia-smi -q | grep -i -A3 "clocks$" > $OUT/clocks_before.txt 2>&1
 timeout 2400 python -m pytest tests -m gpu -q --timeout 1500 > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $OUT/pytest_gpu.log
 tail -3 $OUT/pytest_gpu.log
@@ -30,6 +31,6 @@ for c in C4 C3; do  # the temperature-solve kernels
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"newton|sum_slots" -s 3 -c 1 -o $OUT/newton_$c $B --steps 1 --config $c > $OUT/ncu_newton_$c.log 2>&1
   ncu -i $OUT/newton_$c.ncu-rep --page raw --csv > $OUT/raw_newton_$c.csv 2>/dev/null; rm -f $OUT/newton_$c.ncu-rep
 done
-if [ "$2" != "quick" ]; then bash tools/gpu_sanitize.sh $(basename $OUT)/san; fi
+if [ "$MODE" != "quick" ]; then bash tools/gpu_sanitize.sh $(basename $OUT)/san; fi
 du -sh $OUT
 echo done
