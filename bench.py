@@ -348,8 +348,8 @@ def run_ours(args):
     alg_bytes = BYTES_PER_UPDATE * nc_loc * nd * nb_loc  # per step, this rank
     peak, peak_src = _peaks()
     achieved = alg_bytes / t_flux / 1e9 if t_flux > 0 else None
-    traffic, traffic_src = (_traffic_from_profiles(args.config, alg_bytes) if world == 1 and
-                            not args.rate_law else (None, None))
+    traffic, traffic_src = (_traffic_from_profiles(args.config + ("+law" if args.rate_law else ""), alg_bytes)
+                            if world == 1 else (None, None))
     roof = {"bound": "hbm", "kernel": "bte::flux_*_kernel (all cells; a1+a2+a3)", "achieved": achieved, "peak": peak,
             "unit": "GB/s", "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "peak_source": peak_src, "traffic_source": traffic_src,

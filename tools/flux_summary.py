@@ -37,7 +37,7 @@ def main():
             path, r = path.rsplit(":", 1)
             rows = int(r)
         d = json.load(open(path))
-        cfg = gen.make_config(cfg_name)
+        cfg = gen.make_config(cfg_name[:-4] if cfg_name.endswith("+law") else cfg_name)  # (C4+law: the rate law)
         rows = rows or ROWS_IN_LAUNCH.get(cfg_name, cfg.bands["n_bands"])
         alg = 16.0 * cfg.mesh["n_cells"] * cfg.dirs["n_dirs"] * rows
         k = [k for k in d["kernels"] if "flux" in k["name"]][0]
