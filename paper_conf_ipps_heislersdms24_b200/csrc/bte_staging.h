@@ -20,12 +20,18 @@ namespace bte_host {
 // equal values broadcast (measured on B200: C3t 4.5 wavefronts per warp load
 // before, ncu, against 2 without conflicts).
 // cnt[k] = distinct values of v[0..n) in bank class k.
+// (staged indices are < 1024: kTile + kMaxTileStaged; a 1024-bit set marks the seen ones)
 inline void class_counts(const uint16_t *v, int n, int cnt[16]) {
+    uint64_t seen[16] = {};
     for (int k = 0; k < 16; ++k) cnt[k] = 0;
     for (int a = 0; a < n; ++a) {
-        bool first = true;
-        for (int b = 0; b < a && first; ++b) first = v[b] != v[a];
-        if (first) ++cnt[v[a] & 15];
+        const uint32_t x = v[a];
+        uint64_t &w = seen[(x >> 6) & 15];
+        const uint64_t bit = 1ull << (x & 63);
+        if (!(w & bit)) {
+            w |= bit;
+            ++cnt[x & 15];
+        }
     }
 }
 // Wavefronts of a half-warp's loads of every slot (cost) and a smooth version
